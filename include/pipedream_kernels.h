@@ -1,0 +1,64 @@
+/*
+ * pipedream_kernels.h -- kernel-level entry points of libpipedream.so, for kernel parity
+ * tests and micro-benchmarks.  Same conventions as pipedream.h, except that every pointer
+ * here is a DEVICE pointer owned by the caller and the call is asynchronous on `stream`
+ * (a cudaStream_t passed as void*; NULL = legacy default stream).
+ */
+#ifndef PIPEDREAM_KERNELS_H
+#define PIPEDREAM_KERNELS_H
+
+#include "pipedream.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* C(m, n) = sum_k A(m, k) B(n, k) for 0 <= m < M, 0 <= n < N, 0 <= k < K, fp32 accumulation.
+ *   A(m, k) = a_mn_major ? A[k*lda + m] : A[m*lda + k]      (row-major storage, element units)
+ *   B(n, k) = b_mn_major ? B[k*ldb + n] : B[n*ldb + k]
+ * This one contraction is the forward (X W^T), input gradient (G W) and weight gradient
+ * (G^T X) of a linear layer; the epilogue is fused:
+ *   PD_EPI_STORE  out[m*ldo+n] = act(C + bias[n])            (dtype of the path)
+ *   PD_EPI_MASK   out[m*ldo+n] = C * (mask[m*ldm+n] > 0)     (ReLU derivative from its output)
+ *   PD_EPI_F32    out[m*ldo+n] = C                           (fp32, e.g. replica gradients)
+ *   PD_EPI_SGD    master[i] -= lr*C; slot[i] = bf16(master[i]), i = m*ldo+n  (bf16 only)
+ *   PD_EPI_ADAM   Adam(step) on master/adam_m/adam_v; slot[i] = bf16(master[i]) (bf16 only)
+ * dtype PD_BF16 runs the tcgen05/TMEM/TMA kernel (A, B, out, mask, slot bf16; rows 16-byte
+ * aligned); PD_FP32 the SIMT fp32 kernel (STORE/MASK/F32 only).
+ * Errors: PD_EINVAL (bad sizes/epilogue), PD_ECUDA (launch failure). */
+typedef enum { PD_EPI_STORE = 0, PD_EPI_MASK = 1, PD_EPI_F32 = 2, PD_EPI_SGD = 3, PD_EPI_ADAM = 4 } pd_epilogue;
+
+typedef struct {
+    int dtype;
+    int M, N, K;
+    const void *A;
+    long lda;
+    int a_mn_major;
+    const void *B;
+    long ldb;
+    int b_mn_major;
+    int epilogue;
+    void *out;
+    long ldo;
+    const float *bias;
+    int relu;
+    const void *mask;
+    long ldm;
+    float *master;
+    void *slot;
+    float *adam_m, *adam_v;
+    float lr, beta1, beta2, eps;
+    int step;
+} pd_gemm_desc;
+
+PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *g, void *stream);
+
+/* Mean softmax cross-entropy over `rows` rows of C logits (dtype of the path), labels int32;
+ * dlogits = (softmax - onehot) / rows; *loss (device fp32) += mean loss. */
+PD_API pd_status pd_kernel_softmax_ce(int dtype, const void *logits, const int32_t *labels, long rows, int C,
+                                      void *dlogits, float *loss, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,488 @@
+// gemm_tc.cu -- bf16 x bf16 -> fp32 GEMM on the 5th-generation tensor cores (sm_100a).
+//
+//   C(m, n) = sum_k A(m, k) B(n, k), A/B each K-major or MN-major (so the forward
+//   X W^T, the input gradient G W and the weight gradient G^T X of a linear layer all run
+//   without transposes), with the layer epilogues fused:
+//     EPI_STORE  out = act(acc + bias)            bf16   (forward; may be a peer pointer)
+//     EPI_MASK   out = acc * (mask > 0)           bf16   (dX fused with ReLU derivative)
+//     EPI_F32    out = acc                        fp32   (gradient for replica allreduce)
+//     EPI_SGD    master -= lr acc; slot = bf16(master)   (dW fused with the update that
+//     EPI_ADAM   Adam on master, m, v; slot = bf16(master) writes the next weight version)
+//
+// Structure (persistent, warp-specialised, one CTA per SM):
+//   warp 0      TMA producer: cp.async.bulk.tensor 2-D tiles, 128B swizzle, into a
+//               STAGES-deep shared-memory ring guarded by full/empty mbarriers;
+//   warp 1      MMA issuer: one elected thread issues tcgen05.mma.cta_group::1.kind::f16
+//               (M = 128, N = BN, K = 16) into a double-buffered TMEM accumulator and
+//               tcgen05.commit's the smem slot / accumulator barriers;
+//   warp 2      TMEM allocator (2 * BN columns);
+//   warps 4..7  epilogue: tcgen05.ld 32 lanes x 32 columns -> registers -> fused op ->
+//               16-byte global stores, overlapping the next tile's MMAs.
+#include <cuda.h>
+#include <cuda_bf16.h>
+
+#include <cstdio>
+
+#include "pd_internal.h"
+
+namespace pd {
+namespace {
+
+constexpr int BM = 128;
+constexpr int BK = 64;  // 64 bf16 = 128 B = one swizzle row
+constexpr int UMMA_K = 16;
+constexpr int NUM_THREADS = 256;
+
+template <int BN>
+struct Cfg {
+    static constexpr int A_BYTES = BM * BK * 2;
+    static constexpr int B_BYTES = BN * BK * 2;
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+    static constexpr int STAGES = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
+    static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+struct EpiArgs {
+    void *out;
+    long ldo;
+    const float *bias;
+    int relu;
+    const __nv_bfloat16 *mask;
+    long ldm;
+    float *master;
+    __nv_bfloat16 *slot;
+    float *adam_m, *adam_v;
+    float lr, b1, b2, eps, bc1, bc2;
+};
+
+// ---------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(bar),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map, uint32_t bar, int c0, int c1) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+            dst),
+        "l"(map), "r"(bar), "r"(c0), "r"(c1)
+        : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_commit(uint32_t bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
+    uint32_t r[32];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+          "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+          "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+          "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+// Shared-memory matrix descriptor (tcgen05 "matrix descriptor"): start address >> 4 in
+// bits 0-13, leading byte offset >> 4 in 16-29, stride byte offset >> 4 in 32-45,
+// version 1 in 46-47, base offset 0, swizzle mode in 61-63 (2 = 128B swizzle).
+//   K-major, 128B swizzle: rows of 128 B (64 bf16 of K), 8-row atoms 1024 B apart (SBO);
+//                          LBO unused; K advances by +32 B per UMMA_K inside the atom.
+//   MN-major, 128B swizzle: K rows of 128 B (64 MN elements), 8-row atoms 1024 B apart
+//                          (SBO); successive 64-element MN chunks LBO = BK*128 B apart;
+//                          K advances by 16 rows = 2048 B per UMMA_K.
+__device__ __forceinline__ uint64_t smem_desc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+    uint64_t d = 0;
+    d |= (uint64_t)((addr >> 4) & 0x3FFF);
+    d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+    d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
+    d |= (uint64_t)1 << 46;
+    d |= (uint64_t)2 << 61;
+    return d;
+}
+
+// Instruction descriptor for kind::f16: D fp32 (bits 4-5 = 1), A bf16 (7-9 = 1), B bf16
+// (10-12 = 1), A major (bit 15), B major (bit 16), N >> 3 (17-22), M >> 4 (24-28).
+__host__ __device__ constexpr uint32_t make_idesc(int M, int N, int amaj, int bmaj) {
+    return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)amaj << 15) | ((uint32_t)bmaj << 16) |
+           ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+    return *reinterpret_cast<uint32_t *>(&h);
+}
+
+// ---------------------------------------------------------------- epilogue
+template <int EPI>
+__device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32], int row, int col, int M, int N) {
+    if (row >= M) return;
+    const bool full = (col + 32 <= N);
+    if constexpr (EPI == EPI_STORE || EPI == EPI_MASK) {
+        if constexpr (EPI == EPI_STORE) {
+            if (e.bias) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] += (col + i < N) ? e.bias[col + i] : 0.f;
+            }
+            if (e.relu) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
+            }
+        } else {
+            const __nv_bfloat16 *mk = e.mask + (long)row * e.ldm + col;
+            if (full) {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    uint4 raw = *reinterpret_cast<const uint4 *>(mk + q * 8);
+                    const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[q * 8 + i] = (__bfloat162float(h[i]) > 0.f) ? v[q * 8 + i] : 0.f;
+                }
+            } else {
+                for (int i = 0; i < 32; ++i)
+                    if (col + i < N) v[i] = (__bfloat162float(mk[i]) > 0.f) ? v[i] : 0.f;
+            }
+        }
+        __nv_bfloat16 *o = static_cast<__nv_bfloat16 *>(e.out) + (long)row * e.ldo + col;
+        if (full) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                uint4 w;
+                w.x = pack_bf16(v[q * 8 + 0], v[q * 8 + 1]);
+                w.y = pack_bf16(v[q * 8 + 2], v[q * 8 + 3]);
+                w.z = pack_bf16(v[q * 8 + 4], v[q * 8 + 5]);
+                w.w = pack_bf16(v[q * 8 + 6], v[q * 8 + 7]);
+                *reinterpret_cast<uint4 *>(o + q * 8) = w;
+            }
+        } else {
+            for (int i = 0; i < 32; ++i)
+                if (col + i < N) o[i] = __float2bfloat16_rn(v[i]);
+        }
+    } else if constexpr (EPI == EPI_F32) {
+        float *o = static_cast<float *>(e.out) + (long)row * e.ldo + col;
+        if (full) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                *reinterpret_cast<float4 *>(o + q * 4) = make_float4(v[q * 4], v[q * 4 + 1], v[q * 4 + 2], v[q * 4 + 3]);
+        } else {
+            for (int i = 0; i < 32; ++i)
+                if (col + i < N) o[i] = v[i];
+        }
+    } else {  // EPI_SGD / EPI_ADAM: fused weight update writing the next version
+        const long base = (long)row * e.ldo + col;
+        float *ms = e.master + base;
+        __nv_bfloat16 *sl = e.slot + base;
+        if (full) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                float4 w = *reinterpret_cast<float4 *>(ms + q * 4);
+                float g[4] = {v[q * 4], v[q * 4 + 1], v[q * 4 + 2], v[q * 4 + 3]};
+                float wv[4] = {w.x, w.y, w.z, w.w};
+                if constexpr (EPI == EPI_SGD) {
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) wv[i] = wv[i] - e.lr * g[i];
+                } else {
+                    float4 m4 = *reinterpret_cast<float4 *>(e.adam_m + base + q * 4);
+                    float4 v4 = *reinterpret_cast<float4 *>(e.adam_v + base + q * 4);
+                    float mm[4] = {m4.x, m4.y, m4.z, m4.w}, vv[4] = {v4.x, v4.y, v4.z, v4.w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        mm[i] = e.b1 * mm[i] + (1.f - e.b1) * g[i];
+                        vv[i] = e.b2 * vv[i] + (1.f - e.b2) * g[i] * g[i];
+                        wv[i] = wv[i] - e.lr * (mm[i] / e.bc1) / (sqrtf(vv[i] / e.bc2) + e.eps);
+                    }
+                    *reinterpret_cast<float4 *>(e.adam_m + base + q * 4) = make_float4(mm[0], mm[1], mm[2], mm[3]);
+                    *reinterpret_cast<float4 *>(e.adam_v + base + q * 4) = make_float4(vv[0], vv[1], vv[2], vv[3]);
+                }
+                *reinterpret_cast<float4 *>(ms + q * 4) = make_float4(wv[0], wv[1], wv[2], wv[3]);
+                uint2 p;
+                p.x = pack_bf16(wv[0], wv[1]);
+                p.y = pack_bf16(wv[2], wv[3]);
+                *reinterpret_cast<uint2 *>(sl + q * 4) = p;
+            }
+        } else {
+            for (int i = 0; i < 32; ++i) {
+                if (col + i >= N) continue;
+                float w = ms[i];
+                if constexpr (EPI == EPI_SGD) {
+                    w = w - e.lr * v[i];
+                } else {
+                    float mm = e.adam_m[base + i], vv = e.adam_v[base + i];
+                    mm = e.b1 * mm + (1.f - e.b1) * v[i];
+                    vv = e.b2 * vv + (1.f - e.b2) * v[i] * v[i];
+                    w = w - e.lr * (mm / e.bc1) / (sqrtf(vv / e.bc2) + e.eps);
+                    e.adam_m[base + i] = mm;
+                    e.adam_v[base + i] = vv;
+                }
+                ms[i] = w;
+                sl[i] = __float2bfloat16_rn(w);
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------- the kernel
+template <int BN, int AMAJ, int BMAJ, int EPI>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
+    tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, EpiArgs e,
+                   int M, int N, int K) {
+    using C = Cfg<BN>;
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + C::STAGES * C::STAGE_BYTES);
+    uint64_t *full = bars, *empty = bars + C::STAGES, *tfull = bars + 2 * C::STAGES, *tempty = tfull + 2;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int m_blocks = (M + BM - 1) / BM, n_blocks = (N + BN - 1) / BN;
+    const int tiles = m_blocks * n_blocks;
+    const int kblocks = (K + BK - 1) / BK;
+
+    if (warp == 0 && lane == 0) {
+        asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(&tmB) : "memory");
+        for (int s = 0; s < C::STAGES; ++s) {
+            mbar_init(smem_u32(&full[s]), 1);
+            mbar_init(smem_u32(&empty[s]), 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(smem_u32(&tfull[a]), 1);
+            mbar_init(smem_u32(&tempty[a]), 4);  // one arrival per epilogue warp
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(C::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        // ===== TMA producer =====
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
+                for (int kb = 0; kb < kblocks; ++kb) {
+                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                    const uint32_t fb = smem_u32(&full[stage]);
+                    mbar_expect_tx(fb, C::STAGE_BYTES);
+                    const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
+                    const uint32_t sb = sa + C::A_BYTES;
+                    const int k0 = kb * BK;
+                    if (AMAJ == KMAJ) {
+                        tma_load_2d(sa, &tmA, fb, k0, m0);  // box {64 K, 128 M}
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * BK * 128, &tmA, fb, m0 + 64 * j, k0);
+                    }
+                    if (BMAJ == KMAJ) {
+                        tma_load_2d(sb, &tmB, fb, k0, n0);  // box {64 K, BN N}
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * BK * 128, &tmB, fb, n0 + 64 * j, k0);
+                    }
+                    if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ===== MMA issuer =====
+        if (lane == 0) {
+            constexpr uint32_t idesc = make_idesc(BM, BN, AMAJ, BMAJ);
+            int stage = 0;
+            uint32_t phase = 0;
+            int acc = 0;
+            uint32_t acc_phase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
+                tc_fence_after();
+                const uint32_t d = tmem_base + acc * BN;
+                for (int kb = 0; kb < kblocks; ++kb) {
+                    mbar_wait(smem_u32(&full[stage]), phase);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
+                    const uint32_t sb = sa + C::A_BYTES;
+#pragma unroll
+                    for (int k = 0; k < BK / UMMA_K; ++k) {
+                        const uint64_t ad = AMAJ == KMAJ ? smem_desc(sa + k * 32, 16, 1024)
+                                                         : smem_desc(sa + k * 2048, BK * 128, 1024);
+                        const uint64_t bd = BMAJ == KMAJ ? smem_desc(sb + k * 32, 16, 1024)
+                                                         : smem_desc(sb + k * 2048, BK * 128, 1024);
+                        tc_mma(d, ad, bd, idesc, (kb | k) != 0);
+                    }
+                    tc_commit(smem_u32(&empty[stage]));  // frees the smem slot when these MMAs finish
+                    if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                }
+                tc_commit(smem_u32(&tfull[acc]));  // accumulator ready for the epilogue
+                if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+            }
+        }
+    } else if (warp >= 4) {
+        // ===== epilogue =====
+        const int q = warp & 3;  // TMEM lane quarter this warp may access
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
+            mbar_wait(smem_u32(&tfull[acc]), acc_phase);
+            tc_fence_after();
+            const int row = m0 + q * 32 + lane;
+#pragma unroll 1
+            for (int c = 0; c < BN / 32; ++c) {
+                float v[32];
+                tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, v);
+                if (n0 + c * 32 < N) epilogue_chunk<EPI>(e, v, row, n0 + c * 32, M, N);
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
+            if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(C::TMEM_COLS));
+    }
+}
+
+// ---------------------------------------------------------------- host side
+bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner, int box_outer) {
+    const Driver *d = driver();
+    if (!d) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
+    cuuint64_t strides[1] = {(cuuint64_t)ld_elems * 2};
+    cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = d->tensorMapEncodeTiled(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(base), dims,
+                                         strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                         CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+int num_sms() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+template <int BN, int AMAJ, int BMAJ, int EPI>
+cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e, cudaStream_t s) {
+    using C = Cfg<BN>;
+    auto kern = tc_gemm_kernel<BN, AMAJ, BMAJ, EPI>;
+    static bool attr_set = false;  // per instantiation; benign race (idempotent)
+    if (!attr_set) {
+        cudaError_t err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+        if (err != cudaSuccess) return err;
+        attr_set = true;
+    }
+    const int tiles = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN);
+    const int grid = tiles < num_sms() ? tiles : num_sms();
+    kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, e, g.M, g.N, g.K);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+template <int BN, int AMAJ, int BMAJ>
+cudaError_t dispatch_epi(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e,
+                         cudaStream_t s) {
+    switch (g.epi) {
+    case EPI_STORE: return launch<BN, AMAJ, BMAJ, EPI_STORE>(g, ma, mb, e, s);
+    case EPI_MASK: return launch<BN, AMAJ, BMAJ, EPI_MASK>(g, ma, mb, e, s);
+    case EPI_F32: return launch<BN, AMAJ, BMAJ, EPI_F32>(g, ma, mb, e, s);
+    case EPI_SGD: return launch<BN, AMAJ, BMAJ, EPI_SGD>(g, ma, mb, e, s);
+    case EPI_ADAM: return launch<BN, AMAJ, BMAJ, EPI_ADAM>(g, ma, mb, e, s);
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <int BN>
+cudaError_t dispatch_major(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e,
+                           cudaStream_t s) {
+    if (g.amaj == KMAJ && g.bmaj == KMAJ) return dispatch_epi<BN, KMAJ, KMAJ>(g, ma, mb, e, s);
+    if (g.amaj == KMAJ && g.bmaj == MNMAJ) return dispatch_epi<BN, KMAJ, MNMAJ>(g, ma, mb, e, s);
+    if (g.amaj == MNMAJ && g.bmaj == MNMAJ) return dispatch_epi<BN, MNMAJ, MNMAJ>(g, ma, mb, e, s);
+    return dispatch_epi<BN, MNMAJ, KMAJ>(g, ma, mb, e, s);
+}
+
+}  // namespace
+
+cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
+    if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
+    // tile width: the widest BN that still gives every SM a tile
+    const int sms = num_sms();
+    const int mb = (g.M + BM - 1) / BM;
+    int BN = 256;
+    if ((long)mb * ((g.N + 255) / 256) < sms) BN = 128;
+    if (BN == 128 && (long)mb * ((g.N + 127) / 128) < sms) BN = 64;
+    CUtensorMap ma, mbm;
+    const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
+                                    : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
+    const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, BN)
+                                    : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
+    if (!okA || !okB) return cudaErrorInvalidValue;
+    EpiArgs e{};
+    e.out = g.out;
+    e.ldo = g.ldo;
+    e.bias = g.bias;
+    e.relu = g.relu;
+    e.mask = static_cast<const __nv_bfloat16 *>(g.mask);
+    e.ldm = g.ldm;
+    e.master = g.master;
+    e.slot = static_cast<__nv_bfloat16 *>(g.slot);
+    e.adam_m = g.adam_m;
+    e.adam_v = g.adam_v;
+    e.lr = g.lr;
+    e.b1 = g.b1;
+    e.b2 = g.b2;
+    e.eps = g.eps;
+    e.bc1 = 1.f - powf(g.b1, (float)g.step);
+    e.bc2 = 1.f - powf(g.b2, (float)g.step);
+    if (BN == 256) return dispatch_major<256>(g, ma, mbm, e, s);
+    if (BN == 128) return dispatch_major<128>(g, ma, mbm, e, s);
+    return dispatch_major<64>(g, ma, mbm, e, s);
+}
+
+}  // namespace pd

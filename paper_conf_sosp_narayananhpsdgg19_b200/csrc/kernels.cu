@@ -1,0 +1,300 @@
+// kernels.cu -- fp32 SIMT GEMM (parity path), softmax cross-entropy, bias-gradient column
+// sums, optimizer updates that write the next weight version, casts, and the cross-process
+// flag signal.  The bf16 tensor-core GEMM lives in gemm_tc.cu.
+#include <cuda_bf16.h>
+
+#include "pd_internal.h"
+
+namespace pd {
+
+thread_local uint64_t tl_launches = 0;
+
+namespace {
+
+__device__ __forceinline__ float ld_as_f32(const float *p, long i) { return p[i]; }
+__device__ __forceinline__ float ld_as_f32(const __nv_bfloat16 *p, long i) { return __bfloat162float(p[i]); }
+
+// ------------------------------------------------------------------ fp32 SIMT GEMM
+// 64x64 output tile per 256-thread block, 4x4 per thread, BK = 16, generic operand
+// strides (handles the K-/MN-major views of fwd, dX and dW without transposes).
+constexpr int SB_M = 64, SB_N = 64, SB_K = 16;
+
+__global__ void __launch_bounds__(256) sgemm_kernel(Gemm g) {
+    __shared__ float As[SB_K][SB_M + 4];
+    __shared__ float Bs[SB_K][SB_N + 4];
+    const float *A = static_cast<const float *>(g.A);
+    const float *B = static_cast<const float *>(g.B);
+    const int tid = threadIdx.x;
+    const int m0 = blockIdx.y * SB_M, n0 = blockIdx.x * SB_N;
+    const int tm = (tid / 16) * 4, tn = (tid % 16) * 4;
+    float acc[4][4] = {};
+    for (int k0 = 0; k0 < g.K; k0 += SB_K) {
+        // 1024 elements of each operand tile, 4 per thread; the fastest index follows the
+        // operand's contiguous dimension so global reads coalesce.
+        for (int e = tid; e < SB_M * SB_K; e += 256) {
+            int mm, kk;
+            if (g.amaj == KMAJ) { kk = e % SB_K; mm = e / SB_K; } else { mm = e % SB_M; kk = e / SB_M; }
+            const int m = m0 + mm, k = k0 + kk;
+            float v = 0.f;
+            if (m < g.M && k < g.K) v = g.amaj == KMAJ ? A[(long)m * g.lda + k] : A[(long)k * g.lda + m];
+            As[kk][mm] = v;
+        }
+        for (int e = tid; e < SB_N * SB_K; e += 256) {
+            int nn, kk;
+            if (g.bmaj == KMAJ) { kk = e % SB_K; nn = e / SB_K; } else { nn = e % SB_N; kk = e / SB_N; }
+            const int n = n0 + nn, k = k0 + kk;
+            float v = 0.f;
+            if (n < g.N && k < g.K) v = g.bmaj == KMAJ ? B[(long)n * g.ldb + k] : B[(long)k * g.ldb + n];
+            Bs[kk][nn] = v;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int kk = 0; kk < SB_K; ++kk) {
+            float a[4], b[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) a[i] = As[kk][tm + i];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) b[i] = Bs[kk][tn + i];
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        }
+        __syncthreads();
+    }
+    float *out = static_cast<float *>(g.out);
+    const float *mask = static_cast<const float *>(g.mask);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int m = m0 + tm + i;
+        if (m >= g.M) continue;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int n = n0 + tn + j;
+            if (n >= g.N) continue;
+            float v = acc[i][j];
+            if (g.epi == EPI_STORE) {
+                if (g.bias) v += g.bias[n];
+                if (g.relu && v < 0.f) v = 0.f;
+            } else if (g.epi == EPI_MASK) {
+                if (mask && !(mask[(long)m * g.ldm + n] > 0.f)) v = 0.f;
+            }
+            out[(long)m * g.ldo + n] = v;
+        }
+    }
+}
+
+// ------------------------------------------------------------------ column sums (bias grads)
+// out[c] = sum_r G[r][c]; one thread per column, rows in order (deterministic).
+template <typename T>
+__global__ void col_sum_kernel(const T *G, long rows, long cols, float *out) {
+    const long c = (long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= cols) return;
+    float acc = 0.f;
+    for (long r = 0; r < rows; ++r) acc += ld_as_f32(G, r * cols + c);
+    out[c] = acc;
+}
+
+// ------------------------------------------------------------------ softmax cross-entropy
+// One block per row: max, sum of exp, loss += (lse - z[label]) / rows, and
+// dlogits = (softmax - onehot) / rows written in the logits' dtype (L1217, R8).
+template <typename T>
+__global__ void __launch_bounds__(256) softmax_ce_kernel(const T *z, const int32_t *labels, long rows, int C, T *dz,
+                                                         float *loss) {
+    const long r = blockIdx.x;
+    const T *zr = z + r * C;
+    __shared__ float red[32];
+    float m = -INFINITY;
+    for (int c = threadIdx.x; c < C; c += blockDim.x) m = fmaxf(m, ld_as_f32(zr, c));
+    for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        float v = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : -INFINITY;
+        for (int o = 16; o; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+        if (threadIdx.x == 0) red[0] = v;
+    }
+    __syncthreads();
+    m = red[0];
+    __syncthreads();
+    float s = 0.f;
+    for (int c = threadIdx.x; c < C; c += blockDim.x) s += __expf(ld_as_f32(zr, c) - m);
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        float v = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : 0.f;
+        for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        if (threadIdx.x == 0) red[0] = v;
+    }
+    __syncthreads();
+    s = red[0];
+    const int lab = labels[r];
+    const float inv_rows = 1.0f / (float)rows;
+    const float inv_s = 1.0f / s;
+    for (int c = threadIdx.x; c < C; c += blockDim.x) {
+        const float p = __expf(ld_as_f32(zr, c) - m) * inv_s;
+        const float d = (p - (c == lab ? 1.f : 0.f)) * inv_rows;
+        if constexpr (sizeof(T) == 4) dz[r * C + c] = d;
+        else dz[r * C + c] = __float2bfloat16_rn(d);
+    }
+    if (threadIdx.x == 0) atomicAdd(loss, (m + __logf(s) - ld_as_f32(zr, lab)) * inv_rows);
+}
+
+// ------------------------------------------------------------------ optimizer updates
+__global__ void sgd_f32_kernel(const float *__restrict__ in, const float *__restrict__ g, float *__restrict__ out,
+                               long n, float lr) {
+    const long stride = (long)gridDim.x * blockDim.x;
+    long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
+    if ((n & 3) == 0 && (((uintptr_t)in | (uintptr_t)g | (uintptr_t)out) & 15) == 0) {
+        const long n4 = n >> 2;
+        for (; i < n4; i += stride) {
+            float4 w = reinterpret_cast<const float4 *>(in)[i], d = reinterpret_cast<const float4 *>(g)[i];
+            w.x -= lr * d.x; w.y -= lr * d.y; w.z -= lr * d.z; w.w -= lr * d.w;
+            reinterpret_cast<float4 *>(out)[i] = w;
+        }
+        return;
+    }
+    for (; i < n; i += stride) out[i] = in[i] - lr * g[i];
+}
+
+__device__ __forceinline__ float adam_step(float w, float g, float &m, float &v, float lr, float b1, float b2,
+                                           float eps, float bc1, float bc2) {
+    m = b1 * m + (1.f - b1) * g;
+    v = b2 * v + (1.f - b2) * g * g;
+    const float mh = m / bc1, vh = v / bc2;
+    return w - lr * mh / (sqrtf(vh) + eps);
+}
+
+__global__ void adam_f32_kernel(const float *in, const float *g, float *out, float *m, float *v, long n, float lr,
+                                float b1, float b2, float eps, float bc1, float bc2) {
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        float mm = m[i], vv = v[i];
+        out[i] = adam_step(in[i], g[i], mm, vv, lr, b1, b2, eps, bc1, bc2);
+        m[i] = mm;
+        v[i] = vv;
+    }
+}
+
+// master -= update(mean over replicas of grads); slot = bf16(master) (or fp32 slot)
+__global__ void update_master_kernel(float *master, __nv_bfloat16 *slot_bf16, float *slot_f32,
+                                     const float *const *grads, int R, long goff, long n, int opt, float *m, float *v,
+                                     float lr, float b1, float b2, float eps, float bc1, float bc2) {
+    const long stride = (long)gridDim.x * blockDim.x;
+    const float invR = 1.0f / (float)R;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        float g = 0.f;
+        for (int r = 0; r < R; ++r) g += grads[r][goff + i];  // replica order (R7)
+        if (R > 1) g = g * invR;
+        float w = master[i];
+        if (opt == PD_SGD) {
+            w = w - lr * g;
+        } else {
+            float mm = m[i], vv = v[i];
+            w = adam_step(w, g, mm, vv, lr, b1, b2, eps, bc1, bc2);
+            m[i] = mm;
+            v[i] = vv;
+        }
+        master[i] = w;
+        if (slot_bf16) slot_bf16[i] = __float2bfloat16_rn(w);
+        if (slot_f32) slot_f32[i] = w;
+    }
+}
+
+__global__ void f32_to_bf16_kernel(const float *in, __nv_bfloat16 *out, long n) {
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = __float2bfloat16_rn(in[i]);
+}
+__global__ void bf16_to_f32_kernel(const __nv_bfloat16 *in, float *out, long n) {
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = __bfloat162float(in[i]);
+}
+
+// Release-store of a monotonically increasing counter into (possibly peer-mapped) memory.
+// Stream order makes every earlier kernel's writes complete before this kernel runs; the
+// system-scope fence orders them before the flag for the observing GPU.
+__global__ void signal_kernel(uint32_t *flag, uint32_t value) {
+    __threadfence_system();
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flag), "r"(value) : "memory");
+}
+
+int grid_for(long n, int block = 256) {
+    long b = (n + block - 1) / block;
+    if (b > 148L * 16) b = 148L * 16;  // grid-stride beyond 16 waves of the 148 SMs
+    return (int)(b < 1 ? 1 : b);
+}
+
+}  // namespace
+
+cudaError_t gemm_f32(const Gemm &g, cudaStream_t s) {
+    if (g.epi != EPI_STORE && g.epi != EPI_MASK && g.epi != EPI_F32) return cudaErrorInvalidValue;
+    dim3 grid((g.N + SB_N - 1) / SB_N, (g.M + SB_M - 1) / SB_M);
+    sgemm_kernel<<<grid, 256, 0, s>>>(g);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t col_sum(const void *G, int bf16, long rows, long cols, float *out, cudaStream_t s) {
+    const int blocks = (int)((cols + 255) / 256);
+    if (bf16) col_sum_kernel<<<blocks, 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(G), rows, cols, out);
+    else col_sum_kernel<<<blocks, 256, 0, s>>>(static_cast<const float *>(G), rows, cols, out);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t softmax_ce(const void *logits, int bf16, const int32_t *labels, long rows, int C, void *dlogits,
+                       float *loss_out, cudaStream_t s) {
+    if (bf16)
+        softmax_ce_kernel<<<(unsigned)rows, 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(logits), labels, rows, C,
+                                                         static_cast<__nv_bfloat16 *>(dlogits), loss_out);
+    else
+        softmax_ce_kernel<<<(unsigned)rows, 256, 0, s>>>(static_cast<const float *>(logits), labels, rows, C,
+                                                         static_cast<float *>(dlogits), loss_out);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t sgd_f32(const float *in, const float *g, float *out, long n, float lr, cudaStream_t s) {
+    sgd_f32_kernel<<<grid_for(n / 4 + 1), 256, 0, s>>>(in, g, out, n, lr);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t adam_f32(const float *in, const float *g, float *out, float *m, float *v, long n, float lr, float b1,
+                     float b2, float eps, int step, cudaStream_t s) {
+    const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
+    adam_f32_kernel<<<grid_for(n), 256, 0, s>>>(in, g, out, m, v, n, lr, b1, b2, eps, bc1, bc2);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f32, const float *const *grads,
+                          int R, long goff, long n, int opt, float *m, float *v, float lr, float b1, float b2,
+                          float eps, int step, cudaStream_t s) {
+    const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
+    update_master_kernel<<<grid_for(n), 256, 0, s>>>(master, slot_bf16, slot_f32, grads, R, goff, n, opt, m, v, lr,
+                                                     b1, b2, eps, bc1, bc2);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t f32_to_bf16(const float *in, __nv_bfloat16 *out, long n, cudaStream_t s) {
+    f32_to_bf16_kernel<<<grid_for(n), 256, 0, s>>>(in, out, n);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t bf16_to_f32(const __nv_bfloat16 *in, float *out, long n, cudaStream_t s) {
+    bf16_to_f32_kernel<<<grid_for(n), 256, 0, s>>>(in, out, n);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s) {
+    signal_kernel<<<1, 1, 0, s>>>(flag, value);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+}  // namespace pd

@@ -1,0 +1,104 @@
+// pd_internal.h -- internal declarations of libpipedream (not part of the C ABI).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/pipedream.h"
+
+namespace pd {
+
+// ---------------------------------------------------------------- planner (plan.cpp)
+pd_status plan_partition(const pd_layer_profile *layers, int N, int G, const pd_plan_opts *opts, pd_plan_t *out);
+
+// ---------------------------------------------------------------- schedule (schedule.cpp)
+// One entry of a worker's static 1F1B-RR op list (R3).
+struct Op {
+    char kind;  // 'F', 'B', 'U'
+    int t;      // global minibatch id
+    int j;      // local index of t at this worker (t = replica + j * R_s)
+};
+// k_s per stage (R2 / R19).  Returns PD_EINVAL for an override on a replicated plan.
+pd_status inflight_counts(const pd_plan_t &plan, int depth, std::vector<int> &k);
+// F(t_0..t_{k-1}) then (B(t_j) U F(t_{j+k}))* then (B U)* (L1023-1065, L237-241).
+std::vector<Op> worker_ops(int R_s, int replica, int k_s, int M);
+// receive-ring depth of stage s >= 1: ceil(k_{s-1} R_{s-1} / R_s).
+int recv_ring_depth(const pd_plan_t &plan, const std::vector<int> &k, int s);
+
+// ---------------------------------------------------------------- CUDA driver shim (cudadrv.cpp)
+struct Driver {
+    CUresult (*streamWaitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int) = nullptr;
+    CUresult (*tensorMapEncodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                     const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                     CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill) = nullptr;
+};
+const Driver *driver();  // resolved once through cudaGetDriverEntryPoint; nullptr if unavailable
+
+// ---------------------------------------------------------------- kernels
+// Per-host-thread launch counter (kernels launched by this library).
+extern thread_local uint64_t tl_launches;
+
+enum Major { KMAJ = 0, MNMAJ = 1 };
+enum Epi {
+    EPI_STORE = 0,  // out = act(acc + bias[n])             (dtype of the path)
+    EPI_MASK = 1,   // out = acc * (mask[m][n] > 0)          (dX fused with the ReLU derivative)
+    EPI_F32 = 2,    // out(fp32) = acc                       (gradient buffer)
+    EPI_SGD = 3,    // master -= lr*acc; slot = cast(master) (fused weight update, bf16 path)
+    EPI_ADAM = 4    // Adam on master/m/v; slot = cast(master)
+};
+
+// C(m, n) = sum_k A(m, k) * B(n, k)
+//   A(m, k) = amaj == KMAJ ? A[m*lda + k] : A[k*lda + m]
+//   B(n, k) = bmaj == KMAJ ? B[n*ldb + k] : B[k*ldb + n]
+struct Gemm {
+    int M = 0, N = 0, K = 0;
+    const void *A = nullptr;
+    long lda = 0;
+    int amaj = KMAJ;
+    const void *B = nullptr;
+    long ldb = 0;
+    int bmaj = KMAJ;
+    int epi = EPI_STORE;
+    void *out = nullptr;  // EPI_STORE/MASK: path dtype; EPI_F32: float
+    long ldo = 0;
+    const float *bias = nullptr;
+    int relu = 0;
+    const void *mask = nullptr;  // path dtype, ld = ldm
+    long ldm = 0;
+    // fused update (EPI_SGD / EPI_ADAM), arrays indexed [m*ldo + n]
+    float *master = nullptr;
+    void *slot = nullptr;  // bf16 new version
+    float *adam_m = nullptr, *adam_v = nullptr;
+    float lr = 0.f, b1 = 0.f, b2 = 0.f, eps = 0.f;
+    int step = 0;
+};
+
+// fp32 SIMT GEMM (parity path; no tensor cores, no TF32).  EPI_STORE/MASK/F32 only.
+cudaError_t gemm_f32(const Gemm &g, cudaStream_t s);
+// bf16 tcgen05/TMEM/TMA GEMM, fp32 accumulation.  All epilogues.
+cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s);
+
+// elementwise / reductions (kernels.cu).  T = float or __nv_bfloat16 via `bf16` flag.
+cudaError_t col_sum(const void *G, int bf16, long rows, long cols, float *out, cudaStream_t s);
+cudaError_t softmax_ce(const void *logits, int bf16, const int32_t *labels, long rows, int C, void *dlogits,
+                       float *loss_out, cudaStream_t s);
+// out = in - lr * g  (fp32 versions), n elements
+cudaError_t sgd_f32(const float *in, const float *g, float *out, long n, float lr, cudaStream_t s);
+cudaError_t adam_f32(const float *in, const float *g, float *out, float *m, float *v, long n, float lr, float b1,
+                     float b2, float eps, int step, cudaStream_t s);
+// bf16 path: master -= lr * g (or Adam), slot = bf16(master).  g may be a replica set:
+// g = (sum_r grads[r]) * (1/R), summed in r order (R7).
+// grads is a DEVICE array of R pointers; element i of replica r is grads[r][goff + i].
+cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f32, const float *const *grads,
+                          int R, long goff, long n, int opt, float *m, float *v, float lr, float b1, float b2,
+                          float eps, int step, cudaStream_t s);
+cudaError_t f32_to_bf16(const float *in, __nv_bfloat16 *out, long n, cudaStream_t s);
+cudaError_t bf16_to_f32(const __nv_bfloat16 *in, float *out, long n, cudaStream_t s);
+cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s);
+
+}  // namespace pd

@@ -1,0 +1,1328 @@
+// runtime.cu -- the 1F1B-RR pipeline runtime with weight stashing (§3.2-3.3, §4).
+//
+// One host thread per local worker (stage s, replica r) walks the worker's static op list
+// (schedule.cpp) and issues its kernels on the worker's own CUDA stream, so issue order is
+// execution order (the event trace is exact).  Cross-worker dependencies are the only
+// synchronisation (the schedule is static, "without expensive distributed coordination",
+// L1083-1085):
+//   activation  F(s-1, t) -> F(s, t)   the producing GEMM writes straight into the consumer's
+//                                      receive-ring slot (peer pointer over NVLink when the
+//                                      consumer is another GPU), then posts the link;
+//   gradient    B(s+1, t) -> B(s, t)   the first layer's dX GEMM writes into the upstream
+//                                      worker's gradient ring slot, then posts;
+//   replicas    round j of a replicated stage: every replica posts "gradient ready", each
+//               replica reduces all R gradients (replica order, R7) in one fused
+//               reduce+update kernel reading peer memory, then posts "read done".
+// A link is an event ring + host counters when both ends live in this process (every wait
+// refers to an already-issued record, so any hardware-queue mapping is deadlock free), or
+// a flag word in the consumer's memory written by a release-store kernel and awaited with
+// cuStreamWaitValue32 when the ends are in different processes (CUDA IPC).
+//
+// State per worker (§4 "Parameter State" / "Intermediate State", L1337-1371):
+//   weight-stash ring   k_s versions; version v lives in slot v mod k_s.  F reads the
+//                       latest, B reads the stashed v(s,t); the update writes version v+1
+//                       into slot (v+1) mod k_s -- the slot of the oldest version, which no
+//                       pending backward references any more.
+//                       No copies: stashing a version is remembering its index.
+//   fp32 master + Adam  bf16 path only the master is fp32 (R21); optimizer state is not
+//                       versioned (R9).
+//   receive rings       activations D_s deep (they double as the first layer's stash),
+//                       gradients k_s deep; slot = local index mod depth.
+//   activation stash    inputs of the stage's inner layers, k_s deep.
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <condition_variable>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "pd_internal.h"
+
+using namespace pd;
+
+namespace {
+
+// ---------------------------------------------------------------- errors
+struct CudaFail {
+    cudaError_t e;
+    const char *what;
+};
+#define CK(x)                                              \
+    do {                                                   \
+        cudaError_t _e = (x);                              \
+        if (_e != cudaSuccess) throw CudaFail{_e, #x};     \
+    } while (0)
+struct Abort {};
+
+long numel_params(const pd_layer_desc &d) {
+    switch (d.kind) {
+    case PD_LINEAR: return (long)d.out * d.in + d.out;
+    case PD_LSTM: return 4L * d.out * d.in + 4L * d.out * d.out + 8L * d.out;
+    case PD_CONV3X3: return (long)d.out * d.in * 9 + d.out;
+    case PD_MAXPOOL2: return 0;
+    case PD_EMBEDDING: return (long)d.in * d.out;
+    }
+    return -1;
+}
+long rows_of(const pd_layer_desc &d, int B) { return d.seq_len > 0 ? (long)d.seq_len * B : (long)B; }
+long in_elems(const pd_layer_desc &d, int B) {
+    switch (d.kind) {
+    case PD_LINEAR: return rows_of(d, B) * d.in;
+    case PD_LSTM: return (long)d.seq_len * B * d.in;
+    case PD_CONV3X3:
+    case PD_MAXPOOL2: return (long)B * d.height * d.width * d.in;
+    case PD_EMBEDDING: return (long)d.seq_len * B;
+    }
+    return 0;
+}
+long out_elems(const pd_layer_desc &d, int B) {
+    switch (d.kind) {
+    case PD_LINEAR: return rows_of(d, B) * d.out;
+    case PD_LSTM: return (long)d.seq_len * B * d.out;
+    case PD_CONV3X3: return (long)B * d.height * d.width * d.out;
+    case PD_MAXPOOL2: return (long)B * (d.height / 2) * (d.width / 2) * d.in;
+    case PD_EMBEDDING: return (long)d.seq_len * B * d.out;
+    }
+    return 0;
+}
+
+// ---------------------------------------------------------------- links
+enum LinkType { L_ACT = 0, L_GRAD = 1, L_READY = 2, L_DONE = 3 };
+
+struct Link {
+    bool remote = false;
+    // local (same process): event ring + host counters
+    std::mutex mu;
+    std::condition_variable cv;
+    int64_t posted = 0, waited = 0;
+    std::vector<cudaEvent_t> ev;
+    int device = -1;  // producer's device (events are created there)
+    // remote (other process): flag in the consumer's memory
+    uint32_t *remote_flag = nullptr;  // producer side, IPC-mapped
+    uint32_t *local_flag = nullptr;   // consumer side
+    int64_t rposted = 0;              // producer: messages posted over all runs
+    int64_t rbase = 0, rcount = 0;    // consumer: messages of earlier runs / of this run
+};
+
+// ---------------------------------------------------------------- IPC blob
+struct IpcBlob {
+    uint32_t magic;
+    int32_t stage, replica, device;
+    int32_t has_recv, has_grad, has_rgrad;
+    cudaIpcMemHandle_t recv, grad, rgrad0, rgrad1, flags;
+};
+constexpr uint32_t BLOB_MAGIC = 0x50443031u;  // "PD01"
+
+// Buffers a worker exposes to others (local pointers, or IPC-mapped in this process).
+struct Shared {
+    void *recv = nullptr;      // activation receive ring (stage > 0)
+    void *grad = nullptr;      // gradient receive ring (stage < n-1)
+    float *rgrad[2] = {};      // replica gradient buffers (R_s > 1), round parity
+    uint32_t *flags = nullptr; // flag words (remote links)
+    bool valid = false;
+};
+
+struct Worker;
+
+}  // namespace
+
+struct pd_ctx {
+    pd_plan_t plan{};
+    std::vector<pd_layer_desc> layers;
+    pd_train_cfg cfg{};
+    int n = 0;                       // stages
+    int nw = 0;                      // workers
+    std::vector<int> wbase;          // first worker id per stage
+    std::vector<int> kdef;           // default k_s
+    std::vector<int> kalloc;         // allocated stash depth (max over default and max_depth)
+    std::vector<int> Dalloc, Galloc; // ring depths as allocated
+    std::vector<long> poff;          // parameter offset of each layer inside its stage buffer
+    std::vector<long> pcount;        // parameter count of each layer
+    std::vector<std::unique_ptr<Worker>> W;  // by worker id (null when remote)
+    std::vector<Shared> shared;              // by worker id
+    std::map<std::tuple<int, int, int>, std::unique_ptr<Link>> links;  // (type, src, dst)
+    int esz = 4;                     // element size of the path dtype
+    int n_data = 0;
+    // results of the last run
+    int last_M = 0;
+    std::vector<int32_t> vmap;
+    double host_ms = 0;
+    std::atomic<bool> abort{false};
+    std::mutex err_mu;
+    pd_status sticky = PD_OK;
+    std::string err;
+
+    void fail(pd_status s, const std::string &msg) {
+        std::lock_guard<std::mutex> g(err_mu);
+        if (sticky == PD_OK) {
+            sticky = s;
+            err = msg;
+        }
+        abort = true;
+        for (auto &kv : links) {
+            std::lock_guard<std::mutex> lg(kv.second->mu);
+            kv.second->cv.notify_all();
+        }
+    }
+    int worker_id(int s, int r) const { return wbase[s] + r; }
+    int stage_of(int w) const {
+        int s = 0;
+        while (s + 1 < n && wbase[s + 1] <= w) ++s;
+        return s;
+    }
+    int flag_index(int type, int src_stage, int src_rep, int dst_stage) const;
+    int flag_count(int s) const;
+};
+
+namespace {
+
+struct Worker {
+    pd_ctx *ctx;
+    int id, stage, replica, device;
+    int first, last;   // layer range
+    long P = 0;        // parameters of the stage
+    int k = 1;         // stash slots allocated
+    int D = 0, G = 0;  // receive ring depths
+    cudaStream_t stream = nullptr;
+    // weights
+    std::vector<void *> wslot;  // k versions (path dtype)
+    float *master = nullptr;    // bf16 path
+    float *adam_m = nullptr, *adam_v = nullptr;
+    float *gbuf = nullptr;      // fp32 gradient (unreplicated fp32 path / biases)
+    float *rgrad[2] = {};       // replicated stages: gradient per round parity
+    const float **rgrad_ptrs = nullptr;  // device array [2][R]: peers' rgrad for each parity
+    const float **self_grad_ptr = nullptr;  // device array [1]: gbuf
+    // activations
+    std::vector<void *> act;     // per inner layer l (index l-first, l>first): k slots of in_elems
+    void *recv = nullptr;        // D slots (stage > 0)
+    void *gring = nullptr;       // G slots (stage < n-1)
+    void *scratch[2] = {};       // dY ping-pong
+    void *logits = nullptr, *dlogits = nullptr;  // last stage
+    void *data_in = nullptr;     // stage 0: n_data inputs (path dtype)
+    int32_t *tokens = nullptr;   // stage 0 embedding
+    int32_t *labels = nullptr;   // last stage
+    float *losses = nullptr;     // last stage, per minibatch of the run
+    int losses_cap = 0;
+    uint32_t *flags = nullptr;
+    // bookkeeping
+    int version = 0;
+    std::map<int, int> fwd_version;  // local index -> version used by its forward
+    std::vector<pd_event> events;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> op_ev;  // record_trace 2
+    std::vector<cudaEvent_t> ev_pool;
+    uint64_t launches = 0;
+    uint64_t bytes_sent = 0;
+    int updates_total = 0;  // Adam step counter base (persists across runs)
+
+    ~Worker();
+};
+
+Worker::~Worker() {
+    if (device >= 0) cudaSetDevice(device);
+    if (stream) cudaStreamSynchronize(stream);
+    for (void *p : wslot) cudaFree(p);
+    for (void *p : act) cudaFree(p);
+    void *bufs[] = {master, adam_m, adam_v, gbuf, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
+                    dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
+    for (void *p : bufs)
+        if (p) cudaFree(p);
+    for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
+    if (stream) cudaStreamDestroy(stream);
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+template <typename T>
+T *dalloc(size_t bytes) {
+    void *p = nullptr;
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(&p, align_up(bytes, 256));
+    if (e != cudaSuccess) throw CudaFail{e, "cudaMalloc"};
+    CK(cudaMemset(p, 0, align_up(bytes, 256)));
+    return static_cast<T *>(p);
+}
+
+}  // namespace
+
+// Flag words of the consumer worker of stage `dst_stage`:
+//   [0, R_{s-1})                       activation from producer replica p   (L_ACT)
+//   [R_{s-1}, R_{s-1}+R_{s+1})         gradient from downstream replica c   (L_GRAD)
+//   then R_s "ready" and R_s "done" words from each peer replica           (L_READY / L_DONE)
+int pd_ctx::flag_index(int type, int src_stage, int src_rep, int dst_stage) const {
+    const int s = dst_stage;
+    const int rp = s > 0 ? plan.stage[s - 1].replicas : 0;
+    const int rn = s + 1 < n ? plan.stage[s + 1].replicas : 0;
+    const int rs = plan.stage[s].replicas;
+    (void)src_stage;
+    switch (type) {
+    case L_ACT: return src_rep;
+    case L_GRAD: return rp + src_rep;
+    case L_READY: return rp + rn + src_rep;
+    case L_DONE: return rp + rn + rs + src_rep;
+    }
+    return -1;
+}
+int pd_ctx::flag_count(int s) const {
+    const int rp = s > 0 ? plan.stage[s - 1].replicas : 0;
+    const int rn = s + 1 < n ? plan.stage[s + 1].replicas : 0;
+    return rp + rn + 2 * plan.stage[s].replicas;
+}
+
+namespace {
+
+// ---------------------------------------------------------------- link operations
+Link &get_link(pd_ctx *c, int type, int src, int dst) {
+    auto key = std::make_tuple(type, src, dst);
+    auto it = c->links.find(key);
+    if (it == c->links.end()) throw CudaFail{cudaErrorInvalidValue, "missing link"};
+    return *it->second;
+}
+
+void link_post(pd_ctx *c, Link &L, cudaStream_t s) {
+    if (L.remote) {
+        ++L.rposted;
+        CK(signal_flag(L.remote_flag, (uint32_t)L.rposted, s));
+        return;
+    }
+    const int E = (int)L.ev.size();
+    {
+        std::unique_lock<std::mutex> g(L.mu);
+        L.cv.wait(g, [&] { return L.posted - L.waited < E || c->abort.load(); });
+        if (c->abort) throw Abort{};
+    }
+    CK(cudaEventRecord(L.ev[L.posted % E], s));
+    {
+        std::lock_guard<std::mutex> g(L.mu);
+        ++L.posted;
+    }
+    L.cv.notify_all();
+}
+
+void link_wait(pd_ctx *c, Link &L, cudaStream_t s, int64_t idx) {
+    if (L.remote) {
+        // flags are never reset: run r's message idx is value rbase + idx + 1
+        if (L.rcount < idx + 1) L.rcount = idx + 1;
+        CUresult r = driver()->streamWaitValue32(s, (CUdeviceptr)L.local_flag, (cuuint32_t)(L.rbase + idx + 1),
+                                                 CU_STREAM_WAIT_VALUE_GEQ);
+        if (r != CUDA_SUCCESS) throw CudaFail{cudaErrorUnknown, "cuStreamWaitValue32"};
+        return;
+    }
+    const int E = (int)L.ev.size();
+    {
+        std::unique_lock<std::mutex> g(L.mu);
+        L.cv.wait(g, [&] { return L.posted > idx || c->abort.load(); });
+        if (c->abort) throw Abort{};
+    }
+    CK(cudaStreamWaitEvent(s, L.ev[idx % E], 0));
+    {
+        std::lock_guard<std::mutex> g(L.mu);
+        if (L.waited < idx + 1) L.waited = idx + 1;
+    }
+    L.cv.notify_all();
+}
+
+// ---------------------------------------------------------------- layer kernels
+struct LayerCtx {
+    pd_ctx *c;
+    Worker *w;
+    int bf16;
+};
+
+const void *elem_ptr(const void *base, long idx, int esz) { return static_cast<const char *>(base) + idx * esz; }
+void *elem_ptr(void *base, long idx, int esz) { return static_cast<char *>(base) + idx * esz; }
+
+cudaError_t run_gemm(int bf16, const Gemm &g, cudaStream_t s) { return bf16 ? gemm_bf16(g, s) : gemm_f32(g, s); }
+
+// y = act(x W^T + b)
+void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, const float *bias_f32, const void *x,
+                    void *y) {
+    const int B = L.c->cfg.minibatch;
+    Gemm g;
+    g.M = (int)rows_of(d, B);
+    g.N = d.out;
+    g.K = d.in;
+    g.A = x;
+    g.lda = d.in;
+    g.amaj = KMAJ;
+    g.B = W;
+    g.ldb = d.in;
+    g.bmaj = KMAJ;
+    g.epi = EPI_STORE;
+    g.out = y;
+    g.ldo = d.out;
+    g.bias = bias_f32;
+    g.relu = d.act == PD_ACT_RELU;
+    CK(run_gemm(L.bf16, g, L.w->stream));
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------- worker execution
+namespace {
+
+struct Exec {
+    pd_ctx *c;
+    Worker *w;
+    int M;
+    std::vector<int> k;  // in-flight counts of this run
+    int bf16;
+    int esz;
+    bool timing;
+    int ev_used = 0;
+
+    const pd_layer_desc &layer(int l) const { return c->layers[l]; }
+    int B() const { return c->cfg.minibatch; }
+    int n() const { return c->n; }
+
+    // weights of layer l in stash slot `slot` (path dtype)
+    void *Wl(int l, int slot) const { return elem_ptr(w->wslot[slot], c->poff[l], esz); }
+    // fp32 bias of layer l: the master (bf16 path) or the slot itself (fp32 path)
+    const float *bias_f32(int l, int slot) const {
+        const pd_layer_desc &d = layer(l);
+        const long off = c->poff[l] + (long)d.out * d.in;
+        if (bf16) return w->master + off;  // master holds the latest version
+        return static_cast<const float *>(w->wslot[slot]) + off;
+    }
+
+    // input of layer l for local index j
+    const void *layer_input(int l, int t, int j) const {
+        const pd_layer_desc &d = layer(l);
+        if (l == w->first) {
+            if (w->stage == 0) {
+                const int di = t % c->n_data;
+                if (d.kind == PD_EMBEDDING) return w->tokens + (long)di * in_elems(d, B());
+                return elem_ptr(w->data_in, (long)di * in_elems(d, B()), esz);
+            }
+            return elem_ptr(w->recv, (long)(j % w->D) * in_elems(d, B()), esz);
+        }
+        return elem_ptr(w->act[l - w->first], (long)(j % w->k) * in_elems(d, B()), esz);
+    }
+
+    void record_start() {
+        if (!timing) return;
+        cudaEvent_t a = w->ev_pool[ev_used++];
+        CK(cudaEventRecord(a, w->stream));
+        w->op_ev.push_back({a, nullptr});
+    }
+    void record_end() {
+        if (!timing) return;
+        cudaEvent_t b = w->ev_pool[ev_used++];
+        CK(cudaEventRecord(b, w->stream));
+        w->op_ev.back().second = b;
+    }
+    void trace(char kind, int mb, int vin, int vout) {
+        if (!c->cfg.record_trace) return;
+        pd_event e{};
+        e.worker = (int16_t)w->id;
+        e.stage = (int16_t)w->stage;
+        e.replica = (int16_t)w->replica;
+        e.kind = kind;
+        e.seq = (int32_t)w->events.size();
+        e.minibatch = mb;
+        e.version_in = vin;
+        e.version_out = vout;
+        e.start_us = e.end_us = NAN;
+        w->events.push_back(e);
+    }
+
+    // ---------------- F(s, t)
+    void forward(int t, int j) {
+        const int s = w->stage;
+        if (s > 0) {
+            const int p = t % c->plan.stage[s - 1].replicas;
+            const int src = c->worker_id(s - 1, p);
+            Link &L = get_link(c, L_ACT, src, w->id);
+            // message index on this link: minibatches from p to this replica before t
+            link_wait(c, L, w->stream, act_msg_index(s - 1, t));
+        }
+        const int v = w->version;
+        const int slot = v % w->k;
+        w->fwd_version[j] = v;
+        if (c->cfg.record_trace) c->vmap[(long)s * M + t] = v;
+        trace('F', t, v, v);
+        record_start();
+        for (int l = w->first; l <= w->last; ++l) {
+            const pd_layer_desc &d = layer(l);
+            const void *x = layer_input(l, t, j);
+            void *y;
+            if (l < w->last) {
+                y = elem_ptr(w->act[l + 1 - w->first], (long)(j % w->k) * in_elems(layer(l + 1), B()), esz);
+            } else if (s + 1 < n()) {
+                const int Rn = c->plan.stage[s + 1].replicas;
+                const int cw = c->worker_id(s + 1, t % Rn);
+                const int jc = t / Rn;
+                const Shared &sh = c->shared[cw];
+                y = elem_ptr(sh.recv, (long)(jc % c->Dalloc[s + 1]) * out_elems(d, B()), esz);
+                w->bytes_sent += (uint64_t)out_elems(d, B()) * esz;
+            } else {
+                y = w->logits;
+            }
+            if (d.kind != PD_LINEAR) throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
+            LayerCtx lc{c, w, bf16};
+            linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y);
+        }
+        if (s + 1 == n()) {
+            const pd_layer_desc &d = layer(w->last);
+            const long rows = rows_of(d, B());
+            CK(softmax_ce(w->logits, bf16, w->labels + (long)(t % c->n_data) * rows, rows, d.out, w->dlogits,
+                          w->losses + t, w->stream));
+        } else {
+            const int Rn = c->plan.stage[s + 1].replicas;
+            Link &L = get_link(c, L_ACT, w->id, c->worker_id(s + 1, t % Rn));
+            link_post(c, L, w->stream);
+        }
+        record_end();
+    }
+
+    // message index of minibatch t on the act link (stage ps replica t%Rp) -> (ps+1 replica t%Rc)
+    int64_t act_msg_index(int ps, int t) const {
+        const int Rp = c->plan.stage[ps].replicas, Rc = c->plan.stage[ps + 1].replicas;
+        int64_t cnt = 0;
+        for (int u = 0; u < t; ++u)
+            if (u % Rp == t % Rp && u % Rc == t % Rc) ++cnt;
+        return cnt;
+    }
+
+    // ---------------- B(s, t)
+    void backward(int t, int j) {
+        const int s = w->stage;
+        const int Rs = c->plan.stage[s].replicas;
+        if (s + 1 < n()) {
+            const int Rn = c->plan.stage[s + 1].replicas;
+            Link &L = get_link(c, L_GRAD, c->worker_id(s + 1, t % Rn), w->id);
+            link_wait(c, L, w->stream, act_msg_index(s, t));
+        }
+        const int vst = w->fwd_version[j];
+        const int sslot = vst % w->k;  // stashed version (L1157-1161)
+        trace('B', t, vst, vst);
+        record_start();
+        const int jr = j;  // round index on a replicated stage
+        if (Rs > 1 && jr >= 2) {
+            // gradient buffer parity jr%2 was last read by every replica in round jr-2
+            for (int r = 0; r < Rs; ++r) {
+                if (r == w->replica) continue;
+                Link &L = get_link(c, L_DONE, c->worker_id(s, r), w->id);
+                link_wait(c, L, w->stream, jr - 2);
+            }
+        }
+        // gradient w.r.t. the stage output (pre-activation of the last layer)
+        const void *G = (s + 1 == n()) ? w->dlogits
+                                       : elem_ptr(w->gring, (long)(j % w->G) * out_elems(layer(w->last), B()), esz);
+        int cur = 0;
+        const bool fused = bf16 && Rs == 1;  // dW + optimizer update in one GEMM epilogue
+        float *gdst = Rs > 1 ? w->rgrad[jr & 1] : w->gbuf;
+        const int next_version = w->version + 1;
+        const int nslot = next_version % w->k;
+        for (int l = w->last; l >= w->first; --l) {
+            const pd_layer_desc &d = layer(l);
+            if (d.kind != PD_LINEAR) throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
+            const void *x = layer_input(l, t, j);
+            const long rows = rows_of(d, B());
+            const bool need_dx = !(s == 0 && l == 0);
+            void *dx = nullptr;
+            if (need_dx) {
+                if (l == w->first) {
+                    const int Rp = c->plan.stage[s - 1].replicas;
+                    const int pw = c->worker_id(s - 1, t % Rp);
+                    const int jp = t / Rp;
+                    dx = elem_ptr(c->shared[pw].grad, (long)(jp % c->Galloc[s - 1]) * in_elems(d, B()), esz);
+                    w->bytes_sent += (uint64_t)in_elems(d, B()) * esz;
+                } else {
+                    dx = w->scratch[cur ^ 1];
+                }
+                // dX = G W, fused with the derivative of the previous layer's ReLU, which is
+                // evaluated from this layer's stashed input (post-ReLU, so x > 0 <=> z > 0).
+                const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
+                Gemm g;
+                g.M = (int)rows;
+                g.N = d.in;
+                g.K = d.out;
+                g.A = G;
+                g.lda = d.out;
+                g.amaj = KMAJ;
+                g.B = Wl(l, sslot);
+                g.ldb = d.in;
+                g.bmaj = MNMAJ;
+                g.epi = prev_relu ? EPI_MASK : EPI_STORE;
+                g.out = dx;
+                g.ldo = d.in;
+                g.mask = prev_relu ? x : nullptr;
+                g.ldm = d.in;
+                CK(run_gemm(bf16, g, w->stream));
+            }
+            // dW = G^T X
+            {
+                Gemm g;
+                g.M = d.out;
+                g.N = d.in;
+                g.K = (int)rows;
+                g.A = G;
+                g.lda = d.out;
+                g.amaj = MNMAJ;
+                g.B = x;
+                g.ldb = d.in;
+                g.bmaj = MNMAJ;
+                g.ldo = d.in;
+                const long woff = c->poff[l];
+                if (fused) {
+                    const bool adam = c->cfg.optimizer == PD_ADAM;
+                    g.epi = adam ? EPI_ADAM : EPI_SGD;
+                    g.master = w->master + woff;
+                    g.slot = elem_ptr(w->wslot[nslot], woff, esz);
+                    g.adam_m = adam ? w->adam_m + woff : nullptr;
+                    g.adam_v = adam ? w->adam_v + woff : nullptr;
+                    g.lr = c->cfg.lr;
+                    g.b1 = c->cfg.beta1;
+                    g.b2 = c->cfg.beta2;
+                    g.eps = c->cfg.eps;
+                    g.step = w->updates_total + 1;
+                } else {
+                    g.epi = EPI_F32;
+                    g.out = gdst + woff;
+                }
+                CK(run_gemm(bf16, g, w->stream));
+            }
+            // db = column sums of G
+            const long boff = c->poff[l] + (long)d.out * d.in;
+            CK(col_sum(G, bf16, rows, d.out, gdst + boff, w->stream));
+            if (fused) {
+                CK(update_master(w->master + boff, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[nslot], boff, esz)),
+                                 nullptr, w->self_grad_ptr, 1, boff, d.out, c->cfg.optimizer,
+                                 w->adam_m ? w->adam_m + boff : nullptr, w->adam_v ? w->adam_v + boff : nullptr,
+                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1,
+                                 w->stream));
+            }
+            G = dx;
+            cur ^= 1;
+        }
+        if (s > 0) {
+            const int Rp = c->plan.stage[s - 1].replicas;
+            Link &L = get_link(c, L_GRAD, w->id, c->worker_id(s - 1, t % Rp));
+            link_post(c, L, w->stream);
+        }
+        if (Rs > 1) {
+            for (int r = 0; r < Rs; ++r) {
+                if (r == w->replica) continue;
+                Link &L = get_link(c, L_READY, w->id, c->worker_id(s, r));
+                link_post(c, L, w->stream);
+            }
+        }
+        record_end();
+    }
+
+    // ---------------- U: weight update to the LATEST version (L1341-1353)
+    void update(int t, int j) {
+        const int s = w->stage;
+        const int Rs = c->plan.stage[s].replicas;
+        const int vin = w->version;
+        const int nslot = (vin + 1) % w->k;
+        trace('U', Rs > 1 ? j : t, vin, vin + 1);
+        const bool adam = c->cfg.optimizer == PD_ADAM;
+        const int step = w->updates_total + 1;
+        if (Rs > 1) {
+            // round j: wait for every peer's gradient, then one fused reduce + update kernel
+            for (int r = 0; r < Rs; ++r) {
+                if (r == w->replica) continue;
+                Link &L = get_link(c, L_READY, c->worker_id(s, r), w->id);
+                link_wait(c, L, w->stream, j);
+            }
+            if (bf16) {
+                CK(update_master(w->master, static_cast<__nv_bfloat16 *>(w->wslot[nslot]), nullptr,
+                                 w->rgrad_ptrs + (j & 1) * Rs, Rs, 0, w->P, c->cfg.optimizer, w->adam_m, w->adam_v,
+                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, step, w->stream));
+            } else {
+                // fp32 path: master == latest slot; new version into the next slot
+                const int lslot = vin % w->k;
+                if (nslot != lslot)
+                    CK(cudaMemcpyAsync(w->wslot[nslot], w->wslot[lslot], w->P * 4, cudaMemcpyDeviceToDevice,
+                                       w->stream));
+                CK(update_master(static_cast<float *>(w->wslot[nslot]), nullptr, nullptr, w->rgrad_ptrs + (j & 1) * Rs,
+                                 Rs, 0, w->P, c->cfg.optimizer, w->adam_m, w->adam_v, c->cfg.lr, c->cfg.beta1,
+                                 c->cfg.beta2, c->cfg.eps, step, w->stream));
+            }
+            for (int r = 0; r < Rs; ++r) {
+                if (r == w->replica) continue;
+                Link &L = get_link(c, L_DONE, w->id, c->worker_id(s, r));
+                link_post(c, L, w->stream);
+            }
+        } else if (!bf16) {
+            const float *latest = static_cast<const float *>(w->wslot[vin % w->k]);
+            float *next = static_cast<float *>(w->wslot[nslot]);
+            if (adam)
+                CK(adam_f32(latest, w->gbuf, next, w->adam_m, w->adam_v, w->P, c->cfg.lr, c->cfg.beta1, c->cfg.beta2,
+                            c->cfg.eps, step, w->stream));
+            else
+                CK(sgd_f32(latest, w->gbuf, next, w->P, c->cfg.lr, w->stream));
+        }
+        // (bf16 unreplicated: the update was fused into B's dW epilogues)
+        w->version = vin + 1;
+        w->updates_total += 1;
+        w->fwd_version.erase(j);
+    }
+
+    void run_ops() {
+        const int Rs = c->plan.stage[w->stage].replicas;
+        std::vector<Op> ops = worker_ops(Rs, w->replica, k[w->stage], M);
+        for (const Op &op : ops) {
+            if (c->abort) throw Abort{};
+            if (op.kind == 'F') forward(op.t, op.j);
+            else if (op.kind == 'B') backward(op.t, op.j);
+            else update(op.t, op.j);
+        }
+    }
+};
+
+void worker_thread(pd_ctx *c, Worker *w, int M, std::vector<int> k) {
+    tl_launches = 0;
+    try {
+        CK(cudaSetDevice(w->device));
+        Exec ex{c, w, M, k, c->cfg.dtype == PD_BF16, c->esz, c->cfg.record_trace >= 2};
+        ex.run_ops();
+        CK(cudaStreamSynchronize(w->stream));
+    } catch (const CudaFail &f) {
+        char buf[256];
+        snprintf(buf, sizeof buf, "worker %d: %s failed: %s", w->id, f.what, cudaGetErrorString(f.e));
+        c->fail(f.e == cudaErrorNotSupported ? PD_EUNSUPPORTED : PD_ECUDA, buf);
+    } catch (const Abort &) {
+        if (w->stream) cudaStreamSynchronize(w->stream);
+    }
+    w->launches = tl_launches;
+}
+
+}  // namespace
+
+// ================================================================== C ABI
+#define CHECK_CTX(ctx)                          \
+    do {                                        \
+        if (!(ctx)) return PD_EINVAL;           \
+        if ((ctx)->sticky != PD_OK) return PD_ESTATE; \
+    } while (0)
+
+extern "C" {
+
+const char *pd_strerror(pd_status s) {
+    switch (s) {
+    case PD_OK: return "ok";
+    case PD_EINVAL: return "invalid argument";
+    case PD_ENOMEM: return "out of memory";
+    case PD_ECUDA: return "CUDA error";
+    case PD_ENCCL: return "collective transport error";
+    case PD_ESTATE: return "invalid state (earlier error or wrong call order)";
+    case PD_EUNSUPPORTED: return "unsupported";
+    case PD_EINFEASIBLE: return "no feasible plan";
+    }
+    return "unknown status";
+}
+
+const char *pd_last_error(pd_ctx *ctx) { return ctx ? ctx->err.c_str() : ""; }
+
+pd_status pd_inflight(const pd_plan_t *plan, int noam, int *k_out) {
+    if (!plan || !k_out || plan->num_stages < 1 || plan->num_stages > PD_MAX_STAGES) return PD_EINVAL;
+    std::vector<int> k;
+    pd_status st = inflight_counts(*plan, noam, k);
+    if (st != PD_OK) return st;
+    for (int s = 0; s < plan->num_stages; ++s) k_out[s] = k[s];
+    return PD_OK;
+}
+
+pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *layers, int num_layers,
+                    const pd_train_cfg *cfg) {
+    if (!out || !plan || !layers || !cfg || num_layers < 1) return PD_EINVAL;
+    const int n = plan->num_stages;
+    if (n < 1 || n > PD_MAX_STAGES) return PD_EINVAL;
+    int expect = 0, total_workers = 0;
+    for (int s = 0; s < n; ++s) {
+        const pd_stage_desc &sd = plan->stage[s];
+        if (sd.first_layer != expect || sd.last_layer < sd.first_layer || sd.replicas < 1) return PD_EINVAL;
+        expect = sd.last_layer + 1;
+        total_workers += sd.replicas;
+    }
+    if (expect != num_layers) return PD_EINVAL;
+    if (cfg->minibatch < 1 || (cfg->dtype != PD_FP32 && cfg->dtype != PD_BF16)) return PD_EINVAL;
+    if (cfg->optimizer != PD_SGD && cfg->optimizer != PD_ADAM) return PD_EINVAL;
+    for (int l = 0; l < num_layers; ++l) {
+        const pd_layer_desc &d = layers[l];
+        if (d.in < 1 || d.out < 1 || numel_params(d) < 0) return PD_EINVAL;
+        if (l > 0 && in_elems(d, 1) != out_elems(layers[l - 1], 1) && d.kind != PD_EMBEDDING) return PD_EINVAL;
+        if (d.kind != PD_LINEAR) return PD_EUNSUPPORTED;  // other layer kinds: see DESIGN.md "status"
+        if (cfg->dtype == PD_BF16 && (d.in % 8 || d.out % 8)) return PD_EUNSUPPORTED;  // 16-byte rows for TMA
+    }
+    std::vector<int> kdef, kmax;
+    if (inflight_counts(*plan, 0, kdef) != PD_OK) return PD_EINVAL;
+    kmax = kdef;
+    if (cfg->max_depth > 0) {
+        if (inflight_counts(*plan, cfg->max_depth, kmax) != PD_OK) return PD_EINVAL;
+        for (int s = 0; s < n; ++s) kmax[s] = std::max(kmax[s], kdef[s]);
+    }
+    pd_ctx *c = new pd_ctx;
+    c->plan = *plan;
+    c->layers.assign(layers, layers + num_layers);
+    c->cfg = *cfg;
+    c->n = n;
+    c->nw = total_workers;
+    c->kdef = kdef;
+    c->kalloc = kmax;
+    c->esz = cfg->dtype == PD_BF16 ? 2 : 4;
+    int id = 0;
+    for (int s = 0; s < n; ++s) {
+        c->wbase.push_back(id);
+        id += plan->stage[s].replicas;
+    }
+    c->Dalloc.assign(n, 0);
+    c->Galloc.assign(n, 0);
+    for (int s = 1; s < n; ++s) c->Dalloc[s] = recv_ring_depth(*plan, kmax, s);
+    for (int s = 0; s + 1 < n; ++s) c->Galloc[s] = kmax[s];
+    c->poff.assign(num_layers, 0);
+    c->pcount.assign(num_layers, 0);
+    for (int s = 0; s < n; ++s) {
+        long off = 0;
+        for (int l = plan->stage[s].first_layer; l <= plan->stage[s].last_layer; ++l) {
+            c->poff[l] = off;
+            c->pcount[l] = numel_params(layers[l]);
+            off += align_up(c->pcount[l], 64);  // 256-byte aligned layer blocks
+        }
+    }
+    c->W.resize(total_workers);
+    c->shared.resize(total_workers);
+    *out = c;
+    return PD_OK;
+}
+
+pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float *const *init_params) {
+    CHECK_CTX(c);
+    if (stage < 0 || stage >= c->n || replica < 0 || replica >= c->plan.stage[stage].replicas) return PD_EINVAL;
+    const int id = c->worker_id(stage, replica);
+    if (c->W[id] || c->shared[id].valid) return PD_EINVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        c->fail(PD_ECUDA, "no CUDA device");
+        return PD_ECUDA;
+    }
+    if (dev < 0 || dev >= ndev) return PD_EINVAL;
+    if (!driver()) {
+        c->fail(PD_ECUDA, "CUDA driver entry points unavailable");
+        return PD_ECUDA;
+    }
+    auto w = std::make_unique<Worker>();
+    w->ctx = c;
+    w->id = id;
+    w->stage = stage;
+    w->replica = replica;
+    w->device = dev;
+    w->first = c->plan.stage[stage].first_layer;
+    w->last = c->plan.stage[stage].last_layer;
+    w->k = c->kalloc[stage];
+    w->D = stage > 0 ? c->Dalloc[stage] : 0;
+    w->G = stage + 1 < c->n ? c->Galloc[stage] : 0;
+    const int B = c->cfg.minibatch;
+    const int esz = c->esz;
+    const bool bf16 = c->cfg.dtype == PD_BF16;
+    const int Rs = c->plan.stage[stage].replicas;
+    try {
+        CK(cudaSetDevice(dev));
+        int major = 0;
+        CK(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev));
+        if (major != 10) {
+            c->fail(PD_EUNSUPPORTED, "requires an sm_100 (B200) device");
+            return PD_EUNSUPPORTED;
+        }
+        CK(cudaStreamCreateWithFlags(&w->stream, cudaStreamNonBlocking));
+        long P = 0;
+        for (int l = w->first; l <= w->last; ++l) P = c->poff[l] + align_up(c->pcount[l], 64);
+        w->P = P;
+        // weights: stage buffer in the parameter layout, fp32 staging -> every slot
+        float *stage_f32 = dalloc<float>(P * 4);
+        std::vector<float> host(P, 0.f);
+        for (int l = w->first; l <= w->last; ++l) {
+            const float *src = init_params ? init_params[l - w->first] : nullptr;
+            if (c->pcount[l] > 0) {
+                if (!src) throw CudaFail{cudaErrorInvalidValue, "missing init params"};
+                std::memcpy(host.data() + c->poff[l], src, c->pcount[l] * sizeof(float));
+            }
+        }
+        CK(cudaMemcpy(stage_f32, host.data(), P * 4, cudaMemcpyHostToDevice));
+        for (int q = 0; q < w->k; ++q) {
+            void *slot = dalloc<void>(P * esz);
+            if (bf16) CK(f32_to_bf16(stage_f32, static_cast<__nv_bfloat16 *>(slot), P, nullptr));
+            else CK(cudaMemcpy(slot, stage_f32, P * 4, cudaMemcpyDeviceToDevice));
+            w->wslot.push_back(slot);
+        }
+        if (bf16) w->master = stage_f32;
+        else cudaFree(stage_f32);
+        if (c->cfg.optimizer == PD_ADAM) {
+            w->adam_m = dalloc<float>(P * 4);
+            w->adam_v = dalloc<float>(P * 4);
+        }
+        w->gbuf = dalloc<float>(P * 4);
+        {
+            const float *one[1] = {w->gbuf};
+            w->self_grad_ptr = dalloc<const float *>(sizeof(one));
+            CK(cudaMemcpy(w->self_grad_ptr, one, sizeof(one), cudaMemcpyHostToDevice));
+        }
+        if (Rs > 1) {
+            w->rgrad[0] = dalloc<float>(P * 4);
+            w->rgrad[1] = dalloc<float>(P * 4);
+            w->rgrad_ptrs = dalloc<const float *>(sizeof(float *) * 2 * Rs);
+        }
+        // activation stash for inner layers
+        w->act.assign(w->last - w->first + 1, nullptr);
+        long max_elems = 0;
+        for (int l = w->first; l <= w->last; ++l) {
+            max_elems = std::max(max_elems, std::max(in_elems(c->layers[l], B), out_elems(c->layers[l], B)));
+            if (l > w->first) w->act[l - w->first] = dalloc<void>((size_t)w->k * in_elems(c->layers[l], B) * esz);
+        }
+        w->scratch[0] = dalloc<void>(max_elems * esz);
+        w->scratch[1] = dalloc<void>(max_elems * esz);
+        if (stage > 0) w->recv = dalloc<void>((size_t)w->D * in_elems(c->layers[w->first], B) * esz);
+        if (stage + 1 < c->n) w->gring = dalloc<void>((size_t)w->G * out_elems(c->layers[w->last], B) * esz);
+        if (stage + 1 == c->n) {
+            const long lo = out_elems(c->layers[w->last], B);
+            w->logits = dalloc<void>(lo * esz);
+            w->dlogits = dalloc<void>(lo * esz);
+        }
+        w->flags = dalloc<uint32_t>(sizeof(uint32_t) * std::max(1, c->flag_count(stage)));
+        CK(cudaDeviceSynchronize());
+        // the worker's shareable buffers
+        Shared &sh = c->shared[id];
+        sh.recv = w->recv;
+        sh.grad = w->gring;
+        sh.rgrad[0] = w->rgrad[0];
+        sh.rgrad[1] = w->rgrad[1];
+        sh.flags = w->flags;
+        sh.valid = true;
+    } catch (const CudaFail &f) {
+        cudaGetLastError();
+        c->shared[id] = Shared{};
+        return f.e == cudaErrorMemoryAllocation ? PD_ENOMEM : PD_ECUDA;
+    }
+    c->W[id] = std::move(w);
+    return PD_OK;
+}
+
+pd_status pd_export_worker(pd_ctx *c, int stage, int replica, void *blob, size_t cap, size_t *len) {
+    CHECK_CTX(c);
+    if (!len || stage < 0 || stage >= c->n || replica < 0 || replica >= c->plan.stage[stage].replicas) return PD_EINVAL;
+    *len = sizeof(IpcBlob);
+    const int id = c->worker_id(stage, replica);
+    Worker *w = c->W[id].get();
+    if (!w || !blob || cap < sizeof(IpcBlob)) return PD_EINVAL;
+    IpcBlob b{};
+    b.magic = BLOB_MAGIC;
+    b.stage = stage;
+    b.replica = replica;
+    b.device = w->device;
+    if (cudaSetDevice(w->device) != cudaSuccess) return PD_ECUDA;
+    if (w->recv) {
+        b.has_recv = 1;
+        if (cudaIpcGetMemHandle(&b.recv, w->recv) != cudaSuccess) return PD_ECUDA;
+    }
+    if (w->gring) {
+        b.has_grad = 1;
+        if (cudaIpcGetMemHandle(&b.grad, w->gring) != cudaSuccess) return PD_ECUDA;
+    }
+    if (w->rgrad[0]) {
+        b.has_rgrad = 1;
+        if (cudaIpcGetMemHandle(&b.rgrad0, w->rgrad[0]) != cudaSuccess) return PD_ECUDA;
+        if (cudaIpcGetMemHandle(&b.rgrad1, w->rgrad[1]) != cudaSuccess) return PD_ECUDA;
+    }
+    if (cudaIpcGetMemHandle(&b.flags, w->flags) != cudaSuccess) return PD_ECUDA;
+    std::memcpy(blob, &b, sizeof b);
+    return PD_OK;
+}
+
+pd_status pd_import_worker(pd_ctx *c, const void *blob, size_t len) {
+    CHECK_CTX(c);
+    if (!blob || len < sizeof(IpcBlob)) return PD_EINVAL;
+    IpcBlob b;
+    std::memcpy(&b, blob, sizeof b);
+    if (b.magic != BLOB_MAGIC || b.stage < 0 || b.stage >= c->n || b.replica < 0 ||
+        b.replica >= c->plan.stage[b.stage].replicas)
+        return PD_EINVAL;
+    const int id = c->worker_id(b.stage, b.replica);
+    if (c->W[id]) return PD_EINVAL;  // local worker
+    if (c->shared[id].valid) return PD_OK;
+    // map into the device of a local worker (any; peer pointers are UVA)
+    int dev = -1;
+    for (auto &w : c->W)
+        if (w) { dev = w->device; break; }
+    if (dev < 0) return PD_ESTATE;
+    if (cudaSetDevice(dev) != cudaSuccess) return PD_ECUDA;
+    Shared sh;
+    auto open = [&](const cudaIpcMemHandle_t &h, void **p) {
+        return cudaIpcOpenMemHandle(p, h, cudaIpcMemLazyEnablePeerAccess) == cudaSuccess;
+    };
+    bool ok = true;
+    if (b.has_recv) ok = ok && open(b.recv, &sh.recv);
+    if (b.has_grad) ok = ok && open(b.grad, &sh.grad);
+    if (b.has_rgrad) {
+        ok = ok && open(b.rgrad0, reinterpret_cast<void **>(&sh.rgrad[0]));
+        ok = ok && open(b.rgrad1, reinterpret_cast<void **>(&sh.rgrad[1]));
+    }
+    ok = ok && open(b.flags, reinterpret_cast<void **>(&sh.flags));
+    if (!ok) {
+        cudaGetLastError();
+        return PD_ECUDA;
+    }
+    sh.valid = true;
+    c->shared[id] = sh;
+    return PD_OK;
+}
+
+pd_status pd_set_data(pd_ctx *c, const float *inputs, const int32_t *tokens, const int32_t *labels, int nd) {
+    CHECK_CTX(c);
+    if (nd < 1) return PD_EINVAL;
+    const int B = c->cfg.minibatch;
+    const pd_layer_desc &L0 = c->layers.front();
+    const pd_layer_desc &LL = c->layers.back();
+    const bool emb = L0.kind == PD_EMBEDDING;
+    if (emb ? !tokens : !inputs) return PD_EINVAL;
+    if (!labels) return PD_EINVAL;
+    const long in_n = in_elems(L0, B), rows = rows_of(LL, B);
+    try {
+        for (auto &wp : c->W) {
+            Worker *w = wp.get();
+            if (!w) continue;
+            CK(cudaSetDevice(w->device));
+            if (w->stage == 0) {
+                if (emb) {
+                    if (c->n_data != nd || !w->tokens) {
+                        if (w->tokens) cudaFree(w->tokens);
+                        w->tokens = dalloc<int32_t>((size_t)nd * in_n * 4);
+                    }
+                    CK(cudaMemcpyAsync(w->tokens, tokens, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice, w->stream));
+                } else {
+                    if (c->n_data != nd || !w->data_in) {
+                        if (w->data_in) cudaFree(w->data_in);
+                        w->data_in = dalloc<void>((size_t)nd * in_n * c->esz);
+                    }
+                    if (c->esz == 4) {
+                        CK(cudaMemcpyAsync(w->data_in, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice,
+                                           w->stream));
+                    } else {
+                        float *tmp = nullptr;
+                        CK(cudaMallocAsync(reinterpret_cast<void **>(&tmp), (size_t)nd * in_n * 4, w->stream));
+                        CK(cudaMemcpyAsync(tmp, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice, w->stream));
+                        CK(f32_to_bf16(tmp, static_cast<__nv_bfloat16 *>(w->data_in), (long)nd * in_n, w->stream));
+                        CK(cudaFreeAsync(tmp, w->stream));
+                    }
+                }
+            }
+            if (w->stage + 1 == c->n) {
+                if (c->n_data != nd || !w->labels) {
+                    if (w->labels) cudaFree(w->labels);
+                    w->labels = dalloc<int32_t>((size_t)nd * rows * 4);
+                }
+                CK(cudaMemcpyAsync(w->labels, labels, (size_t)nd * rows * 4, cudaMemcpyHostToDevice, w->stream));
+            }
+        }
+    } catch (const CudaFail &f) {
+        c->fail(PD_ECUDA, std::string("pd_set_data: ") + f.what + ": " + cudaGetErrorString(f.e));
+        return PD_ECUDA;
+    }
+    c->n_data = nd;
+    return PD_OK;
+}
+
+pd_status pd_run(pd_ctx *c, int M, int noam) {
+    CHECK_CTX(c);
+    if (M < 1) return PD_EINVAL;
+    for (int s = 0; s < c->n; ++s)
+        if (M % c->plan.stage[s].replicas) return PD_EINVAL;
+    std::vector<int> k;
+    if (inflight_counts(c->plan, noam, k) != PD_OK) return PD_EINVAL;
+    for (int s = 0; s < c->n; ++s)
+        if (k[s] > c->kalloc[s]) return PD_EINVAL;
+    if (c->n_data < 1) return PD_ESTATE;
+    for (int id = 0; id < c->nw; ++id)
+        if (!c->shared[id].valid) return PD_ESTATE;
+    bool any_local = false;
+    for (auto &w : c->W) any_local = any_local || (bool)w;
+    if (!any_local) return PD_ESTATE;
+    // with a depth override the stash ring must still hold k_s versions at every worker
+    try {
+        // links (created once; local when both ends are in this process)
+        auto make_link = [&](int type, int src, int dst) {
+            auto key = std::make_tuple(type, src, dst);
+            if (c->links.count(key)) return;
+            auto L = std::make_unique<Link>();
+            Worker *ws = c->W[src].get(), *wd = c->W[dst].get();
+            if (ws && wd) {
+                L->remote = false;
+                L->device = ws->device;
+                CK(cudaSetDevice(ws->device));
+                const int E = 2 * std::max(8, std::max(c->Dalloc[wd->stage], c->kalloc[ws->stage])) + 4;
+                L->ev.resize(E);
+                for (auto &e : L->ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+                if (ws->device != wd->device) {
+                    int can = 0;
+                    CK(cudaDeviceCanAccessPeer(&can, ws->device, wd->device));
+                    if (can) {
+                        cudaError_t e = cudaDeviceEnablePeerAccess(wd->device, 0);
+                        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CK(e);
+                        cudaGetLastError();
+                        CK(cudaSetDevice(wd->device));
+                        e = cudaDeviceEnablePeerAccess(ws->device, 0);
+                        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CK(e);
+                        cudaGetLastError();
+                    }
+                }
+            } else {
+                L->remote = true;
+                const int ds = c->stage_of(dst), sst = c->stage_of(src);
+                const int sr = src - c->wbase[sst];
+                const int fi = c->flag_index(type, sst, sr, ds);
+                if (ws) L->remote_flag = c->shared[dst].flags + fi;  // IPC-mapped
+                if (wd) L->local_flag = wd->flags + fi;
+            }
+            c->links[key] = std::move(L);
+        };
+        for (int s = 0; s < c->n; ++s) {
+            const int Rs = c->plan.stage[s].replicas;
+            for (int r = 0; r < Rs; ++r) {
+                const int id = c->worker_id(s, r);
+                if (s + 1 < c->n) {
+                    const int Rn = c->plan.stage[s + 1].replicas;
+                    for (int q = 0; q < Rn; ++q) {
+                        const int od = c->worker_id(s + 1, q);
+                        if (c->W[id] || c->W[od]) {
+                            make_link(L_ACT, id, od);
+                            make_link(L_GRAD, od, id);
+                        }
+                    }
+                }
+                for (int q = 0; q < Rs; ++q) {
+                    const int od = c->worker_id(s, q);
+                    if (q != r && (c->W[id] || c->W[od])) {
+                        make_link(L_READY, id, od);
+                        make_link(L_DONE, id, od);
+                    }
+                }
+            }
+        }
+        // reset the host-side counters of local links; remote flags are monotonic across
+        // runs (no reset, so no cross-process barrier is needed before a run)
+        for (auto &kv : c->links) {
+            Link &L = *kv.second;
+            L.posted = L.waited = 0;
+            L.rbase += L.rcount;
+            L.rcount = 0;
+        }
+        for (auto &wp : c->W) {
+            Worker *w = wp.get();
+            if (!w) continue;
+            CK(cudaSetDevice(w->device));
+            if (w->stage + 1 == c->n && w->losses_cap < M) {
+                if (w->losses) cudaFree(w->losses);
+                w->losses = dalloc<float>((size_t)M * 4);
+                w->losses_cap = M;
+            }
+            if (w->stage + 1 == c->n) CK(cudaMemsetAsync(w->losses, 0, (size_t)M * 4, w->stream));
+            const int Rs = c->plan.stage[w->stage].replicas;
+            if (Rs > 1) {
+                std::vector<const float *> ptrs(2 * Rs);
+                for (int par = 0; par < 2; ++par)
+                    for (int r = 0; r < Rs; ++r) ptrs[par * Rs + r] = c->shared[c->worker_id(w->stage, r)].rgrad[par];
+                CK(cudaMemcpy(w->rgrad_ptrs, ptrs.data(), sizeof(float *) * ptrs.size(), cudaMemcpyHostToDevice));
+            }
+            w->events.clear();
+            w->op_ev.clear();
+            const size_t need = c->cfg.record_trace >= 2 ? (size_t)6 * M + 16 : 0;
+            while (w->ev_pool.size() < need) {
+                cudaEvent_t e;
+                CK(cudaEventCreate(&e));
+                w->ev_pool.push_back(e);
+            }
+            CK(cudaStreamSynchronize(w->stream));
+        }
+    } catch (const CudaFail &f) {
+        c->fail(PD_ECUDA, std::string("pd_run setup: ") + f.what + ": " + cudaGetErrorString(f.e));
+        return PD_ECUDA;
+    }
+    c->last_M = M;
+    c->vmap.assign((size_t)c->n * M, -1);
+    auto t0 = std::chrono::steady_clock::now();
+    std::vector<std::thread> th;
+    for (auto &wp : c->W)
+        if (wp) th.emplace_back(worker_thread, c, wp.get(), M, k);
+    for (auto &t : th) t.join();
+    c->host_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    if (c->sticky != PD_OK) return c->sticky;
+    return PD_OK;
+}
+
+pd_status pd_get_params(pd_ctx *c, int layer, float *host_out, size_t count) {
+    CHECK_CTX(c);
+    if (layer < 0 || layer >= (int)c->layers.size() || !host_out) return PD_EINVAL;
+    if (count != (size_t)c->pcount[layer]) return PD_EINVAL;
+    int s = 0;
+    while (c->plan.stage[s].last_layer < layer) ++s;
+    Worker *w = nullptr;
+    for (int r = 0; r < c->plan.stage[s].replicas && !w; ++r) w = c->W[c->worker_id(s, r)].get();
+    if (!w) return PD_EINVAL;
+    if (count == 0) return PD_OK;
+    if (cudaSetDevice(w->device) != cudaSuccess) return PD_ECUDA;
+    const float *src = (c->cfg.dtype == PD_BF16) ? w->master : static_cast<const float *>(w->wslot[w->version % w->k]);
+    if (cudaMemcpy(host_out, src + c->poff[layer], count * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+        c->fail(PD_ECUDA, "pd_get_params copy");
+        return PD_ECUDA;
+    }
+    return PD_OK;
+}
+
+pd_status pd_get_trace(pd_ctx *c, pd_event *out, size_t cap, size_t *written) {
+    CHECK_CTX(c);
+    if (!written) return PD_EINVAL;
+    size_t total = 0;
+    for (auto &w : c->W)
+        if (w) total += w->events.size();
+    *written = total;
+    if (!out) return PD_OK;
+    if (cap < total) return PD_EINVAL;
+    size_t i = 0;
+    for (auto &wp : c->W) {
+        Worker *w = wp.get();
+        if (!w) continue;
+        const bool timed = c->cfg.record_trace >= 2 && w->op_ev.size() * 3 >= w->events.size() * 2;
+        size_t opi = 0;
+        for (auto &e : w->events) {
+            pd_event x = e;
+            if (timed && e.kind != 'U' && opi < w->op_ev.size() && w->op_ev[opi].second) {
+                float a = 0, b = 0;
+                cudaSetDevice(w->device);
+                if (cudaEventElapsedTime(&a, w->op_ev[0].first, w->op_ev[opi].first) == cudaSuccess &&
+                    cudaEventElapsedTime(&b, w->op_ev[0].first, w->op_ev[opi].second) == cudaSuccess) {
+                    x.start_us = a * 1000.f;
+                    x.end_us = b * 1000.f;
+                }
+                ++opi;
+            }
+            out[i++] = x;
+        }
+    }
+    return PD_OK;
+}
+
+pd_status pd_get_version_map(pd_ctx *c, int32_t *out, size_t cap) {
+    CHECK_CTX(c);
+    if (!out || cap < c->vmap.size()) return PD_EINVAL;
+    std::memcpy(out, c->vmap.data(), c->vmap.size() * 4);
+    return PD_OK;
+}
+
+pd_status pd_get_losses(pd_ctx *c, float *out, size_t cap) {
+    CHECK_CTX(c);
+    if (!out || cap < (size_t)c->last_M) return PD_EINVAL;
+    for (int t = 0; t < c->last_M; ++t) out[t] = NAN;
+    for (auto &wp : c->W) {
+        Worker *w = wp.get();
+        if (!w || w->stage + 1 != c->n || !w->losses) continue;
+        std::vector<float> tmp(c->last_M);
+        if (cudaSetDevice(w->device) != cudaSuccess ||
+            cudaMemcpy(tmp.data(), w->losses, (size_t)c->last_M * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            c->fail(PD_ECUDA, "pd_get_losses copy");
+            return PD_ECUDA;
+        }
+        const int Rs = c->plan.stage[w->stage].replicas;
+        for (int t = w->replica; t < c->last_M; t += Rs) out[t] = tmp[t];
+    }
+    return PD_OK;
+}
+
+pd_status pd_get_stats(pd_ctx *c, pd_stats *out) {
+    CHECK_CTX(c);
+    if (!out) return PD_EINVAL;
+    std::memset(out, 0, sizeof *out);
+    out->host_ms = c->host_ms;
+    double busy_sum = 0, span_max = 0;
+    int nl = 0;
+    for (auto &wp : c->W) {
+        Worker *w = wp.get();
+        if (!w) continue;
+        out->kernel_launches += w->launches;
+        out->bytes_sent += w->bytes_sent;
+        double busy = 0, span = 0;
+        if (!w->op_ev.empty() && w->op_ev.back().second) {
+            cudaSetDevice(w->device);
+            for (auto &pr : w->op_ev) {
+                float ms = 0;
+                if (pr.second && cudaEventElapsedTime(&ms, pr.first, pr.second) == cudaSuccess) busy += ms;
+            }
+            float sp = 0;
+            if (cudaEventElapsedTime(&sp, w->op_ev.front().first, w->op_ev.back().second) == cudaSuccess) span = sp;
+        }
+        if (nl < PD_MAX_LOCAL_WORKERS) {
+            out->worker_id[nl] = w->id;
+            out->busy_ms[nl] = busy;
+            out->span_ms[nl] = span;
+        }
+        busy_sum += busy;
+        span_max = std::max(span_max, span);
+        ++nl;
+    }
+    out->num_local_workers = nl;
+    out->device_ms = span_max;
+    out->bubble = (span_max > 0 && nl > 0) ? 1.0 - busy_sum / (nl * span_max) : 0.0;
+    return PD_OK;
+}
+
+void pd_destroy(pd_ctx *c) {
+    if (!c) return;
+    for (auto &w : c->W)
+        if (w) {
+            cudaSetDevice(w->device);
+            cudaStreamSynchronize(w->stream);
+        }
+    for (auto &kv : c->links)
+        for (auto e : kv.second->ev) cudaEventDestroy(e);
+    c->links.clear();
+    for (int id = 0; id < c->nw; ++id) {
+        if (c->W[id] || !c->shared[id].valid) continue;
+        Shared &sh = c->shared[id];
+        void *ps[] = {sh.recv, sh.grad, sh.rgrad[0], sh.rgrad[1], sh.flags};
+        for (void *p : ps)
+            if (p) cudaIpcCloseMemHandle(p);
+    }
+    c->W.clear();
+    delete c;
+}
+
+}  // extern "C"
+
+// ================================================================== kernel-level C ABI
+#include "../../include/pipedream_kernels.h"
+
+extern "C" PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *d, void *stream) {
+    if (!d || d->M < 1 || d->N < 1 || d->K < 1 || !d->A || !d->B) return PD_EINVAL;
+    if (d->epilogue < PD_EPI_STORE || d->epilogue > PD_EPI_ADAM) return PD_EINVAL;
+    if (d->dtype == PD_FP32 && d->epilogue > PD_EPI_F32) return PD_EINVAL;
+    Gemm g;
+    g.M = d->M; g.N = d->N; g.K = d->K;
+    g.A = d->A; g.lda = d->lda; g.amaj = d->a_mn_major ? MNMAJ : KMAJ;
+    g.B = d->B; g.ldb = d->ldb; g.bmaj = d->b_mn_major ? MNMAJ : KMAJ;
+    g.epi = d->epilogue;
+    g.out = d->out; g.ldo = d->ldo;
+    g.bias = d->bias; g.relu = d->relu;
+    g.mask = d->mask; g.ldm = d->ldm;
+    g.master = d->master; g.slot = d->slot; g.adam_m = d->adam_m; g.adam_v = d->adam_v;
+    g.lr = d->lr; g.b1 = d->beta1; g.b2 = d->beta2; g.eps = d->eps; g.step = d->step;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    cudaError_t e = d->dtype == PD_BF16 ? gemm_bf16(g, s) : gemm_f32(g, s);
+    if (e == cudaErrorInvalidValue) return PD_EINVAL;
+    return e == cudaSuccess ? PD_OK : PD_ECUDA;
+}
+
+extern "C" PD_API pd_status pd_kernel_softmax_ce(int dtype, const void *logits, const int32_t *labels, long rows,
+                                                 int C, void *dlogits, float *loss, void *stream) {
+    if (!logits || !labels || !dlogits || !loss || rows < 1 || C < 1) return PD_EINVAL;
+    cudaError_t e = softmax_ce(logits, dtype == PD_BF16, labels, rows, C, dlogits, loss,
+                               static_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? PD_OK : PD_ECUDA;
+}

@@ -1,0 +1,99 @@
+"""Pipeline session: wires the C-ABI calls together for one process (all workers local,
+several "virtual" workers may share a GPU) or one process per GPU (torch.distributed
+exchanges the CUDA-IPC blobs; plumbing only, no data-path collective)."""
+from __future__ import annotations
+
+from typing import Callable, Dict, List, Optional, Sequence
+
+import numpy as np
+
+from . import (PD_BF16, PD_SGD, Plan, pd_create, pd_destroy, pd_export_worker, pd_get_losses, pd_get_params,
+               pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data, pd_stage_init, pd_run)
+
+
+def workers_of(plan: Plan):
+    """(worker id, stage, replica, gpu) in plan order (consecutive GPUs per stage, R18)."""
+    out, wid = [], 0
+    for s, (first, last, reps, gpu0) in enumerate(plan.stages):
+        for r in range(reps):
+            out.append((wid, s, r, gpu0 + r))
+            wid += 1
+    return out
+
+
+class Pipeline:
+    def __init__(self, plan: Plan, layers, params: Sequence[np.ndarray], *, dtype=PD_BF16, optimizer=PD_SGD,
+                 lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8, minibatch=1, record_trace=1, max_depth=0,
+                 device_of: Optional[Callable[[int], int]] = None, local: Optional[Callable[[int], bool]] = None,
+                 allgather: Optional[Callable[[list], list]] = None):
+        """device_of(worker_gpu) -> CUDA ordinal (default: everything on device 0, i.e. virtual
+        workers); local(worker_id) -> whether this process owns the worker (default all);
+        allgather(list_of_bytes) -> list over processes of lists (needed when not all local)."""
+        self.plan, self.layers = plan, list(layers)
+        self.ctx = pd_create(plan, self.layers, dtype, optimizer, lr, beta1, beta2, eps, minibatch, record_trace,
+                             max_depth)
+        device_of = device_of or (lambda g: 0)
+        local = local or (lambda w: True)
+        self.workers = workers_of(plan)
+        self.local_ids = [w for w, s, r, g in self.workers if local(w)]
+        for wid, s, r, g in self.workers:
+            if not local(wid):
+                continue
+            first, last = plan.stages[s][0], plan.stages[s][1]
+            pd_stage_init(self.ctx, s, r, device_of(g), [params[l] for l in range(first, last + 1)])
+        if len(self.local_ids) < len(self.workers):
+            if allgather is None:
+                raise ValueError("remote workers need an allgather for the IPC blobs")
+            mine = [pd_export_worker(self.ctx, s, r) for wid, s, r, g in self.workers if local(wid)]
+            for blobs in allgather(mine):
+                for b in blobs:
+                    try:
+                        pd_import_worker(self.ctx, b)
+                    except Exception:
+                        # our own blobs come back too; the library rejects local workers
+                        pass
+
+    def set_data(self, inputs, tokens, labels, n):
+        pd_set_data(self.ctx, inputs, tokens, labels, n)
+
+    def run(self, M, noam=0):
+        pd_run(self.ctx, M, noam)
+
+    def params(self, layer_sizes: Sequence[int], layers: Optional[Sequence[int]] = None) -> Dict[int, np.ndarray]:
+        layers = range(len(self.layers)) if layers is None else layers
+        return {l: pd_get_params(self.ctx, l, layer_sizes[l]) for l in layers}
+
+    def trace(self):
+        return pd_get_trace(self.ctx)
+
+    def version_map(self, M):
+        return pd_get_version_map(self.ctx, len(self.plan.stages), M)
+
+    def losses(self, M):
+        return pd_get_losses(self.ctx, M)
+
+    def stats(self):
+        return pd_get_stats(self.ctx)
+
+    def close(self):
+        if self.ctx is not None:
+            pd_destroy(self.ctx)
+            self.ctx = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+def torch_allgather(group=None):
+    """allgather over torch.distributed (gloo or nccl), for Pipeline(allgather=...)."""
+    import torch.distributed as dist
+
+    def ag(obj):
+        out = [None] * dist.get_world_size(group)
+        dist.all_gather_object(out, obj, group=group)
+        return out
+
+    return ag

@@ -1,0 +1,133 @@
+"""Kernel parity on a B200: the tcgen05 bf16 GEMM (all operand majors and fused epilogues)
+and the fp32 SIMT GEMM against plain PyTorch fp32 references of the same op, and the
+softmax-CE kernel against the oracle.  Called through the C ABI (pd_kernel_*)."""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+
+pytestmark = pytest.mark.gpu
+
+torch.backends.cuda.matmul.allow_tf32 = False
+
+
+def _operands(M, N, K, amn, bmn, dtype, seed=0):
+    g = torch.Generator(device="cuda").manual_seed(seed)
+    A = torch.randn(M, K, device="cuda", generator=g).to(dtype)  # logical A(m, k)
+    B = torch.randn(N, K, device="cuda", generator=g).to(dtype)  # logical B(n, k)
+    As = A.t().contiguous() if amn else A.contiguous()
+    Bs = B.t().contiguous() if bmn else B.contiguous()
+    return A, B, As, Bs
+
+
+def _rel(x, ref):
+    return float((x.float() - ref.float()).abs().max() / ref.float().abs().max().clamp_min(1e-30))
+
+
+SHAPES = [
+    (256, 4096, 4096, 0, 0),   # forward of an MLP-4096 layer, X W^T
+    (256, 4096, 4096, 0, 1),   # dX = G W
+    (4096, 4096, 256, 1, 1),   # dW = G^T X
+    (200, 520, 264, 0, 0),     # ragged M/N/K tails
+    (200, 520, 264, 0, 1),
+    (520, 200, 72, 1, 1),
+    (32, 64, 64, 0, 0),        # tiny (parity-size layers)
+    (3200, 1024, 4096, 1, 0),  # the fourth major combination
+]
+
+
+@pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES)
+def test_tc_gemm_f32_out(M, N, K, amn, bmn):
+    A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16)
+    out = torch.empty(M, N, device="cuda", dtype=torch.float32)
+    pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], out.data_ptr(),
+                      N, amn, bmn, pd.PD_EPI_F32)
+    torch.cuda.synchronize()
+    ref = A.float() @ B.float().t()
+    assert _rel(out, ref) < 1e-5
+
+
+@pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES[:4])
+def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn):
+    A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16, seed=1)
+    bias = torch.randn(N, device="cuda")
+    out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], out.data_ptr(),
+                      N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1)
+    torch.cuda.synchronize()
+    ref = torch.relu(A.float() @ B.float().t() + bias)
+    assert _rel(out, ref) < 1e-2
+
+
+def test_tc_gemm_mask_epilogue():
+    M, N, K = 256, 1024, 512
+    A, B, As, Bs = _operands(M, N, K, 0, 1, torch.bfloat16, seed=2)
+    mask = torch.relu(torch.randn(M, N, device="cuda")).to(torch.bfloat16)
+    out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), K, Bs.data_ptr(), N, out.data_ptr(), N, 0, 1,
+                      pd.PD_EPI_MASK, mask=mask.data_ptr(), ldm=N)
+    torch.cuda.synchronize()
+    ref = (A.float() @ B.float().t()) * (mask.float() > 0)
+    assert _rel(out, ref) < 1e-2
+    assert bool(((out.float() == 0) | (mask.float() > 0)).all())
+
+
+@pytest.mark.parametrize("adam", [False, True])
+def test_tc_gemm_fused_update(adam):
+    M, N, K = 512, 384, 256  # dW of a 384 -> 512 layer over 256 rows
+    A, B, As, Bs = _operands(M, N, K, 1, 1, torch.bfloat16, seed=3)
+    master = torch.randn(M, N, device="cuda")
+    slot = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    m = torch.randn(M, N, device="cuda").abs() * 0.1
+    v = torch.rand(M, N, device="cuda") * 0.1
+    ref_w, ref_m, ref_v = master.clone(), m.clone(), v.clone()
+    lr, b1, b2, eps, step = 0.01, 0.9, 0.999, 1e-8, 3
+    pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), M, Bs.data_ptr(), N, None, N, 1, 1,
+                      pd.PD_EPI_ADAM if adam else pd.PD_EPI_SGD, master=master.data_ptr(), slot=slot.data_ptr(),
+                      adam_m=m.data_ptr(), adam_v=v.data_ptr(), lr=lr, beta1=b1, beta2=b2, eps=eps, step=step)
+    torch.cuda.synchronize()
+    g = A.float() @ B.float().t()
+    if adam:
+        ref_m = b1 * ref_m + (1 - b1) * g
+        ref_v = b2 * ref_v + (1 - b2) * g * g
+        ref_w = ref_w - lr * (ref_m / (1 - b1 ** step)) / ((ref_v / (1 - b2 ** step)).sqrt() + eps)
+        assert _rel(m, ref_m) < 1e-5 and _rel(v, ref_v) < 1e-5
+    else:
+        ref_w = ref_w - lr * g
+    assert float((master - ref_w).abs().max()) < 1e-4
+    assert _rel(slot, ref_w) < 1e-2
+
+
+@pytest.mark.parametrize("M,N,K,amn,bmn", [(16, 512, 784, 0, 0), (16, 784, 512, 0, 1), (512, 784, 16, 1, 1),
+                                           (70, 130, 33, 1, 0)])
+def test_simt_fp32_gemm(M, N, K, amn, bmn):
+    A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.float32, seed=4)
+    out = torch.empty(M, N, device="cuda")
+    bias = torch.randn(N, device="cuda")
+    pd.pd_kernel_gemm(pd.PD_FP32, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], out.data_ptr(),
+                      N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1)
+    torch.cuda.synchronize()
+    ref = torch.relu(A.double() @ B.double().t() + bias.double())
+    assert _rel(out, ref) < 1e-5
+
+
+@pytest.mark.parametrize("dtype", [pd.PD_FP32, pd.PD_BF16])
+def test_softmax_ce_kernel_vs_oracle(dtype):
+    import oracle
+    rng = np.random.default_rng(5)
+    R, Cn = 48, 1000
+    z = (rng.standard_normal((R, Cn)) * 3).astype(np.float32)
+    lab = rng.integers(0, Cn, R).astype(np.int32)
+    tdt = torch.bfloat16 if dtype == pd.PD_BF16 else torch.float32
+    zt = torch.tensor(z).to(tdt).cuda()
+    zq = zt.float().cpu().numpy()  # oracle sees the same (possibly rounded) logits
+    lt = torch.tensor(lab).cuda()
+    dz = torch.empty_like(zt)
+    loss = torch.zeros(1, device="cuda")
+    pd.pd_kernel_softmax_ce(dtype, zt.data_ptr(), lt.data_ptr(), R, Cn, dz.data_ptr(), loss.data_ptr())
+    torch.cuda.synchronize()
+    ref_loss, ref_dz = oracle.softmax_ce(zq, lab)
+    assert abs(loss.item() - ref_loss) < 1e-4 * max(1, abs(ref_loss))
+    tol = 1e-2 if dtype == pd.PD_BF16 else 1e-5
+    assert np.abs(dz.float().cpu().numpy() - ref_dz).max() / np.abs(ref_dz).max() < tol

@@ -1,0 +1,108 @@
+"""Pipeline parity on one B200 (several "virtual" workers share the GPU, each with its own
+stream): event trace, weight-version map and parameters of pd_run against the oracle."""
+import numpy as np
+import pytest
+
+import synth
+import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+from gpu_helpers import run_both, assert_schedule_exact, param_errors, FP32_TOL, BF16_TOL
+
+pytestmark = pytest.mark.gpu
+
+
+def test_cfg1_full_size_two_stages_fp32():
+    # BASELINE.json configs[0]: MLP 784-512-512-10 fp32, 2 stages, B=16, 8 minibatches, NOAM=2
+    wl = synth.workload("mlp_small")
+    res = run_both(wl, [1, 2], [1, 1], 8, pd.PD_FP32, n_data=8)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL, perr
+    assert derr < 1e-3, derr
+    assert np.allclose(res["losses"], res["ref"].losses, rtol=1e-4, atol=1e-5)
+
+
+@pytest.mark.parametrize("last", [[3, 7, 11, 15], [0, 1, 2, 15], [15]])
+def test_mlp_reduced_straight_fp32(last):
+    wl = synth.workload("mlp4096", reduced=True)
+    M = 4 * len(last) + 3  # startup, steady state, drain, ragged tail
+    res = run_both(wl, last, [1] * len(last), M, pd.PD_FP32)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+@pytest.mark.parametrize("reps", [[2, 1], [3, 1], [4]])
+def test_replicated_stage_fp32(reps):
+    wl = synth.workload("mlp4096", reduced=True)
+    last = [7, 15] if len(reps) == 2 else [15]
+    M = 4 * reps[0]
+    res = run_both(wl, last, reps, M, pd.PD_FP32)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+@pytest.mark.parametrize("depth", [1, 2, 6])
+def test_depth_override_fp32(depth):
+    wl = synth.workload("mlp4096", reduced=True)
+    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 14, pd.PD_FP32, noam=depth)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+def test_mlp_reduced_four_stages_bf16():
+    wl = synth.workload("mlp4096", reduced=True)
+    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 16, pd.PD_BF16)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
+
+
+def test_replicated_bf16():
+    wl = synth.workload("mlp4096", reduced=True)
+    res = run_both(wl, [7, 15], [2, 1], 8, pd.PD_BF16)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
+
+
+def test_full_width_4096_bf16_two_stages():
+    # full MLP-4096 width (16 N-tiles, 64 K-blocks per GEMM), two layers per stage, B = 32
+    layers = synth.mlp([4096] * 5, 32)
+    wl = synth.Workload("mlp4096_w", layers, 32, synth.SGD, 0.05)
+    res = run_both(wl, [1, 3], [1, 1], 4, pd.PD_BF16, n_data=2)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
+
+
+def test_second_run_continues_training_fp32():
+    # versions and optimizer state persist across pd_run calls
+    wl = synth.workload("mlp_small")
+    p0 = synth.init_params(wl.layers)
+    data = synth.make_data(wl, 8)
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline
+    import oracle
+    plan = pd.Plan.manual([1, 2], [1, 1])
+    with Pipeline(plan, wl.layers, p0, dtype=pd.PD_FP32, lr=wl.lr, minibatch=wl.batch) as P:
+        P.set_data(*data, 8)
+        P.run(8)
+        P.run(8)
+        got = P.params([synth.param_count(L) for L in wl.layers])
+    r1 = oracle.run(wl.layers, [1, 2], [1, 1], wl.batch, 8, p0, data, lr=wl.lr)
+    r2 = oracle.run(wl.layers, [1, 2], [1, 1], wl.batch, 8, r1.params, data, lr=wl.lr)
+    import torchref
+    assert torchref.max_rel_err([got[l] for l in range(3)], r2.params) < FP32_TOL
+
+
+def test_timing_trace_and_bubble():
+    wl = synth.workload("mlp4096", reduced=True)
+    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 16, pd.PD_BF16, record_trace=2)
+    st = res["stats"]
+    assert st["num_local_workers"] == 4
+    assert 0.0 <= st["bubble"] < 1.0
+    assert st["kernel_launches"] > 0
+    for e in res["trace"]:
+        if e[4] != "U":
+            assert e[8] <= e[9]

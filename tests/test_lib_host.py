@@ -1,0 +1,116 @@
+"""Host-side checks of libpipedream.so that need no GPU: it loads, exports every symbol the
+headers declare, its planner is bit-exact with the oracle's, its in-flight counts match,
+input validation works, and device calls fail loudly without a B200 (no CPU fallback)."""
+import os
+import re
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_symbols():
+    names = set()
+    for h in ("pipedream.h", "pipedream_kernels.h"):
+        src = open(os.path.join(ROOT, "include", h)).read()
+        names |= set(re.findall(r"PD_API[^;(]*?\b(pd_\w+)\s*\(", src))
+    return names
+
+
+def test_library_exports_every_declared_symbol():
+    names = declared_symbols()
+    assert len(names) >= 18
+    for n in names:
+        assert hasattr(pd.lib, n), n
+    assert set(pd.EXPORTED) == names
+
+
+def test_library_has_no_libcuda_link_dependency():
+    # must load on a GPU-less host; the driver is resolved at run time
+    import subprocess
+    out = subprocess.run(["ldd", pd.LIB_PATH], capture_output=True, text=True).stdout
+    assert "libcuda.so" not in out
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_pd_plan_bit_exact_with_oracle(seed):
+    rng = np.random.default_rng(100 + seed)
+    N = int(rng.integers(1, 12))
+    G = int(rng.integers(1, 9))
+    T, a, w = synth.random_profile(rng, N)
+    bw = float(rng.choice([1e9, 25e9, 900e9]))
+    for max_rep in (0, 1, 2):
+        for cm in (0, 1):
+            try:
+                ref = oracle.plan(T, a, w, G, bw, max_rep, cm)
+            except ValueError:
+                with pytest.raises(pd.PDError) as ei:
+                    pd.pd_plan(T, a, w, G, bw, max_rep, cm)
+                assert ei.value.status == pd.PD_EINFEASIBLE
+                continue
+            got = pd.pd_plan(T, a, w, G, bw, max_rep, cm)
+            assert got.stage_last == ref.stage_last
+            assert got.replicas == ref.replicas
+            assert got.noam == ref.noam
+            assert got.slowest_stage_s == ref.slowest  # bit-exact (same arithmetic order, R16)
+            assert got.stages[0][0] == 0 and got.stages[-1][1] == N - 1
+            assert [s[3] for s in got.stages] == list(np.cumsum([0] + got.replicas[:-1]))
+
+
+def test_pd_plan_full_size_configs_run_fast():
+    # FLOP-proportional profiles of the BASELINE configs (see bench.py), < 8 s (L985)
+    import time
+    rng = np.random.default_rng(0)
+    T, a, w = synth.random_profile(rng, 40)
+    t0 = time.time()
+    pd.pd_plan(T, a, w, 8)
+    assert time.time() - t0 < 8
+
+
+@pytest.mark.parametrize("reps,depth", [([1, 1, 1, 1], 0), ([2, 1], 0), ([7, 1], 0), ([3, 2, 1], 0),
+                                         ([1] * 5, 2), ([1] * 5, 7), ([1, 1], 1)])
+def test_inflight_matches_oracle(reps, depth):
+    plan = pd.Plan.manual(list(range(len(reps))), reps)
+    assert pd.pd_inflight(plan, depth) == oracle.inflight(reps, depth)
+
+
+def test_inflight_override_rejected_on_replicated_plan():
+    plan = pd.Plan.manual([0, 1], [2, 1])
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_inflight(plan, 3)
+    assert ei.value.status == pd.PD_EINVAL
+
+
+def test_create_validation():
+    wl = synth.workload("mlp_small")
+    good = pd.Plan.manual([1, 2], [1, 1])
+    ctx = pd.pd_create(good, wl.layers, pd.PD_FP32, minibatch=16)
+    pd.pd_destroy(ctx)
+    bad_cover = pd.Plan.manual([1], [1])  # does not cover layer 2
+    with pytest.raises(pd.PDError):
+        pd.pd_create(bad_cover, wl.layers, pd.PD_FP32, minibatch=16)
+    bad_shape = list(wl.layers)
+    bad_shape[1] = synth.Layer(synth.LINEAR, 500, 512, synth.ACT_RELU)
+    with pytest.raises(pd.PDError):
+        pd.pd_create(good, bad_shape, pd.PD_FP32, minibatch=16)
+    with pytest.raises(pd.PDError):
+        pd.pd_create(good, wl.layers, pd.PD_FP32, minibatch=0)
+
+
+@pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU failure mode")
+def test_device_calls_fail_loudly_without_gpu():
+    wl = synth.workload("mlp_small")
+    ctx = pd.pd_create(pd.Plan.manual([2], [1]), wl.layers, pd.PD_FP32, minibatch=16)
+    params = synth.init_params(wl.layers)
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_stage_init(ctx, 0, 0, 0, params)
+    assert ei.value.status in (pd.PD_ECUDA, pd.PD_EUNSUPPORTED)
+    with pytest.raises(pd.PDError):
+        pd.pd_run(ctx, 4)
+    pd.pd_destroy(ctx)
