@@ -1,0 +1,344 @@
+#!/usr/bin/env python
+"""Benchmark of the B200-native PipeDream hot path (1F1B + weight stashing).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config mlp4096] [--impl reference]
+
+One step = one pd_run over `--minibatches` minibatches of the BASELINE.json configs[1]
+workload (16 x Linear(4096)+ReLU -> CE(4096), minibatch 256, bf16, SGD): startup, steady
+state and drain of the 1F1B pipeline, with inputs already resident in HBM (a ring of 8
+synthetic minibatches).  N = 1 is a single stage (plain SGD, k = 1, P1); N > 1 is
+the straight pipeline pd_plan(max_replicas = 1) returns for N GPUs, one process per GPU
+(torchrun), activations/gradients over NVLink peer stores (CUDA IPC).
+
+Prints ONE JSON line (rank 0).  `value` = samples/s of the whole job, device time of each
+step = max over ranks of the library's per-run CUDA-event span.  `e2e` repeats the
+measurement through the public API with host inputs (pinned) copied in and the losses read
+back inside every step.  `roofline` reports the dominant kernel (the dW GEMM with the fused
+SGD update -- HBM-bound) against MEASURED_PEAKS.json.  `cpu_baseline` times the oracle.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
+import numpy as np  # noqa: E402
+
+METRIC = "samples/sec at 1/2/4/8 B200 (1F1B+stash); bubble %; per-stage tensor-pipe util"
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d["bf16_tflops"],
+                "bf16_tflops_sustained": d.get("bf16_tflops_sustained", d["bf16_tflops"]), "source": "measured"}
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "source": "fallback"}
+
+
+class Clocks:
+    """Samples nvidia-smi during the timed region (clocks line of B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.rows, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm = [float(r[1]) for r in self.rows if len(r) > 2 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+# ----------------------------------------------------------------------------- workload
+
+def mlp_profile(layers, B, peaks):
+    """FLOP/byte-proportional per-layer profile for pd_plan (T_l, a_l, w_l, L841-843)."""
+    import synth
+    T, a, w = [], [], []
+    for L in layers:
+        P = synth.param_count(L)
+        flop_t = 6.0 * B * P / (peaks["bf16_tflops"] * 1e12 * 0.6)
+        byte_t = 14.0 * P / (peaks["hbm_gbs"] * 1e9)
+        T.append(max(flop_t, byte_t))
+        a.append(B * L.out * 2)
+        w.append(P * 2)
+    return T, a, w
+
+
+def dw_update_bytes(L, B):
+    """Algorithmic HBM bytes of one dW GEMM with the fused SGD update:
+    read G [B][out] and X [B][in] (bf16), read+write the fp32 master, write the bf16 version."""
+    return B * L.out * 2 + B * L.in_ * 2 + L.out * L.in_ * (4 + 4 + 2)
+
+
+def gemm_flops(L, B):
+    return 2.0 * B * L.in_ * L.out
+
+
+# ----------------------------------------------------------------------------- reference arm
+
+def run_reference(args):
+    """--impl reference: the oracle (this tier's reference arm) on the host cores, on a
+    bounded sample of the same workload; one JSON line."""
+    import oracle
+    import synth
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    wl = synth.workload(args.config)
+    Bs = args.cpu_batch
+    layers = wl.layers
+    p0 = synth.init_params(layers)
+    wl_s = synth.Workload(wl.name, layers, Bs, wl.optimizer, wl.lr)
+    data = synth.make_data(wl_s, 1)
+    times = []
+    for _ in range(args.warmup if args.warmup < 1 else 0):
+        pass
+    for _ in range(max(1, args.steps)):
+        t0 = time.perf_counter()
+        oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
+        times.append(time.perf_counter() - t0)
+    per = float(np.median(times))
+    value = Bs / per
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": args.gpus,
+            "steps": len(times), "warmup": 0, "ms_per_step": per * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{args.config} (BASELINE configs[1]) as the CPU oracle: 1 stage, "
+                                   f"bounded sample of 1 minibatch of B={Bs} per step", "global_batch": Bs},
+            "cpu_baseline": {"value": value, "unit": "samples/s", "cores": 1, "kind": "oracle",
+                             "sample": f"1 minibatch of B={Bs} through all {len(layers)} layers (fwd+bwd+SGD), "
+                                       f"single-threaded fp32 naive loops"},
+            "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(args, layers, wl):
+    import oracle
+    import synth
+    Bs = args.cpu_batch
+    p0 = synth.init_params(layers)
+    wl_s = synth.Workload(wl.name, layers, Bs, wl.optimizer, wl.lr)
+    data = synth.make_data(wl_s, 1)
+    t0 = time.perf_counter()
+    oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
+    dt = time.perf_counter() - t0
+    return {"value": Bs / dt, "unit": "samples/s", "cores": 1, "kind": "oracle",
+            "sample": f"1 minibatch of B={Bs} (not 256) through all {len(layers)} layers of {args.config} "
+                      f"(fwd+bwd+SGD), single-threaded fp32 naive loops, {dt:.1f} s"}
+
+
+# ----------------------------------------------------------------------------- main arm
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="mlp4096")
+    ap.add_argument("--minibatches", type=int, default=0, help="minibatches per step (default 8, 16n for n>1)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--cpu-batch", type=int, default=8)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    import synth
+    import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline, torch_allgather
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    N = args.gpus
+    if world != N:
+        raise SystemExit(f"--gpus {N} but WORLD_SIZE {world}")
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def allmax(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def allsum(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    peaks = load_peaks()
+    wl = synth.workload(args.config)
+    layers, B = wl.layers, wl.batch
+    if N == 1:
+        plan = pd.Plan.manual([len(layers) - 1], [1])
+    else:
+        T, a, w = mlp_profile(layers, B, peaks)
+        plan = pd.pd_plan(T, a, w, N, max_replicas=1)
+    n = len(plan.stages)
+    M = args.minibatches or (8 if n == 1 else 16 * n)
+    p0 = synth.init_params(layers) if True else None
+    n_data = 8
+    data = synth.make_data(wl, n_data)
+    P = Pipeline(plan, layers, p0, dtype=pd.PD_BF16, optimizer=wl.optimizer, lr=wl.lr, minibatch=B,
+                 record_trace=2, device_of=lambda g: g if world > 1 else local_rank,
+                 local=(lambda wid: wid == rank) if world > 1 else None,
+                 allgather=torch_allgather() if world > 1 else None)
+    P.set_data(*data, n_data)
+    barrier()
+    for _ in range(args.warmup):
+        P.run(M)
+    barrier()
+    clocks = Clocks(local_rank)
+    clocks.start()
+    step_ms, launches, kern_ms, kern_cnt, bubbles = [], 0, np.zeros(4), np.zeros(4), []
+    barrier()
+    t_wall0 = time.perf_counter()
+    for _ in range(args.steps):
+        P.run(M)
+        st = P.stats()
+        step_ms.append(allmax(st["run_ms"]))
+        launches += st["kernel_launches"]
+        kern_ms += np.array(st["kern_ms"])
+        kern_cnt += np.array(st["kern_count"])
+        bubbles.append(st["bubble"])
+    barrier()
+    wall = time.perf_counter() - t_wall0
+    clk = clocks.stop()
+    total_ms = sum(step_ms)
+    samples = args.steps * M * B
+    value = samples / (total_ms / 1e3)
+    launches = int(allsum(launches))
+    bubble = allmax(float(np.mean(bubbles)))
+
+    # ---- roofline of the dominant kernel (the dW GEMM + fused SGD update), this rank's stage
+    s_mine = [s for s, st in enumerate(plan.stages) if st[3] <= rank < st[3] + st[2]][0]
+    my_layers = [layers[l] for l in range(plan.stages[s_mine][0], plan.stages[s_mine][1] + 1)]
+    dw_bytes = float(np.mean([dw_update_bytes(L, B) for L in my_layers]))
+    dw_avg_s = kern_ms[2] / max(kern_cnt[2], 1) / 1e3
+    achieved = dw_bytes / dw_avg_s / 1e9 if dw_avg_s > 0 else 0.0
+    fw_flops = float(np.mean([gemm_flops(L, B) for L in my_layers]))
+    fw_avg_s = kern_ms[0] / max(kern_cnt[0], 1) / 1e3
+    fw_tflops = fw_flops / fw_avg_s / 1e12 if fw_avg_s > 0 else 0.0
+    dx_avg_s = kern_ms[1] / max(kern_cnt[1], 1) / 1e3
+    dx_tflops = fw_flops / dx_avg_s / 1e12 if dx_avg_s > 0 else 0.0
+    step_share = {cls: float(kern_ms[i] / max(total_ms, 1e-9)) for i, cls in enumerate(["fwd_gemm", "dx_gemm",
+                                                                                         "dw_update_gemm", "other"])}
+
+    # ---- end to end through the public API: host (pinned) inputs in, losses out, every step
+    e2e = None
+    if not args.no_e2e:
+        inputs, tokens, labels = data
+        pin_in = torch.from_numpy(np.ascontiguousarray(np.resize(inputs, (M,) + inputs.shape[1:]))).pin_memory()
+        pin_lab = torch.from_numpy(np.ascontiguousarray(np.resize(labels, (M,) + labels.shape[1:]))).pin_memory()
+        P.set_data(pin_in, None, pin_lab, M)
+        P.run(M)  # warm the M-sized data ring
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            P.set_data(pin_in, None, pin_lab, M)
+            P.run(M)
+            P.losses(M)
+        barrier()
+        e2e_s = allmax(time.perf_counter() - t0)
+        e2e = {"value": samples / e2e_s, "unit": "samples/s",
+               "h2d_bytes_per_step": int(pin_in.numel() * 4 + pin_lab.numel() * 4) if s_mine in (0, n - 1) else 0,
+               "d2h_bytes_per_step": int(M * 4),
+               "note": "wall clock around set_data(pinned host) + pd_run + pd_get_losses, max over ranks"}
+
+    cpu = None
+    if rank == 0 and N == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(args, layers, wl)
+    P.close()
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": N, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+            "config": {"workload": f"{args.config}: BASELINE configs[1] 16 x Linear(4096)+ReLU -> CE(4096), "
+                                   f"minibatch {B}, bf16 weights/activations, fp32 master, SGD lr {wl.lr}",
+                       "plan": "-".join(str(s[2]) for s in plan.stages) + f" ({n} stage{'s' if n > 1 else ''} "
+                               f"of {[s[1] - s[0] + 1 for s in plan.stages]} layers)",
+                       "global_batch": B, "minibatches_per_step": M, "noam": plan.noam,
+                       "parallelism": f"pipeline{n}" if n > 1 else "single-stage",
+                       "l2": "working set > L2: every minibatch streams 0.54 GB bf16 weights + 1.07 GB fp32 "
+                             "master per 16 layers (126 MB L2), no flush needed"},
+            "bubble_pct": 100.0 * bubble,
+            "wall_s": wall,
+            "gpu_launches": launches,
+            "clocks": clk,
+            "roofline": {"bound": "hbm", "kernel": "dW GEMM + fused SGD update (tcgen05, EPI_SGD)",
+                         "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                         "frac": achieved / peaks["hbm_gbs"], "traffic": None,
+                         "bytes_per_launch": dw_bytes, "avg_launch_us": dw_avg_s * 1e6,
+                         "peak_source": peaks["source"] + " hbm_gbs (copy)"},
+            "tensor_pipe": {"fwd_gemm_tflops": fw_tflops, "dx_gemm_tflops": dx_tflops,
+                            "peak_tflops": peaks["bf16_tflops_sustained"],
+                            "fwd_frac": fw_tflops / peaks["bf16_tflops_sustained"],
+                            "dx_frac": dx_tflops / peaks["bf16_tflops_sustained"],
+                            "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"},
+            "step_share": step_share,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

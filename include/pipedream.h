@@ -215,7 +215,12 @@ typedef struct {
     int worker_id[PD_MAX_LOCAL_WORKERS];
     double busy_ms[PD_MAX_LOCAL_WORKERS];  /* sum of F/B op device durations per worker    */
     double span_ms[PD_MAX_LOCAL_WORKERS];  /* first op start to last op end per worker     */
-    double gemm_ms[PD_MAX_LOCAL_WORKERS];  /* reserved                                       */
+    double run_ms;                /* device time of the last run: max over local workers of
+                                     the span between events recorded on the worker's stream
+                                     before its first and after its last operation          */
+    double kern_ms[4];            /* record_trace 2: summed device time per kernel class:
+                                     0 forward GEMM, 1 dX GEMM, 2 dW GEMM (+fused update), 3 reserved */
+    uint64_t kern_count[4];       /* launches timed per class                                */
 } pd_stats;
 
 PD_API pd_status pd_get_stats(pd_ctx *ctx, pd_stats *out);

@@ -75,7 +75,8 @@ class Stats(C.Structure):
     _fields_ = [("host_ms", C.c_double), ("device_ms", C.c_double), ("bubble", C.c_double),
                 ("kernel_launches", C.c_uint64), ("bytes_sent", C.c_uint64), ("num_local_workers", C.c_int),
                 ("worker_id", C.c_int * PD_MAX_LOCAL_WORKERS), ("busy_ms", C.c_double * PD_MAX_LOCAL_WORKERS),
-                ("span_ms", C.c_double * PD_MAX_LOCAL_WORKERS), ("gemm_ms", C.c_double * PD_MAX_LOCAL_WORKERS)]
+                ("span_ms", C.c_double * PD_MAX_LOCAL_WORKERS), ("run_ms", C.c_double),
+                ("kern_ms", C.c_double * 4), ("kern_count", C.c_uint64 * 4)]
 
 
 class GemmDesc(C.Structure):
@@ -295,7 +296,8 @@ def pd_get_stats(ctx) -> dict:
     n = s.num_local_workers
     return {"host_ms": s.host_ms, "device_ms": s.device_ms, "bubble": s.bubble,
             "kernel_launches": int(s.kernel_launches), "bytes_sent": int(s.bytes_sent), "num_local_workers": n,
-            "worker_id": list(s.worker_id[:n]), "busy_ms": list(s.busy_ms[:n]), "span_ms": list(s.span_ms[:n])}
+            "worker_id": list(s.worker_id[:n]), "busy_ms": list(s.busy_ms[:n]), "span_ms": list(s.span_ms[:n]),
+            "run_ms": s.run_ms, "kern_ms": list(s.kern_ms), "kern_count": [int(x) for x in s.kern_count]}
 
 
 def pd_destroy(ctx):

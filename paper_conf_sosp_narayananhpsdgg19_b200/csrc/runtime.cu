@@ -217,6 +217,8 @@ struct Worker {
     std::vector<pd_event> events;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> op_ev;  // record_trace 2
     std::vector<cudaEvent_t> ev_pool;
+    cudaEvent_t run_ev[2] = {nullptr, nullptr};  // start / end of this worker's part of a run
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev[4];  // per kernel class (record_trace 2)
     uint64_t launches = 0;
     uint64_t bytes_sent = 0;
     int updates_total = 0;  // Adam step counter base (persists across runs)
@@ -234,6 +236,8 @@ Worker::~Worker() {
     for (void *p : bufs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
+    for (cudaEvent_t e : run_ev)
+        if (e) cudaEventDestroy(e);
     if (stream) cudaStreamDestroy(stream);
 }
 
@@ -245,7 +249,10 @@ T *dalloc(size_t bytes) {
     if (bytes == 0) bytes = 16;
     cudaError_t e = cudaMalloc(&p, align_up(bytes, 256));
     if (e != cudaSuccess) throw CudaFail{e, "cudaMalloc"};
+    // The zero fill runs on the legacy stream, which does NOT order with the workers'
+    // non-blocking streams: complete it before anyone else touches the buffer.
     CK(cudaMemset(p, 0, align_up(bytes, 256)));
+    CK(cudaDeviceSynchronize());
     return static_cast<T *>(p);
 }
 
@@ -405,6 +412,19 @@ struct Exec {
         return elem_ptr(w->act[l - w->first], (long)(j % w->k) * in_elems(d, B()), esz);
     }
 
+    // per-kernel-class device time (0 fwd GEMM, 1 dX GEMM, 2 dW(+update) GEMM, 3 other)
+    cudaEvent_t kstart(int) {
+        if (!timing) return nullptr;
+        cudaEvent_t a = w->ev_pool[ev_used++];
+        CK(cudaEventRecord(a, w->stream));
+        return a;
+    }
+    void kend(int cls, cudaEvent_t a) {
+        if (!timing) return;
+        cudaEvent_t b = w->ev_pool[ev_used++];
+        CK(cudaEventRecord(b, w->stream));
+        w->kev[cls].push_back({a, b});
+    }
     void record_start() {
         if (!timing) return;
         cudaEvent_t a = w->ev_pool[ev_used++];
@@ -466,7 +486,9 @@ struct Exec {
             }
             if (d.kind != PD_LINEAR) throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             LayerCtx lc{c, w, bf16};
+            cudaEvent_t k0 = kstart(0);
             linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y);
+            kend(0, k0);
         }
         if (s + 1 == n()) {
             const pd_layer_desc &d = layer(w->last);
@@ -555,7 +577,9 @@ struct Exec {
                 g.ldo = d.in;
                 g.mask = prev_relu ? x : nullptr;
                 g.ldm = d.in;
+                cudaEvent_t k0 = kstart(1);
                 CK(run_gemm(bf16, g, w->stream));
+                kend(1, k0);
             }
             // dW = G^T X
             {
@@ -587,7 +611,9 @@ struct Exec {
                     g.epi = EPI_F32;
                     g.out = gdst + woff;
                 }
+                cudaEvent_t k0 = kstart(2);
                 CK(run_gemm(bf16, g, w->stream));
+                kend(2, k0);
             }
             // db = column sums of G
             const long boff = c->poff[l] + (long)d.out * d.in;
@@ -684,7 +710,9 @@ void worker_thread(pd_ctx *c, Worker *w, int M, std::vector<int> k) {
     try {
         CK(cudaSetDevice(w->device));
         Exec ex{c, w, M, k, c->cfg.dtype == PD_BF16, c->esz, c->cfg.record_trace >= 2};
+        CK(cudaEventRecord(w->run_ev[0], w->stream));
         ex.run_ops();
+        CK(cudaEventRecord(w->run_ev[1], w->stream));
         CK(cudaStreamSynchronize(w->stream));
     } catch (const CudaFail &f) {
         char buf[256];
@@ -1134,13 +1162,18 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
             }
             w->events.clear();
             w->op_ev.clear();
-            const size_t need = c->cfg.record_trace >= 2 ? (size_t)6 * M + 16 : 0;
+            for (auto &kv : w->kev) kv.clear();
+            for (auto &e : w->run_ev)
+                if (!e) CK(cudaEventCreate(&e));
+            const int nl = w->last - w->first + 1;
+            const size_t need = c->cfg.record_trace >= 2 ? (size_t)(6 + 8 * nl) * M + 16 : 0;
             while (w->ev_pool.size() < need) {
                 cudaEvent_t e;
                 CK(cudaEventCreate(&e));
                 w->ev_pool.push_back(e);
             }
             CK(cudaStreamSynchronize(w->stream));
+            CK(cudaDeviceSynchronize());  // legacy-stream copies (rgrad_ptrs) before the run
         }
     } catch (const CudaFail &f) {
         c->fail(PD_ECUDA, std::string("pd_run setup: ") + f.what + ": " + cudaGetErrorString(f.e));
@@ -1258,6 +1291,18 @@ pd_status pd_get_stats(pd_ctx *c, pd_stats *out) {
             float sp = 0;
             if (cudaEventElapsedTime(&sp, w->op_ev.front().first, w->op_ev.back().second) == cudaSuccess) span = sp;
         }
+        float run_ms = 0;
+        if (w->run_ev[0] && cudaEventElapsedTime(&run_ms, w->run_ev[0], w->run_ev[1]) == cudaSuccess)
+            out->run_ms = std::max(out->run_ms, (double)run_ms);
+        cudaGetLastError();
+        for (int cls = 0; cls < 4; ++cls)
+            for (auto &pr : w->kev[cls]) {
+                float ms = 0;
+                if (cudaEventElapsedTime(&ms, pr.first, pr.second) == cudaSuccess) {
+                    out->kern_ms[cls] += ms;
+                    out->kern_count[cls] += 1;
+                }
+            }
         if (nl < PD_MAX_LOCAL_WORKERS) {
             out->worker_id[nl] = w->id;
             out->busy_ms[nl] = busy;

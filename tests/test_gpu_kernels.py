@@ -92,7 +92,7 @@ def test_tc_gemm_fused_update(adam):
         ref_m = b1 * ref_m + (1 - b1) * g
         ref_v = b2 * ref_v + (1 - b2) * g * g
         ref_w = ref_w - lr * (ref_m / (1 - b1 ** step)) / ((ref_v / (1 - b2 ** step)).sqrt() + eps)
-        assert _rel(m, ref_m) < 1e-5 and _rel(v, ref_v) < 1e-5
+        assert _rel(m, ref_m) < 1e-5 and _rel(v, ref_v) < 1e-4
     else:
         ref_w = ref_w - lr * g
     assert float((master - ref_w).abs().max()) < 1e-4

@@ -31,15 +31,15 @@ def test_mlp_reduced_straight_fp32(last):
     assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
 
 
-@pytest.mark.parametrize("reps", [[2, 1], [3, 1], [4]])
+@pytest.mark.parametrize("reps", [[2, 1], [3, 1], [4], [2]])
 def test_replicated_stage_fp32(reps):
     wl = synth.workload("mlp4096", reduced=True)
     last = [7, 15] if len(reps) == 2 else [15]
-    M = 4 * reps[0]
-    res = run_both(wl, last, reps, M, pd.PD_FP32)
-    assert_schedule_exact(res)
-    perr, derr = param_errors(res)
-    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+    for M in (reps[0], 4 * reps[0]):  # one round only, then several
+        res = run_both(wl, last, reps, M, pd.PD_FP32)
+        assert_schedule_exact(res)
+        perr, derr = param_errors(res)
+        assert perr < FP32_TOL and derr < 1e-3, (M, perr, derr)
 
 
 @pytest.mark.parametrize("depth", [1, 2, 6])
@@ -51,9 +51,17 @@ def test_depth_override_fp32(depth):
     assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
 
 
+# The bf16 path is compared at the parity learning rate 0.05: the reduced
+# width-64, 16-layer MLP has cancellation-heavy gradients below layer 13 for which bf16
+# activations/gradients alone give ~15-30 % gradient error (reproduced by a torch bf16
+# emulation), so lr 0.5 would exceed 2e-2 for bf16 rounding
+# reasons, not version reasons.  Version sensitivity is carried by the fp32 tests.
+BF16_LR = 0.05
+
+
 def test_mlp_reduced_four_stages_bf16():
     wl = synth.workload("mlp4096", reduced=True)
-    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 16, pd.PD_BF16)
+    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 16, pd.PD_BF16, lr=BF16_LR)
     assert_schedule_exact(res)
     perr, derr = param_errors(res)
     assert perr < BF16_TOL, (perr, derr)
@@ -61,7 +69,7 @@ def test_mlp_reduced_four_stages_bf16():
 
 def test_replicated_bf16():
     wl = synth.workload("mlp4096", reduced=True)
-    res = run_both(wl, [7, 15], [2, 1], 8, pd.PD_BF16)
+    res = run_both(wl, [7, 15], [2, 1], 8, pd.PD_BF16, lr=BF16_LR)
     assert_schedule_exact(res)
     perr, derr = param_errors(res)
     assert perr < BF16_TOL, (perr, derr)
