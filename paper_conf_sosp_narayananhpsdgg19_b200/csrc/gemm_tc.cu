@@ -382,15 +382,260 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
 }
 
+// ---------------------------------------------------------------- dW GEMM + fused optimizer update
+// The weight-gradient GEMM of an unreplicated stage never leaves the chip: its accumulator
+// tile is consumed in TMEM by the update, which reads the fp32 master tile (and Adam m, v),
+// writes the new master and the new bf16 weight version.  That epilogue is pure HBM
+// traffic (10 B/param for SGD, 26 B for Adam), so it is staged through shared memory with
+// TMA: the producer warp prefetches the master (m, v) tile with cp.async.bulk.tensor into a
+// 128B-swizzled buffer while the MMAs run, the epilogue warps update it in place (bank-
+// conflict-free thanks to the swizzle) and one thread writes the tiles back with TMA bulk
+// stores.  Everything moves as full lines with the TMA engine's queue depth instead of
+// per-thread 16-byte accesses.
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t src, int c0, int c1) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(map), "r"(src),
+                 "r"(c0), "r"(c1)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+template <int BN, bool ADAM>
+struct UpdCfg {
+    static constexpr int A_BYTES = BM * BK * 2;
+    static constexpr int B_BYTES = BN * BK * 2;
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+    static constexpr int STAGES = 3;
+    static constexpr int F32_TILE = BM * BN * 4;           // one fp32 [128][BN] tile
+    static constexpr int NF32 = ADAM ? 3 : 1;              // master (+ m, v)
+    static constexpr int BF_TILE = BM * BN * 2;            // bf16 version tile
+    static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + NF32 * F32_TILE + BF_TILE + 1024 + 256;
+};
+
+struct UpdArgs {
+    float lr, b1, b2, eps, bc1, bc2;
+};
+
+template <int BN, int AMAJ, int BMAJ, bool ADAM>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
+    tc_gemm_update_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                          const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmM,
+                          const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmS, UpdArgs u,
+                          int M, int N, int K) {
+    using C = UpdCfg<BN, ADAM>;
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *f32_tiles = smem + C::STAGES * C::STAGE_BYTES;      // master [, m, v]
+    uint8_t *bf_tile = f32_tiles + C::NF32 * C::F32_TILE;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(bf_tile + C::BF_TILE);
+    uint64_t *full = bars, *empty = bars + C::STAGES, *tfull = bars + 2 * C::STAGES, *tempty = tfull + 2;
+    uint64_t *wfull = tempty + 2, *wempty = wfull + 1;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(wempty + 1);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int m_blocks = (M + BM - 1) / BM, n_blocks = (N + BN - 1) / BN;
+    const int tiles = m_blocks * n_blocks;
+    const int kblocks = (K + BK - 1) / BK;
+    constexpr int F32_BOXES = BN / 32;   // 32 fp32 = 128 B per swizzled box row
+    constexpr int BF_BOXES = BN / 64;    // 64 bf16 = 128 B
+
+    if (warp == 0 && lane == 0) {
+        const CUtensorMap *maps[6] = {&tmA, &tmB, &tmW, &tmM, &tmV, &tmS};
+        for (int i = 0; i < 6; ++i) asm volatile("prefetch.tensormap [%0];" ::"l"(maps[i]) : "memory");
+        for (int s2 = 0; s2 < C::STAGES; ++s2) {
+            mbar_init(smem_u32(&full[s2]), 1);
+            mbar_init(smem_u32(&empty[s2]), 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(smem_u32(&tfull[a]), 1);
+            mbar_init(smem_u32(&tempty[a]), 4);
+        }
+        mbar_init(smem_u32(wfull), 1);
+        mbar_init(smem_u32(wempty), 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(C::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t phase = 0, wphase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
+                for (int kb = 0; kb < kblocks; ++kb) {
+                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                    const uint32_t fb = smem_u32(&full[stage]);
+                    mbar_expect_tx(fb, C::STAGE_BYTES);
+                    const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
+                    const uint32_t sb = sa + C::A_BYTES;
+                    const int k0 = kb * BK;
+                    if (AMAJ == KMAJ) tma_load_2d(sa, &tmA, fb, k0, m0);
+                    else
+#pragma unroll
+                        for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * BK * 128, &tmA, fb, m0 + 64 * j, k0);
+                    if (BMAJ == KMAJ) tma_load_2d(sb, &tmB, fb, k0, n0);
+                    else
+#pragma unroll
+                        for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * BK * 128, &tmB, fb, n0 + 64 * j, k0);
+                    if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                }
+                // the optimizer-state tile(s) of this output tile, once the previous tile's
+                // write-back has finished reading the buffer
+                mbar_wait(smem_u32(wempty), wphase ^ 1);
+                wphase ^= 1;
+                const uint32_t wb = smem_u32(wfull);
+                mbar_expect_tx(wb, C::NF32 * C::F32_TILE);
+                const CUtensorMap *fm[3] = {&tmW, &tmM, &tmV};
+#pragma unroll
+                for (int t3 = 0; t3 < C::NF32; ++t3)
+#pragma unroll
+                    for (int q = 0; q < F32_BOXES; ++q)
+                        tma_load_2d(smem_u32(f32_tiles + t3 * C::F32_TILE + q * BM * 128), fm[t3], wb, n0 + 32 * q, m0);
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            constexpr uint32_t idesc = make_idesc(BM, BN, AMAJ, BMAJ);
+            int stage = 0;
+            uint32_t phase = 0;
+            int acc = 0;
+            uint32_t acc_phase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
+                tc_fence_after();
+                const uint32_t d = tmem_base + acc * BN;
+                for (int kb = 0; kb < kblocks; ++kb) {
+                    mbar_wait(smem_u32(&full[stage]), phase);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
+                    const uint32_t sb = sa + C::A_BYTES;
+#pragma unroll
+                    for (int k = 0; k < BK / UMMA_K; ++k) {
+                        const uint64_t ad = AMAJ == KMAJ ? smem_desc(sa + k * 32, 16, 1024)
+                                                         : smem_desc(sa + k * 2048, BK * 128, 1024);
+                        const uint64_t bd = BMAJ == KMAJ ? smem_desc(sb + k * 32, 16, 1024)
+                                                         : smem_desc(sb + k * 2048, BK * 128, 1024);
+                        tc_mma(d, ad, bd, idesc, (kb | k) != 0);
+                    }
+                    tc_commit(smem_u32(&empty[stage]));
+                    if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                }
+                tc_commit(smem_u32(&tfull[acc]));
+                if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+            }
+        }
+    } else if (warp >= 4) {
+        const int q4 = warp & 3;
+        const int r = q4 * 32 + lane;  // tile row owned by this thread (TMEM lane)
+        const uint32_t rsw = (uint32_t)(r & 7);
+        int acc = 0;
+        uint32_t acc_phase = 0, wphase = 0;
+        const bool leader = (warp == 4 && lane == 0);
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
+            mbar_wait(smem_u32(&tfull[acc]), acc_phase);
+            tc_fence_after();
+            mbar_wait(smem_u32(wfull), wphase);
+            wphase ^= 1;
+#pragma unroll 1
+            for (int c = 0; c < BN / 32; ++c) {
+                float g[32];
+                tmem_ld32(tmem_base + ((uint32_t)(q4 * 32) << 16) + acc * BN + c * 32, g);
+                // fp32 box c, row r: 16-byte chunk j lives at chunk (j ^ (r & 7))
+                float *wrow = reinterpret_cast<float *>(f32_tiles + c * BM * 128 + r * 128);
+                float *mrow = reinterpret_cast<float *>(f32_tiles + C::F32_TILE + c * BM * 128 + r * 128);
+                float *vrow = reinterpret_cast<float *>(f32_tiles + 2 * C::F32_TILE + c * BM * 128 + r * 128);
+                uint32_t packed[16];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    const int pj = (int)((uint32_t)j ^ rsw) * 4;
+                    float4 w4 = *reinterpret_cast<float4 *>(wrow + pj);
+                    float wv[4] = {w4.x, w4.y, w4.z, w4.w};
+                    if constexpr (ADAM) {
+                        float4 m4 = *reinterpret_cast<float4 *>(mrow + pj);
+                        float4 v4 = *reinterpret_cast<float4 *>(vrow + pj);
+                        float mm[4] = {m4.x, m4.y, m4.z, m4.w}, vv[4] = {v4.x, v4.y, v4.z, v4.w};
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) {
+                            const float gi = g[j * 4 + i];
+                            mm[i] = u.b1 * mm[i] + (1.f - u.b1) * gi;
+                            vv[i] = u.b2 * vv[i] + (1.f - u.b2) * gi * gi;
+                            wv[i] = wv[i] - u.lr * (mm[i] / u.bc1) / (sqrtf(vv[i] / u.bc2) + u.eps);
+                        }
+                        *reinterpret_cast<float4 *>(mrow + pj) = make_float4(mm[0], mm[1], mm[2], mm[3]);
+                        *reinterpret_cast<float4 *>(vrow + pj) = make_float4(vv[0], vv[1], vv[2], vv[3]);
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) wv[i] = wv[i] - u.lr * g[j * 4 + i];
+                    }
+                    *reinterpret_cast<float4 *>(wrow + pj) = make_float4(wv[0], wv[1], wv[2], wv[3]);
+                    packed[j * 2] = pack_bf16(wv[0], wv[1]);
+                    packed[j * 2 + 1] = pack_bf16(wv[2], wv[3]);
+                }
+                // bf16 box c/2 (64 columns), this chunk = 4 logical 16-byte chunks
+                uint8_t *brow = bf_tile + (c >> 1) * BM * 128 + r * 128;
+#pragma unroll
+                for (int u4 = 0; u4 < 4; ++u4) {
+                    const uint32_t lj = (uint32_t)((c & 1) * 4 + u4);
+                    *reinterpret_cast<uint4 *>(brow + ((lj ^ rsw) << 4)) =
+                        make_uint4(packed[u4 * 4], packed[u4 * 4 + 1], packed[u4 * 4 + 2], packed[u4 * 4 + 3]);
+                }
+            }
+            // accumulator consumed: hand TMEM back to the MMA warp
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
+            if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+            // write the new master (m, v) and the new bf16 version back with TMA
+            fence_proxy_async();
+            epi_bar();
+            if (leader) {
+                const CUtensorMap *fm[3] = {&tmW, &tmM, &tmV};
+#pragma unroll
+                for (int t3 = 0; t3 < C::NF32; ++t3)
+#pragma unroll
+                    for (int q = 0; q < F32_BOXES; ++q)
+                        tma_store_2d(fm[t3], smem_u32(f32_tiles + t3 * C::F32_TILE + q * BM * 128), n0 + 32 * q, m0);
+#pragma unroll
+                for (int q = 0; q < BF_BOXES; ++q) tma_store_2d(&tmS, smem_u32(bf_tile + q * BM * 128), n0 + 64 * q, m0);
+                bulk_commit();
+                bulk_wait_read0();
+                mbar_arrive(smem_u32(wempty));
+            }
+        }
+        if (leader) bulk_wait0();
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(C::TMEM_COLS));
+    }
+}
+
 // ---------------------------------------------------------------- host side
-bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner, int box_outer) {
+bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner, int box_outer,
+              bool f32 = false) {
     const Driver *d = driver();
     if (!d) return false;
     cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
-    cuuint64_t strides[1] = {(cuuint64_t)ld_elems * 2};
+    cuuint64_t strides[1] = {(cuuint64_t)ld_elems * (f32 ? 4 : 2)};
     cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer};
     cuuint32_t estr[2] = {1, 1};
-    CUresult r = d->tensorMapEncodeTiled(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(base), dims,
+    CUresult r = d->tensorMapEncodeTiled(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
+                                         2, const_cast<void *>(base), dims,
                                          strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                                          CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -447,9 +692,61 @@ cudaError_t dispatch_major(const Gemm &g, const CUtensorMap &ma, const CUtensorM
     return dispatch_epi<BN, MNMAJ, KMAJ>(g, ma, mb, e, s);
 }
 
+template <int BN, int AMAJ, int BMAJ, bool ADAM>
+cudaError_t launch_update(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const CUtensorMap &mw,
+                          const CUtensorMap &mm, const CUtensorMap &mv, const CUtensorMap &ms, const UpdArgs &u,
+                          cudaStream_t s) {
+    using C = UpdCfg<BN, ADAM>;
+    auto kern = tc_gemm_update_kernel<BN, AMAJ, BMAJ, ADAM>;
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaError_t err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+        if (err != cudaSuccess) return err;
+        attr_set = true;
+    }
+    const int tiles = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN);
+    const int grid = tiles < num_sms() ? tiles : num_sms();
+    kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, mw, mm, mv, ms, u, g.M, g.N, g.K);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+template <int BN, bool ADAM>
+cudaError_t update_major(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const CUtensorMap &mw,
+                         const CUtensorMap &mm, const CUtensorMap &mv, const CUtensorMap &ms, const UpdArgs &u,
+                         cudaStream_t s) {
+    if (g.amaj == MNMAJ && g.bmaj == MNMAJ) return launch_update<BN, MNMAJ, MNMAJ, ADAM>(g, ma, mb, mw, mm, mv, ms, u, s);
+    if (g.amaj == KMAJ && g.bmaj == KMAJ) return launch_update<BN, KMAJ, KMAJ, ADAM>(g, ma, mb, mw, mm, mv, ms, u, s);
+    if (g.amaj == KMAJ) return launch_update<BN, KMAJ, MNMAJ, ADAM>(g, ma, mb, mw, mm, mv, ms, u, s);
+    return launch_update<BN, MNMAJ, KMAJ, ADAM>(g, ma, mb, mw, mm, mv, ms, u, s);
+}
+
+// dW GEMM with the optimizer update fused (TMA-staged epilogue).  Requirements: ldo == N
+// rows 16-byte aligned (N % 8 == 0 for bf16, % 4 for fp32).
+cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
+    const bool adam = g.epi == EPI_ADAM;
+    constexpr int BN_SGD = 128, BN_ADAM = 64;
+    const int BN = adam ? BN_ADAM : BN_SGD;
+    CUtensorMap ma, mbm, mw, mm, mv, ms;
+    const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
+                                    : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
+    const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, BN)
+                                    : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
+    bool ok = okA && okB && make_map(&mw, g.master, g.N, g.M, g.ldo, 32, BM, true) &&
+              make_map(&ms, g.slot, g.N, g.M, g.ldo, 64, BM, false);
+    if (adam) ok = ok && make_map(&mm, g.adam_m, g.N, g.M, g.ldo, 32, BM, true) &&
+                   make_map(&mv, g.adam_v, g.N, g.M, g.ldo, 32, BM, true);
+    else mm = mv = mw;
+    if (!ok) return cudaErrorInvalidValue;
+    UpdArgs u{g.lr, g.b1, g.b2, g.eps, 1.f - powf(g.b1, (float)g.step), 1.f - powf(g.b2, (float)g.step)};
+    if (adam) return update_major<BN_ADAM, true>(g, ma, mbm, mw, mm, mv, ms, u, s);
+    return update_major<BN_SGD, false>(g, ma, mbm, mw, mm, mv, ms, u, s);
+}
+
 }  // namespace
 
 cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
+    if ((g.epi == EPI_SGD || g.epi == EPI_ADAM) && g.ldo == g.N && g.N % 8 == 0) return gemm_bf16_update(g, s);
     if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
     // tile width: the widest BN that still gives every SM a tile
     const int sms = num_sms();

@@ -95,6 +95,46 @@ __global__ void col_sum_kernel(const T *G, long rows, long cols, float *out) {
     out[c] = acc;
 }
 
+// ------------------------------------------------------------------ bias gradient (+ update)
+// db[c] = sum_r G[r][c] for 32 columns per block: 8 row groups x 32 columns, coalesced
+// 64-byte row segments, partials reduced in a fixed order (deterministic).  When `master`
+// is given the optimizer update of the bias is applied in the same kernel (bf16 path,
+// unreplicated stage); otherwise db is written to grad_out.
+template <typename T>
+__global__ void __launch_bounds__(256) bias_grad_kernel(const T *__restrict__ G, long rows, long cols,
+                                                        float *grad_out, float *master, __nv_bfloat16 *slot, int opt,
+                                                        float *m, float *v, float lr, float b1, float b2, float eps,
+                                                        float bc1, float bc2) {
+    __shared__ float part[8][33];
+    const int cl = threadIdx.x & 31, rg = threadIdx.x >> 5;
+    const long c = (long)blockIdx.x * 32 + cl;
+    float acc = 0.f;
+    if (c < cols)
+        for (long r = rg; r < rows; r += 8) acc += ld_as_f32(G, r * cols + c);
+    part[rg][cl] = acc;
+    __syncthreads();
+    if (rg == 0 && c < cols) {
+        float g = part[0][cl];
+#pragma unroll
+        for (int q = 1; q < 8; ++q) g += part[q][cl];
+        if (grad_out) grad_out[c] = g;
+        if (master) {
+            float w = master[c];
+            if (opt == PD_SGD) {
+                w = w - lr * g;
+            } else {
+                float mm = b1 * m[c] + (1.f - b1) * g;
+                float vv = b2 * v[c] + (1.f - b2) * g * g;
+                m[c] = mm;
+                v[c] = vv;
+                w = w - lr * (mm / bc1) / (sqrtf(vv / bc2) + eps);
+            }
+            master[c] = w;
+            if (slot) slot[c] = __float2bfloat16_rn(w);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ softmax cross-entropy
 // One block per row: max, sum of exp, loss += (lse - z[label]) / rows, and
 // dlogits = (softmax - onehot) / rows written in the logits' dtype (L1217, R8).
@@ -239,6 +279,21 @@ cudaError_t col_sum(const void *G, int bf16, long rows, long cols, float *out, c
     const int blocks = (int)((cols + 255) / 256);
     if (bf16) col_sum_kernel<<<blocks, 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(G), rows, cols, out);
     else col_sum_kernel<<<blocks, 256, 0, s>>>(static_cast<const float *>(G), rows, cols, out);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t bias_grad(const void *G, int bf16, long rows, long cols, float *grad_out, float *master,
+                      __nv_bfloat16 *slot, int opt, float *m, float *v, float lr, float b1, float b2, float eps,
+                      int step, cudaStream_t s) {
+    const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
+    const unsigned blocks = (unsigned)((cols + 31) / 32);
+    if (bf16)
+        bias_grad_kernel<<<blocks, 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(G), rows, cols, grad_out, master,
+                                                slot, opt, m, v, lr, b1, b2, eps, bc1, bc2);
+    else
+        bias_grad_kernel<<<blocks, 256, 0, s>>>(static_cast<const float *>(G), rows, cols, grad_out, master, slot, opt,
+                                                m, v, lr, b1, b2, eps, bc1, bc2);
     ++tl_launches;
     return cudaGetLastError();
 }

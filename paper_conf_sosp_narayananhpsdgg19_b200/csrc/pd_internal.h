@@ -85,6 +85,11 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s);
 
 // elementwise / reductions (kernels.cu).  T = float or __nv_bfloat16 via `bf16` flag.
 cudaError_t col_sum(const void *G, int bf16, long rows, long cols, float *out, cudaStream_t s);
+// bias gradient db = column sums of G [rows][cols]; written to grad_out if non-null; if
+// master is non-null the SGD/Adam update of the bias is fused (slot receives bf16(master)).
+cudaError_t bias_grad(const void *G, int bf16, long rows, long cols, float *grad_out, float *master,
+                      __nv_bfloat16 *slot, int opt, float *m, float *v, float lr, float b1, float b2, float eps,
+                      int step, cudaStream_t s);
 cudaError_t softmax_ce(const void *logits, int bf16, const int32_t *labels, long rows, int C, void *dlogits,
                        float *loss_out, cudaStream_t s);
 // out = in - lr * g  (fp32 versions), n elements

@@ -615,15 +615,19 @@ struct Exec {
                 CK(run_gemm(bf16, g, w->stream));
                 kend(2, k0);
             }
-            // db = column sums of G
+            // db = column sums of G (+ the bias update itself on the fused path)
             const long boff = c->poff[l] + (long)d.out * d.in;
-            CK(col_sum(G, bf16, rows, d.out, gdst + boff, w->stream));
-            if (fused) {
-                CK(update_master(w->master + boff, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[nslot], boff, esz)),
-                                 nullptr, w->self_grad_ptr, 1, boff, d.out, c->cfg.optimizer,
+            {
+                cudaEvent_t k0 = kstart(3);
+                if (fused)
+                    CK(bias_grad(G, bf16, rows, d.out, nullptr, w->master + boff,
+                                 static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[nslot], boff, esz)), c->cfg.optimizer,
                                  w->adam_m ? w->adam_m + boff : nullptr, w->adam_v ? w->adam_v + boff : nullptr,
-                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1,
-                                 w->stream));
+                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+                else
+                    CK(bias_grad(G, bf16, rows, d.out, gdst + boff, nullptr, nullptr, 0, nullptr, nullptr, 0.f, 0.f,
+                                 0.f, 0.f, 1, w->stream));
+                kend(3, k0);
             }
             G = dx;
             cur ^= 1;

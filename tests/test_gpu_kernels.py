@@ -74,8 +74,9 @@ def test_tc_gemm_mask_epilogue():
 
 
 @pytest.mark.parametrize("adam", [False, True])
-def test_tc_gemm_fused_update(adam):
-    M, N, K = 512, 384, 256  # dW of a 384 -> 512 layer over 256 rows
+@pytest.mark.parametrize("M,N,K", [(512, 384, 256), (4096, 4096, 256), (200, 72, 40), (1000, 4096, 64)])
+def test_tc_gemm_fused_update(adam, M, N, K):
+    # dW of an N -> M layer over K rows, optimizer fused (TMA-staged epilogue)
     A, B, As, Bs = _operands(M, N, K, 1, 1, torch.bfloat16, seed=3)
     master = torch.randn(M, N, device="cuda")
     slot = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
