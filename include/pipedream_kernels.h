@@ -49,6 +49,9 @@ typedef struct {
     float *adam_m, *adam_v;
     float lr, beta1, beta2, eps;
     int step;
+    float *workspace;      /* optional fp32 scratch (device) for split-K partial sums of small-M
+                              STORE/MASK GEMMs (bf16); NULL disables split-K           */
+    long workspace_bytes;
 } pd_gemm_desc;
 
 PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *g, void *stream);

@@ -22,6 +22,7 @@
 #include <cuda_bf16.h>
 
 #include <cstdio>
+#include <cstdlib>
 
 #include "pd_internal.h"
 
@@ -46,6 +47,8 @@ struct Cfg {
 struct EpiArgs {
     void *out;
     long ldo;
+    long split_stride;  // elements between the fp32 partial outputs of K-splits (EPI_F32)
+    int ksplit;         // K is cut into ksplit contiguous ranges; work unit = (tile, split)
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
@@ -266,6 +269,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int m_blocks = (M + BM - 1) / BM, n_blocks = (N + BN - 1) / BN;
     const int tiles = m_blocks * n_blocks;
     const int kblocks = (K + BK - 1) / BK;
+    const int units = tiles * e.ksplit;
+    const int kper = (kblocks + e.ksplit - 1) / e.ksplit;
 
     if (warp == 0 && lane == 0) {
         asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
@@ -295,9 +300,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+                const int tile = unit % tiles, split = unit / tiles;
                 const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
-                for (int kb = 0; kb < kblocks; ++kb) {
+                const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
+                for (int kb = kb0; kb < kb1; ++kb) {
                     mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
                     const uint32_t fb = smem_u32(&full[stage]);
                     mbar_expect_tx(fb, C::STAGE_BYTES);
@@ -328,11 +335,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             uint32_t phase = 0;
             int acc = 0;
             uint32_t acc_phase = 0;
-            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+                const int split = unit / tiles;
+                const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
                 mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
                 tc_fence_after();
                 const uint32_t d = tmem_base + acc * BN;
-                for (int kb = 0; kb < kblocks; ++kb) {
+                for (int kb = kb0; kb < kb1; ++kb) {
                     mbar_wait(smem_u32(&full[stage]), phase);
                     tc_fence_after();
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
@@ -343,7 +352,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                                                          : smem_desc(sa + k * 2048, BK * 128, 1024);
                         const uint64_t bd = BMAJ == KMAJ ? smem_desc(sb + k * 32, 16, 1024)
                                                          : smem_desc(sb + k * 2048, BK * 128, 1024);
-                        tc_mma(d, ad, bd, idesc, (kb | k) != 0);
+                        tc_mma(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
                     }
                     tc_commit(smem_u32(&empty[stage]));  // frees the smem slot when these MMAs finish
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
@@ -357,16 +366,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int q = warp & 3;  // TMEM lane quarter this warp may access
         int acc = 0;
         uint32_t acc_phase = 0;
-        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+            const int tile = unit % tiles, split = unit / tiles;
             const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
             tc_fence_after();
             const int row = m0 + q * 32 + lane;
+            EpiArgs es = e;
+            if (EPI == EPI_F32) es.out = static_cast<float *>(e.out) + (long)split * e.split_stride;
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
                 float v[32];
                 tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, v);
-                if (n0 + c * 32 < N) epilogue_chunk<EPI>(e, v, row, n0 + c * 32, M, N);
+                if (n0 + c * 32 < N) epilogue_chunk<EPI>(es, v, row, n0 + c * 32, M, N);
             }
             tc_fence_before();
             __syncwarp();
@@ -409,11 +421,16 @@ struct UpdCfg {
     static constexpr int B_BYTES = BN * BK * 2;
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
     static constexpr int STAGES = 3;
-    static constexpr int F32_TILE = BM * BN * 4;           // one fp32 [128][BN] tile
-    static constexpr int NF32 = ADAM ? 3 : 1;              // master (+ m, v)
-    static constexpr int BF_TILE = BM * BN * 2;            // bf16 version tile
+    // epilogue sub-tiles: ECOLS columns of the [128][BN] tile, double-buffered so the TMA
+    // load of sub-tile k+1 and the TMA store of sub-tile k-1 overlap the update of k
+    static constexpr int ECOLS = ADAM ? 32 : 64;
+    static constexpr int ESTAGES = 2;
+    static constexpr int NF32 = ADAM ? 3 : 1;           // master (+ m, v)
+    static constexpr int F32_SUB = BM * ECOLS * 4;       // one fp32 sub-tile
+    static constexpr int BF_SUB = BM * ECOLS * 2;        // one bf16 sub-tile
+    static constexpr int EBUF = NF32 * F32_SUB + BF_SUB; // one epilogue stage
     static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
-    static constexpr int SMEM = STAGES * STAGE_BYTES + NF32 * F32_TILE + BF_TILE + 1024 + 256;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + ESTAGES * EBUF + 1024 + 256;
 };
 
 struct UpdArgs {
@@ -427,21 +444,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                           const __grid_constant__ CUtensorMap tmV, const __grid_constant__ CUtensorMap tmS, UpdArgs u,
                           int M, int N, int K) {
     using C = UpdCfg<BN, ADAM>;
+    constexpr int SUBS = BN / C::ECOLS;        // epilogue sub-tiles per tile
+    constexpr int F32_BOXES = C::ECOLS / 32;   // 32 fp32 = 128 B per swizzled box row
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint8_t *f32_tiles = smem + C::STAGES * C::STAGE_BYTES;      // master [, m, v]
-    uint8_t *bf_tile = f32_tiles + C::NF32 * C::F32_TILE;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(bf_tile + C::BF_TILE);
+    uint8_t *ebuf = smem + C::STAGES * C::STAGE_BYTES;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ebuf + C::ESTAGES * C::EBUF);
     uint64_t *full = bars, *empty = bars + C::STAGES, *tfull = bars + 2 * C::STAGES, *tempty = tfull + 2;
-    uint64_t *wfull = tempty + 2, *wempty = wfull + 1;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(wempty + 1);
+    uint64_t *wfull = tempty + 2, *wempty = wfull + C::ESTAGES;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(wempty + C::ESTAGES);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int m_blocks = (M + BM - 1) / BM, n_blocks = (N + BN - 1) / BN;
     const int tiles = m_blocks * n_blocks;
     const int kblocks = (K + BK - 1) / BK;
-    constexpr int F32_BOXES = BN / 32;   // 32 fp32 = 128 B per swizzled box row
-    constexpr int BF_BOXES = BN / 64;    // 64 bf16 = 128 B
 
     if (warp == 0 && lane == 0) {
         const CUtensorMap *maps[6] = {&tmA, &tmB, &tmW, &tmM, &tmV, &tmS};
@@ -454,8 +470,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             mbar_init(smem_u32(&tfull[a]), 1);
             mbar_init(smem_u32(&tempty[a]), 4);
         }
-        mbar_init(smem_u32(wfull), 1);
-        mbar_init(smem_u32(wempty), 1);
+        for (int e = 0; e < C::ESTAGES; ++e) {
+            mbar_init(smem_u32(&wfull[e]), 1);
+            mbar_init(smem_u32(&wempty[e]), 1);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 2) {
@@ -470,8 +488,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
     if (warp == 0) {
         if (lane == 0) {
-            int stage = 0;
-            uint32_t phase = 0, wphase = 0;
+            int stage = 0, es = 0;
+            uint32_t phase = 0, ephase = 0;
+            const CUtensorMap *fm[3] = {&tmW, &tmM, &tmV};
             for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
                 const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
                 for (int kb = 0; kb < kblocks; ++kb) {
@@ -491,18 +510,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * BK * 128, &tmB, fb, n0 + 64 * j, k0);
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
                 }
-                // the optimizer-state tile(s) of this output tile, once the previous tile's
-                // write-back has finished reading the buffer
-                mbar_wait(smem_u32(wempty), wphase ^ 1);
-                wphase ^= 1;
-                const uint32_t wb = smem_u32(wfull);
-                mbar_expect_tx(wb, C::NF32 * C::F32_TILE);
-                const CUtensorMap *fm[3] = {&tmW, &tmM, &tmV};
+                // optimizer-state sub-tiles of this output tile into the epilogue ring
+                for (int sub = 0; sub < SUBS; ++sub) {
+                    mbar_wait(smem_u32(&wempty[es]), ephase ^ 1);
+                    const uint32_t wb = smem_u32(&wfull[es]);
+                    mbar_expect_tx(wb, C::NF32 * C::F32_SUB);
+                    uint8_t *buf = ebuf + es * C::EBUF;
 #pragma unroll
-                for (int t3 = 0; t3 < C::NF32; ++t3)
+                    for (int t3 = 0; t3 < C::NF32; ++t3)
 #pragma unroll
-                    for (int q = 0; q < F32_BOXES; ++q)
-                        tma_load_2d(smem_u32(f32_tiles + t3 * C::F32_TILE + q * BM * 128), fm[t3], wb, n0 + 32 * q, m0);
+                        for (int q = 0; q < F32_BOXES; ++q)
+                            tma_load_2d(smem_u32(buf + t3 * C::F32_SUB + q * BM * 128), fm[t3], wb,
+                                        n0 + sub * C::ECOLS + 32 * q, m0);
+                    if (++es == C::ESTAGES) { es = 0; ephase ^= 1; }
+                }
             }
         }
     } else if (warp == 1) {
@@ -540,80 +561,89 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int q4 = warp & 3;
         const int r = q4 * 32 + lane;  // tile row owned by this thread (TMEM lane)
         const uint32_t rsw = (uint32_t)(r & 7);
-        int acc = 0;
-        uint32_t acc_phase = 0, wphase = 0;
         const bool leader = (warp == 4 && lane == 0);
+        int acc = 0, es = 0;
+        uint32_t acc_phase = 0, ephase = 0;
         for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
             const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
             tc_fence_after();
-            mbar_wait(smem_u32(wfull), wphase);
-            wphase ^= 1;
+            for (int sub = 0; sub < SUBS; ++sub) {
+                uint8_t *buf = ebuf + es * C::EBUF;
+                uint8_t *bf_tile = buf + C::NF32 * C::F32_SUB;
+                mbar_wait(smem_u32(&wfull[es]), ephase);
 #pragma unroll 1
-            for (int c = 0; c < BN / 32; ++c) {
-                float g[32];
-                tmem_ld32(tmem_base + ((uint32_t)(q4 * 32) << 16) + acc * BN + c * 32, g);
-                // fp32 box c, row r: 16-byte chunk j lives at chunk (j ^ (r & 7))
-                float *wrow = reinterpret_cast<float *>(f32_tiles + c * BM * 128 + r * 128);
-                float *mrow = reinterpret_cast<float *>(f32_tiles + C::F32_TILE + c * BM * 128 + r * 128);
-                float *vrow = reinterpret_cast<float *>(f32_tiles + 2 * C::F32_TILE + c * BM * 128 + r * 128);
-                uint32_t packed[16];
+                for (int cc = 0; cc < C::ECOLS / 32; ++cc) {
+                    float g[32];
+                    tmem_ld32(tmem_base + ((uint32_t)(q4 * 32) << 16) + acc * BN + sub * C::ECOLS + cc * 32, g);
+                    // fp32 box cc, row r: 16-byte chunk j lives at chunk (j ^ (r & 7))
+                    float *wrow = reinterpret_cast<float *>(buf + cc * BM * 128 + r * 128);
+                    float *mrow = reinterpret_cast<float *>(buf + C::F32_SUB + cc * BM * 128 + r * 128);
+                    float *vrow = reinterpret_cast<float *>(buf + 2 * C::F32_SUB + cc * BM * 128 + r * 128);
+                    uint32_t packed[16];
 #pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                    const int pj = (int)((uint32_t)j ^ rsw) * 4;
-                    float4 w4 = *reinterpret_cast<float4 *>(wrow + pj);
-                    float wv[4] = {w4.x, w4.y, w4.z, w4.w};
-                    if constexpr (ADAM) {
-                        float4 m4 = *reinterpret_cast<float4 *>(mrow + pj);
-                        float4 v4 = *reinterpret_cast<float4 *>(vrow + pj);
-                        float mm[4] = {m4.x, m4.y, m4.z, m4.w}, vv[4] = {v4.x, v4.y, v4.z, v4.w};
+                    for (int j = 0; j < 8; ++j) {
+                        const int pj = (int)((uint32_t)j ^ rsw) * 4;
+                        float4 w4 = *reinterpret_cast<float4 *>(wrow + pj);
+                        float wv[4] = {w4.x, w4.y, w4.z, w4.w};
+                        if constexpr (ADAM) {
+                            float4 m4 = *reinterpret_cast<float4 *>(mrow + pj);
+                            float4 v4 = *reinterpret_cast<float4 *>(vrow + pj);
+                            float mm[4] = {m4.x, m4.y, m4.z, m4.w}, vv[4] = {v4.x, v4.y, v4.z, v4.w};
 #pragma unroll
-                        for (int i = 0; i < 4; ++i) {
-                            const float gi = g[j * 4 + i];
-                            mm[i] = u.b1 * mm[i] + (1.f - u.b1) * gi;
-                            vv[i] = u.b2 * vv[i] + (1.f - u.b2) * gi * gi;
-                            wv[i] = wv[i] - u.lr * (mm[i] / u.bc1) / (sqrtf(vv[i] / u.bc2) + u.eps);
+                            for (int i = 0; i < 4; ++i) {
+                                const float gi = g[j * 4 + i];
+                                mm[i] = u.b1 * mm[i] + (1.f - u.b1) * gi;
+                                vv[i] = u.b2 * vv[i] + (1.f - u.b2) * gi * gi;
+                                wv[i] = wv[i] - u.lr * (mm[i] / u.bc1) / (sqrtf(vv[i] / u.bc2) + u.eps);
+                            }
+                            *reinterpret_cast<float4 *>(mrow + pj) = make_float4(mm[0], mm[1], mm[2], mm[3]);
+                            *reinterpret_cast<float4 *>(vrow + pj) = make_float4(vv[0], vv[1], vv[2], vv[3]);
+                        } else {
+#pragma unroll
+                            for (int i = 0; i < 4; ++i) wv[i] = wv[i] - u.lr * g[j * 4 + i];
                         }
-                        *reinterpret_cast<float4 *>(mrow + pj) = make_float4(mm[0], mm[1], mm[2], mm[3]);
-                        *reinterpret_cast<float4 *>(vrow + pj) = make_float4(vv[0], vv[1], vv[2], vv[3]);
-                    } else {
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) wv[i] = wv[i] - u.lr * g[j * 4 + i];
+                        *reinterpret_cast<float4 *>(wrow + pj) = make_float4(wv[0], wv[1], wv[2], wv[3]);
+                        packed[j * 2] = pack_bf16(wv[0], wv[1]);
+                        packed[j * 2 + 1] = pack_bf16(wv[2], wv[3]);
                     }
-                    *reinterpret_cast<float4 *>(wrow + pj) = make_float4(wv[0], wv[1], wv[2], wv[3]);
-                    packed[j * 2] = pack_bf16(wv[0], wv[1]);
-                    packed[j * 2 + 1] = pack_bf16(wv[2], wv[3]);
-                }
-                // bf16 box c/2 (64 columns), this chunk = 4 logical 16-byte chunks
-                uint8_t *brow = bf_tile + (c >> 1) * BM * 128 + r * 128;
+                    // bf16 sub-tile: one 64-column box when ECOLS = 64, a 32-column box otherwise
+                    constexpr int BF_ROW = C::ECOLS * 2;  // bytes per bf16 row of the sub-tile box
+                    uint8_t *brow = bf_tile + r * BF_ROW;
 #pragma unroll
-                for (int u4 = 0; u4 < 4; ++u4) {
-                    const uint32_t lj = (uint32_t)((c & 1) * 4 + u4);
-                    *reinterpret_cast<uint4 *>(brow + ((lj ^ rsw) << 4)) =
-                        make_uint4(packed[u4 * 4], packed[u4 * 4 + 1], packed[u4 * 4 + 2], packed[u4 * 4 + 3]);
+                    for (int u4 = 0; u4 < 4; ++u4) {
+                        const uint32_t lj = (uint32_t)(cc * 4 + u4);
+                        const uint32_t pjb = BF_ROW == 128 ? (lj ^ rsw) : (lj ^ ((rsw >> 1) & 3));
+                        *reinterpret_cast<uint4 *>(brow + (pjb << 4)) =
+                            make_uint4(packed[u4 * 4], packed[u4 * 4 + 1], packed[u4 * 4 + 2], packed[u4 * 4 + 3]);
+                    }
                 }
+                if (sub == SUBS - 1) {
+                    // accumulator fully consumed: hand TMEM back to the MMA warp
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
+                }
+                fence_proxy_async();
+                epi_bar();
+                if (leader) {
+                    const CUtensorMap *fm[3] = {&tmW, &tmM, &tmV};
+                    const int c0 = n0 + sub * C::ECOLS;
+#pragma unroll
+                    for (int t3 = 0; t3 < C::NF32; ++t3)
+#pragma unroll
+                        for (int q = 0; q < F32_BOXES; ++q)
+                            tma_store_2d(fm[t3], smem_u32(buf + t3 * C::F32_SUB + q * BM * 128), c0 + 32 * q, m0);
+                    tma_store_2d(&tmS, smem_u32(bf_tile), c0, m0);
+                    bulk_commit();
+                    // the bulk store reads shared memory quickly; once it has, the buffer can
+                    // take the next sub-tile's load while the global writes drain
+                    bulk_wait_read0();
+                    mbar_arrive(smem_u32(&wempty[es]));
+                }
+                if (++es == C::ESTAGES) { es = 0; ephase ^= 1; }
             }
-            // accumulator consumed: hand TMEM back to the MMA warp
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
             if (++acc == 2) { acc = 0; acc_phase ^= 1; }
-            // write the new master (m, v) and the new bf16 version back with TMA
-            fence_proxy_async();
-            epi_bar();
-            if (leader) {
-                const CUtensorMap *fm[3] = {&tmW, &tmM, &tmV};
-#pragma unroll
-                for (int t3 = 0; t3 < C::NF32; ++t3)
-#pragma unroll
-                    for (int q = 0; q < F32_BOXES; ++q)
-                        tma_store_2d(fm[t3], smem_u32(f32_tiles + t3 * C::F32_TILE + q * BM * 128), n0 + 32 * q, m0);
-#pragma unroll
-                for (int q = 0; q < BF_BOXES; ++q) tma_store_2d(&tmS, smem_u32(bf_tile + q * BM * 128), n0 + 64 * q, m0);
-                bulk_commit();
-                bulk_wait_read0();
-                mbar_arrive(smem_u32(wempty));
-            }
         }
         if (leader) bulk_wait0();
     }
@@ -627,7 +657,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
 // ---------------------------------------------------------------- host side
 bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner, int box_outer,
-              bool f32 = false) {
+              bool f32 = false, int swizzle_bytes = 128) {
     const Driver *d = driver();
     if (!d) return false;
     cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
@@ -637,7 +667,8 @@ bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long l
     CUresult r = d->tensorMapEncodeTiled(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
                                          2, const_cast<void *>(base), dims,
                                          strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                         CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                         swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
 }
@@ -663,8 +694,8 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         if (err != cudaSuccess) return err;
         attr_set = true;
     }
-    const int tiles = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN);
-    const int grid = tiles < num_sms() ? tiles : num_sms();
+    const int units = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * e.ksplit;
+    const int grid = units < num_sms() ? units : num_sms();
     kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, e, g.M, g.N, g.K);
     ++tl_launches;
     return cudaGetLastError();
@@ -732,8 +763,9 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
     const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, BN)
                                     : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
+    const int ecols = adam ? 32 : 64;  // UpdCfg::ECOLS
     bool ok = okA && okB && make_map(&mw, g.master, g.N, g.M, g.ldo, 32, BM, true) &&
-              make_map(&ms, g.slot, g.N, g.M, g.ldo, 64, BM, false);
+              make_map(&ms, g.slot, g.N, g.M, g.ldo, ecols, BM, false, ecols == 64 ? 128 : 64);
     if (adam) ok = ok && make_map(&mm, g.adam_m, g.N, g.M, g.ldo, 32, BM, true) &&
                    make_map(&mv, g.adam_v, g.N, g.M, g.ldo, 32, BM, true);
     else mm = mv = mw;
@@ -743,9 +775,98 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
     return update_major<BN_SGD, false>(g, ma, mbm, mw, mm, mv, ms, u, s);
 }
 
+// out = act(sum_s ws[s] + bias) or (sum_s ws[s]) * (mask > 0), bf16; partials summed in
+// split order (deterministic).  4 columns per thread, 16-byte loads.
+__global__ void splitk_epilogue_kernel(const float *__restrict__ ws, int S, long split_stride, int M, int N,
+                                       const float *__restrict__ bias, int relu, const __nv_bfloat16 *__restrict__ mask,
+                                       long ldm, __nv_bfloat16 *__restrict__ out, long ldo) {
+    const long n4 = N / 4;
+    const long total = (long)M * n4;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long)gridDim.x * blockDim.x) {
+        const long m = i / n4, c = (i % n4) * 4;
+        float4 a = *reinterpret_cast<const float4 *>(ws + m * N + c);
+        for (int sp = 1; sp < S; ++sp) {
+            const float4 b = *reinterpret_cast<const float4 *>(ws + sp * split_stride + m * N + c);
+            a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+        }
+        float v[4] = {a.x, a.y, a.z, a.w};
+        if (bias) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) v[j] += bias[c + j];
+        }
+        if (relu) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) v[j] = fmaxf(v[j], 0.f);
+        }
+        if (mask) {
+            const uint2 mr = *reinterpret_cast<const uint2 *>(mask + m * ldm + c);
+            const __nv_bfloat16 *mh = reinterpret_cast<const __nv_bfloat16 *>(&mr);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) v[j] = (__bfloat162float(mh[j]) > 0.f) ? v[j] : 0.f;
+        }
+        uint2 o;
+        o.x = pack_bf16(v[0], v[1]);
+        o.y = pack_bf16(v[2], v[3]);
+        *reinterpret_cast<uint2 *>(out + m * ldo + c) = o;
+    }
+}
+
 }  // namespace
 
+// Split-K is used for the small-M GEMMs of a minibatch (forward X W^T and dX = G W at
+// M = B = 256): with one output tile per SM they are L2->SM bandwidth bound because every
+// N-tile re-reads the activations; fewer, wider (BN = 256) tiles cut that traffic and the
+// K splits restore the parallelism.  Returns the split count (1 = not used).
+static int env_int(const char *name, int dflt) {
+    const char *v = getenv(name);
+    return v ? atoi(v) : dflt;
+}
+
+static int choose_ksplit(const Gemm &g, int sms) {
+    if (!(g.epi == EPI_STORE || g.epi == EPI_MASK) || !g.workspace || g.N % 4 || g.ldo != g.N) return 1;
+    const int forced = env_int("PD_GEMM_SPLIT", 0);  // tuning override (tools/gemm_bench.py)
+    if (forced > 0) return forced;
+    const long tiles = (long)((g.M + BM - 1) / BM) * ((g.N + 255) / 256);
+    const int kblocks = (g.K + BK - 1) / BK;
+    if (tiles * 2 > sms) return 1;
+    int S = (int)(sms / tiles);
+    if (S > 8) S = 8;
+    while (S > 1 && kblocks / S < 8) --S;
+    while (S > 1 && (long)S * g.M * g.N * 4 > g.workspace_bytes) --S;
+    return S;
+}
+
 cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
+    if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
+    {
+        const int S = choose_ksplit(g, num_sms());
+        if (S > 1) {
+            CUtensorMap ma, mbm;
+            const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
+                                            : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
+            const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, 256)
+                                            : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
+            if (!okA || !okB) return cudaErrorInvalidValue;
+            EpiArgs e{};
+            e.out = g.workspace;
+            e.ldo = g.N;
+            e.ksplit = S;
+            e.split_stride = (long)g.M * g.N;
+            Gemm gf = g;
+            gf.epi = EPI_F32;
+            cudaError_t err = dispatch_major<256>(gf, ma, mbm, e, s);
+            if (err != cudaSuccess) return err;
+            const long total = (long)g.M * (g.N / 4);
+            long blocks = (total + 255) / 256;
+            if (blocks > 148L * 8) blocks = 148L * 8;
+            splitk_epilogue_kernel<<<(unsigned)blocks, 256, 0, s>>>(
+                g.workspace, S, (long)g.M * g.N, g.M, g.N, g.epi == EPI_STORE ? g.bias : nullptr,
+                g.epi == EPI_STORE ? g.relu : 0, g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr,
+                g.ldm, static_cast<__nv_bfloat16 *>(g.out), g.ldo);
+            ++tl_launches;
+            return cudaGetLastError();
+        }
+    }
     if ((g.epi == EPI_SGD || g.epi == EPI_ADAM) && g.ldo == g.N && g.N % 8 == 0) return gemm_bf16_update(g, s);
     if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
     // tile width: the widest BN that still gives every SM a tile
@@ -754,6 +875,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     int BN = 256;
     if ((long)mb * ((g.N + 255) / 256) < sms) BN = 128;
     if (BN == 128 && (long)mb * ((g.N + 127) / 128) < sms) BN = 64;
+    BN = env_int("PD_GEMM_BN", BN);  // tuning override (tools/gemm_bench.py)
     CUtensorMap ma, mbm;
     const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
@@ -763,6 +885,8 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     EpiArgs e{};
     e.out = g.out;
     e.ldo = g.ldo;
+    e.ksplit = 1;
+    e.split_stride = 0;
     e.bias = g.bias;
     e.relu = g.relu;
     e.mask = static_cast<const __nv_bfloat16 *>(g.mask);

@@ -76,6 +76,9 @@ struct Gemm {
     float *adam_m = nullptr, *adam_v = nullptr;
     float lr = 0.f, b1 = 0.f, b2 = 0.f, eps = 0.f;
     int step = 0;
+    // optional fp32 scratch for split-K partials (bf16 EPI_STORE / EPI_MASK); nullptr = off
+    float *workspace = nullptr;
+    long workspace_bytes = 0;
 };
 
 // fp32 SIMT GEMM (parity path; no tensor cores, no TF32).  EPI_STORE/MASK/F32 only.

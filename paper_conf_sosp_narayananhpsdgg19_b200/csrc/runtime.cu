@@ -196,6 +196,8 @@ struct Worker {
     float *master = nullptr;    // bf16 path
     float *adam_m = nullptr, *adam_v = nullptr;
     float *gbuf = nullptr;      // fp32 gradient (unreplicated fp32 path / biases)
+    float *ws = nullptr;        // split-K partials of the bf16 GEMMs
+    long ws_bytes = 0;
     float *rgrad[2] = {};       // replicated stages: gradient per round parity
     const float **rgrad_ptrs = nullptr;  // device array [2][R]: peers' rgrad for each parity
     const float **self_grad_ptr = nullptr;  // device array [1]: gbuf
@@ -231,7 +233,7 @@ Worker::~Worker() {
     if (stream) cudaStreamSynchronize(stream);
     for (void *p : wslot) cudaFree(p);
     for (void *p : act) cudaFree(p);
-    void *bufs[] = {master, adam_m, adam_v, gbuf, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
+    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
     for (void *p : bufs)
         if (p) cudaFree(p);
@@ -349,7 +351,7 @@ cudaError_t run_gemm(int bf16, const Gemm &g, cudaStream_t s) { return bf16 ? ge
 
 // y = act(x W^T + b)
 void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, const float *bias_f32, const void *x,
-                    void *y) {
+                    void *y, float *ws, long ws_bytes) {
     const int B = L.c->cfg.minibatch;
     Gemm g;
     g.M = (int)rows_of(d, B);
@@ -366,6 +368,8 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.ldo = d.out;
     g.bias = bias_f32;
     g.relu = d.act == PD_ACT_RELU;
+    g.workspace = ws;
+    g.workspace_bytes = ws_bytes;
     CK(run_gemm(L.bf16, g, L.w->stream));
 }
 
@@ -487,7 +491,7 @@ struct Exec {
             if (d.kind != PD_LINEAR) throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             LayerCtx lc{c, w, bf16};
             cudaEvent_t k0 = kstart(0);
-            linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y);
+            linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes);
             kend(0, k0);
         }
         if (s + 1 == n()) {
@@ -577,6 +581,8 @@ struct Exec {
                 g.ldo = d.in;
                 g.mask = prev_relu ? x : nullptr;
                 g.ldm = d.in;
+                g.workspace = w->ws;
+                g.workspace_bytes = w->ws_bytes;
                 cudaEvent_t k0 = kstart(1);
                 CK(run_gemm(bf16, g, w->stream));
                 kend(1, k0);
@@ -913,6 +919,10 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         }
         w->scratch[0] = dalloc<void>(max_elems * esz);
         w->scratch[1] = dalloc<void>(max_elems * esz);
+        if (bf16) {
+            w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
+            w->ws = dalloc<float>(w->ws_bytes);
+        }
         if (stage > 0) w->recv = dalloc<void>((size_t)w->D * in_elems(c->layers[w->first], B) * esz);
         if (stage + 1 < c->n) w->gring = dalloc<void>((size_t)w->G * out_elems(c->layers[w->last], B) * esz);
         if (stage + 1 == c->n) {
@@ -1362,6 +1372,7 @@ extern "C" PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *d, void *stream) 
     g.mask = d->mask; g.ldm = d->ldm;
     g.master = d->master; g.slot = d->slot; g.adam_m = d->adam_m; g.adam_v = d->adam_v;
     g.lr = d->lr; g.b1 = d->beta1; g.b2 = d->beta2; g.eps = d->eps; g.step = d->step;
+    g.workspace = d->workspace; g.workspace_bytes = d->workspace_bytes;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     cudaError_t e = d->dtype == PD_BF16 ? gemm_bf16(g, s) : gemm_f32(g, s);
     if (e == cudaErrorInvalidValue) return PD_EINVAL;

@@ -48,25 +48,31 @@ def test_tc_gemm_f32_out(M, N, K, amn, bmn):
     assert _rel(out, ref) < 1e-5
 
 
+@pytest.mark.parametrize("split", [False, True])
 @pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES[:4])
-def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn):
+def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split):
     A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16, seed=1)
     bias = torch.randn(N, device="cuda")
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    ws = torch.empty(8 * M * N, device="cuda") if split else None
     pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], out.data_ptr(),
-                      N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1)
+                      N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1,
+                      workspace=ws.data_ptr() if split else None, workspace_bytes=ws.numel() * 4 if split else 0)
     torch.cuda.synchronize()
     ref = torch.relu(A.float() @ B.float().t() + bias)
     assert _rel(out, ref) < 1e-2
 
 
-def test_tc_gemm_mask_epilogue():
-    M, N, K = 256, 1024, 512
+@pytest.mark.parametrize("split", [False, True])
+def test_tc_gemm_mask_epilogue(split):
+    M, N, K = 256, 1024, 4096
     A, B, As, Bs = _operands(M, N, K, 0, 1, torch.bfloat16, seed=2)
     mask = torch.relu(torch.randn(M, N, device="cuda")).to(torch.bfloat16)
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    ws = torch.empty(8 * M * N, device="cuda") if split else None
     pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), K, Bs.data_ptr(), N, out.data_ptr(), N, 0, 1,
-                      pd.PD_EPI_MASK, mask=mask.data_ptr(), ldm=N)
+                      pd.PD_EPI_MASK, mask=mask.data_ptr(), ldm=N,
+                      workspace=ws.data_ptr() if split else None, workspace_bytes=ws.numel() * 4 if split else 0)
     torch.cuda.synchronize()
     ref = (A.float() @ B.float().t()) * (mask.float() > 0)
     assert _rel(out, ref) < 1e-2

@@ -1,0 +1,62 @@
+"""GEMM micro-benchmark through the C ABI (pd_kernel_gemm), CUDA events on the launching
+stream, L2 flushed between iterations; for tuning tile width / split-K on the MLP shapes.
+usage: gemm_bench.py [fwd|dx|dw] BN SPLIT [M N K]"""
+import os, sys
+sys.path.insert(0, os.path.join(os.path.dirname(os.path.abspath(__file__)), ".."))
+import torch
+import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+
+
+def bench(M, N, K, amn, bmn, epi, split_ws, iters=20):
+    A = (torch.randn(K, M, device="cuda") if amn else torch.randn(M, K, device="cuda")).to(torch.bfloat16)
+    B = (torch.randn(K, N, device="cuda") if bmn else torch.randn(N, K, device="cuda")).to(torch.bfloat16)
+    out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    master = torch.randn(M, N, device="cuda")
+    slot = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    bias = torch.zeros(N, device="cuda")
+    ws = torch.empty(8 * M * N, device="cuda")
+    s = torch.cuda.current_stream()
+    if epi == pd.PD_EPI_STORE:
+        kw = dict(bias=bias.data_ptr(), relu=1)
+    else:
+        kw = dict(master=master.data_ptr(), slot=slot.data_ptr(), lr=1e-3)
+    if split_ws:
+        kw.update(workspace=ws.data_ptr(), workspace_bytes=ws.numel() * 4)
+    f = lambda: pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, A.data_ptr(), A.shape[1], B.data_ptr(), B.shape[1],
+                                  out.data_ptr(), N, amn, bmn, epi, stream=s.cuda_stream, **kw)
+    for _ in range(3):
+        f()
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda")
+    ts = []
+    for _ in range(iters):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        f()
+        e1.record(s)
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1) * 1e3)
+    ts.sort()
+    return ts[len(ts) // 2]
+
+
+if __name__ == "__main__":
+    kind = sys.argv[1] if len(sys.argv) > 1 else "all"
+    if kind == "all":
+        for (bn, split) in [(64, 0), (128, 0), (256, 0), (256, 2), (256, 4), (256, 8)]:
+            os.environ["PD_GEMM_BN"], os.environ["PD_GEMM_SPLIT"] = str(bn), str(split)
+            t = bench(256, 4096, 4096, 0, 0, pd.PD_EPI_STORE, split > 0)
+            print(("fwd", bn, split, round(t, 2), "us", round(2 * 256 * 4096 ** 2 / t / 1e6, 1), "TF"), flush=True)
+            t = bench(256, 4096, 4096, 0, 1, pd.PD_EPI_STORE, split > 0)
+            print(("dx", bn, split, round(t, 2), "us", round(2 * 256 * 4096 ** 2 / t / 1e6, 1), "TF"), flush=True)
+        os.environ.pop("PD_GEMM_BN")
+        os.environ.pop("PD_GEMM_SPLIT")
+        t = bench(4096, 4096, 256, 1, 1, pd.PD_EPI_SGD, False)
+        print(("dw_sgd", round(t, 2), "us", round(171966464 / t / 1e3, 1), "GB/s"))
+    else:
+        bn, split = int(sys.argv[2]), int(sys.argv[3])
+        os.environ["PD_GEMM_BN"], os.environ["PD_GEMM_SPLIT"] = str(bn), str(split)
+        M, N, K = (int(x) for x in sys.argv[4:7]) if len(sys.argv) > 6 else (256, 4096, 4096)
+        amn, bmn, epi = {"fwd": (0, 0, pd.PD_EPI_STORE), "dx": (0, 1, pd.PD_EPI_STORE),
+                         "dw": (1, 1, pd.PD_EPI_SGD)}[kind]
+        print(kind, bn, split, bench(M, N, K, amn, bmn, epi, split > 0, iters=5))
