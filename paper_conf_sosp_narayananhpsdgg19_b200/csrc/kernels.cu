@@ -96,41 +96,68 @@ __global__ void col_sum_kernel(const T *G, long rows, long cols, float *out) {
 }
 
 // ------------------------------------------------------------------ bias gradient (+ update)
-// db[c] = sum_r G[r][c] for 32 columns per block: 8 row groups x 32 columns, coalesced
-// 64-byte row segments, partials reduced in a fixed order (deterministic).  When `master`
-// is given the optimizer update of the bias is applied in the same kernel (bf16 path,
-// unreplicated stage); otherwise db is written to grad_out.
+// db[c] = sum_r G[r][c].  A 1024-thread block covers 64 columns (a lane reads 2 adjacent
+// columns, so a warp reads one 128-byte row segment) x 32 row groups; each thread sums its
+// rows with 8 independent loads in flight, then the 32 partials are added in a fixed order
+// (deterministic).  When `master` is given the optimizer update of the bias is applied in
+// the same kernel (bf16 path, unreplicated stage); otherwise db is written to grad_out.
 template <typename T>
-__global__ void __launch_bounds__(256) bias_grad_kernel(const T *__restrict__ G, long rows, long cols,
-                                                        float *grad_out, float *master, __nv_bfloat16 *slot, int opt,
-                                                        float *m, float *v, float lr, float b1, float b2, float eps,
-                                                        float bc1, float bc2) {
-    __shared__ float part[8][33];
-    const int cl = threadIdx.x & 31, rg = threadIdx.x >> 5;
-    const long c = (long)blockIdx.x * 32 + cl;
-    float acc = 0.f;
-    if (c < cols)
-        for (long r = rg; r < rows; r += 8) acc += ld_as_f32(G, r * cols + c);
-    part[rg][cl] = acc;
-    __syncthreads();
-    if (rg == 0 && c < cols) {
-        float g = part[0][cl];
+__device__ __forceinline__ float2 ld2_as_f32(const T *p, long i) {
+    if constexpr (sizeof(T) == 4) return make_float2(p[i], p[i + 1]);
+    else {
+        const __nv_bfloat162 h = *reinterpret_cast<const __nv_bfloat162 *>(p + i);
+        return __bfloat1622float2(h);
+    }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(1024) bias_grad_kernel(const T *__restrict__ G, long rows, long cols,
+                                                         float *grad_out, float *master, __nv_bfloat16 *slot, int opt,
+                                                         float *m, float *v, float lr, float b1, float b2, float eps,
+                                                         float bc1, float bc2) {
+    __shared__ float part[32][65];
+    const int lane = threadIdx.x & 31, rg = threadIdx.x >> 5;
+    const long c = (long)blockIdx.x * 64 + 2 * lane;
+    float a0 = 0.f, a1 = 0.f;
+    if (c + 1 < cols) {
+        long r = rg;
+        for (; r + 7 * 32 < rows; r += 8 * 32) {
+            float2 x[8];
 #pragma unroll
-        for (int q = 1; q < 8; ++q) g += part[q][cl];
-        if (grad_out) grad_out[c] = g;
+            for (int u = 0; u < 8; ++u) x[u] = ld2_as_f32(G, (r + u * 32) * cols + c);
+#pragma unroll
+            for (int u = 0; u < 8; ++u) { a0 += x[u].x; a1 += x[u].y; }
+        }
+        for (; r < rows; r += 32) {
+            const float2 x = ld2_as_f32(G, r * cols + c);
+            a0 += x.x;
+            a1 += x.y;
+        }
+    } else if (c < cols) {
+        for (long r = rg; r < rows; r += 32) a0 += ld_as_f32(G, r * cols + c);
+    }
+    part[rg][2 * lane] = a0;
+    part[rg][2 * lane + 1] = a1;
+    __syncthreads();
+    if (threadIdx.x < 64) {
+        const long cc = (long)blockIdx.x * 64 + threadIdx.x;
+        if (cc >= cols) return;
+        float g = part[0][threadIdx.x];
+        for (int q = 1; q < 32; ++q) g += part[q][threadIdx.x];
+        if (grad_out) grad_out[cc] = g;
         if (master) {
-            float w = master[c];
+            float w = master[cc];
             if (opt == PD_SGD) {
                 w = w - lr * g;
             } else {
-                float mm = b1 * m[c] + (1.f - b1) * g;
-                float vv = b2 * v[c] + (1.f - b2) * g * g;
-                m[c] = mm;
-                v[c] = vv;
+                const float mm = b1 * m[cc] + (1.f - b1) * g;
+                const float vv = b2 * v[cc] + (1.f - b2) * g * g;
+                m[cc] = mm;
+                v[cc] = vv;
                 w = w - lr * (mm / bc1) / (sqrtf(vv / bc2) + eps);
             }
-            master[c] = w;
-            if (slot) slot[c] = __float2bfloat16_rn(w);
+            master[cc] = w;
+            if (slot) slot[cc] = __float2bfloat16_rn(w);
         }
     }
 }
@@ -244,7 +271,19 @@ __global__ void update_master_kernel(float *master, __nv_bfloat16 *slot_bf16, fl
 
 __global__ void f32_to_bf16_kernel(const float *in, __nv_bfloat16 *out, long n) {
     const long stride = (long)gridDim.x * blockDim.x;
-    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = __float2bfloat16_rn(in[i]);
+    long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
+    if ((n & 3) == 0 && ((uintptr_t)in & 15) == 0 && ((uintptr_t)out & 7) == 0) {
+        for (; i < n / 4; i += stride) {
+            const float4 x = reinterpret_cast<const float4 *>(in)[i];
+            __nv_bfloat162 lo = __floats2bfloat162_rn(x.x, x.y), hi = __floats2bfloat162_rn(x.z, x.w);
+            uint2 o;
+            o.x = *reinterpret_cast<uint32_t *>(&lo);
+            o.y = *reinterpret_cast<uint32_t *>(&hi);
+            reinterpret_cast<uint2 *>(out)[i] = o;
+        }
+        return;
+    }
+    for (; i < n; i += stride) out[i] = __float2bfloat16_rn(in[i]);
 }
 __global__ void bf16_to_f32_kernel(const __nv_bfloat16 *in, float *out, long n) {
     const long stride = (long)gridDim.x * blockDim.x;
@@ -287,13 +326,13 @@ cudaError_t bias_grad(const void *G, int bf16, long rows, long cols, float *grad
                       __nv_bfloat16 *slot, int opt, float *m, float *v, float lr, float b1, float b2, float eps,
                       int step, cudaStream_t s) {
     const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
-    const unsigned blocks = (unsigned)((cols + 31) / 32);
+    const unsigned blocks = (unsigned)((cols + 63) / 64);
     if (bf16)
-        bias_grad_kernel<<<blocks, 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(G), rows, cols, grad_out, master,
-                                                slot, opt, m, v, lr, b1, b2, eps, bc1, bc2);
+        bias_grad_kernel<<<blocks, 1024, 0, s>>>(static_cast<const __nv_bfloat16 *>(G), rows, cols, grad_out, master,
+                                                 slot, opt, m, v, lr, b1, b2, eps, bc1, bc2);
     else
-        bias_grad_kernel<<<blocks, 256, 0, s>>>(static_cast<const float *>(G), rows, cols, grad_out, master, slot, opt,
-                                                m, v, lr, b1, b2, eps, bc1, bc2);
+        bias_grad_kernel<<<blocks, 1024, 0, s>>>(static_cast<const float *>(G), rows, cols, grad_out, master, slot,
+                                                 opt, m, v, lr, b1, b2, eps, bc1, bc2);
     ++tl_launches;
     return cudaGetLastError();
 }

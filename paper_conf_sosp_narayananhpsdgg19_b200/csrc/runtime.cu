@@ -210,6 +210,8 @@ struct Worker {
     void *data_in = nullptr;     // stage 0: n_data inputs (path dtype)
     int32_t *tokens = nullptr;   // stage 0 embedding
     int32_t *labels = nullptr;   // last stage
+    float *stage_in = nullptr;   // fp32 upload staging for pd_set_data (bf16 path)
+    long stage_in_elems = 0;
     float *losses = nullptr;     // last stage, per minibatch of the run
     int losses_cap = 0;
     uint32_t *flags = nullptr;
@@ -233,7 +235,7 @@ Worker::~Worker() {
     if (stream) cudaStreamSynchronize(stream);
     for (void *p : wslot) cudaFree(p);
     for (void *p : act) cudaFree(p);
-    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
+    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
     for (void *p : bufs)
         if (p) cudaFree(p);
@@ -1049,11 +1051,17 @@ pd_status pd_set_data(pd_ctx *c, const float *inputs, const int32_t *tokens, con
                         CK(cudaMemcpyAsync(w->data_in, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice,
                                            w->stream));
                     } else {
-                        float *tmp = nullptr;
-                        CK(cudaMallocAsync(reinterpret_cast<void **>(&tmp), (size_t)nd * in_n * 4, w->stream));
-                        CK(cudaMemcpyAsync(tmp, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice, w->stream));
-                        CK(f32_to_bf16(tmp, static_cast<__nv_bfloat16 *>(w->data_in), (long)nd * in_n, w->stream));
-                        CK(cudaFreeAsync(tmp, w->stream));
+                        // persistent fp32 staging (no allocation on the per-step path)
+                        if (w->stage_in_elems < (long)nd * in_n) {
+                            CK(cudaStreamSynchronize(w->stream));
+                            if (w->stage_in) cudaFree(w->stage_in);
+                            w->stage_in = dalloc<float>((size_t)nd * in_n * 4);
+                            w->stage_in_elems = (long)nd * in_n;
+                        }
+                        CK(cudaMemcpyAsync(w->stage_in, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice,
+                                           w->stream));
+                        CK(f32_to_bf16(w->stage_in, static_cast<__nv_bfloat16 *>(w->data_in), (long)nd * in_n,
+                                       w->stream));
                     }
                 }
             }
