@@ -109,4 +109,13 @@ cudaError_t f32_to_bf16(const float *in, __nv_bfloat16 *out, long n, cudaStream_
 cudaError_t bf16_to_f32(const __nv_bfloat16 *in, float *out, long n, cudaStream_t s);
 cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s);
 
+// LSTM / embedding (lstm.cu); `bf16` selects the path dtype of h / dy / da / y / E
+cudaError_t lstm_cell_fwd(int bf16, const float *gx, const float *gh, const float *b_ih, const float *b_hh,
+                          const float *c_prev, float *gates, float *c_out, void *h_out, void *y_out, int B, int H,
+                          cudaStream_t s);
+cudaError_t lstm_cell_bwd(int bf16, const void *dy, const float *dh_rec, const float *gates, const float *c,
+                          const float *c_prev, float *dc, void *da, int B, int H, cudaStream_t s);
+cudaError_t embedding_fwd(int bf16, const int32_t *tok, const void *E, void *y, long rows, int H, cudaStream_t s);
+cudaError_t embedding_bwd(int bf16, const int32_t *tok, const void *dy, float *dE, long rows, int H, cudaStream_t s);
+
 }  // namespace pd

@@ -210,6 +210,12 @@ struct Worker {
     void *data_in = nullptr;     // stage 0: n_data inputs (path dtype)
     int32_t *tokens = nullptr;   // stage 0 embedding
     int32_t *labels = nullptr;   // last stage
+    // LSTM layers: per layer a k-deep ring of saved state {gates fp32 [T*B][4H], c fp32
+    // [T*B][H], h (path dtype) [T*B][H]}; per worker transient scratch for the recurrence
+    std::vector<void *> aux;     // index l - first (nullptr for other kinds)
+    std::vector<long> aux_bytes;
+    float *lstm_gx = nullptr, *lstm_gh = nullptr, *lstm_dh = nullptr, *lstm_dc = nullptr;
+    void *lstm_da = nullptr;
     float *stage_in = nullptr;   // fp32 upload staging for pd_set_data (bf16 path)
     long stage_in_elems = 0;
     float *losses = nullptr;     // last stage, per minibatch of the run
@@ -235,6 +241,11 @@ Worker::~Worker() {
     if (stream) cudaStreamSynchronize(stream);
     for (void *p : wslot) cudaFree(p);
     for (void *p : act) cudaFree(p);
+    for (void *p : aux)
+        if (p) cudaFree(p);
+    void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da};
+    for (void *p : lb)
+        if (p) cudaFree(p);
     void *bufs[] = {master, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
     for (void *p : bufs)
@@ -490,10 +501,18 @@ struct Exec {
             } else {
                 y = w->logits;
             }
-            if (d.kind != PD_LINEAR) throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
-            LayerCtx lc{c, w, bf16};
             cudaEvent_t k0 = kstart(0);
-            linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes);
+            if (d.kind == PD_LINEAR) {
+                LayerCtx lc{c, w, bf16};
+                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes);
+            } else if (d.kind == PD_LSTM) {
+                lstm_forward(l, j, slot, x, y);
+            } else if (d.kind == PD_EMBEDDING) {
+                CK(embedding_fwd(bf16, static_cast<const int32_t *>(x), Wl(l, slot), y, rows_of(d, B()), d.out,
+                                 w->stream));
+            } else {
+                throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
+            }
             kend(0, k0);
         }
         if (s + 1 == n()) {
@@ -516,6 +535,225 @@ struct Exec {
         for (int u = 0; u < t; ++u)
             if (u % Rp == t % Rp && u % Rc == t % Rc) ++cnt;
         return cnt;
+    }
+
+    struct BwdCtx {
+        bool fused;   // bf16 unreplicated: optimizer update fused into the dW GEMMs
+        float *gdst;  // fp32 gradient buffer otherwise (gbuf or replica round buffer)
+        int nslot;    // slot receiving the next version
+        int sslot;    // stashed version's slot
+    };
+
+    // dX = G W (B(n,k) given by the caller) fused with the previous layer's ReLU derivative
+    void gemm_dx(int l, int M, int N, int K, const void *G, long ldg, const void *W, long ldw, const void *x, void *dx) {
+        const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
+        Gemm g;
+        g.M = M;
+        g.N = N;
+        g.K = K;
+        g.A = G;
+        g.lda = ldg;
+        g.amaj = KMAJ;
+        g.B = W;
+        g.ldb = ldw;
+        g.bmaj = MNMAJ;
+        g.epi = prev_relu ? EPI_MASK : EPI_STORE;
+        g.out = dx;
+        g.ldo = N;
+        g.mask = prev_relu ? x : nullptr;
+        g.ldm = N;
+        g.workspace = w->ws;
+        g.workspace_bytes = w->ws_bytes;
+        CK(run_gemm(bf16, g, w->stream));
+    }
+
+    // dW (M x N, row-major at parameter offset woff) = A^T B over K rows, either fused with
+    // the optimizer update (writing the next version) or stored as an fp32 gradient
+    void gemm_dw(const BwdCtx &bc, long woff, int M, int N, int K, const void *A, long lda, const void *Bm, long ldb) {
+        Gemm g;
+        g.M = M;
+        g.N = N;
+        g.K = K;
+        g.A = A;
+        g.lda = lda;
+        g.amaj = MNMAJ;
+        g.B = Bm;
+        g.ldb = ldb;
+        g.bmaj = MNMAJ;
+        g.ldo = N;
+        if (bc.fused) {
+            const bool adam = c->cfg.optimizer == PD_ADAM;
+            g.epi = adam ? EPI_ADAM : EPI_SGD;
+            g.master = w->master + woff;
+            g.slot = elem_ptr(w->wslot[bc.nslot], woff, esz);
+            g.adam_m = adam ? w->adam_m + woff : nullptr;
+            g.adam_v = adam ? w->adam_v + woff : nullptr;
+            g.lr = c->cfg.lr;
+            g.b1 = c->cfg.beta1;
+            g.b2 = c->cfg.beta2;
+            g.eps = c->cfg.eps;
+            g.step = w->updates_total + 1;
+        } else {
+            g.epi = EPI_F32;
+            g.out = bc.gdst + woff;
+        }
+        CK(run_gemm(bf16, g, w->stream));
+    }
+
+    // bias gradient = column sums of G [rows][cols] (+ fused update)
+    void bias_update(const BwdCtx &bc, long boff, const void *G, long rows, int cols) {
+        if (bc.fused)
+            CK(bias_grad(G, bf16, rows, cols, nullptr, w->master + boff,
+                         static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], boff, esz)), c->cfg.optimizer,
+                         w->adam_m ? w->adam_m + boff : nullptr, w->adam_v ? w->adam_v + boff : nullptr, c->cfg.lr,
+                         c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+        else
+            CK(bias_grad(G, bf16, rows, cols, bc.gdst + boff, nullptr, nullptr, 0, nullptr, nullptr, 0.f, 0.f, 0.f,
+                         0.f, 1, w->stream));
+    }
+
+    void linear_backward(int l, const void *x, const void *G, void *dx, const BwdCtx &bc) {
+        const pd_layer_desc &d = layer(l);
+        const long rows = rows_of(d, B());
+        if (dx) {
+            cudaEvent_t k0 = kstart(1);
+            gemm_dx(l, (int)rows, d.in, d.out, G, d.out, Wl(l, bc.sslot), d.in, x, dx);
+            kend(1, k0);
+        }
+        cudaEvent_t k0 = kstart(2);
+        gemm_dw(bc, c->poff[l], d.out, d.in, (int)rows, G, d.out, x, d.in);
+        kend(2, k0);
+        k0 = kstart(3);
+        bias_update(bc, c->poff[l] + (long)d.out * d.in, G, rows, d.out);
+        kend(3, k0);
+    }
+
+    // LSTM saved state of layer l for local index j
+    struct LstmState {
+        float *gates, *c;
+        void *h;
+    };
+    LstmState lstm_state(int l, int j) const {
+        const pd_layer_desc &d = layer(l);
+        const long TB = (long)d.seq_len * B(), H = d.out;
+        char *base = static_cast<char *>(w->aux[l - w->first]) + (long)(j % w->k) * w->aux_bytes[l - w->first];
+        LstmState st;
+        st.gates = reinterpret_cast<float *>(base);
+        st.c = reinterpret_cast<float *>(base + align_up(TB * 4 * H * 4, 256));
+        st.h = base + align_up(TB * 4 * H * 4, 256) + align_up(TB * H * 4, 256);
+        return st;
+    }
+    // parameter offsets of W_ih, W_hh, b_ih, b_hh
+    long lstm_off(int l, int which) const {
+        const pd_layer_desc &d = layer(l);
+        const long H = d.out, I = d.in;
+        const long o[4] = {0, 4 * H * I, 4 * H * I + 4 * H * H, 4 * H * I + 4 * H * H + 4 * H};
+        return c->poff[l] + o[which];
+    }
+    const float *param_f32(long off, int slot) const {
+        if (bf16) return w->master + off;
+        return static_cast<const float *>(w->wslot[slot]) + off;
+    }
+
+    void lstm_forward(int l, int j, int slot, const void *x, void *y) {
+        const pd_layer_desc &d = layer(l);
+        const int T = d.seq_len, Bn = B(), H = d.out, I = d.in;
+        const long TB = (long)T * Bn;
+        LstmState st = lstm_state(l, j);
+        // Gx = X W_ih^T for all T*B rows at once
+        Gemm g;
+        g.M = (int)TB;
+        g.N = 4 * H;
+        g.K = I;
+        g.A = x;
+        g.lda = I;
+        g.B = elem_ptr(w->wslot[slot], lstm_off(l, 0), esz);
+        g.ldb = I;
+        g.epi = EPI_F32;
+        g.out = w->lstm_gx;
+        g.ldo = 4 * H;
+        CK(run_gemm(bf16, g, w->stream));
+        const float *bih = param_f32(lstm_off(l, 2), slot), *bhh = param_f32(lstm_off(l, 3), slot);
+        for (int t = 0; t < T; ++t) {
+            if (t > 0) {
+                Gemm r;
+                r.M = Bn;
+                r.N = 4 * H;
+                r.K = H;
+                r.A = elem_ptr(st.h, (long)(t - 1) * Bn * H, esz);
+                r.lda = H;
+                r.B = elem_ptr(w->wslot[slot], lstm_off(l, 1), esz);
+                r.ldb = H;
+                r.epi = EPI_F32;
+                r.out = w->lstm_gh;
+                r.ldo = 4 * H;
+                CK(run_gemm(bf16, r, w->stream));
+            }
+            CK(lstm_cell_fwd(bf16, w->lstm_gx + (long)t * Bn * 4 * H, t > 0 ? w->lstm_gh : nullptr, bih, bhh,
+                             t > 0 ? st.c + (long)(t - 1) * Bn * H : nullptr, st.gates + (long)t * Bn * 4 * H,
+                             st.c + (long)t * Bn * H, elem_ptr(st.h, (long)t * Bn * H, esz),
+                             elem_ptr(y, (long)t * Bn * H, esz), Bn, H, w->stream));
+        }
+    }
+
+    void lstm_backward(int l, int j, const void *x, const void *G, void *dx, const BwdCtx &bc) {
+        const pd_layer_desc &d = layer(l);
+        const int T = d.seq_len, Bn = B(), H = d.out, I = d.in;
+        const long TB = (long)T * Bn;
+        LstmState st = lstm_state(l, j);
+        const void *Wih = elem_ptr(w->wslot[bc.sslot], lstm_off(l, 0), esz);
+        const void *Whh = elem_ptr(w->wslot[bc.sslot], lstm_off(l, 1), esz);
+        cudaEvent_t k0 = kstart(1);
+        CK(cudaMemsetAsync(w->lstm_dc, 0, (size_t)Bn * H * 4, w->stream));
+        for (int t = T - 1; t >= 0; --t) {
+            if (t < T - 1) {
+                // dh_rec = da_{t+1} W_hh
+                Gemm r;
+                r.M = Bn;
+                r.N = H;
+                r.K = 4 * H;
+                r.A = elem_ptr(w->lstm_da, (long)(t + 1) * Bn * 4 * H, esz);
+                r.lda = 4 * H;
+                r.amaj = KMAJ;
+                r.B = Whh;
+                r.ldb = H;
+                r.bmaj = MNMAJ;
+                r.epi = EPI_F32;
+                r.out = w->lstm_dh;
+                r.ldo = H;
+                CK(run_gemm(bf16, r, w->stream));
+            }
+            CK(lstm_cell_bwd(bf16, elem_ptr(G, (long)t * Bn * H, esz), t < T - 1 ? w->lstm_dh : nullptr,
+                             st.gates + (long)t * Bn * 4 * H, st.c + (long)t * Bn * H,
+                             t > 0 ? st.c + (long)(t - 1) * Bn * H : nullptr, w->lstm_dc,
+                             elem_ptr(w->lstm_da, (long)t * Bn * 4 * H, esz), Bn, H, w->stream));
+        }
+        if (dx) gemm_dx(l, (int)TB, I, 4 * H, w->lstm_da, 4 * H, Wih, I, x, dx);
+        kend(1, k0);
+        k0 = kstart(2);
+        gemm_dw(bc, lstm_off(l, 0), 4 * H, I, (int)TB, w->lstm_da, 4 * H, x, I);
+        gemm_dw(bc, lstm_off(l, 1), 4 * H, H, (int)((T - 1) * (long)Bn), elem_ptr(w->lstm_da, (long)Bn * 4 * H, esz),
+                4 * H, st.h, H);
+        kend(2, k0);
+        k0 = kstart(3);
+        bias_update(bc, lstm_off(l, 2), w->lstm_da, TB, 4 * H);
+        bias_update(bc, lstm_off(l, 3), w->lstm_da, TB, 4 * H);
+        kend(3, k0);
+    }
+
+    void embedding_backward(int l, const void *tok, const void *G, const BwdCtx &bc) {
+        const pd_layer_desc &d = layer(l);
+        const long off = c->poff[l], n = (long)d.in * d.out;
+        float *gE = bc.fused ? w->gbuf + off : bc.gdst + off;
+        cudaEvent_t k0 = kstart(2);
+        CK(cudaMemsetAsync(gE, 0, (size_t)n * 4, w->stream));
+        CK(embedding_bwd(bf16, static_cast<const int32_t *>(tok), G, gE, rows_of(d, B()), d.out, w->stream));
+        if (bc.fused)
+            CK(update_master(w->master + off, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], off, esz)),
+                             nullptr, w->self_grad_ptr, 1, off, n, c->cfg.optimizer,
+                             w->adam_m ? w->adam_m + off : nullptr, w->adam_v ? w->adam_v + off : nullptr, c->cfg.lr,
+                             c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+        kend(2, k0);
     }
 
     // ---------------- B(s, t)
@@ -548,12 +786,11 @@ struct Exec {
         float *gdst = Rs > 1 ? w->rgrad[jr & 1] : w->gbuf;
         const int next_version = w->version + 1;
         const int nslot = next_version % w->k;
+        BwdCtx bc{fused, gdst, nslot, sslot};
         for (int l = w->last; l >= w->first; --l) {
             const pd_layer_desc &d = layer(l);
-            if (d.kind != PD_LINEAR) throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             const void *x = layer_input(l, t, j);
-            const long rows = rows_of(d, B());
-            const bool need_dx = !(s == 0 && l == 0);
+            const bool need_dx = !(s == 0 && l == 0) && d.kind != PD_EMBEDDING;
             void *dx = nullptr;
             if (need_dx) {
                 if (l == w->first) {
@@ -565,78 +802,11 @@ struct Exec {
                 } else {
                     dx = w->scratch[cur ^ 1];
                 }
-                // dX = G W, fused with the derivative of the previous layer's ReLU, which is
-                // evaluated from this layer's stashed input (post-ReLU, so x > 0 <=> z > 0).
-                const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
-                Gemm g;
-                g.M = (int)rows;
-                g.N = d.in;
-                g.K = d.out;
-                g.A = G;
-                g.lda = d.out;
-                g.amaj = KMAJ;
-                g.B = Wl(l, sslot);
-                g.ldb = d.in;
-                g.bmaj = MNMAJ;
-                g.epi = prev_relu ? EPI_MASK : EPI_STORE;
-                g.out = dx;
-                g.ldo = d.in;
-                g.mask = prev_relu ? x : nullptr;
-                g.ldm = d.in;
-                g.workspace = w->ws;
-                g.workspace_bytes = w->ws_bytes;
-                cudaEvent_t k0 = kstart(1);
-                CK(run_gemm(bf16, g, w->stream));
-                kend(1, k0);
             }
-            // dW = G^T X
-            {
-                Gemm g;
-                g.M = d.out;
-                g.N = d.in;
-                g.K = (int)rows;
-                g.A = G;
-                g.lda = d.out;
-                g.amaj = MNMAJ;
-                g.B = x;
-                g.ldb = d.in;
-                g.bmaj = MNMAJ;
-                g.ldo = d.in;
-                const long woff = c->poff[l];
-                if (fused) {
-                    const bool adam = c->cfg.optimizer == PD_ADAM;
-                    g.epi = adam ? EPI_ADAM : EPI_SGD;
-                    g.master = w->master + woff;
-                    g.slot = elem_ptr(w->wslot[nslot], woff, esz);
-                    g.adam_m = adam ? w->adam_m + woff : nullptr;
-                    g.adam_v = adam ? w->adam_v + woff : nullptr;
-                    g.lr = c->cfg.lr;
-                    g.b1 = c->cfg.beta1;
-                    g.b2 = c->cfg.beta2;
-                    g.eps = c->cfg.eps;
-                    g.step = w->updates_total + 1;
-                } else {
-                    g.epi = EPI_F32;
-                    g.out = gdst + woff;
-                }
-                cudaEvent_t k0 = kstart(2);
-                CK(run_gemm(bf16, g, w->stream));
-                kend(2, k0);
-            }
-            // db = column sums of G (+ the bias update itself on the fused path)
-            const long boff = c->poff[l] + (long)d.out * d.in;
-            {
-                cudaEvent_t k0 = kstart(3);
-                if (fused)
-                    CK(bias_grad(G, bf16, rows, d.out, nullptr, w->master + boff,
-                                 static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[nslot], boff, esz)), c->cfg.optimizer,
-                                 w->adam_m ? w->adam_m + boff : nullptr, w->adam_v ? w->adam_v + boff : nullptr,
-                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
-                else
-                    CK(bias_grad(G, bf16, rows, d.out, gdst + boff, nullptr, nullptr, 0, nullptr, nullptr, 0.f, 0.f,
-                                 0.f, 0.f, 1, w->stream));
-                kend(3, k0);
-            }
+            if (d.kind == PD_LINEAR) linear_backward(l, x, G, dx, bc);
+            else if (d.kind == PD_LSTM) lstm_backward(l, j, x, G, dx, bc);
+            else if (d.kind == PD_EMBEDDING) embedding_backward(l, x, G, bc);
+            else throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             G = dx;
             cur ^= 1;
         }
@@ -791,8 +961,12 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
         const pd_layer_desc &d = layers[l];
         if (d.in < 1 || d.out < 1 || numel_params(d) < 0) return PD_EINVAL;
         if (l > 0 && in_elems(d, 1) != out_elems(layers[l - 1], 1) && d.kind != PD_EMBEDDING) return PD_EINVAL;
-        if (d.kind != PD_LINEAR) return PD_EUNSUPPORTED;  // other layer kinds: see DESIGN.md "status"
-        if (cfg->dtype == PD_BF16 && (d.in % 8 || d.out % 8)) return PD_EUNSUPPORTED;  // 16-byte rows for TMA
+        if (d.kind != PD_LINEAR && d.kind != PD_LSTM && d.kind != PD_EMBEDDING)
+            return PD_EUNSUPPORTED;  // conv / pool: see DESIGN.md "status"
+        if (d.kind == PD_EMBEDDING && l != 0) return PD_EUNSUPPORTED;  // token ids enter at layer 0 only
+        if (d.kind == PD_LSTM && d.seq_len < 2) return PD_EUNSUPPORTED;
+        if (cfg->dtype == PD_BF16 && ((d.in % 8 && d.kind != PD_EMBEDDING) || d.out % 8))
+            return PD_EUNSUPPORTED;  // 16-byte rows for TMA
     }
     std::vector<int> kdef, kmax;
     if (inflight_counts(*plan, 0, kdef) != PD_OK) return PD_EINVAL;
@@ -921,6 +1095,26 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         }
         w->scratch[0] = dalloc<void>(max_elems * esz);
         w->scratch[1] = dalloc<void>(max_elems * esz);
+        w->aux.assign(w->last - w->first + 1, nullptr);
+        w->aux_bytes.assign(w->last - w->first + 1, 0);
+        long gx_elems = 0, bh_elems = 0;
+        for (int l = w->first; l <= w->last; ++l) {
+            const pd_layer_desc &d = c->layers[l];
+            if (d.kind != PD_LSTM) continue;
+            const long TB = (long)d.seq_len * B, H = d.out;
+            const long bytes = align_up(TB * 4 * H * 4, 256) + align_up(TB * H * 4, 256) + align_up(TB * H * esz, 256);
+            w->aux_bytes[l - w->first] = bytes;
+            w->aux[l - w->first] = dalloc<void>((size_t)w->k * bytes);
+            gx_elems = std::max(gx_elems, TB * 4 * H);
+            bh_elems = std::max(bh_elems, (long)B * H);
+        }
+        if (gx_elems) {
+            w->lstm_gx = dalloc<float>(gx_elems * 4);
+            w->lstm_da = dalloc<void>(gx_elems * esz);
+            w->lstm_gh = dalloc<float>(4 * bh_elems * 4);
+            w->lstm_dh = dalloc<float>(bh_elems * 4);
+            w->lstm_dc = dalloc<float>(bh_elems * 4);
+        }
         if (bf16) {
             w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
             w->ws = dalloc<float>(w->ws_bytes);
