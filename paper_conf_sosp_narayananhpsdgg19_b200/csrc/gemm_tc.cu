@@ -49,6 +49,8 @@ struct EpiArgs {
     long ldo;
     long split_stride;  // elements between the fp32 partial outputs of K-splits (EPI_F32)
     int ksplit;         // K is cut into ksplit contiguous ranges; work unit = (tile, split)
+    ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
+    int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
@@ -150,6 +152,13 @@ template <int EPI>
 __device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32], int row, int col, int M, int N) {
     if (row >= M) return;
     const bool full = (col + 32 <= N);
+    // conv output on the zero-padded grid: border pixels are written as 0 so buffers never
+    // need clearing and the next layer's halo stays zero
+    bool border = false;
+    if (e.conv.Hp) {
+        const int wp = row % e.conv.Wp, hp = (row / e.conv.Wp) % e.conv.Hp;
+        border = hp == 0 || hp == e.conv.Hp - 1 || wp == 0 || wp == e.conv.Wp - 1;
+    }
     if constexpr (EPI == EPI_STORE || EPI == EPI_MASK) {
         if constexpr (EPI == EPI_STORE) {
             if (e.bias) {
@@ -160,7 +169,15 @@ __device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32],
 #pragma unroll
                 for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
             }
+            if (border) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = 0.f;
+            }
         } else {
+            if (border) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = 0.f;
+            }
             const __nv_bfloat16 *mk = e.mask + (long)row * e.ldm + col;
             if (full) {
 #pragma unroll
@@ -192,6 +209,11 @@ __device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32],
         }
     } else if constexpr (EPI == EPI_F32) {
         float *o = static_cast<float *>(e.out) + (long)row * e.ldo + col;
+        if (e.atomic_out) {
+            for (int i = 0; i < 32; ++i)
+                if (col + i < N) atomicAdd(o + i, v[i]);
+            return;
+        }
         if (full) {
 #pragma unroll
             for (int q = 0; q < 8; ++q)
@@ -311,17 +333,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
                     const uint32_t sb = sa + C::A_BYTES;
                     const int k0 = kb * BK;
+                    // implicit-GEMM convolution: K-block kb = (tap, 64-channel block); the A rows
+                    // (padded-grid pixels) shift by the tap's offset, B moves to the tap's slice
+                    int ka = k0, ma = m0, kbk = k0, nb = n0;
+                    if (e.conv.taps) {
+                        const int tap = kb / e.conv.kpt, cblk = (kb % e.conv.kpt) * BK;
+                        ka = cblk;
+                        ma = m0 + e.conv.a_shift[tap];
+                        kbk = cblk + tap * e.conv.b_koff;
+                        nb = n0 + tap * e.conv.b_noff;
+                    }
+                    kbk += e.conv.b_kshift;
                     if (AMAJ == KMAJ) {
-                        tma_load_2d(sa, &tmA, fb, k0, m0);  // box {64 K, 128 M}
+                        tma_load_2d(sa, &tmA, fb, ka, ma);  // box {64 K, 128 M}
                     } else {
 #pragma unroll
-                        for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * BK * 128, &tmA, fb, m0 + 64 * j, k0);
+                        for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * BK * 128, &tmA, fb, ma + 64 * j, ka);
                     }
                     if (BMAJ == KMAJ) {
-                        tma_load_2d(sb, &tmB, fb, k0, n0);  // box {64 K, BN N}
+                        tma_load_2d(sb, &tmB, fb, kbk, nb);  // box {64 K, BN N}
                     } else {
 #pragma unroll
-                        for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * BK * 128, &tmB, fb, n0 + 64 * j, k0);
+                        for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * BK * 128, &tmB, fb, nb + 64 * j, kbk);
                     }
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
                 }
@@ -374,10 +407,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const int row = m0 + q * 32 + lane;
             EpiArgs es = e;
             if (EPI == EPI_F32) es.out = static_cast<float *>(e.out) + (long)split * e.split_stride;
+            const bool empty_range = split * kper >= kblocks;  // (host avoids it; be safe)
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
                 float v[32];
                 tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, v);
+                if (empty_range) {
+                    if (e.atomic_out) continue;
+#pragma unroll
+                    for (int i = 0; i < 32; ++i) v[i] = 0.f;
+                }
                 if (n0 + c * 32 < N) epilogue_chunk<EPI>(es, v, row, n0 + c * 32, M, N);
             }
             tc_fence_before();
@@ -823,7 +862,8 @@ static int env_int(const char *name, int dflt) {
 }
 
 static int choose_ksplit(const Gemm &g, int sms) {
-    if (!(g.epi == EPI_STORE || g.epi == EPI_MASK) || !g.workspace || g.N % 4 || g.ldo != g.N) return 1;
+    if (!(g.epi == EPI_STORE || g.epi == EPI_MASK) || !g.workspace || g.N % 4 || g.ldo != g.N || g.conv.taps)
+        return 1;
     const int forced = env_int("PD_GEMM_SPLIT", 0);  // tuning override (tools/gemm_bench.py)
     if (forced > 0) return forced;
     const long tiles = (long)((g.M + BM - 1) / BM) * ((g.N + 255) / 256);
@@ -833,7 +873,8 @@ static int choose_ksplit(const Gemm &g, int sms) {
     if (S > 8) S = 8;
     while (S > 1 && kblocks / S < 8) --S;
     while (S > 1 && (long)S * g.M * g.N * 4 > g.workspace_bytes) --S;
-    return S;
+    const int kper = (kblocks + S - 1) / S;
+    return (kblocks + kper - 1) / kper;  // no empty K range
 }
 
 cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
@@ -848,6 +889,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
                                             : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
             if (!okA || !okB) return cudaErrorInvalidValue;
             EpiArgs e{};
+            e.conv = g.conv;
             e.out = g.workspace;
             e.ldo = g.N;
             e.ksplit = S;
@@ -877,15 +919,37 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     if (BN == 128 && (long)mb * ((g.N + 127) / 128) < sms) BN = 64;
     BN = env_int("PD_GEMM_BN", BN);  // tuning override (tools/gemm_bench.py)
     CUtensorMap ma, mbm;
-    const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
+    // implicit-GEMM conv: the tensors are [rows][channels] / [Cout][9*Cp]; the K walk over
+    // (tap, channel block) is done by the producer's coordinates, not by the map extents
+    const long aK = g.conv.taps ? g.conv.a_inner : g.K;
+    const long bK = g.conv.taps && g.bmaj == KMAJ ? g.conv.b_inner : g.K;
+    const long bN = g.conv.taps && g.bmaj == MNMAJ ? g.conv.b_inner : g.N;
+    const long bKo = g.conv.taps && g.bmaj == MNMAJ ? g.conv.a_inner : g.K;  // dX: k = Cout rows of W
+    const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, aK, g.M, g.lda, 64, BM)
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
-    const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, BN)
-                                    : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
+    const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, bK, g.N, g.ldb, 64, BN)
+                                    : make_map(&mbm, g.B, bN, bKo, g.ldb, 64, BK);
     if (!okA || !okB) return cudaErrorInvalidValue;
     EpiArgs e{};
+    e.conv = g.conv;
+    e.atomic_out = g.atomic_out;
     e.out = g.out;
     e.ldo = g.ldo;
-    e.ksplit = 1;
+    e.ksplit = g.ksplit > 1 ? g.ksplit : 1;
+    if (g.atomic_out && g.ksplit == 0) {  // long-K reductions (conv dW): fill the machine
+        const long tiles = (long)mb * ((g.N + BN - 1) / BN);
+        const int kb = (g.K + BK - 1) / BK;
+        long S = (2L * sms + tiles - 1) / tiles;
+        if (S > kb / 4) S = kb / 4;
+        if (S < 1) S = 1;
+        const long kper = (kb + S - 1) / S;
+        e.ksplit = (int)((kb + kper - 1) / kper);  // no empty K range
+    }
+    if (e.ksplit > 1) {
+        const int kb = (g.K + BK - 1) / BK;
+        const int kper = (kb + e.ksplit - 1) / e.ksplit;
+        e.ksplit = (kb + kper - 1) / kper;
+    }
     e.split_stride = 0;
     e.bias = g.bias;
     e.relu = g.relu;

@@ -52,6 +52,20 @@ enum Epi {
     EPI_ADAM = 4    // Adam on master/m/v; slot = cast(master)
 };
 
+// Implicit-GEMM 3x3 convolution on a zero-padded NHWC grid (Hp = H+2, Wp = W+2): GEMM rows
+// are padded-grid pixels, K-block kb covers tap kb / kpt and 64 channels (kb % kpt).
+struct ConvGeom {
+    int taps = 0;          // 9 for fwd / dX, 0 otherwise
+    int kpt = 0;           // 64-wide K-blocks per tap
+    int a_shift[9] = {};   // A row offset of each tap (fwd: +delta, dX: -delta)
+    int b_koff = 0;        // B K-coordinate offset per tap (fwd, K-major weights)
+    int b_noff = 0;        // B N-coordinate offset per tap (dX, MN-major weights)
+    int b_kshift = 0;      // constant B K-coordinate shift (per-tap dW launch)
+    int Hp = 0, Wp = 0;    // padded grid of the OUTPUT rows (epilogue zeroes borders); 0 = off
+    int a_inner = 0;       // inner extents of the A / B tensors for the TMA maps (taps > 0)
+    int b_inner = 0;
+};
+
 // C(m, n) = sum_k A(m, k) * B(n, k)
 //   A(m, k) = amaj == KMAJ ? A[m*lda + k] : A[k*lda + m]
 //   B(n, k) = bmaj == KMAJ ? B[n*ldb + k] : B[k*ldb + n]
@@ -79,6 +93,9 @@ struct Gemm {
     // optional fp32 scratch for split-K partials (bf16 EPI_STORE / EPI_MASK); nullptr = off
     float *workspace = nullptr;
     long workspace_bytes = 0;
+    ConvGeom conv;        // implicit-GEMM convolution (bf16 path only)
+    int ksplit = 1;       // explicit split-K (EPI_F32 with atomic_out)
+    int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
 };
 
 // fp32 SIMT GEMM (parity path; no tensor cores, no TF32).  EPI_STORE/MASK/F32 only.
@@ -117,5 +134,18 @@ cudaError_t lstm_cell_bwd(int bf16, const void *dy, const float *dh_rec, const f
                           const float *c_prev, float *dc, void *da, int B, int H, cudaStream_t s);
 cudaError_t embedding_fwd(int bf16, const int32_t *tok, const void *E, void *y, long rows, int H, cudaStream_t s);
 cudaError_t embedding_bwd(int bf16, const int32_t *tok, const void *dy, float *dE, long rows, int H, cudaStream_t s);
+
+// conv / pool on the zero-padded NHWC layout (conv.cu)
+cudaError_t pad_nhwc(const float *in, void *out, int bf16, int B, int H, int W, int C, int Cp, cudaStream_t s);
+cudaError_t pool_fwd(int bf16, const void *x, void *y, int B, int H, int W, int C, int out_padded, cudaStream_t s);
+cudaError_t pool_bwd(int bf16, const void *x, const void *dy, void *dx, int B, int H, int W, int C, int dy_padded,
+                     int mask_relu, cudaStream_t s);
+cudaError_t col_sum_tall(const void *G, int bf16, long rows, int cols, float *out, cudaStream_t s);
+cudaError_t conv_fwd_f32(const float *x, const float *Wd, const float *bias, float *y, int B, int H, int W, int Cp,
+                         int Cout, int relu, cudaStream_t s);
+cudaError_t conv_dx_f32(const float *dy, const float *Wd, const float *xmask, float *dx, int B, int H, int W, int Cp,
+                        int Cout, cudaStream_t s);
+cudaError_t conv_dw_f32(const float *dy, const float *x, float *dW, int B, int H, int W, int Cp, int Cout,
+                        cudaStream_t s);
 
 }  // namespace pd

@@ -93,6 +93,51 @@ long out_elems(const pd_layer_desc &d, int B) {
     return 0;
 }
 
+// Device layouts.  Conv / pool inputs live on a zero-padded NHWC grid [B][H+2][W+2][Cp]
+// (Cp = channels rounded up to 8 for conv inputs, so rows are 16-byte aligned for TMA);
+// everything else is the contract layout.  A layer writes its output in the layout of the
+// layer that consumes it.
+int cpad8(int c) { return (c + 7) / 8 * 8; }
+bool padded_in(const pd_layer_desc &d) { return d.kind == PD_CONV3X3 || d.kind == PD_MAXPOOL2; }
+int dev_channels(const pd_layer_desc &d) { return d.kind == PD_CONV3X3 ? cpad8(d.in) : d.in; }
+long dev_in_elems(const std::vector<pd_layer_desc> &L, int l, int B) {
+    const pd_layer_desc &d = L[l];
+    if (padded_in(d)) return (long)B * (d.height + 2) * (d.width + 2) * dev_channels(d);
+    return in_elems(d, B);
+}
+long dev_out_elems(const std::vector<pd_layer_desc> &L, int l, int B) {
+    return l + 1 < (int)L.size() ? dev_in_elems(L, l + 1, B) : out_elems(L[l], B);
+}
+// device parameter count (conv weights are stored [Cout][3][3][Cp], K-major for the GEMM)
+long dev_params(const pd_layer_desc &d) {
+    if (d.kind == PD_CONV3X3) return (long)d.out * 9 * cpad8(d.in) + d.out;
+    return numel_params(d);
+}
+// contract layout <-> device layout of one layer's parameters (host side)
+void params_to_dev(const pd_layer_desc &d, const float *src, float *dst) {
+    if (d.kind != PD_CONV3X3) {
+        std::memcpy(dst, src, sizeof(float) * numel_params(d));
+        return;
+    }
+    const int Ci = d.in, Cp = cpad8(d.in), Co = d.out;
+    for (int co = 0; co < Co; ++co)
+        for (int tap = 0; tap < 9; ++tap)
+            for (int ci = 0; ci < Cp; ++ci)
+                dst[((long)co * 9 + tap) * Cp + ci] = ci < Ci ? src[((long)co * Ci + ci) * 9 + tap] : 0.f;
+    std::memcpy(dst + (long)Co * 9 * Cp, src + (long)Co * Ci * 9, sizeof(float) * Co);
+}
+void params_from_dev(const pd_layer_desc &d, const float *src, float *dst) {
+    if (d.kind != PD_CONV3X3) {
+        std::memcpy(dst, src, sizeof(float) * numel_params(d));
+        return;
+    }
+    const int Ci = d.in, Cp = cpad8(d.in), Co = d.out;
+    for (int co = 0; co < Co; ++co)
+        for (int ci = 0; ci < Ci; ++ci)
+            for (int tap = 0; tap < 9; ++tap) dst[((long)co * Ci + ci) * 9 + tap] = src[((long)co * 9 + tap) * Cp + ci];
+    std::memcpy(dst + (long)Co * Ci * 9, src + (long)Co * 9 * Cp, sizeof(float) * Co);
+}
+
 // ---------------------------------------------------------------- links
 enum LinkType { L_ACT = 0, L_GRAD = 1, L_READY = 2, L_DONE = 3 };
 
@@ -144,7 +189,8 @@ struct pd_ctx {
     std::vector<int> kalloc;         // allocated stash depth (max over default and max_depth)
     std::vector<int> Dalloc, Galloc; // ring depths as allocated
     std::vector<long> poff;          // parameter offset of each layer inside its stage buffer
-    std::vector<long> pcount;        // parameter count of each layer
+    std::vector<long> pcount;        // parameter count of each layer in the device layout
+    std::vector<long> hcount;        // ... in the contract layout (pd_stage_init / pd_get_params)
     std::vector<std::unique_ptr<Worker>> W;  // by worker id (null when remote)
     std::vector<Shared> shared;              // by worker id
     std::map<std::tuple<int, int, int>, std::unique_ptr<Link>> links;  // (type, src, dst)
@@ -422,11 +468,11 @@ struct Exec {
             if (w->stage == 0) {
                 const int di = t % c->n_data;
                 if (d.kind == PD_EMBEDDING) return w->tokens + (long)di * in_elems(d, B());
-                return elem_ptr(w->data_in, (long)di * in_elems(d, B()), esz);
+                return elem_ptr(w->data_in, (long)di * dev_in_elems(c->layers, l, B()), esz);
             }
-            return elem_ptr(w->recv, (long)(j % w->D) * in_elems(d, B()), esz);
+            return elem_ptr(w->recv, (long)(j % w->D) * dev_in_elems(c->layers, l, B()), esz);
         }
-        return elem_ptr(w->act[l - w->first], (long)(j % w->k) * in_elems(d, B()), esz);
+        return elem_ptr(w->act[l - w->first], (long)(j % w->k) * dev_in_elems(c->layers, l, B()), esz);
     }
 
     // per-kernel-class device time (0 fwd GEMM, 1 dX GEMM, 2 dW(+update) GEMM, 3 other)
@@ -490,14 +536,14 @@ struct Exec {
             const void *x = layer_input(l, t, j);
             void *y;
             if (l < w->last) {
-                y = elem_ptr(w->act[l + 1 - w->first], (long)(j % w->k) * in_elems(layer(l + 1), B()), esz);
+                y = elem_ptr(w->act[l + 1 - w->first], (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz);
             } else if (s + 1 < n()) {
                 const int Rn = c->plan.stage[s + 1].replicas;
                 const int cw = c->worker_id(s + 1, t % Rn);
                 const int jc = t / Rn;
                 const Shared &sh = c->shared[cw];
-                y = elem_ptr(sh.recv, (long)(jc % c->Dalloc[s + 1]) * out_elems(d, B()), esz);
-                w->bytes_sent += (uint64_t)out_elems(d, B()) * esz;
+                y = elem_ptr(sh.recv, (long)(jc % c->Dalloc[s + 1]) * dev_out_elems(c->layers, l, B()), esz);
+                w->bytes_sent += (uint64_t)dev_out_elems(c->layers, l, B()) * esz;
             } else {
                 y = w->logits;
             }
@@ -510,6 +556,11 @@ struct Exec {
             } else if (d.kind == PD_EMBEDDING) {
                 CK(embedding_fwd(bf16, static_cast<const int32_t *>(x), Wl(l, slot), y, rows_of(d, B()), d.out,
                                  w->stream));
+            } else if (d.kind == PD_CONV3X3) {
+                conv_forward(l, slot, x, y);
+            } else if (d.kind == PD_MAXPOOL2) {
+                const bool outpad = l + 1 < (int)c->layers.size() && padded_in(layer(l + 1));
+                CK(pool_fwd(bf16, x, y, B(), d.height, d.width, d.in, outpad, w->stream));
             } else {
                 throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             }
@@ -741,6 +792,126 @@ struct Exec {
         kend(3, k0);
     }
 
+    // ---------------- 3x3 convolution as an implicit GEMM on the padded grid
+    ConvGeom conv_geom(const pd_layer_desc &d, int sign) const {
+        ConvGeom g;
+        const int Wp = d.width + 2;
+        g.taps = 9;
+        for (int tap = 0; tap < 9; ++tap) g.a_shift[tap] = sign * (((tap / 3) - 1) * Wp + (tap % 3) - 1);
+        g.Hp = d.height + 2;
+        g.Wp = Wp;
+        return g;
+    }
+
+    void conv_forward(int l, int slot, const void *x, void *y) {
+        const pd_layer_desc &d = layer(l);
+        const int Cp = cpad8(d.in), Co = d.out, Hp = d.height + 2, Wp = d.width + 2;
+        const long M = (long)B() * Hp * Wp;
+        const long boff = c->poff[l] + (long)Co * 9 * Cp;
+        if (!bf16) {
+            const float *Wd = static_cast<const float *>(w->wslot[slot]) + c->poff[l];
+            CK(conv_fwd_f32(static_cast<const float *>(x), Wd, Wd + (long)Co * 9 * Cp, static_cast<float *>(y), B(),
+                            d.height, d.width, Cp, Co, d.act == PD_ACT_RELU, w->stream));
+            return;
+        }
+        Gemm g;
+        g.conv = conv_geom(d, +1);
+        g.conv.kpt = (Cp + 63) / 64;
+        g.conv.b_koff = Cp;
+        g.conv.a_inner = Cp;
+        g.conv.b_inner = 9 * Cp;
+        g.M = (int)M;
+        g.N = Co;
+        g.K = 9 * g.conv.kpt * 64;
+        g.A = x;
+        g.lda = Cp;
+        g.B = Wl(l, slot);
+        g.ldb = 9L * Cp;
+        g.epi = EPI_STORE;
+        g.out = y;
+        g.ldo = Co;
+        g.bias = w->master + boff;  // latest version (forward)
+        g.relu = d.act == PD_ACT_RELU;
+        CK(run_gemm(1, g, w->stream));
+    }
+
+    void conv_backward(int l, const void *x, const void *G, void *dx, const BwdCtx &bc) {
+        const pd_layer_desc &d = layer(l);
+        const int Cp = cpad8(d.in), Co = d.out, Hp = d.height + 2, Wp = d.width + 2;
+        const long M = (long)B() * Hp * Wp;
+        const long n = c->pcount[l];
+        const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
+        float *gW = (bc.fused ? w->gbuf : bc.gdst) + c->poff[l];
+        if (dx) {
+            cudaEvent_t k0 = kstart(1);
+            if (!bf16) {
+                CK(conv_dx_f32(static_cast<const float *>(G),
+                               static_cast<const float *>(w->wslot[bc.sslot]) + c->poff[l],
+                               prev_relu ? static_cast<const float *>(x) : nullptr, static_cast<float *>(dx), B(),
+                               d.height, d.width, Cp, Co, w->stream));
+            } else {
+                Gemm g;
+                g.conv = conv_geom(d, -1);
+                g.conv.kpt = (Co + 63) / 64;
+                g.conv.b_noff = Cp;
+                g.conv.a_inner = Co;
+                g.conv.b_inner = 9 * Cp;
+                g.M = (int)M;
+                g.N = Cp;
+                g.K = 9 * g.conv.kpt * 64;
+                g.A = G;
+                g.lda = Co;
+                g.amaj = KMAJ;
+                g.B = Wl(l, bc.sslot);
+                g.ldb = 9L * Cp;
+                g.bmaj = MNMAJ;
+                g.epi = prev_relu ? EPI_MASK : EPI_STORE;
+                g.mask = prev_relu ? x : nullptr;
+                g.ldm = Cp;
+                g.out = dx;
+                g.ldo = Cp;
+                CK(run_gemm(1, g, w->stream));
+            }
+            kend(1, k0);
+        }
+        cudaEvent_t k0 = kstart(2);
+        CK(cudaMemsetAsync(gW, 0, (size_t)n * 4, w->stream));
+        if (!bf16) {
+            CK(conv_dw_f32(static_cast<const float *>(G), static_cast<const float *>(x), gW, B(), d.height, d.width,
+                           Cp, Co, w->stream));
+        } else {
+            const int Wpp = Wp;
+            for (int tap = 0; tap < 9; ++tap) {
+                // dW[:, tap, :] = dY^T X_shifted over every padded-grid pixel (halo rows are 0)
+                Gemm g;
+                g.M = Co;
+                g.N = Cp;
+                g.K = (int)M;
+                g.A = G;
+                g.lda = Co;
+                g.amaj = MNMAJ;
+                g.B = x;
+                g.ldb = Cp;
+                g.bmaj = MNMAJ;
+                g.conv.b_kshift = ((tap / 3) - 1) * Wpp + (tap % 3) - 1;
+                g.epi = EPI_F32;
+                g.atomic_out = 1;
+                g.ksplit = 0;  // auto
+                g.out = gW + tap * Cp;
+                g.ldo = 9L * Cp;
+                CK(run_gemm(1, g, w->stream));
+            }
+        }
+        CK(col_sum_tall(G, bf16, M, Co, gW + (long)Co * 9 * Cp, w->stream));
+        if (bc.fused)
+            CK(update_master(w->master + c->poff[l],
+                             static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], c->poff[l], esz)), nullptr,
+                             w->self_grad_ptr, 1, c->poff[l], n, c->cfg.optimizer,
+                             w->adam_m ? w->adam_m + c->poff[l] : nullptr, w->adam_v ? w->adam_v + c->poff[l] : nullptr,
+                             c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+        kend(2, k0);
+    }
+
     void embedding_backward(int l, const void *tok, const void *G, const BwdCtx &bc) {
         const pd_layer_desc &d = layer(l);
         const long off = c->poff[l], n = (long)d.in * d.out;
@@ -780,7 +951,7 @@ struct Exec {
         }
         // gradient w.r.t. the stage output (pre-activation of the last layer)
         const void *G = (s + 1 == n()) ? w->dlogits
-                                       : elem_ptr(w->gring, (long)(j % w->G) * out_elems(layer(w->last), B()), esz);
+                                       : elem_ptr(w->gring, (long)(j % w->G) * dev_out_elems(c->layers, w->last, B()), esz);
         int cur = 0;
         const bool fused = bf16 && Rs == 1;  // dW + optimizer update in one GEMM epilogue
         float *gdst = Rs > 1 ? w->rgrad[jr & 1] : w->gbuf;
@@ -797,8 +968,8 @@ struct Exec {
                     const int Rp = c->plan.stage[s - 1].replicas;
                     const int pw = c->worker_id(s - 1, t % Rp);
                     const int jp = t / Rp;
-                    dx = elem_ptr(c->shared[pw].grad, (long)(jp % c->Galloc[s - 1]) * in_elems(d, B()), esz);
-                    w->bytes_sent += (uint64_t)in_elems(d, B()) * esz;
+                    dx = elem_ptr(c->shared[pw].grad, (long)(jp % c->Galloc[s - 1]) * dev_in_elems(c->layers, l, B()), esz);
+                    w->bytes_sent += (uint64_t)dev_in_elems(c->layers, l, B()) * esz;
                 } else {
                     dx = w->scratch[cur ^ 1];
                 }
@@ -806,7 +977,16 @@ struct Exec {
             if (d.kind == PD_LINEAR) linear_backward(l, x, G, dx, bc);
             else if (d.kind == PD_LSTM) lstm_backward(l, j, x, G, dx, bc);
             else if (d.kind == PD_EMBEDDING) embedding_backward(l, x, G, bc);
-            else throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
+            else if (d.kind == PD_CONV3X3) conv_backward(l, x, G, dx, bc);
+            else if (d.kind == PD_MAXPOOL2) {
+                if (dx) {
+                    const bool dypad = l + 1 < (int)c->layers.size() && padded_in(layer(l + 1));
+                    const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
+                    cudaEvent_t k0 = kstart(1);
+                    CK(pool_bwd(bf16, x, G, dx, B(), d.height, d.width, d.in, dypad, prev_relu, w->stream));
+                    kend(1, k0);
+                }
+            } else throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             G = dx;
             cur ^= 1;
         }
@@ -961,11 +1141,16 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
         const pd_layer_desc &d = layers[l];
         if (d.in < 1 || d.out < 1 || numel_params(d) < 0) return PD_EINVAL;
         if (l > 0 && in_elems(d, 1) != out_elems(layers[l - 1], 1) && d.kind != PD_EMBEDDING) return PD_EINVAL;
-        if (d.kind != PD_LINEAR && d.kind != PD_LSTM && d.kind != PD_EMBEDDING)
-            return PD_EUNSUPPORTED;  // conv / pool: see DESIGN.md "status"
+        if (d.kind == PD_CONV3X3 || d.kind == PD_MAXPOOL2) {
+            if (d.height < 2 || d.width < 2 || (d.kind == PD_MAXPOOL2 && ((d.height | d.width) & 1)))
+                return PD_EINVAL;
+            // a conv writes the padded layout: its consumer must be a conv or a pool
+            if (d.kind == PD_CONV3X3 && (l + 1 >= num_layers || !padded_in(layers[l + 1]))) return PD_EUNSUPPORTED;
+            if (cfg->dtype == PD_BF16 && d.kind == PD_MAXPOOL2 && d.in % 8) return PD_EUNSUPPORTED;
+        }
         if (d.kind == PD_EMBEDDING && l != 0) return PD_EUNSUPPORTED;  // token ids enter at layer 0 only
         if (d.kind == PD_LSTM && d.seq_len < 2) return PD_EUNSUPPORTED;
-        if (cfg->dtype == PD_BF16 && ((d.in % 8 && d.kind != PD_EMBEDDING) || d.out % 8))
+        if (cfg->dtype == PD_BF16 && ((d.in % 8 && d.kind != PD_EMBEDDING && d.kind != PD_CONV3X3) || d.out % 8))
             return PD_EUNSUPPORTED;  // 16-byte rows for TMA
     }
     std::vector<int> kdef, kmax;
@@ -995,11 +1180,13 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
     for (int s = 0; s + 1 < n; ++s) c->Galloc[s] = kmax[s];
     c->poff.assign(num_layers, 0);
     c->pcount.assign(num_layers, 0);
+    c->hcount.assign(num_layers, 0);
     for (int s = 0; s < n; ++s) {
         long off = 0;
         for (int l = plan->stage[s].first_layer; l <= plan->stage[s].last_layer; ++l) {
             c->poff[l] = off;
-            c->pcount[l] = numel_params(layers[l]);
+            c->hcount[l] = numel_params(layers[l]);
+            c->pcount[l] = dev_params(layers[l]);
             off += align_up(c->pcount[l], 64);  // 256-byte aligned layer blocks
         }
     }
@@ -1059,7 +1246,7 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             const float *src = init_params ? init_params[l - w->first] : nullptr;
             if (c->pcount[l] > 0) {
                 if (!src) throw CudaFail{cudaErrorInvalidValue, "missing init params"};
-                std::memcpy(host.data() + c->poff[l], src, c->pcount[l] * sizeof(float));
+                params_to_dev(c->layers[l], src, host.data() + c->poff[l]);
             }
         }
         CK(cudaMemcpy(stage_f32, host.data(), P * 4, cudaMemcpyHostToDevice));
@@ -1090,8 +1277,8 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         w->act.assign(w->last - w->first + 1, nullptr);
         long max_elems = 0;
         for (int l = w->first; l <= w->last; ++l) {
-            max_elems = std::max(max_elems, std::max(in_elems(c->layers[l], B), out_elems(c->layers[l], B)));
-            if (l > w->first) w->act[l - w->first] = dalloc<void>((size_t)w->k * in_elems(c->layers[l], B) * esz);
+            max_elems = std::max(max_elems, std::max(dev_in_elems(c->layers, l, B), dev_out_elems(c->layers, l, B)));
+            if (l > w->first) w->act[l - w->first] = dalloc<void>((size_t)w->k * dev_in_elems(c->layers, l, B) * esz);
         }
         w->scratch[0] = dalloc<void>(max_elems * esz);
         w->scratch[1] = dalloc<void>(max_elems * esz);
@@ -1119,8 +1306,8 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
             w->ws = dalloc<float>(w->ws_bytes);
         }
-        if (stage > 0) w->recv = dalloc<void>((size_t)w->D * in_elems(c->layers[w->first], B) * esz);
-        if (stage + 1 < c->n) w->gring = dalloc<void>((size_t)w->G * out_elems(c->layers[w->last], B) * esz);
+        if (stage > 0) w->recv = dalloc<void>((size_t)w->D * dev_in_elems(c->layers, w->first, B) * esz);
+        if (stage + 1 < c->n) w->gring = dalloc<void>((size_t)w->G * dev_out_elems(c->layers, w->last, B) * esz);
         if (stage + 1 == c->n) {
             const long lo = out_elems(c->layers[w->last], B);
             w->logits = dalloc<void>(lo * esz);
@@ -1237,11 +1424,12 @@ pd_status pd_set_data(pd_ctx *c, const float *inputs, const int32_t *tokens, con
                     }
                     CK(cudaMemcpyAsync(w->tokens, tokens, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice, w->stream));
                 } else {
+                    const long dev_n = dev_in_elems(c->layers, 0, B);  // padded for a conv first layer
                     if (c->n_data != nd || !w->data_in) {
                         if (w->data_in) cudaFree(w->data_in);
-                        w->data_in = dalloc<void>((size_t)nd * in_n * c->esz);
+                        w->data_in = dalloc<void>((size_t)nd * dev_n * c->esz);
                     }
-                    if (c->esz == 4) {
+                    if (c->esz == 4 && !padded_in(L0)) {
                         CK(cudaMemcpyAsync(w->data_in, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice,
                                            w->stream));
                     } else {
@@ -1254,8 +1442,12 @@ pd_status pd_set_data(pd_ctx *c, const float *inputs, const int32_t *tokens, con
                         }
                         CK(cudaMemcpyAsync(w->stage_in, inputs, (size_t)nd * in_n * 4, cudaMemcpyHostToDevice,
                                            w->stream));
-                        CK(f32_to_bf16(w->stage_in, static_cast<__nv_bfloat16 *>(w->data_in), (long)nd * in_n,
-                                       w->stream));
+                        if (padded_in(L0))
+                            CK(pad_nhwc(w->stage_in, w->data_in, c->esz == 2, nd * B, L0.height, L0.width, L0.in,
+                                        dev_channels(L0), w->stream));
+                        else
+                            CK(f32_to_bf16(w->stage_in, static_cast<__nv_bfloat16 *>(w->data_in), (long)nd * in_n,
+                                           w->stream));
                     }
                 }
             }
@@ -1410,7 +1602,7 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
 pd_status pd_get_params(pd_ctx *c, int layer, float *host_out, size_t count) {
     CHECK_CTX(c);
     if (layer < 0 || layer >= (int)c->layers.size() || !host_out) return PD_EINVAL;
-    if (count != (size_t)c->pcount[layer]) return PD_EINVAL;
+    if (count != (size_t)c->hcount[layer]) return PD_EINVAL;
     int s = 0;
     while (c->plan.stage[s].last_layer < layer) ++s;
     Worker *w = nullptr;
@@ -1419,10 +1611,12 @@ pd_status pd_get_params(pd_ctx *c, int layer, float *host_out, size_t count) {
     if (count == 0) return PD_OK;
     if (cudaSetDevice(w->device) != cudaSuccess) return PD_ECUDA;
     const float *src = (c->cfg.dtype == PD_BF16) ? w->master : static_cast<const float *>(w->wslot[w->version % w->k]);
-    if (cudaMemcpy(host_out, src + c->poff[layer], count * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+    std::vector<float> dev(c->pcount[layer]);
+    if (cudaMemcpy(dev.data(), src + c->poff[layer], dev.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
         c->fail(PD_ECUDA, "pd_get_params copy");
         return PD_ECUDA;
     }
+    params_from_dev(c->layers[layer], dev.data(), host_out);
     return PD_OK;
 }
 

@@ -149,3 +149,46 @@ def test_gnmt16_reduced_eight_stages_fp32():
     assert_schedule_exact(res)
     perr, derr = param_errors(res)
     assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+# ---------------------------------------------------------------- VGG-like conv stacks (cfg 4)
+VGG_PLANS = [([5], [1]), ([2, 5], [1, 1]), ([1, 5], [1, 1]), ([3, 5], [1, 1]), ([3, 5], [3, 1])]
+
+
+@pytest.mark.parametrize("last,reps", VGG_PLANS)
+def test_vgg_reduced_fp32(last, reps):
+    wl = synth.workload("vgg16", reduced=True)  # conv3x3(3->8)+pool, conv(8->16)+pool, FC 32, FC 10
+    M = 4 * len(last) * reps[0] + reps[0]
+    res = run_both(wl, last, reps, M, pd.PD_FP32)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+def _vgg_bf16_workload():
+    # 16 classes: 16-byte logit rows for TMA.  lr = the paper's VGG rate 0.01 (L1571-1573):
+    # bf16 activations alone give ~10 % error on these tiny convolutions' weight gradients
+    # (max-pool argmax flips; reproduced by a torch bf16 emulation)
+    layers = synth.vgg([[8], [16]], 8, 3, [32], 16)
+    return synth.Workload("vgg_r16", layers, 4, synth.SGD, 0.01)
+
+
+@pytest.mark.parametrize("last,reps", VGG_PLANS)
+def test_vgg_reduced_bf16(last, reps):
+    wl = _vgg_bf16_workload()
+    M = 4 * len(last) * reps[0] + reps[0]
+    res = run_both(wl, last, reps, M, pd.PD_BF16)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
+
+
+def test_vgg_wider_bf16_two_blocks():
+    # 64-channel convolutions on 16x16 images: several 64-channel K-blocks per tap, M tiles
+    # spanning images, split-K per-tap weight gradients
+    layers = synth.vgg([[64, 64], [128]], 16, 3, [64], 16)
+    wl = synth.Workload("vgg_w", layers, 8, synth.SGD, 0.01)
+    res = run_both(wl, [2, len(layers) - 1], [1, 1], 6, pd.PD_BF16, n_data=3)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
