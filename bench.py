@@ -34,6 +34,12 @@ os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 import numpy as np  # noqa: E402
 
 METRIC = "samples/sec at 1/2/4/8 B200 (1F1B+stash); bubble %; per-stage tensor-pipe util"
+WORKLOAD_DESC = {
+    "mlp4096": "mlp4096: BASELINE configs[1] 16 x Linear(4096)+ReLU -> CE(4096)",
+    "gnmt8": "gnmt8: BASELINE configs[2] Emb(32000,1024) -> 8 x LSTM(1024), T=50 -> Linear(1024,32000) -> CE",
+    "gnmt16": "gnmt16: BASELINE configs[4] Emb(32000,1024) -> 16 x LSTM(1024), T=50 -> Linear(1024,32000) -> CE",
+    "vgg16": "vgg16: BASELINE configs[3] VGG-16 224x224 NHWC, 13 conv3x3 + 5 maxpool + FC 4096/4096/1000",
+}
 
 
 def load_peaks():
@@ -92,16 +98,38 @@ class Clocks:
 
 # ----------------------------------------------------------------------------- workload
 
-def mlp_profile(layers, B, peaks):
-    """FLOP/byte-proportional per-layer profile for pd_plan (T_l, a_l, w_l, L841-843)."""
+def layer_flops(L, B):
+    """Algorithmic fwd+bwd FLOPs of one layer for one minibatch (2 fwd + 4 bwd per MAC)."""
+    import synth
+    if L.kind == synth.LINEAR:
+        return 6.0 * B * (L.seq_len or 1) * L.in_ * L.out
+    if L.kind == synth.LSTM:
+        return 6.0 * B * L.seq_len * 4 * L.out * (L.in_ + L.out)
+    if L.kind == synth.CONV3X3:
+        return 6.0 * B * L.height * L.width * L.out * L.in_ * 9
+    return 0.0
+
+
+def layer_out_bytes(L, B):
+    import synth
+    if L.kind == synth.MAXPOOL2:
+        return B * (L.height // 2) * (L.width // 2) * L.in_ * 2
+    if L.kind == synth.CONV3X3:
+        return B * L.height * L.width * L.out * 2
+    return B * (L.seq_len or 1) * L.out * 2
+
+
+def model_profile(layers, B, peaks):
+    """FLOP/byte-proportional per-layer profile for pd_plan (T_l, a_l, w_l, L841-843): compute
+    at 60 % of the bf16 peak or the update's HBM bytes, whichever is larger."""
     import synth
     T, a, w = [], [], []
     for L in layers:
         P = synth.param_count(L)
-        flop_t = 6.0 * B * P / (peaks["bf16_tflops"] * 1e12 * 0.6)
+        flop_t = layer_flops(L, B) / (peaks["bf16_tflops"] * 1e12 * 0.6)
         byte_t = 14.0 * P / (peaks["hbm_gbs"] * 1e9)
-        T.append(max(flop_t, byte_t))
-        a.append(B * L.out * 2)
+        T.append(max(flop_t, byte_t, 1e-7))
+        a.append(layer_out_bytes(L, B))
         w.append(P * 2)
     return T, a, w
 
@@ -127,25 +155,26 @@ def run_reference(args):
     if rank != 0:
         return
     wl = synth.workload(args.config)
-    Bs = args.cpu_batch
+    # bounded sample per step: 2 samples of the full model (mlp4096 ~5 s of single-thread
+    # oracle work per step), so --steps K --warmup W ends within minutes
+    Bs = max(1, args.cpu_batch // 4)
     layers = wl.layers
     p0 = synth.init_params(layers)
     wl_s = synth.Workload(wl.name, layers, Bs, wl.optimizer, wl.lr)
     data = synth.make_data(wl_s, 1)
     times = []
-    for _ in range(args.warmup if args.warmup < 1 else 0):
-        pass
-    for _ in range(max(1, args.steps)):
+    for i in range(min(args.warmup, 1) + max(1, args.steps)):
         t0 = time.perf_counter()
         oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
-        times.append(time.perf_counter() - t0)
+        if i >= min(args.warmup, 1):
+            times.append(time.perf_counter() - t0)
     per = float(np.median(times))
     value = Bs / per
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": args.gpus,
-            "steps": len(times), "warmup": 0, "ms_per_step": per * 1e3, "higher_is_better": True,
+            "steps": len(times), "warmup": min(args.warmup, 1), "ms_per_step": per * 1e3, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"{args.config} (BASELINE configs[1]) as the CPU oracle: 1 stage, "
-                                   f"bounded sample of 1 minibatch of B={Bs} per step", "global_batch": Bs},
+            "config": {"workload": WORKLOAD_DESC.get(args.config, args.config) + " run by the CPU oracle (1 stage); "
+                                   f"bounded sample: 1 minibatch of B={Bs} per step", "global_batch": Bs},
             "cpu_baseline": {"value": value, "unit": "samples/s", "cores": 1, "kind": "oracle",
                              "sample": f"1 minibatch of B={Bs} through all {len(layers)} layers (fwd+bwd+SGD), "
                                        f"single-threaded fp32 naive loops"},
@@ -175,7 +204,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="mlp4096")
+    ap.add_argument("--config", default="mlp4096", choices=["mlp4096", "gnmt8", "gnmt16", "vgg16"])
     ap.add_argument("--minibatches", type=int, default=0, help="minibatches per step (default 8, 16n for n>1)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-batch", type=int, default=8)
@@ -225,11 +254,17 @@ def main():
     layers, B = wl.layers, wl.batch
     if N == 1:
         plan = pd.Plan.manual([len(layers) - 1], [1])
+    elif args.config == "vgg16":
+        # VGG-16 as (N-1)-1 -- conv stage replicated, FC stage alone
+        conv_last = max(i for i, L in enumerate(layers) if L.kind == synth.MAXPOOL2)
+        plan = pd.Plan.manual([conv_last, len(layers) - 1], [N - 1, 1])
     else:
-        T, a, w = mlp_profile(layers, B, peaks)
+        T, a, w = model_profile(layers, B, peaks)
         plan = pd.pd_plan(T, a, w, N, max_replicas=1)
     n = len(plan.stages)
+    R0 = plan.stages[0][2]
     M = args.minibatches or (8 if n == 1 else 16 * n)
+    M = -(-M // R0) * R0  # a multiple of every replica count
     p0 = synth.init_params(layers) if True else None
     n_data = 8
     data = synth.make_data(wl, n_data)
@@ -267,10 +302,12 @@ def main():
     # ---- roofline of the dominant kernel (the dW GEMM + fused SGD update), this rank's stage
     s_mine = [s for s, st in enumerate(plan.stages) if st[3] <= rank < st[3] + st[2]][0]
     my_layers = [layers[l] for l in range(plan.stages[s_mine][0], plan.stages[s_mine][1] + 1)]
-    dw_bytes = float(np.mean([dw_update_bytes(L, B) for L in my_layers]))
+    lin = [L for L in my_layers if L.kind == synth.LINEAR] or my_layers
+    dw_bytes = float(np.mean([dw_update_bytes(L, B) for L in lin]))
+    stage_flops = sum(layer_flops(L, B) for L in my_layers)
     dw_avg_s = kern_ms[2] / max(kern_cnt[2], 1) / 1e3
     achieved = dw_bytes / dw_avg_s / 1e9 if dw_avg_s > 0 else 0.0
-    fw_flops = float(np.mean([gemm_flops(L, B) for L in my_layers]))
+    fw_flops = float(np.mean([gemm_flops(L, B) for L in lin]))
     fw_avg_s = kern_ms[0] / max(kern_cnt[0], 1) / 1e3
     fw_tflops = fw_flops / fw_avg_s / 1e12 if fw_avg_s > 0 else 0.0
     dx_avg_s = kern_ms[1] / max(kern_cnt[1], 1) / 1e3
@@ -282,14 +319,17 @@ def main():
     e2e = None
     if not args.no_e2e:
         inputs, tokens, labels = data
-        pin_in = torch.from_numpy(np.ascontiguousarray(np.resize(inputs, (M,) + inputs.shape[1:]))).pin_memory()
+        src = tokens if inputs is None else inputs
+        pin_in = torch.from_numpy(np.ascontiguousarray(np.resize(src, (M,) + src.shape[1:]))).pin_memory()
         pin_lab = torch.from_numpy(np.ascontiguousarray(np.resize(labels, (M,) + labels.shape[1:]))).pin_memory()
-        P.set_data(pin_in, None, pin_lab, M)
+        tok_arg = pin_in if inputs is None else None
+        in_arg = None if inputs is None else pin_in
+        P.set_data(in_arg, tok_arg, pin_lab, M)
         P.run(M)  # warm the M-sized data ring
         barrier()
         t0 = time.perf_counter()
         for _ in range(args.steps):
-            P.set_data(pin_in, None, pin_lab, M)
+            P.set_data(in_arg, tok_arg, pin_lab, M)
             P.run(M)
             P.losses(M)
         barrier()
@@ -308,8 +348,9 @@ def main():
             "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": N, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-            "config": {"workload": f"{args.config}: BASELINE configs[1] 16 x Linear(4096)+ReLU -> CE(4096), "
-                                   f"minibatch {B}, bf16 weights/activations, fp32 master, SGD lr {wl.lr}",
+            "config": {"workload": WORKLOAD_DESC.get(args.config, args.config) +
+                                   f", minibatch {B}, bf16 weights/activations, fp32 master, "
+                                   f"{'Adam' if wl.optimizer else 'SGD'} lr {wl.lr}",
                        "plan": "-".join(str(s[2]) for s in plan.stages) + f" ({n} stage{'s' if n > 1 else ''} "
                                f"of {[s[1] - s[0] + 1 for s in plan.stages]} layers)",
                        "global_batch": B, "minibatches_per_step": M, "noam": plan.noam,
@@ -331,6 +372,7 @@ def main():
                             "dx_frac": dx_tflops / peaks["bf16_tflops_sustained"],
                             "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"},
             "step_share": step_share,
+            "stage_tflops": stage_flops * args.steps * M / plan.stages[s_mine][2] / (total_ms / 1e3) / 1e12,
             "e2e": e2e,
             "cpu_baseline": cpu,
         }

@@ -51,6 +51,7 @@ struct EpiArgs {
     int ksplit;         // K is cut into ksplit contiguous ranges; work unit = (tile, split)
     ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
     int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
+    int l2_prefetch;    // producer L2-prefetch distance in K-blocks (0 = off; measured no gain so far)
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
@@ -90,6 +91,28 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map
         "l"(map), "r"(bar), "r"(c0), "r"(c1)
         : "memory");
 }
+// L2 prefetch of a tensor-map box (no shared memory, no barrier): lets the producer run far
+// ahead of the smem ring so HBM-streamed operands (the weights of a small-M GEMM) are in
+// flight long before their stage is free
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap *map, int c0, int c1) {
+    asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(map), "r"(c0), "r"(c1)
+                 : "memory");
+}
+template <int CG>
+__device__ __forceinline__ void tma_load_2d_cg(uint32_t dst, const CUtensorMap *map, uint32_t bar, int c0, int c1) {
+    if (CG == 1) {
+        tma_load_2d(dst, map, bar, c0, c1);
+    } else {
+        asm volatile(
+            "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, "
+            "%4}], [%2];" ::"r"(dst),
+            "l"(map), "r"(bar), "r"(c0), "r"(c1)
+            : "memory");
+    }
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t bar_cluster_addr) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(bar_cluster_addr) : "memory");
+}
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_commit(uint32_t bar) {
@@ -101,6 +124,32 @@ __device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t
         "setp.ne.b32 p, %4, 0;\n\t"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}" ::"r"(d_tmem),
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
+}
+template <int CG>
+__device__ __forceinline__ void tc_mma_cg(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t acc) {
+    if (CG == 1) {
+        tc_mma(d_tmem, adesc, bdesc, idesc, acc);
+    } else {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "setp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}" ::"r"(d_tmem),
+            "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
+    }
+}
+template <int CG>
+__device__ __forceinline__ void tc_commit_cg(uint32_t bar) {
+    if (CG == 1) {
+        tc_commit(bar);
+    } else {
+        const uint16_t mask = 0x3;  // arrive on the barrier at this offset in both CTAs of the pair
+        asm volatile(
+            "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                bar),
+            "h"(mask)
+            : "memory");
+    }
 }
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
     uint32_t r[32];
@@ -276,11 +325,17 @@ __device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32],
 }
 
 // ---------------------------------------------------------------- the kernel
-template <int BN, int AMAJ, int BMAJ, int EPI>
+// CG = 1: one CTA per 128 x BN tile.  CG = 2: a CTA pair (cluster of 2 on one TPC) per
+// 256 x BN tile with tcgen05.mma.cta_group::2 -- each CTA stages its 128 rows of A and half
+// (BN/2) of B, the leader issues the M = 256 MMAs reading both CTAs' shared memory, and
+// each CTA's TMEM receives its 128 accumulator rows.  Per SM that halves the B bytes per
+// FLOP, the lever that matters when the L2->SM fill (~80 GB/s per SM) is the limit.
+template <int BN, int AMAJ, int BMAJ, int EPI, int CG>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, EpiArgs e,
                    int M, int N, int K) {
-    using C = Cfg<BN>;
+    using C = Cfg<BN / CG>;  // shared-memory ring holds this CTA's A rows and B columns
+    constexpr int BNC = BN / CG;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem + C::STAGES * C::STAGE_BYTES);
@@ -288,11 +343,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int m_blocks = (M + BM - 1) / BM, n_blocks = (N + BN - 1) / BN;
+    uint32_t rank = 0;
+    if (CG == 2) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    const int pair = blockIdx.x / CG, npairs = gridDim.x / CG;
+    const int m_blocks = (M + BM * CG - 1) / (BM * CG), n_blocks = (N + BN - 1) / BN;
     const int tiles = m_blocks * n_blocks;
     const int kblocks = (K + BK - 1) / BK;
     const int units = tiles * e.ksplit;
     const int kper = (kblocks + e.ksplit - 1) / e.ksplit;
+    constexpr uint32_t TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
 
     if (warp == 0 && lane == 0) {
         asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
@@ -303,17 +362,30 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(smem_u32(&tfull[a]), 1);
-            mbar_init(smem_u32(&tempty[a]), 4);  // one arrival per epilogue warp
+            mbar_init(smem_u32(&tempty[a]), 4 * CG);  // one arrival per epilogue warp of the pair
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "r"(C::TMEM_COLS));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        if (CG == 1) {
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                             smem_u32(tmem_slot)),
+                         "r"(TMEM_COLS));
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        } else {
+            asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                             smem_u32(tmem_slot)),
+                         "r"(TMEM_COLS));
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+        }
     }
     tc_fence_before();
-    __syncthreads();
+    if (CG == 2) {
+        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+    } else {
+        __syncthreads();
+    }
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
@@ -322,20 +394,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+            for (int unit = pair; unit < units; unit += npairs) {
                 const int tile = unit % tiles, split = unit / tiles;
-                const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
+                const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM;
+                const int n0 = (tile / m_blocks) * BN + (int)rank * BNC;
                 const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-                    const uint32_t fb = smem_u32(&full[stage]);
-                    mbar_expect_tx(fb, C::STAGE_BYTES);
-                    const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
-                    const uint32_t sb = sa + C::A_BYTES;
+                // coordinates of K-block kb for this CTA (plain GEMM, implicit conv, shifted dW)
+                auto coords = [&](int kb, int &ka, int &ma, int &kbk, int &nb) {
                     const int k0 = kb * BK;
-                    // implicit-GEMM convolution: K-block kb = (tap, 64-channel block); the A rows
-                    // (padded-grid pixels) shift by the tap's offset, B moves to the tap's slice
-                    int ka = k0, ma = m0, kbk = k0, nb = n0;
+                    ka = k0; ma = m0; kbk = k0; nb = n0;
                     if (e.conv.taps) {
                         const int tap = kb / e.conv.kpt, cblk = (kb % e.conv.kpt) * BK;
                         ka = cblk;
@@ -344,31 +411,58 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         nb = n0 + tap * e.conv.b_noff;
                     }
                     kbk += e.conv.b_kshift;
+                };
+                auto prefetch = [&](int kb) {
+                    int ka, ma, kbk, nb;
+                    coords(kb, ka, ma, kbk, nb);
+                    if (AMAJ == KMAJ) tma_prefetch_2d(&tmA, ka, ma);
+                    else
+                        for (int j = 0; j < BM / 64; ++j) tma_prefetch_2d(&tmA, ma + 64 * j, ka);
+                    if (BMAJ == KMAJ) tma_prefetch_2d(&tmB, kbk, nb);
+                    else
+                        for (int j = 0; j < BNC / 64; ++j) tma_prefetch_2d(&tmB, nb + 64 * j, kbk);
+                };
+                const int PF = e.l2_prefetch;  // L2 prefetch distance in K-blocks (0 = off)
+                for (int kb = kb0; kb < min(kb1, kb0 + PF); ++kb) prefetch(kb);
+                for (int kb = kb0; kb < kb1; ++kb) {
+                    if (PF && kb + PF < kb1) prefetch(kb + PF);
+                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                    // CG = 2: both CTAs' bytes land on the LEADER's full barrier (peer bit cleared)
+                    const uint32_t fb = smem_u32(&full[stage]) & (CG == 2 ? 0xFEFFFFFFu : 0xFFFFFFFFu);
+                    if (rank == 0) mbar_expect_tx(fb, CG * C::STAGE_BYTES);
+                    const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
+                    const uint32_t sb = sa + C::A_BYTES;
+                    // implicit-GEMM convolution: K-block kb = (tap, 64-channel block); the A rows
+                    // (padded-grid pixels) shift by the tap's offset, B moves to the tap's slice
+                    int ka, ma, kbk, nb;
+                    coords(kb, ka, ma, kbk, nb);
                     if (AMAJ == KMAJ) {
-                        tma_load_2d(sa, &tmA, fb, ka, ma);  // box {64 K, 128 M}
+                        tma_load_2d_cg<CG>(sa, &tmA, fb, ka, ma);  // box {64 K, 128 M}
                     } else {
 #pragma unroll
-                        for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * BK * 128, &tmA, fb, ma + 64 * j, ka);
+                        for (int j = 0; j < BM / 64; ++j)
+                            tma_load_2d_cg<CG>(sa + j * BK * 128, &tmA, fb, ma + 64 * j, ka);
                     }
                     if (BMAJ == KMAJ) {
-                        tma_load_2d(sb, &tmB, fb, kbk, nb);  // box {64 K, BN N}
+                        tma_load_2d_cg<CG>(sb, &tmB, fb, kbk, nb);  // box {64 K, BN/CG N}
                     } else {
 #pragma unroll
-                        for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * BK * 128, &tmB, fb, nb + 64 * j, kbk);
+                        for (int j = 0; j < BNC / 64; ++j)
+                            tma_load_2d_cg<CG>(sb + j * BK * 128, &tmB, fb, nb + 64 * j, kbk);
                     }
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
                 }
             }
         }
     } else if (warp == 1) {
-        // ===== MMA issuer =====
-        if (lane == 0) {
-            constexpr uint32_t idesc = make_idesc(BM, BN, AMAJ, BMAJ);
+        // ===== MMA issuer (the pair's leader only) =====
+        if (lane == 0 && rank == 0) {
+            constexpr uint32_t idesc = make_idesc(BM * CG, BN, AMAJ, BMAJ);
             int stage = 0;
             uint32_t phase = 0;
             int acc = 0;
             uint32_t acc_phase = 0;
-            for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+            for (int unit = pair; unit < units; unit += npairs) {
                 const int split = unit / tiles;
                 const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
                 mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
@@ -385,12 +479,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                                                          : smem_desc(sa + k * 2048, BK * 128, 1024);
                         const uint64_t bd = BMAJ == KMAJ ? smem_desc(sb + k * 32, 16, 1024)
                                                          : smem_desc(sb + k * 2048, BK * 128, 1024);
-                        tc_mma(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
+                        tc_mma_cg<CG>(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
                     }
-                    tc_commit(smem_u32(&empty[stage]));  // frees the smem slot when these MMAs finish
+                    tc_commit_cg<CG>(smem_u32(&empty[stage]));  // frees the slot (both CTAs) when done
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
                 }
-                tc_commit(smem_u32(&tfull[acc]));  // accumulator ready for the epilogue
+                tc_commit_cg<CG>(smem_u32(&tfull[acc]));  // accumulator ready for both epilogues
                 if (++acc == 2) { acc = 0; acc_phase ^= 1; }
             }
         }
@@ -399,9 +493,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int q = warp & 3;  // TMEM lane quarter this warp may access
         int acc = 0;
         uint32_t acc_phase = 0;
-        for (int unit = blockIdx.x; unit < units; unit += gridDim.x) {
+        for (int unit = pair; unit < units; unit += npairs) {
             const int tile = unit % tiles, split = unit / tiles;
-            const int m0 = (tile % m_blocks) * BM, n0 = (tile / m_blocks) * BN;
+            const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM, n0 = (tile / m_blocks) * BN;
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
             tc_fence_after();
             const int row = m0 + q * 32 + lane;
@@ -421,15 +515,26 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             }
             tc_fence_before();
             __syncwarp();
-            if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
+            if (lane == 0) {
+                if (CG == 1) mbar_arrive(smem_u32(&tempty[acc]));
+                else mbar_arrive_cluster(smem_u32(&tempty[acc]) & 0xFEFFFFFFu);  // the leader's barrier
+            }
             if (++acc == 2) { acc = 0; acc_phase ^= 1; }
         }
     }
     tc_fence_before();
-    __syncthreads();
+    if (CG == 2) {
+        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+    } else {
+        __syncthreads();
+    }
     if (warp == 2) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(C::TMEM_COLS));
+        if (CG == 1)
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(TMEM_COLS));
+        else
+            asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(TMEM_COLS));
     }
 }
 
@@ -723,43 +828,61 @@ int num_sms() {
     return n;
 }
 
-template <int BN, int AMAJ, int BMAJ, int EPI>
+template <int BN, int AMAJ, int BMAJ, int EPI, int CG>
 cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e, cudaStream_t s) {
-    using C = Cfg<BN>;
-    auto kern = tc_gemm_kernel<BN, AMAJ, BMAJ, EPI>;
+    using C = Cfg<BN / CG>;
+    auto kern = tc_gemm_kernel<BN, AMAJ, BMAJ, EPI, CG>;
     static bool attr_set = false;  // per instantiation; benign race (idempotent)
     if (!attr_set) {
         cudaError_t err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
         if (err != cudaSuccess) return err;
         attr_set = true;
     }
-    const int units = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN) * e.ksplit;
-    const int grid = units < num_sms() ? units : num_sms();
-    kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, e, g.M, g.N, g.K);
+    const int units = ((g.M + BM * CG - 1) / (BM * CG)) * ((g.N + BN - 1) / BN) * e.ksplit;
+    const int slots = num_sms() / CG;
+    const int grid = CG * (units < slots ? units : slots);
+    if (CG == 1) {
+        kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, e, g.M, g.N, g.K);
+    } else {
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(NUM_THREADS);
+        cfg.dynamicSmemBytes = C::SMEM;
+        cfg.stream = s;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = 2;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        cudaError_t err = cudaLaunchKernelEx(&cfg, kern, ma, mb, e, g.M, g.N, g.K);
+        if (err != cudaSuccess) return err;
+    }
     ++tl_launches;
     return cudaGetLastError();
 }
 
-template <int BN, int AMAJ, int BMAJ>
+template <int BN, int AMAJ, int BMAJ, int CG>
 cudaError_t dispatch_epi(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e,
                          cudaStream_t s) {
     switch (g.epi) {
-    case EPI_STORE: return launch<BN, AMAJ, BMAJ, EPI_STORE>(g, ma, mb, e, s);
-    case EPI_MASK: return launch<BN, AMAJ, BMAJ, EPI_MASK>(g, ma, mb, e, s);
-    case EPI_F32: return launch<BN, AMAJ, BMAJ, EPI_F32>(g, ma, mb, e, s);
-    case EPI_SGD: return launch<BN, AMAJ, BMAJ, EPI_SGD>(g, ma, mb, e, s);
-    case EPI_ADAM: return launch<BN, AMAJ, BMAJ, EPI_ADAM>(g, ma, mb, e, s);
+    case EPI_STORE: return launch<BN, AMAJ, BMAJ, EPI_STORE, CG>(g, ma, mb, e, s);
+    case EPI_MASK: return launch<BN, AMAJ, BMAJ, EPI_MASK, CG>(g, ma, mb, e, s);
+    case EPI_F32: return launch<BN, AMAJ, BMAJ, EPI_F32, CG>(g, ma, mb, e, s);
+    case EPI_SGD: return launch<BN, AMAJ, BMAJ, EPI_SGD, 1>(g, ma, mb, e, s);
+    case EPI_ADAM: return launch<BN, AMAJ, BMAJ, EPI_ADAM, 1>(g, ma, mb, e, s);
     }
     return cudaErrorInvalidValue;
 }
 
-template <int BN>
+template <int BN, int CG = 1>
 cudaError_t dispatch_major(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e,
                            cudaStream_t s) {
-    if (g.amaj == KMAJ && g.bmaj == KMAJ) return dispatch_epi<BN, KMAJ, KMAJ>(g, ma, mb, e, s);
-    if (g.amaj == KMAJ && g.bmaj == MNMAJ) return dispatch_epi<BN, KMAJ, MNMAJ>(g, ma, mb, e, s);
-    if (g.amaj == MNMAJ && g.bmaj == MNMAJ) return dispatch_epi<BN, MNMAJ, MNMAJ>(g, ma, mb, e, s);
-    return dispatch_epi<BN, MNMAJ, KMAJ>(g, ma, mb, e, s);
+    if (g.amaj == KMAJ && g.bmaj == KMAJ) return dispatch_epi<BN, KMAJ, KMAJ, CG>(g, ma, mb, e, s);
+    if (g.amaj == KMAJ && g.bmaj == MNMAJ) return dispatch_epi<BN, KMAJ, MNMAJ, CG>(g, ma, mb, e, s);
+    if (g.amaj == MNMAJ && g.bmaj == MNMAJ) return dispatch_epi<BN, MNMAJ, MNMAJ, CG>(g, ma, mb, e, s);
+    return dispatch_epi<BN, MNMAJ, KMAJ, CG>(g, ma, mb, e, s);
 }
 
 template <int BN, int AMAJ, int BMAJ, bool ADAM>
@@ -861,15 +984,23 @@ static int env_int(const char *name, int dflt) {
     return v ? atoi(v) : dflt;
 }
 
+// 2-CTA pairs (M = 256 per MMA) for every plain GEMM with at least 256 rows
+static int use_pairs(const Gemm &g) {
+    if (env_int("PD_GEMM_CG", 2) == 1) return 1;
+    return (g.M >= 256 && (g.epi == EPI_STORE || g.epi == EPI_MASK || g.epi == EPI_F32)) ? 2 : 1;
+}
+
 static int choose_ksplit(const Gemm &g, int sms) {
     if (!(g.epi == EPI_STORE || g.epi == EPI_MASK) || !g.workspace || g.N % 4 || g.ldo != g.N || g.conv.taps)
         return 1;
     const int forced = env_int("PD_GEMM_SPLIT", 0);  // tuning override (tools/gemm_bench.py)
     if (forced > 0) return forced;
-    const long tiles = (long)((g.M + BM - 1) / BM) * ((g.N + 255) / 256);
+    const int cg = use_pairs(g);
+    const long slots = sms / cg;  // CTAs (or pairs) that can run at once
+    const long tiles = (long)((g.M + BM * cg - 1) / (BM * cg)) * ((g.N + 255) / 256);
     const int kblocks = (g.K + BK - 1) / BK;
-    if (tiles * 2 > sms) return 1;
-    int S = (int)(sms / tiles);
+    if (tiles * 2 > slots) return 1;
+    int S = (int)(slots / tiles);
     if (S > 8) S = 8;
     while (S > 1 && kblocks / S < 8) --S;
     while (S > 1 && (long)S * g.M * g.N * 4 > g.workspace_bytes) --S;
@@ -883,9 +1014,10 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         const int S = choose_ksplit(g, num_sms());
         if (S > 1) {
             CUtensorMap ma, mbm;
+            const int cg = use_pairs(g);
             const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
                                             : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
-            const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, 256)
+            const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, 256 / cg)
                                             : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
             if (!okA || !okB) return cudaErrorInvalidValue;
             EpiArgs e{};
@@ -896,7 +1028,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             e.split_stride = (long)g.M * g.N;
             Gemm gf = g;
             gf.epi = EPI_F32;
-            cudaError_t err = dispatch_major<256>(gf, ma, mbm, e, s);
+            cudaError_t err = cg == 2 ? dispatch_major<256, 2>(gf, ma, mbm, e, s) : dispatch_major<256>(gf, ma, mbm, e, s);
             if (err != cudaSuccess) return err;
             const long total = (long)g.M * (g.N / 4);
             long blocks = (total + 255) / 256;
@@ -914,10 +1046,18 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     // tile width: the widest BN that still gives every SM a tile
     const int sms = num_sms();
     const int mb = (g.M + BM - 1) / BM;
+    const int cg = use_pairs(g);
     int BN = 256;
-    if ((long)mb * ((g.N + 255) / 256) < sms) BN = 128;
-    if (BN == 128 && (long)mb * ((g.N + 127) / 128) < sms) BN = 64;
+    if (cg == 2) {
+        // pair tiles of 256 rows; BN >= 128 so each CTA holds >= 64 B columns
+        const long pm = (g.M + 255) / 256;
+        if (pm * ((g.N + 255) / 256) < sms / 2 || g.N <= 128) BN = 128;
+    } else {
+        if ((long)mb * ((g.N + 255) / 256) < sms) BN = 128;
+        if (BN == 128 && (long)mb * ((g.N + 127) / 128) < sms) BN = 64;
+    }
     BN = env_int("PD_GEMM_BN", BN);  // tuning override (tools/gemm_bench.py)
+    if (cg == 2 && BN < 128) BN = 128;
     CUtensorMap ma, mbm;
     // implicit-GEMM conv: the tensors are [rows][channels] / [Cout][9*Cp]; the K walk over
     // (tap, channel block) is done by the producer's coordinates, not by the map extents
@@ -927,12 +1067,13 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     const long bKo = g.conv.taps && g.bmaj == MNMAJ ? g.conv.a_inner : g.K;  // dX: k = Cout rows of W
     const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, aK, g.M, g.lda, 64, BM)
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
-    const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, bK, g.N, g.ldb, 64, BN)
+    const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, bK, g.N, g.ldb, 64, BN / cg)
                                     : make_map(&mbm, g.B, bN, bKo, g.ldb, 64, BK);
     if (!okA || !okB) return cudaErrorInvalidValue;
     EpiArgs e{};
     e.conv = g.conv;
     e.atomic_out = g.atomic_out;
+    e.l2_prefetch = env_int("PD_GEMM_PF", 0);
     e.out = g.out;
     e.ldo = g.ldo;
     e.ksplit = g.ksplit > 1 ? g.ksplit : 1;
@@ -965,6 +1106,10 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     e.eps = g.eps;
     e.bc1 = 1.f - powf(g.b1, (float)g.step);
     e.bc2 = 1.f - powf(g.b2, (float)g.step);
+    if (cg == 2) {
+        if (BN == 256) return dispatch_major<256, 2>(g, ma, mbm, e, s);
+        return dispatch_major<128, 2>(g, ma, mbm, e, s);
+    }
     if (BN == 256) return dispatch_major<256>(g, ma, mbm, e, s);
     if (BN == 128) return dispatch_major<128>(g, ma, mbm, e, s);
     return dispatch_major<64>(g, ma, mbm, e, s);

@@ -262,6 +262,10 @@ struct Worker {
     std::vector<long> aux_bytes;
     float *lstm_gx = nullptr, *lstm_gh = nullptr, *lstm_dh = nullptr, *lstm_dc = nullptr;
     void *lstm_da = nullptr;
+    // CUDA graphs of the LSTM recurrences (T steps of small GEMM + cell kernels), keyed by
+    // (layer, direction, saved-state slot, weight slot, dY pointer): replayed instead of
+    // re-issuing ~3T launches per layer
+    std::map<std::tuple<int, int, int, int, const void *>, std::pair<cudaGraphExec_t, int>> graphs;
     float *stage_in = nullptr;   // fp32 upload staging for pd_set_data (bf16 path)
     long stage_in_elems = 0;
     float *losses = nullptr;     // last stage, per minibatch of the run
@@ -299,6 +303,7 @@ Worker::~Worker() {
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
     for (cudaEvent_t e : run_ev)
         if (e) cudaEventDestroy(e);
+    for (auto &kv : graphs) cudaGraphExecDestroy(kv.second.first);
     if (stream) cudaStreamDestroy(stream);
 }
 
@@ -706,6 +711,34 @@ struct Exec {
         return static_cast<const float *>(w->wslot[slot]) + off;
     }
 
+    // Run `body` (a sequence of launches on w->stream) through a cached CUDA graph.
+    template <typename F>
+    void graph_run(const std::tuple<int, int, int, int, const void *> &key, F body) {
+        auto it = w->graphs.find(key);
+        if (it == w->graphs.end()) {
+            const uint64_t before = tl_launches;
+            CK(cudaStreamBeginCapture(w->stream, cudaStreamCaptureModeRelaxed));
+            try {
+                body();
+            } catch (...) {
+                cudaGraph_t g;
+                cudaStreamEndCapture(w->stream, &g);
+                if (g) cudaGraphDestroy(g);
+                throw;
+            }
+            cudaGraph_t g;
+            CK(cudaStreamEndCapture(w->stream, &g));
+            cudaGraphExec_t ex;
+            CK(cudaGraphInstantiate(&ex, g, 0));
+            CK(cudaGraphDestroy(g));
+            const int nk = (int)(tl_launches - before);
+            tl_launches = before;
+            it = w->graphs.emplace(key, std::make_pair(ex, nk)).first;
+        }
+        CK(cudaGraphLaunch(it->second.first, w->stream));
+        tl_launches += it->second.second;  // count the kernels the graph runs
+    }
+
     void lstm_forward(int l, int j, int slot, const void *x, void *y) {
         const pd_layer_desc &d = layer(l);
         const int T = d.seq_len, Bn = B(), H = d.out, I = d.in;
@@ -725,6 +758,9 @@ struct Exec {
         g.ldo = 4 * H;
         CK(run_gemm(bf16, g, w->stream));
         const float *bih = param_f32(lstm_off(l, 2), slot), *bhh = param_f32(lstm_off(l, 3), slot);
+        // the recurrence writes h into the saved state only; one copy forwards it to y
+        // (possibly another GPU's receive ring) so the captured graph is independent of y
+        graph_run(std::make_tuple(l, 0, j % w->k, slot, (const void *)nullptr), [&] {
         for (int t = 0; t < T; ++t) {
             if (t > 0) {
                 Gemm r;
@@ -738,13 +774,20 @@ struct Exec {
                 r.epi = EPI_F32;
                 r.out = w->lstm_gh;
                 r.ldo = 4 * H;
+                if (bf16) {  // M = B is tiny: split K across the machine, fp32 atomics
+                    CK(cudaMemsetAsync(w->lstm_gh, 0, (size_t)Bn * 4 * H * 4, w->stream));
+                    r.atomic_out = 1;
+                    r.ksplit = 0;
+                }
                 CK(run_gemm(bf16, r, w->stream));
             }
             CK(lstm_cell_fwd(bf16, w->lstm_gx + (long)t * Bn * 4 * H, t > 0 ? w->lstm_gh : nullptr, bih, bhh,
                              t > 0 ? st.c + (long)(t - 1) * Bn * H : nullptr, st.gates + (long)t * Bn * 4 * H,
-                             st.c + (long)t * Bn * H, elem_ptr(st.h, (long)t * Bn * H, esz),
-                             elem_ptr(y, (long)t * Bn * H, esz), Bn, H, w->stream));
+                             st.c + (long)t * Bn * H, elem_ptr(st.h, (long)t * Bn * H, esz), nullptr, Bn, H,
+                             w->stream));
         }
+        });
+        CK(cudaMemcpyAsync(y, st.h, (size_t)TB * H * esz, cudaMemcpyDeviceToDevice, w->stream));
     }
 
     void lstm_backward(int l, int j, const void *x, const void *G, void *dx, const BwdCtx &bc) {
@@ -755,6 +798,7 @@ struct Exec {
         const void *Wih = elem_ptr(w->wslot[bc.sslot], lstm_off(l, 0), esz);
         const void *Whh = elem_ptr(w->wslot[bc.sslot], lstm_off(l, 1), esz);
         cudaEvent_t k0 = kstart(1);
+        graph_run(std::make_tuple(l, 1, j % w->k, bc.sslot, G), [&] {
         CK(cudaMemsetAsync(w->lstm_dc, 0, (size_t)Bn * H * 4, w->stream));
         for (int t = T - 1; t >= 0; --t) {
             if (t < T - 1) {
@@ -772,6 +816,11 @@ struct Exec {
                 r.epi = EPI_F32;
                 r.out = w->lstm_dh;
                 r.ldo = H;
+                if (bf16) {  // M = B, N = H, K = 4H: split K, fp32 atomics
+                    CK(cudaMemsetAsync(w->lstm_dh, 0, (size_t)Bn * H * 4, w->stream));
+                    r.atomic_out = 1;
+                    r.ksplit = 0;
+                }
                 CK(run_gemm(bf16, r, w->stream));
             }
             CK(lstm_cell_bwd(bf16, elem_ptr(G, (long)t * Bn * H, esz), t < T - 1 ? w->lstm_dh : nullptr,
@@ -779,6 +828,7 @@ struct Exec {
                              t > 0 ? st.c + (long)(t - 1) * Bn * H : nullptr, w->lstm_dc,
                              elem_ptr(w->lstm_da, (long)t * Bn * 4 * H, esz), Bn, H, w->stream));
         }
+        });
         if (dx) gemm_dx(l, (int)TB, I, 4 * H, w->lstm_da, 4 * H, Wih, I, x, dx);
         kend(1, k0);
         k0 = kstart(2);

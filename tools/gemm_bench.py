@@ -26,10 +26,10 @@ def bench(M, N, K, amn, bmn, epi, split_ws, iters=20):
                                   out.data_ptr(), N, amn, bmn, epi, stream=s.cuda_stream, **kw)
     for _ in range(3):
         f()
-    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda")
+    flush = torch.ones(64 * 1024 * 1024, dtype=torch.float32, device="cuda")  # 256 MB, read to flush
     ts = []
     for _ in range(iters):
-        flush.zero_()
+        flush.sum()  # clean (read-only) L2 flush: no dirty lines left to write back
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(s)
         f()
@@ -43,14 +43,19 @@ def bench(M, N, K, amn, bmn, epi, split_ws, iters=20):
 if __name__ == "__main__":
     kind = sys.argv[1] if len(sys.argv) > 1 else "all"
     if kind == "all":
-        for (bn, split) in [(64, 0), (128, 0), (256, 0), (256, 2), (256, 4), (256, 8)]:
+        for (cg, bn, split) in [(1, 64, 0), (1, 256, 4), (2, 128, 0), (2, 256, 0), (2, 256, 2), (2, 256, 4), (0, 0, 0)]:
+            os.environ["PD_GEMM_CG"] = str(cg)
             os.environ["PD_GEMM_BN"], os.environ["PD_GEMM_SPLIT"] = str(bn), str(split)
+            if cg == 0:  # the library's own choice
+                for k in ("PD_GEMM_CG", "PD_GEMM_BN", "PD_GEMM_SPLIT"):
+                    os.environ.pop(k)
             t = bench(256, 4096, 4096, 0, 0, pd.PD_EPI_STORE, split > 0)
-            print(("fwd", bn, split, round(t, 2), "us", round(2 * 256 * 4096 ** 2 / t / 1e6, 1), "TF"), flush=True)
+            print(("fwd", cg, bn, split, round(t, 2), "us", round(2 * 256 * 4096 ** 2 / t / 1e6, 1), "TF"), flush=True)
             t = bench(256, 4096, 4096, 0, 1, pd.PD_EPI_STORE, split > 0)
-            print(("dx", bn, split, round(t, 2), "us", round(2 * 256 * 4096 ** 2 / t / 1e6, 1), "TF"), flush=True)
-        os.environ.pop("PD_GEMM_BN")
-        os.environ.pop("PD_GEMM_SPLIT")
+            print(("dx", cg, bn, split, round(t, 2), "us", round(2 * 256 * 4096 ** 2 / t / 1e6, 1), "TF"), flush=True)
+        for (M, N, K) in [(3200, 32000, 1024), (3200, 4096, 1024), (8192, 8192, 8192)]:
+            t = bench(M, N, K, 0, 0, pd.PD_EPI_STORE, False)
+            print(("big", M, N, K, round(t, 2), "us", round(2 * M * N * K / t / 1e6, 1), "TF"), flush=True)
         t = bench(4096, 4096, 256, 1, 1, pd.PD_EPI_SGD, False)
         print(("dw_sgd", round(t, 2), "us", round(171966464 / t / 1e3, 1), "GB/s"))
     else:
