@@ -898,7 +898,8 @@ cudaError_t launch_update(const Gemm &g, const CUtensorMap &ma, const CUtensorMa
         attr_set = true;
     }
     const int tiles = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN);
-    const int grid = tiles < num_sms() ? tiles : num_sms();
+    const int cap = g.max_ctas > 0 && g.max_ctas < num_sms() ? g.max_ctas : num_sms();
+    const int grid = tiles < cap ? tiles : cap;
     kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, mw, mm, mv, ms, u, g.M, g.N, g.K);
     ++tl_launches;
     return cudaGetLastError();

@@ -95,6 +95,7 @@ struct Gemm {
     long workspace_bytes = 0;
     ConvGeom conv;        // implicit-GEMM convolution (bf16 path only)
     int ksplit = 1;       // explicit split-K (EPI_F32 with atomic_out)
+    int max_ctas = 0;     // cap on resident CTAs (0 = every SM): leaves SMs to a concurrent kernel
     int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
 };
 

@@ -237,6 +237,8 @@ struct Worker {
     int k = 1;         // stash slots allocated
     int D = 0, G = 0;  // receive ring depths
     cudaStream_t stream = nullptr;
+    cudaStream_t side = nullptr;           // second stream: dW+update overlapping the next dX
+    std::vector<cudaEvent_t> ev_dx, ev_dw; // per stage layer, reused by every backward
     // weights
     std::vector<void *> wslot;  // k versions (path dtype)
     float *master = nullptr;    // bf16 path
@@ -251,7 +253,7 @@ struct Worker {
     std::vector<void *> act;     // per inner layer l (index l-first, l>first): k slots of in_elems
     void *recv = nullptr;        // D slots (stage > 0)
     void *gring = nullptr;       // G slots (stage < n-1)
-    void *scratch[2] = {};       // dY ping-pong
+    void *scratch[3] = {};       // dY rotation (3 deep so a dW on the side stream can still read it)
     void *logits = nullptr, *dlogits = nullptr;  // last stage
     void *data_in = nullptr;     // stage 0: n_data inputs (path dtype)
     int32_t *tokens = nullptr;   // stage 0 embedding
@@ -296,7 +298,7 @@ Worker::~Worker() {
     void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da};
     for (void *p : lb)
         if (p) cudaFree(p);
-    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], logits,
+    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
     for (void *p : bufs)
         if (p) cudaFree(p);
@@ -304,6 +306,9 @@ Worker::~Worker() {
     for (cudaEvent_t e : run_ev)
         if (e) cudaEventDestroy(e);
     for (auto &kv : graphs) cudaGraphExecDestroy(kv.second.first);
+    for (cudaEvent_t e : ev_dx) cudaEventDestroy(e);
+    for (cudaEvent_t e : ev_dw) cudaEventDestroy(e);
+    if (side) cudaStreamDestroy(side);
     if (stream) cudaStreamDestroy(stream);
 }
 
@@ -977,6 +982,99 @@ struct Exec {
         kend(2, k0);
     }
 
+    static bool concurrent_dw() {
+        static const int v = [] {
+            const char *e = getenv("PD_OVERLAP_DW");
+            return e ? atoi(e) : 1;
+        }();
+        return v != 0;
+    }
+    static int dw_ctas() {
+        static const int v = [] {
+            const char *e = getenv("PD_DW_CTAS");
+            return e ? atoi(e) : 0;
+        }();
+        return v;
+    }
+
+    // Backward of an all-linear stage on the bf16 fused path with the weight-gradient GEMM +
+    // optimizer update of layer l (HBM-bound) on a side stream, overlapping the input-gradient
+    // GEMM of layer l-1 (L2/latency-bound) on the main stream.  Hazards: dW_l rewrites W_l
+    // (k_s = 1: in place) so it waits for dX_l; dX_{l-2} reuses dW_l's input buffer G_l, so it
+    // waits for dW_l (3-deep rotation of the gradient scratch).
+    void backward_linear_overlapped(int t, int j, const void *G_ext, const BwdCtx &bc) {
+        const int s = w->stage;
+        const int first = w->first, last = w->last;
+        auto Gof = [&](int l) -> const void * {
+            return l == last ? G_ext : w->scratch[(last - l - 1) % 3];
+        };
+        for (int l = last; l >= first; --l) {
+            const pd_layer_desc &d = layer(l);
+            const void *x = layer_input(l, t, j);
+            const long rows = rows_of(d, B());
+            const void *Gl = Gof(l);
+            const bool need_dx = !(s == 0 && l == 0);
+            if (need_dx) {
+                void *dx;
+                if (l == first) {
+                    const int Rp = c->plan.stage[s - 1].replicas;
+                    const int pw = c->worker_id(s - 1, t % Rp);
+                    const int jp = t / Rp;
+                    dx = elem_ptr(c->shared[pw].grad, (long)(jp % c->Galloc[s - 1]) * dev_in_elems(c->layers, l, B()),
+                                  esz);
+                    w->bytes_sent += (uint64_t)dev_in_elems(c->layers, l, B()) * esz;
+                } else {
+                    dx = w->scratch[(last - l) % 3];
+                    if (l + 2 <= last) CK(cudaStreamWaitEvent(w->stream, w->ev_dw[l + 2 - first], 0));
+                }
+                cudaEvent_t k0 = kstart(1);
+                gemm_dx(l, (int)rows, d.in, d.out, Gl, d.out, Wl(l, bc.sslot), d.in, x, dx);
+                kend(1, k0);
+                CK(cudaEventRecord(w->ev_dx[l - first], w->stream));
+                CK(cudaStreamWaitEvent(w->side, w->ev_dx[l - first], 0));
+            }
+            // side stream: dW_l + fused update, bias
+            cudaStream_t main = w->stream;
+            w->stream = w->side;
+            cudaEvent_t k0 = kstart(2);
+            {
+                Gemm g;
+                g.M = d.out;
+                g.N = d.in;
+                g.K = (int)rows;
+                g.A = Gl;
+                g.lda = d.out;
+                g.amaj = MNMAJ;
+                g.B = x;
+                g.ldb = d.in;
+                g.bmaj = MNMAJ;
+                g.ldo = d.in;
+                const bool adam = c->cfg.optimizer == PD_ADAM;
+                const long woff = c->poff[l];
+                g.epi = adam ? EPI_ADAM : EPI_SGD;
+                g.master = w->master + woff;
+                g.slot = elem_ptr(w->wslot[bc.nslot], woff, esz);
+                g.adam_m = adam ? w->adam_m + woff : nullptr;
+                g.adam_v = adam ? w->adam_v + woff : nullptr;
+                g.lr = c->cfg.lr;
+                g.b1 = c->cfg.beta1;
+                g.b2 = c->cfg.beta2;
+                g.eps = c->cfg.eps;
+                g.step = w->updates_total + 1;
+                g.max_ctas = dw_ctas();
+                CK(run_gemm(1, g, w->stream));
+            }
+            kend(2, k0);
+            k0 = kstart(3);
+            bias_update(bc, c->poff[l] + (long)d.out * d.in, Gl, rows, d.out);
+            kend(3, k0);
+            CK(cudaEventRecord(w->ev_dw[l - first], w->side));
+            w->stream = main;
+        }
+        // join: everything of this backward is complete on the main stream
+        CK(cudaStreamWaitEvent(w->stream, w->ev_dw[0], 0));
+    }
+
     // ---------------- B(s, t)
     void backward(int t, int j) {
         const int s = w->stage;
@@ -1008,6 +1106,11 @@ struct Exec {
         const int next_version = w->version + 1;
         const int nslot = next_version % w->k;
         BwdCtx bc{fused, gdst, nslot, sslot};
+        bool all_linear = true;
+        for (int l = w->first; l <= w->last; ++l) all_linear = all_linear && layer(l).kind == PD_LINEAR;
+        if (fused && all_linear && concurrent_dw()) {
+            backward_linear_overlapped(t, j, G, bc);
+        } else
         for (int l = w->last; l >= w->first; --l) {
             const pd_layer_desc &d = layer(l);
             const void *x = layer_input(l, t, j);
@@ -1332,6 +1435,12 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         }
         w->scratch[0] = dalloc<void>(max_elems * esz);
         w->scratch[1] = dalloc<void>(max_elems * esz);
+        w->scratch[2] = dalloc<void>(max_elems * esz);
+        CK(cudaStreamCreateWithFlags(&w->side, cudaStreamNonBlocking));
+        w->ev_dx.resize(w->last - w->first + 1);
+        w->ev_dw.resize(w->last - w->first + 1);
+        for (auto &e : w->ev_dx) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        for (auto &e : w->ev_dw) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         w->aux.assign(w->last - w->first + 1, nullptr);
         w->aux_bytes.assign(w->last - w->first + 1, 0);
         long gx_elems = 0, bh_elems = 0;
