@@ -225,6 +225,12 @@ typedef struct {
 
 PD_API pd_status pd_get_stats(pd_ctx *ctx, pd_stats *out);
 
+/* Changes the instrumentation of later pd_run calls: record_trace as in pd_train_cfg;
+ * kernel_timing_mask bit c times every kernel of class c with CUDA events on its stream
+ * (0 forward GEMMs, 1 dX GEMMs, 2 dW GEMMs incl. the fused update, 3 bias / other); each timed
+ * launch costs two event records, so time only what is needed inside a timed region. */
+PD_API pd_status pd_set_timing(pd_ctx *ctx, int record_trace, int kernel_timing_mask);
+
 /* Releases everything the context owns.  Safe on NULL. */
 PD_API void pd_destroy(pd_ctx *ctx);
 

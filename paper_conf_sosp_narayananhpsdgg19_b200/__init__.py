@@ -108,6 +108,7 @@ def _load():
         "pd_get_losses": [vp, vp, st],
         "pd_get_stats": [vp, vp],
         "pd_inflight": [vp, i, vp],
+        "pd_set_timing": [vp, i, i],
         "pd_kernel_gemm": [vp, vp],
         "pd_kernel_softmax_ce": [i, vp, vp, C.c_long, i, vp, vp, vp],
     }
@@ -128,7 +129,8 @@ lib = _load()
 
 EXPORTED = ["pd_plan", "pd_create", "pd_stage_init", "pd_export_worker", "pd_import_worker", "pd_set_data", "pd_run",
             "pd_get_params", "pd_get_trace", "pd_get_version_map", "pd_get_losses", "pd_get_stats", "pd_destroy",
-            "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce"]
+            "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce",
+            "pd_set_timing"]
 
 
 def _strerror(s):
@@ -298,6 +300,10 @@ def pd_get_stats(ctx) -> dict:
             "kernel_launches": int(s.kernel_launches), "bytes_sent": int(s.bytes_sent), "num_local_workers": n,
             "worker_id": list(s.worker_id[:n]), "busy_ms": list(s.busy_ms[:n]), "span_ms": list(s.span_ms[:n]),
             "run_ms": s.run_ms, "kern_ms": list(s.kern_ms), "kern_count": [int(x) for x in s.kern_count]}
+
+
+def pd_set_timing(ctx, record_trace: int, kernel_timing_mask: int = 0xF):
+    _check(lib.pd_set_timing(ctx, record_trace, kernel_timing_mask), ctx)
 
 
 def pd_destroy(ctx):

@@ -23,6 +23,7 @@
 
 #include <cstdio>
 #include <cstdlib>
+#include <unordered_map>
 
 #include "pd_internal.h"
 
@@ -52,6 +53,13 @@ struct EpiArgs {
     ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
     int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
     int l2_prefetch;    // producer L2-prefetch distance in K-blocks (0 = off; measured no gain so far)
+    // in-kernel split-K: each (tile, split) writes its fp32 partial to ws[split]; the last CTA
+    // to finish a tile (per-tile counter) sums the partials in split order and applies the
+    // final epilogue (final_epi = EPI_STORE or EPI_MASK) -- no separate reduction launch
+    void *ws;               // final output (bf16) when reducing in-kernel
+    long split_stride_out;  // its row stride
+    int *counters;
+    int final_epi;
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
@@ -502,6 +510,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             EpiArgs es = e;
             if (EPI == EPI_F32) es.out = static_cast<float *>(e.out) + (long)split * e.split_stride;
             const bool empty_range = split * kper >= kblocks;  // (host avoids it; be safe)
+            const bool reduce = EPI == EPI_F32 && e.counters != nullptr;  // in-kernel split-K
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
                 float v[32];
@@ -520,6 +529,53 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 else mbar_arrive_cluster(smem_u32(&tempty[acc]) & 0xFEFFFFFFu);  // the leader's barrier
             }
             if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+            if (reduce) {
+                // publish this partial; the tile's last arriving split reduces all of them
+                __threadfence();
+                asm volatile("bar.sync 1, 128;" ::: "memory");
+                __shared__ int s_last;
+                const int cidx = tile * CG + (int)rank;
+                if (warp == 4 && lane == 0) {
+                    const int old = atomicAdd(e.counters + cidx, 1);
+                    s_last = (old == e.ksplit - 1);
+                    if (s_last) e.counters[cidx] = 0;  // ready for the next launch (stream order)
+                }
+                asm volatile("bar.sync 1, 128;" ::: "memory");
+                if (s_last) {
+                    __threadfence();
+                    EpiArgs ef = e;
+                    for (int c = 0; c < BN / 32; ++c) {
+                        const int col = n0 + c * 32;
+                        if (col >= N || row >= M) continue;
+                        float v[32];
+                        const float *p0 = static_cast<const float *>(e.out) + (long)row * e.ldo + col;
+                        const bool fullc = col + 32 <= N;
+                        for (int sp = 0; sp < e.ksplit; ++sp) {
+                            const float *p = p0 + (long)sp * e.split_stride;
+                            if (fullc) {
+#pragma unroll
+                                for (int q4 = 0; q4 < 8; ++q4) {
+                                    const float4 f = __ldcg(reinterpret_cast<const float4 *>(p) + q4);
+                                    if (sp == 0) {
+                                        v[q4 * 4] = f.x; v[q4 * 4 + 1] = f.y; v[q4 * 4 + 2] = f.z; v[q4 * 4 + 3] = f.w;
+                                    } else {
+                                        v[q4 * 4] += f.x; v[q4 * 4 + 1] += f.y; v[q4 * 4 + 2] += f.z; v[q4 * 4 + 3] += f.w;
+                                    }
+                                }
+                            } else {
+                                for (int i = 0; i < 32; ++i) {
+                                    const float f = (col + i < N) ? __ldcg(p + i) : 0.f;
+                                    v[i] = sp == 0 ? f : v[i] + f;
+                                }
+                            }
+                        }
+                        ef.out = e.ws;  // the final bf16 output
+                        ef.ldo = e.split_stride_out;
+                        if (e.final_epi == EPI_MASK) epilogue_chunk<EPI_MASK>(ef, v, row, col, M, N);
+                        else epilogue_chunk<EPI_STORE>(ef, v, row, col, M, N);
+                    }
+                }
+            }
         }
     }
     tc_fence_before();
@@ -800,8 +856,46 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 }
 
 // ---------------------------------------------------------------- host side
+struct MapKey {
+    const void *base;
+    long inner, outer, ld;
+    int bi, bo, f32, sw;
+    bool operator==(const MapKey &o) const {
+        return base == o.base && inner == o.inner && outer == o.outer && ld == o.ld && bi == o.bi && bo == o.bo &&
+               f32 == o.f32 && sw == o.sw;
+    }
+};
+struct MapKeyHash {
+    size_t operator()(const MapKey &k) const {
+        size_t h = std::hash<const void *>()(k.base);
+        for (long v : {k.inner, k.outer, k.ld, (long)k.bi, (long)k.bo, (long)(k.f32 * 1024 + k.sw)})
+            h = h * 1000003u ^ std::hash<long>()(v);
+        return h;
+    }
+};
+
+bool encode_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner,
+                int box_outer, bool f32, int swizzle_bytes);
+
+// Tensor maps are encoded once per (buffer, shape, box) and reused: encoding costs a driver
+// call on every launch otherwise, and the runtime's buffers are stable for a context's life.
 bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner, int box_outer,
               bool f32 = false, int swizzle_bytes = 128) {
+    thread_local std::unordered_map<MapKey, CUtensorMap, MapKeyHash> cache;
+    const MapKey key{base, inner, outer, ld_elems, box_inner, box_outer, (int)f32, swizzle_bytes};
+    auto it = cache.find(key);
+    if (it != cache.end()) {
+        *map = it->second;
+        return true;
+    }
+    if (!encode_map(map, base, inner, outer, ld_elems, box_inner, box_outer, f32, swizzle_bytes)) return false;
+    if (cache.size() > 65536) cache.clear();
+    cache.emplace(key, *map);
+    return true;
+}
+
+bool encode_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner,
+                int box_outer, bool f32, int swizzle_bytes) {
     const Driver *d = driver();
     if (!d) return false;
     cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
@@ -1027,10 +1121,21 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             e.ldo = g.N;
             e.ksplit = S;
             e.split_stride = (long)g.M * g.N;
+            const bool inkernel = g.split_counters != nullptr && env_int("PD_SPLIT_INKERNEL", 0);
+            if (inkernel) {
+                e.counters = g.split_counters;
+                e.ws = g.out;
+                e.split_stride_out = g.ldo;
+                e.final_epi = g.epi;
+                e.bias = g.epi == EPI_STORE ? g.bias : nullptr;
+                e.relu = g.epi == EPI_STORE ? g.relu : 0;
+                e.mask = g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr;
+                e.ldm = g.ldm;
+            }
             Gemm gf = g;
             gf.epi = EPI_F32;
             cudaError_t err = cg == 2 ? dispatch_major<256, 2>(gf, ma, mbm, e, s) : dispatch_major<256>(gf, ma, mbm, e, s);
-            if (err != cudaSuccess) return err;
+            if (err != cudaSuccess || inkernel) return err;
             const long total = (long)g.M * (g.N / 4);
             long blocks = (total + 255) / 256;
             if (blocks > 148L * 8) blocks = 148L * 8;

@@ -96,6 +96,7 @@ struct Gemm {
     ConvGeom conv;        // implicit-GEMM convolution (bf16 path only)
     int ksplit = 1;       // explicit split-K (EPI_F32 with atomic_out)
     int max_ctas = 0;     // cap on resident CTAs (0 = every SM): leaves SMs to a concurrent kernel
+    int *split_counters = nullptr;  // >= 8192 zeroed ints: split-K tiles reduce in-kernel (last CTA)
     int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
 };
 

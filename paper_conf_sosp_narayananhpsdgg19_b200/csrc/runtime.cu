@@ -200,6 +200,7 @@ struct pd_ctx {
     int last_M = 0;
     std::vector<int32_t> vmap;
     double host_ms = 0;
+    int ktime_mask = 0xF;            // kernel classes timed when record_trace >= 2
     std::atomic<bool> abort{false};
     std::mutex err_mu;
     pd_status sticky = PD_OK;
@@ -246,6 +247,7 @@ struct Worker {
     float *gbuf = nullptr;      // fp32 gradient (unreplicated fp32 path / biases)
     float *ws = nullptr;        // split-K partials of the bf16 GEMMs
     long ws_bytes = 0;
+    int *split_counters = nullptr;  // per-tile arrival counters of in-kernel split-K
     float *rgrad[2] = {};       // replicated stages: gradient per round parity
     const float **rgrad_ptrs = nullptr;  // device array [2][R]: peers' rgrad for each parity
     const float **self_grad_ptr = nullptr;  // device array [1]: gbuf
@@ -298,7 +300,7 @@ Worker::~Worker() {
     void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da};
     for (void *p : lb)
         if (p) cudaFree(p);
-    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
+    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, (void *)split_counters, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
     for (void *p : bufs)
         if (p) cudaFree(p);
@@ -439,6 +441,7 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.relu = d.act == PD_ACT_RELU;
     g.workspace = ws;
     g.workspace_bytes = ws_bytes;
+    g.split_counters = L.w->split_counters;
     CK(run_gemm(L.bf16, g, L.w->stream));
 }
 
@@ -486,14 +489,14 @@ struct Exec {
     }
 
     // per-kernel-class device time (0 fwd GEMM, 1 dX GEMM, 2 dW(+update) GEMM, 3 other)
-    cudaEvent_t kstart(int) {
-        if (!timing) return nullptr;
+    cudaEvent_t kstart(int cls) {
+        if (!timing || !((c->ktime_mask >> cls) & 1)) return nullptr;
         cudaEvent_t a = w->ev_pool[ev_used++];
         CK(cudaEventRecord(a, w->stream));
         return a;
     }
     void kend(int cls, cudaEvent_t a) {
-        if (!timing) return;
+        if (!a) return;
         cudaEvent_t b = w->ev_pool[ev_used++];
         CK(cudaEventRecord(b, w->stream));
         w->kev[cls].push_back({a, b});
@@ -625,6 +628,7 @@ struct Exec {
         g.ldm = N;
         g.workspace = w->ws;
         g.workspace_bytes = w->ws_bytes;
+        g.split_counters = w->split_counters;
         CK(run_gemm(bf16, g, w->stream));
     }
 
@@ -1464,6 +1468,7 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         if (bf16) {
             w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
             w->ws = dalloc<float>(w->ws_bytes);
+            w->split_counters = dalloc<int>(8192 * sizeof(int));
         }
         if (stage > 0) w->recv = dalloc<void>((size_t)w->D * dev_in_elems(c->layers, w->first, B) * esz);
         if (stage + 1 < c->n) w->gring = dalloc<void>((size_t)w->G * dev_out_elems(c->layers, w->last, B) * esz);
@@ -1887,6 +1892,14 @@ pd_status pd_get_stats(pd_ctx *c, pd_stats *out) {
     return PD_OK;
 }
 
+pd_status pd_set_timing(pd_ctx *c, int record_trace, int mask) {
+    CHECK_CTX(c);
+    if (record_trace < 0 || record_trace > 2) return PD_EINVAL;
+    c->cfg.record_trace = record_trace;
+    c->ktime_mask = mask & 0xF;
+    return PD_OK;
+}
+
 void pd_destroy(pd_ctx *c) {
     if (!c) return;
     for (auto &w : c->W)
@@ -1928,6 +1941,13 @@ extern "C" PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *d, void *stream) 
     g.master = d->master; g.slot = d->slot; g.adam_m = d->adam_m; g.adam_v = d->adam_v;
     g.lr = d->lr; g.b1 = d->beta1; g.b2 = d->beta2; g.eps = d->eps; g.step = d->step;
     g.workspace = d->workspace; g.workspace_bytes = d->workspace_bytes;
+    static int *counters = nullptr;  // kernel-level API: one zeroed counter array per process
+    if (d->dtype == PD_BF16 && d->workspace && !counters) {
+        if (cudaMalloc(&counters, 8192 * sizeof(int)) != cudaSuccess || cudaMemset(counters, 0, 8192 * sizeof(int)) != cudaSuccess ||
+            cudaDeviceSynchronize() != cudaSuccess)
+            return PD_ECUDA;
+    }
+    g.split_counters = counters;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     cudaError_t e = d->dtype == PD_BF16 ? gemm_bf16(g, s) : gemm_f32(g, s);
     if (e == cudaErrorInvalidValue) return PD_EINVAL;

@@ -8,7 +8,8 @@ from typing import Callable, Dict, List, Optional, Sequence
 import numpy as np
 
 from . import (PD_BF16, PD_SGD, Plan, pd_create, pd_destroy, pd_export_worker, pd_get_losses, pd_get_params,
-               pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data, pd_stage_init, pd_run)
+               pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data, pd_set_timing,
+               pd_stage_init, pd_run)
 
 
 def workers_of(plan: Plan):
@@ -74,6 +75,9 @@ class Pipeline:
 
     def stats(self):
         return pd_get_stats(self.ctx)
+
+    def set_timing(self, record_trace, kernel_timing_mask=0xF):
+        pd_set_timing(self.ctx, record_trace, kernel_timing_mask)
 
     def close(self):
         if self.ctx is not None:
