@@ -270,6 +270,9 @@ struct Worker {
     // (layer, direction, saved-state slot, weight slot, dY pointer): replayed instead of
     // re-issuing ~3T launches per layer
     std::map<std::tuple<int, int, int, int, const void *>, std::pair<cudaGraphExec_t, int>> graphs;
+    // whole-op graphs (F / B of an all-linear bf16 SGD stage), keyed by every pointer the op uses
+    std::map<std::vector<uintptr_t>, std::pair<cudaGraphExec_t, int>> opgraphs;
+    float *loss_scratch = nullptr;  // CE writes here inside a graph; copied to losses[t] after
     float *stage_in = nullptr;   // fp32 upload staging for pd_set_data (bf16 path)
     long stage_in_elems = 0;
     float *losses = nullptr;     // last stage, per minibatch of the run
@@ -308,6 +311,8 @@ Worker::~Worker() {
     for (cudaEvent_t e : run_ev)
         if (e) cudaEventDestroy(e);
     for (auto &kv : graphs) cudaGraphExecDestroy(kv.second.first);
+    for (auto &kv : opgraphs) cudaGraphExecDestroy(kv.second.first);
+    if (loss_scratch) cudaFree(loss_scratch);
     for (cudaEvent_t e : ev_dx) cudaEventDestroy(e);
     for (cudaEvent_t e : ev_dw) cudaEventDestroy(e);
     if (side) cudaStreamDestroy(side);
@@ -489,8 +494,9 @@ struct Exec {
     }
 
     // per-kernel-class device time (0 fwd GEMM, 1 dX GEMM, 2 dW(+update) GEMM, 3 other)
+    bool capturing = false;
     cudaEvent_t kstart(int cls) {
-        if (!timing || !((c->ktime_mask >> cls) & 1)) return nullptr;
+        if (capturing || !timing || !((c->ktime_mask >> cls) & 1)) return nullptr;
         cudaEvent_t a = w->ev_pool[ev_used++];
         CK(cudaEventRecord(a, w->stream));
         return a;
@@ -544,22 +550,24 @@ struct Exec {
         if (c->cfg.record_trace) c->vmap[(long)s * M + t] = v;
         trace('F', t, v, v);
         record_start();
+        void *y_last = w->logits;
+        if (s + 1 < n()) {
+            const int Rn = c->plan.stage[s + 1].replicas;
+            const int cw = c->worker_id(s + 1, t % Rn);
+            const int jc = t / Rn;
+            y_last = elem_ptr(c->shared[cw].recv, (long)(jc % c->Dalloc[s + 1]) * dev_out_elems(c->layers, w->last, B()),
+                              esz);
+            w->bytes_sent += (uint64_t)dev_out_elems(c->layers, w->last, B()) * esz;
+        }
+        const long lrows = rows_of(layer(w->last), B());
+        const int32_t *labels = (s + 1 == n()) ? w->labels + (long)(t % c->n_data) * lrows : nullptr;
+        auto body = [&](float *loss_dst) {
         for (int l = w->first; l <= w->last; ++l) {
             const pd_layer_desc &d = layer(l);
             const void *x = layer_input(l, t, j);
-            void *y;
-            if (l < w->last) {
-                y = elem_ptr(w->act[l + 1 - w->first], (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz);
-            } else if (s + 1 < n()) {
-                const int Rn = c->plan.stage[s + 1].replicas;
-                const int cw = c->worker_id(s + 1, t % Rn);
-                const int jc = t / Rn;
-                const Shared &sh = c->shared[cw];
-                y = elem_ptr(sh.recv, (long)(jc % c->Dalloc[s + 1]) * dev_out_elems(c->layers, l, B()), esz);
-                w->bytes_sent += (uint64_t)dev_out_elems(c->layers, l, B()) * esz;
-            } else {
-                y = w->logits;
-            }
+            void *y = l < w->last ? elem_ptr(w->act[l + 1 - w->first],
+                                             (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz)
+                                  : y_last;
             cudaEvent_t k0 = kstart(0);
             if (d.kind == PD_LINEAR) {
                 LayerCtx lc{c, w, bf16};
@@ -580,10 +588,21 @@ struct Exec {
             kend(0, k0);
         }
         if (s + 1 == n()) {
-            const pd_layer_desc &d = layer(w->last);
-            const long rows = rows_of(d, B());
-            CK(softmax_ce(w->logits, bf16, w->labels + (long)(t % c->n_data) * rows, rows, d.out, w->dlogits,
-                          w->losses + t, w->stream));
+            if (loss_dst == w->loss_scratch) CK(cudaMemsetAsync(loss_dst, 0, 4, w->stream));
+            CK(softmax_ce(w->logits, bf16, labels, lrows, layer(w->last).out, w->dlogits, loss_dst, w->stream));
+        }
+        };
+        if (op_graphs_ok()) {
+            const std::vector<uintptr_t> key = {0, (uintptr_t)slot, (uintptr_t)(j % w->k),
+                                                (uintptr_t)layer_input(w->first, t, j), (uintptr_t)y_last,
+                                                (uintptr_t)labels};
+            opgraph_run(key, [&] { body(w->loss_scratch); });
+            if (s + 1 == n())
+                CK(cudaMemcpyAsync(w->losses + t, w->loss_scratch, 4, cudaMemcpyDeviceToDevice, w->stream));
+        } else {
+            body(w->losses + t);
+        }
+        if (s + 1 == n()) {
         } else {
             const int Rn = c->plan.stage[s + 1].replicas;
             Link &L = get_link(c, L_ACT, w->id, c->worker_id(s + 1, t % Rn));
@@ -746,6 +765,55 @@ struct Exec {
         }
         CK(cudaGraphLaunch(it->second.first, w->stream));
         tl_launches += it->second.second;  // count the kernels the graph runs
+    }
+
+    template <typename F>
+    void opgraph_run(const std::vector<uintptr_t> &key, F body) {
+        auto it = w->opgraphs.find(key);
+        if (it == w->opgraphs.end()) {
+            const uint64_t before = tl_launches;
+            capturing = true;
+            CK(cudaStreamBeginCapture(w->stream, cudaStreamCaptureModeRelaxed));
+            try {
+                body();
+            } catch (...) {
+                cudaGraph_t g = nullptr;
+                cudaStreamEndCapture(w->stream, &g);
+                if (g) cudaGraphDestroy(g);
+                capturing = false;
+                throw;
+            }
+            cudaGraph_t g;
+            CK(cudaStreamEndCapture(w->stream, &g));
+            capturing = false;
+            cudaGraphExec_t ex;
+            CK(cudaGraphInstantiate(&ex, g, 0));
+            CK(cudaGraphDestroy(g));
+            const int nk = (int)(tl_launches - before);
+            tl_launches = before;
+            if (w->opgraphs.size() > 4096) {
+                for (auto &kv : w->opgraphs) cudaGraphExecDestroy(kv.second.first);
+                w->opgraphs.clear();
+            }
+            it = w->opgraphs.emplace(key, std::make_pair(ex, nk)).first;
+        }
+        CK(cudaGraphLaunch(it->second.first, w->stream));
+        tl_launches += it->second.second;
+    }
+
+    // whole-op graphs: bf16 fused all-linear SGD stages (the launch-bound MLP path), and only
+    // when no per-kernel timing is requested (event timing cannot live inside a graph)
+    bool op_graphs_ok() const {
+        static const int env = [] {
+            const char *e = getenv("PD_OP_GRAPHS");
+            return e ? atoi(e) : 1;
+        }();
+        if (!env || !bf16 || c->cfg.optimizer != PD_SGD) return false;
+        if (c->plan.stage[w->stage].replicas != 1) return false;
+        if (timing && c->ktime_mask) return false;
+        for (int l = w->first; l <= w->last; ++l)
+            if (layer(l).kind != PD_LINEAR) return false;
+        return true;
     }
 
     void lstm_forward(int l, int j, int slot, const void *x, void *y) {
@@ -1006,7 +1074,7 @@ struct Exec {
     // GEMM of layer l-1 (L2/latency-bound) on the main stream.  Hazards: dW_l rewrites W_l
     // (k_s = 1: in place) so it waits for dX_l; dX_{l-2} reuses dW_l's input buffer G_l, so it
     // waits for dW_l (3-deep rotation of the gradient scratch).
-    void backward_linear_overlapped(int t, int j, const void *G_ext, const BwdCtx &bc) {
+    void backward_linear_overlapped(int t, int j, const void *G_ext, const BwdCtx &bc, const void *dx_first) {
         const int s = w->stage;
         const int first = w->first, last = w->last;
         auto Gof = [&](int l) -> const void * {
@@ -1021,12 +1089,7 @@ struct Exec {
             if (need_dx) {
                 void *dx;
                 if (l == first) {
-                    const int Rp = c->plan.stage[s - 1].replicas;
-                    const int pw = c->worker_id(s - 1, t % Rp);
-                    const int jp = t / Rp;
-                    dx = elem_ptr(c->shared[pw].grad, (long)(jp % c->Galloc[s - 1]) * dev_in_elems(c->layers, l, B()),
-                                  esz);
-                    w->bytes_sent += (uint64_t)dev_in_elems(c->layers, l, B()) * esz;
+                    dx = const_cast<void *>(dx_first);
                 } else {
                     dx = w->scratch[(last - l) % 3];
                     if (l + 2 <= last) CK(cudaStreamWaitEvent(w->stream, w->ev_dw[l + 2 - first], 0));
@@ -1113,7 +1176,22 @@ struct Exec {
         bool all_linear = true;
         for (int l = w->first; l <= w->last; ++l) all_linear = all_linear && layer(l).kind == PD_LINEAR;
         if (fused && all_linear && concurrent_dw()) {
-            backward_linear_overlapped(t, j, G, bc);
+            const void *dx_first = nullptr;
+            if (!(s == 0 && w->first == 0)) {
+                const int Rp = c->plan.stage[s - 1].replicas;
+                const int pw = c->worker_id(s - 1, t % Rp);
+                dx_first = elem_ptr(c->shared[pw].grad,
+                                    (long)((t / Rp) % c->Galloc[s - 1]) * dev_in_elems(c->layers, w->first, B()), esz);
+                w->bytes_sent += (uint64_t)dev_in_elems(c->layers, w->first, B()) * esz;
+            }
+            if (op_graphs_ok()) {
+                const std::vector<uintptr_t> key = {1, (uintptr_t)sslot, (uintptr_t)nslot, (uintptr_t)(j % w->k),
+                                                    (uintptr_t)G, (uintptr_t)layer_input(w->first, t, j),
+                                                    (uintptr_t)dx_first};
+                opgraph_run(key, [&] { backward_linear_overlapped(t, j, G, bc, dx_first); });
+            } else {
+                backward_linear_overlapped(t, j, G, bc, dx_first);
+            }
         } else
         for (int l = w->last; l >= w->first; --l) {
             const pd_layer_desc &d = layer(l);
@@ -1469,6 +1547,7 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
             w->ws = dalloc<float>(w->ws_bytes);
             w->split_counters = dalloc<int>(8192 * sizeof(int));
+            w->loss_scratch = dalloc<float>(256);
         }
         if (stage > 0) w->recv = dalloc<void>((size_t)w->D * dev_in_elems(c->layers, w->first, B) * esz);
         if (stage + 1 < c->n) w->gring = dalloc<void>((size_t)w->G * dev_out_elems(c->layers, w->last, B) * esz);
