@@ -453,6 +453,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     }
                     if (BMAJ == KMAJ) {
                         tma_load_2d_cg<CG>(sb, &tmB, fb, kbk, nb);  // box {64 K, BN/CG N}
+                    } else if (e.conv.b_tapchunk) {
+                        // implicit im2col on B: column chunk (tap, 64 channels) = X rows shifted by the tap
+                        const int Cp = e.conv.b_tapchunk;
+#pragma unroll
+                        for (int j = 0; j < BNC / 64; ++j) {
+                            const int col = nb + 64 * j, tap = col / Cp;
+                            if (tap < 9) tma_load_2d_cg<CG>(sb + j * BK * 128, &tmB, fb, col % Cp, kbk + e.conv.a_shift[tap]);
+                            else tma_load_2d_cg<CG>(sb + j * BK * 128, &tmB, fb, Cp, kbk);  // past N: zero fill
+                        }
                     } else {
 #pragma unroll
                         for (int j = 0; j < BNC / 64; ++j)
@@ -1174,7 +1183,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, aK, g.M, g.lda, 64, BM)
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
     const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, bK, g.N, g.ldb, 64, BN / cg)
-                                    : make_map(&mbm, g.B, bN, bKo, g.ldb, 64, BK);
+                                    : make_map(&mbm, g.B, g.conv.b_tapchunk ? g.conv.b_tapchunk : bN, bKo, g.ldb, 64, BK);
     if (!okA || !okB) return cudaErrorInvalidValue;
     EpiArgs e{};
     e.conv = g.conv;

@@ -62,6 +62,8 @@ struct ConvGeom {
     int b_noff = 0;        // B N-coordinate offset per tap (dX, MN-major weights)
     int b_kshift = 0;      // constant B K-coordinate shift (per-tap dW launch)
     int Hp = 0, Wp = 0;    // padded grid of the OUTPUT rows (epilogue zeroes borders); 0 = off
+    int b_tapchunk = 0;    // dW over all 9 taps in one GEMM: B column n = tap*Cp + ci, each 64-column
+                           // chunk reads X shifted by a_shift[tap] (value = Cp, multiple of 64; 0 = off)
     int a_inner = 0;       // inner extents of the A / B tensors for the TMA maps (taps > 0)
     int b_inner = 0;
 };

@@ -930,6 +930,14 @@ struct Exec {
         return g;
     }
 
+    static bool tapchunk_dw() {
+        static const int v = [] {
+            const char *e = getenv("PD_CONV_DW_ONEGEMM");
+            return e ? atoi(e) : 1;
+        }();
+        return v != 0;
+    }
+
     void conv_forward(int l, int slot, const void *x, void *y) {
         const pd_layer_desc &d = layer(l);
         const int Cp = cpad8(d.in), Co = d.out, Hp = d.height + 2, Wp = d.width + 2;
@@ -1006,6 +1014,27 @@ struct Exec {
         if (!bf16) {
             CK(conv_dw_f32(static_cast<const float *>(G), static_cast<const float *>(x), gW, B(), d.height, d.width,
                            Cp, Co, w->stream));
+        } else if (Cp % 64 == 0 && tapchunk_dw()) {
+            // dW[co][tap*Cp + ci] for all 9 taps in ONE GEMM (N = 9*Cp): the dY tile is loaded
+            // once per K-block for every tap of the tile instead of once per tap
+            Gemm g;
+            g.M = Co;
+            g.N = 9 * Cp;
+            g.K = (int)M;
+            g.A = G;
+            g.lda = Co;
+            g.amaj = MNMAJ;
+            g.B = x;
+            g.ldb = Cp;
+            g.bmaj = MNMAJ;
+            g.conv.b_tapchunk = Cp;
+            for (int tap = 0; tap < 9; ++tap) g.conv.a_shift[tap] = ((tap / 3) - 1) * Wp + (tap % 3) - 1;
+            g.epi = EPI_F32;
+            g.atomic_out = 1;
+            g.ksplit = 0;
+            g.out = gW;
+            g.ldo = 9L * Cp;
+            CK(run_gemm(1, g, w->stream));
         } else {
             const int Wpp = Wp;
             for (int tap = 0; tap < 9; ++tap) {
