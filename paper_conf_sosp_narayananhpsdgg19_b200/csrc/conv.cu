@@ -9,6 +9,8 @@
 // path's direct convolution kernels.
 #include <cuda_bf16.h>
 
+#include <algorithm>
+
 #include "pd_internal.h"
 
 namespace pd {
@@ -129,6 +131,33 @@ __global__ void __launch_bounds__(256) col_sum_tall_kernel(const T *__restrict__
     }
 }
 
+// bf16, cols % 8 == 0, cols <= 2048: thread = 8 consecutive columns (one 16-byte load) of
+// every (256 / (cols/8))-th row of the block's chunk; per-column partials reduced in smem
+__global__ void __launch_bounds__(256) col_sum_tall8_kernel(const __nv_bfloat16 *__restrict__ G, long rows,
+                                                            int cols, long rows_per_block, float *out) {
+    extern __shared__ float red[];  // [256][8]
+    const int tpr = cols / 8, rpp = 256 / tpr;  // threads per row, rows per pass
+    const int t = threadIdx.x, cg = t % tpr, rr = t / tpr;
+    const long r0 = (long)blockIdx.x * rows_per_block, r1 = min(rows, r0 + rows_per_block);
+    float a[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+    if (rr < rpp)
+        for (long r = r0 + rr; r < r1; r += rpp) {
+            const uint4 q = *reinterpret_cast<const uint4 *>(G + r * cols + cg * 8);
+            const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&q);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) a[i] += __bfloat162float(h[i]);
+        }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) red[t * 8 + i] = a[i];
+    __syncthreads();
+    for (int c = t; c < cols; c += 256) {
+        const int g = c / 8, i = c % 8;
+        float sum = 0.f;
+        for (int q = 0; q < rpp; ++q) sum += red[(q * tpr + g) * 8 + i];
+        atomicAdd(out + c, sum);
+    }
+}
+
 // ---------------- fp32 parity path: direct convolutions on the padded layout
 // W_dev [Cout][9][Cp] (tap = kh*3 + kw), bias [Cout]
 __global__ void conv_fwd_direct_kernel(const float *__restrict__ x, const float *__restrict__ Wd,
@@ -201,6 +230,97 @@ __global__ void conv_dw_direct_kernel(const float *__restrict__ dy, const float 
     }
 }
 
+// 8-channel vectorised variants (bf16, C % 8 == 0): one thread = one pooling window x 8
+// channels; fwd reads the 4 inputs once, bwd writes all 4 input gradients (no re-reads)
+__device__ __forceinline__ void ld8(const __nv_bfloat16 *p, float (&v)[8]) {
+    const uint4 r = *reinterpret_cast<const uint4 *>(p);
+    const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&r);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = __bfloat162float(h[i]);
+}
+__device__ __forceinline__ void st8(__nv_bfloat16 *p, const float (&v)[8]) {
+    uint4 r;
+    __nv_bfloat16 *h = reinterpret_cast<__nv_bfloat16 *>(&r);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) h[i] = __float2bfloat16_rn(v[i]);
+    *reinterpret_cast<uint4 *>(p) = r;
+}
+
+__global__ void pool_fwd8_kernel(const __nv_bfloat16 *__restrict__ x, __nv_bfloat16 *__restrict__ y, int B, int H,
+                                 int W, int C, int out_padded) {
+    const int Ho = H / 2, Wo = W / 2, Hp = H + 2, Wp = W + 2, C8 = C / 8;
+    const int Hq = out_padded ? Ho + 2 : Ho, Wq = out_padded ? Wo + 2 : Wo, off = out_padded ? 1 : 0;
+    const long n = (long)B * Hq * Wq * C8;
+    GRID_STRIDE(i, n) {
+        const int c8 = (int)(i % C8);
+        const long p = i / C8;
+        const int wq = (int)(p % Wq), hq = (int)((p / Wq) % Hq), b = (int)(p / ((long)Wq * Hq));
+        const int ho = hq - off, wo = wq - off;
+        float best[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+        if (ho >= 0 && ho < Ho && wo >= 0 && wo < Wo) {
+            for (int dh = 0; dh < 2; ++dh)
+                for (int dw = 0; dw < 2; ++dw) {
+                    float v[8];
+                    ld8(x + (((long)b * Hp + 2 * ho + dh + 1) * Wp + 2 * wo + dw + 1) * C + c8 * 8, v);
+#pragma unroll
+                    for (int k = 0; k < 8; ++k)
+                        if ((dh | dw) == 0 || v[k] > best[k]) best[k] = v[k];
+                }
+        }
+        st8(y + p * C + c8 * 8, best);
+    }
+}
+
+// one thread per input 2x2 window (and the halo pixels, written as 0)
+__global__ void pool_bwd8_kernel(const __nv_bfloat16 *__restrict__ x, const __nv_bfloat16 *__restrict__ dy,
+                                 __nv_bfloat16 *__restrict__ dx, int B, int H, int W, int C, int dy_padded,
+                                 int mask_relu) {
+    const int Ho = H / 2, Wo = W / 2, Hp = H + 2, Wp = W + 2, C8 = C / 8;
+    const int Hq = dy_padded ? Ho + 2 : Ho, Wq = dy_padded ? Wo + 2 : Wo, off = dy_padded ? 1 : 0;
+    const long nwin = (long)B * Ho * Wo * C8;
+    GRID_STRIDE(i, nwin) {
+        const int c8 = (int)(i % C8);
+        const long p = i / C8;
+        const int wo = (int)(p % Wo), ho = (int)((p / Wo) % Ho), b = (int)(p / ((long)Wo * Ho));
+        float v[4][8];
+        long idx[4];
+        for (int q = 0; q < 4; ++q) {
+            idx[q] = (((long)b * Hp + 2 * ho + (q >> 1) + 1) * Wp + 2 * wo + (q & 1) + 1) * C + c8 * 8;
+            ld8(x + idx[q], v[q]);
+        }
+        float g[8];
+        ld8(dy + (((long)b * Hq + ho + off) * Wq + wo + off) * C + c8 * 8, g);
+        float o[4][8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            int arg = 0;
+            float best = v[0][k];
+            for (int q = 1; q < 4; ++q)
+                if (v[q][k] > best) { best = v[q][k]; arg = q; }
+            for (int q = 0; q < 4; ++q) {
+                float gv = q == arg ? g[k] : 0.f;
+                if (mask_relu && !(v[q][k] > 0.f)) gv = 0.f;
+                o[q][k] = gv;
+            }
+        }
+        for (int q = 0; q < 4; ++q) st8(dx + idx[q], o[q]);
+    }
+    // halo of dx (and the odd last row/column when H or W is odd: not supported by pd_create)
+    const long nh = (long)B * (2 * Wp + 2 * H) * C8;
+    GRID_STRIDE(i, nh) {
+        const int c8 = (int)(i % C8);
+        const long p = i / C8;
+        const int per = 2 * Wp + 2 * H, b = (int)(p / per), e = (int)(p % per);
+        int hp, wp;
+        if (e < Wp) { hp = 0; wp = e; }
+        else if (e < 2 * Wp) { hp = Hp - 1; wp = e - Wp; }
+        else if (e < 2 * Wp + H) { hp = e - 2 * Wp + 1; wp = 0; }
+        else { hp = e - 2 * Wp - H + 1; wp = Wp - 1; }
+        const float z[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+        st8(dx + (((long)b * Hp + hp) * Wp + wp) * C + c8 * 8, z);
+    }
+}
+
 }  // namespace
 
 cudaError_t pad_nhwc(const float *in, void *out, int bf16, int B, int H, int W, int C, int Cp, cudaStream_t s) {
@@ -213,7 +333,10 @@ cudaError_t pad_nhwc(const float *in, void *out, int bf16, int B, int H, int W, 
 
 cudaError_t pool_fwd(int bf16, const void *x, void *y, int B, int H, int W, int C, int out_padded, cudaStream_t s) {
     const long n = (long)B * (out_padded ? H / 2 + 2 : H / 2) * (out_padded ? W / 2 + 2 : W / 2) * C;
-    if (bf16)
+    if (bf16 && C % 8 == 0) {
+        pool_fwd8_kernel<<<blocks_for(n / 8), 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(x),
+                                                           static_cast<__nv_bfloat16 *>(y), B, H, W, C, out_padded);
+    } else if (bf16)
         pool_fwd_kernel<<<blocks_for(n), 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(x),
                                                       static_cast<__nv_bfloat16 *>(y), B, H, W, C, out_padded);
     else
@@ -226,7 +349,11 @@ cudaError_t pool_fwd(int bf16, const void *x, void *y, int B, int H, int W, int 
 cudaError_t pool_bwd(int bf16, const void *x, const void *dy, void *dx, int B, int H, int W, int C, int dy_padded,
                      int mask_relu, cudaStream_t s) {
     const long n = (long)B * (H + 2) * (W + 2) * C;
-    if (bf16)
+    if (bf16 && C % 8 == 0) {
+        pool_bwd8_kernel<<<blocks_for((long)B * (H / 2) * (W / 2) * (C / 8)), 256, 0, s>>>(
+            static_cast<const __nv_bfloat16 *>(x), static_cast<const __nv_bfloat16 *>(dy),
+            static_cast<__nv_bfloat16 *>(dx), B, H, W, C, dy_padded, mask_relu);
+    } else if (bf16)
         pool_bwd_kernel<<<blocks_for(n), 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(x),
                                                       static_cast<const __nv_bfloat16 *>(dy),
                                                       static_cast<__nv_bfloat16 *>(dx), B, H, W, C, dy_padded,
@@ -239,6 +366,15 @@ cudaError_t pool_bwd(int bf16, const void *x, const void *dy, void *dx, int B, i
 }
 
 cudaError_t col_sum_tall(const void *G, int bf16, long rows, int cols, float *out, cudaStream_t s) {
+    if (bf16 && cols % 8 == 0 && cols <= 2048) {
+        // ~8 blocks per SM, each reducing a contiguous row chunk
+        const long nb = std::max(1L, std::min((rows + 63) / 64, 148L * 8));
+        const long rpb8 = (rows + nb - 1) / nb;
+        col_sum_tall8_kernel<<<(unsigned)((rows + rpb8 - 1) / rpb8), 256, 256 * 8 * sizeof(float), s>>>(
+            static_cast<const __nv_bfloat16 *>(G), rows, cols, rpb8, out);
+        ++tl_launches;
+        return cudaGetLastError();
+    }
     long rpb = 2048;
     long ychunks = (rows + rpb - 1) / rpb;
     if (ychunks > 1024) {

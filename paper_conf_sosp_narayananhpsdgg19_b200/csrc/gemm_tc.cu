@@ -192,6 +192,16 @@ __device__ __forceinline__ uint64_t smem_desc(uint32_t addr, uint32_t lbo, uint3
     return d;
 }
 
+// unswizzled (interleaved core-matrix) layout: 8 rows x 16 B core matrices
+__device__ __forceinline__ uint64_t smem_desc_ns(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+    uint64_t d = 0;
+    d |= (uint64_t)((addr >> 4) & 0x3FFF);
+    d |= (uint64_t)((lbo >> 4) & 0x3FFF) << 16;
+    d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;
+    d |= (uint64_t)1 << 46;
+    return d;
+}
+
 // Instruction descriptor for kind::f16: D fp32 (bits 4-5 = 1), A bf16 (7-9 = 1), B bf16
 // (10-12 = 1), A major (bit 15), B major (bit 16), N >> 3 (17-22), M >> 4 (24-28).
 __host__ __device__ constexpr uint32_t make_idesc(int M, int N, int amaj, int bmaj) {
@@ -387,6 +397,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
         }
     }
+    if (e.conv.c8 == 1) {
+        // packed-tap forward: A slot 9 (K 72..79) is never loaded; it meets zero weights,
+        // so it only has to be finite -- zero it once
+        for (int s = 0; s < C::STAGES; ++s)
+            for (int i = threadIdx.x; i < 2048 / 16; i += NUM_THREADS)
+                reinterpret_cast<uint4 *>(smem + s * C::STAGE_BYTES + 9 * 2048)[i] = make_uint4(0, 0, 0, 0);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
     tc_fence_before();
     if (CG == 2) {
         asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
@@ -437,9 +455,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
                     // CG = 2: both CTAs' bytes land on the LEADER's full barrier (peer bit cleared)
                     const uint32_t fb = smem_u32(&full[stage]) & (CG == 2 ? 0xFEFFFFFFu : 0xFFFFFFFFu);
-                    if (rank == 0) mbar_expect_tx(fb, CG * C::STAGE_BYTES);
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
                     const uint32_t sb = sa + C::A_BYTES;
+                    if (CG == 1 && e.conv.c8 == 1) {
+                        // packed-tap forward: A slot t = X rows shifted by tap t (2 KB each),
+                        // B slot j = W[:, 8j .. 8j+7] (slot 9 past K = 72: zero fill)
+                        mbar_expect_tx(fb, 9 * 2048 + 10 * BN / 2 * 16);
+                        for (int t = 0; t < 9; ++t) tma_load_2d(sa + t * 2048, &tmA, fb, 0, m0 + e.conv.a_shift[t]);
+                        for (int j = 0; j < 10; ++j) tma_load_2d(sa + 20480 + j * (BN / 2) * 16, &tmB, fb, 8 * j, n0);
+                        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                        continue;
+                    }
+                    if (CG == 1 && e.conv.c8 == 2) {
+                        // packed-tap dW: B slot t = 64 pixels of X shifted by tap t, 8 channels
+                        const int k0 = kb * BK;
+                        mbar_expect_tx(fb, C::A_BYTES + 9 * 1024);
+#pragma unroll
+                        for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * BK * 128, &tmA, fb, m0 + 64 * j, k0);
+                        for (int t = 0; t < 9; ++t) tma_load_2d(sb + t * 1024, &tmB, fb, 0, k0 + e.conv.a_shift[t]);
+                        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                        continue;
+                    }
+                    if (rank == 0) mbar_expect_tx(fb, CG * C::STAGE_BYTES);
                     // implicit-GEMM convolution: K-block kb = (tap, 64-channel block); the A rows
                     // (padded-grid pixels) shift by the tap's offset, B moves to the tap's slice
                     int ka, ma, kbk, nb;
@@ -490,6 +527,31 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     tc_fence_after();
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
                     const uint32_t sb = sa + C::A_BYTES;
+                    if (CG == 1 && e.conv.c8 == 1) {
+                        // K = 80 in 5 steps; each step's two 8-wide K chunks are 2 slots apart
+                        constexpr uint32_t id64 = make_idesc(BM, BN / 2, KMAJ, KMAJ);
+                        for (int k = 0; k < 5; ++k) {
+                            const uint64_t ad = smem_desc_ns(sa + k * 4096, 2048, 128);
+                            const uint64_t bd = smem_desc_ns(sa + 20480 + k * 2 * (BN / 2) * 16, (BN / 2) * 16, 128);
+                            tc_mma(d, ad, bd, id64, k > 0 ? 1u : 0u);
+                        }
+                        tc_commit(smem_u32(&empty[stage]));
+                        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                        continue;
+                    }
+                    if (CG == 1 && e.conv.c8 == 2) {
+                        // N = 80 (72 used): B is MN-major unswizzled, 8-pixel K groups 128 B apart,
+                        // 8-channel N groups (taps) 1 KB apart
+                        constexpr uint32_t id80 = make_idesc(BM, 80, MNMAJ, MNMAJ);
+                        for (int k = 0; k < BK / UMMA_K; ++k) {
+                            const uint64_t ad = smem_desc(sa + k * 2048, BK * 128, 1024);
+                            const uint64_t bd = smem_desc_ns(sb + k * 256, 128, 1024);
+                            tc_mma(d, ad, bd, id80, (kb > kb0 || k > 0) ? 1u : 0u);
+                        }
+                        tc_commit(smem_u32(&empty[stage]));
+                        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+                        continue;
+                    }
 #pragma unroll
                     for (int k = 0; k < BK / UMMA_K; ++k) {
                         const uint64_t ad = AMAJ == KMAJ ? smem_desc(sa + k * 32, 16, 1024)
@@ -914,7 +976,9 @@ bool encode_map(CUtensorMap *map, const void *base, long inner, long outer, long
     CUresult r = d->tensorMapEncodeTiled(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
                                          2, const_cast<void *>(base), dims,
                                          strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                                         swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                                         swizzle_bytes == 64    ? CU_TENSOR_MAP_SWIZZLE_64B
+                                         : swizzle_bytes == 0 ? CU_TENSOR_MAP_SWIZZLE_NONE
+                                                              : CU_TENSOR_MAP_SWIZZLE_128B,
                                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
@@ -1091,7 +1155,8 @@ static int env_int(const char *name, int dflt) {
 // 2-CTA pairs (M = 256 per MMA) for every plain GEMM with at least 256 rows
 static int use_pairs(const Gemm &g) {
     if (env_int("PD_GEMM_CG", 2) == 1) return 1;
-    return (g.M >= 256 && (g.epi == EPI_STORE || g.epi == EPI_MASK || g.epi == EPI_F32)) ? 2 : 1;
+    // N <= 64 would leave the second CTA's half of B empty (zero columns): single CTAs there
+    return (g.M >= 256 && g.N > 64 && (g.epi == EPI_STORE || g.epi == EPI_MASK || g.epi == EPI_F32)) ? 2 : 1;
 }
 
 static int choose_ksplit(const Gemm &g, int sms) {
@@ -1110,6 +1175,44 @@ static int choose_ksplit(const Gemm &g, int sms) {
     while (S > 1 && (long)S * g.M * g.N * 4 > g.workspace_bytes) --S;
     const int kper = (kblocks + S - 1) / S;
     return (kblocks + kper - 1) / kper;  // no empty K range
+}
+
+// packed-tap convolution GEMMs for Cp = 8 inputs (ConvGeom::c8); single CTAs, BN = 128
+// template (ring stages of 32 KB hold the 20 KB A + 10 KB B packed K-block)
+static cudaError_t gemm_c8(const Gemm &g, cudaStream_t s) {
+    CUtensorMap ma, mbm;
+    EpiArgs e{};
+    e.conv = g.conv;
+    e.out = g.out;
+    e.ldo = g.ldo;
+    e.bias = g.bias;
+    e.relu = g.relu;
+    e.ksplit = 1;
+    if (g.conv.c8 == 1) {
+        // forward: A = X [M][8] (box {8, 128}), B = W [N][72] (box {8, N}); N <= 64
+        if (g.N > 64 || g.amaj != KMAJ || g.bmaj != KMAJ || g.epi != EPI_STORE) return cudaErrorInvalidValue;
+        if (!make_map(&ma, g.A, 8, g.M, g.lda, 8, BM, false, 0) ||
+            !make_map(&mbm, g.B, 72, g.N, g.ldb, 8, 64, false, 0))
+            return cudaErrorInvalidValue;
+        Gemm gg = g;
+        gg.K = BK;  // one packed K-block per tile
+        return dispatch_epi<128, KMAJ, KMAJ, 1>(gg, ma, mbm, e, s);
+    }
+    // weight gradient: A = dY [K pixels][M = Cout] MN-major, B = X [K pixels][8] shifted per tap
+    if (g.N != 72 || g.amaj != MNMAJ || g.bmaj != MNMAJ || g.epi != EPI_F32 || !g.atomic_out)
+        return cudaErrorInvalidValue;
+    if (!make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK) || !make_map(&mbm, g.B, 8, g.K, g.ldb, 8, BK, false, 0))
+        return cudaErrorInvalidValue;
+    e.atomic_out = 1;
+    const int sms = num_sms();
+    const long tiles = (g.M + BM - 1) / BM;
+    const int kb = (g.K + BK - 1) / BK;
+    long S = (2L * sms + tiles - 1) / tiles;
+    if (S > kb / 4) S = kb / 4;
+    if (S < 1) S = 1;
+    const long kper = (kb + S - 1) / S;
+    e.ksplit = (int)((kb + kper - 1) / kper);
+    return dispatch_epi<128, MNMAJ, MNMAJ, 1>(g, ma, mbm, e, s);
 }
 
 cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
@@ -1157,6 +1260,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         }
     }
     if ((g.epi == EPI_SGD || g.epi == EPI_ADAM) && g.ldo == g.N && g.N % 8 == 0) return gemm_bf16_update(g, s);
+    if (g.conv.c8) return gemm_c8(g, s);
     if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
     // tile width: the widest BN that still gives every SM a tile
     const int sms = num_sms();
@@ -1168,8 +1272,8 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         const long pm = (g.M + 255) / 256;
         if (pm * ((g.N + 255) / 256) < sms / 2 || g.N <= 128) BN = 128;
     } else {
-        if ((long)mb * ((g.N + 255) / 256) < sms) BN = 128;
-        if (BN == 128 && (long)mb * ((g.N + 127) / 128) < sms) BN = 64;
+        if ((long)mb * ((g.N + 255) / 256) < sms || g.N <= 128) BN = 128;
+        if (BN == 128 && ((long)mb * ((g.N + 127) / 128) < sms || g.N <= 64)) BN = 64;
     }
     BN = env_int("PD_GEMM_BN", BN);  // tuning override (tools/gemm_bench.py)
     if (cg == 2 && BN < 128) BN = 128;

@@ -66,6 +66,13 @@ struct ConvGeom {
                            // chunk reads X shifted by a_shift[tap] (value = Cp, multiple of 64; 0 = off)
     int a_inner = 0;       // inner extents of the A / B tensors for the TMA maps (taps > 0)
     int b_inner = 0;
+    // packed-tap mode for Cp = 8 inputs (the RGB first layer): the 9 taps' 8-channel slices
+    // are packed side by side along K in unswizzled core-matrix layout (one 16-byte TMA box
+    // per tap) instead of one mostly-zero 64-wide K-block per tap.
+    //   1 = forward (A = X, 9 boxes {8, 128 rows}; B = W [Co][72], 10 boxes {8, Co}; K = 80)
+    //   2 = weight gradient (A = dY MN-major; B = X shifted per tap, 9 boxes {8, 64 pixels};
+    //       N = 72 (MMA N = 80))
+    int c8 = 0;
 };
 
 // C(m, n) = sum_k A(m, k) * B(n, k)

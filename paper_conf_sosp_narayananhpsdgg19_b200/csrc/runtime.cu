@@ -930,6 +930,14 @@ struct Exec {
         return g;
     }
 
+    static bool packed_taps() {
+        static const int v = [] {
+            const char *e = getenv("PD_CONV_C8");
+            return e ? atoi(e) : 1;
+        }();
+        return v != 0;
+    }
+
     static bool tapchunk_dw() {
         static const int v = [] {
             const char *e = getenv("PD_CONV_DW_ONEGEMM");
@@ -951,6 +959,24 @@ struct Exec {
         }
         Gemm g;
         g.conv = conv_geom(d, +1);
+        if (Cp == 8 && Co <= 64 && packed_taps()) {
+            // RGB first layer: 9 taps x 8 channels packed into one K = 80 block
+            g.conv.c8 = 1;
+            g.M = (int)M;
+            g.N = Co;
+            g.K = 72;
+            g.A = x;
+            g.lda = 8;
+            g.B = Wl(l, slot);
+            g.ldb = 72;
+            g.epi = EPI_STORE;
+            g.out = y;
+            g.ldo = Co;
+            g.bias = w->master + boff;
+            g.relu = d.act == PD_ACT_RELU;
+            CK(run_gemm(1, g, w->stream));
+            return;
+        }
         g.conv.kpt = (Cp + 63) / 64;
         g.conv.b_koff = Cp;
         g.conv.a_inner = Cp;
@@ -1014,6 +1040,25 @@ struct Exec {
         if (!bf16) {
             CK(conv_dw_f32(static_cast<const float *>(G), static_cast<const float *>(x), gW, B(), d.height, d.width,
                            Cp, Co, w->stream));
+        } else if (Cp == 8 && packed_taps()) {
+            // dW[co][tap*8 + ci] for all 9 taps of an 8-channel input in ONE GEMM (N = 72)
+            Gemm g;
+            g.M = Co;
+            g.N = 72;
+            g.K = (int)M;
+            g.A = G;
+            g.lda = Co;
+            g.amaj = MNMAJ;
+            g.B = x;
+            g.ldb = 8;
+            g.bmaj = MNMAJ;
+            g.conv.c8 = 2;
+            for (int tap = 0; tap < 9; ++tap) g.conv.a_shift[tap] = ((tap / 3) - 1) * Wp + (tap % 3) - 1;
+            g.epi = EPI_F32;
+            g.atomic_out = 1;
+            g.out = gW;
+            g.ldo = 72;
+            CK(run_gemm(1, g, w->stream));
         } else if (Cp % 64 == 0 && tapchunk_dw()) {
             // dW[co][tap*Cp + ci] for all 9 taps in ONE GEMM (N = 9*Cp): the dY tile is loaded
             // once per K-block for every tap of the tile instead of once per tap
