@@ -62,7 +62,7 @@ def lib():
                               C.c_int, C.c_int, C.c_float, C.c_float, C.c_float, C.c_float, C.c_int,
                               C.c_void_p, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p, C.c_void_p,
                               C.c_void_p, C.c_void_p, C.c_int, C.c_void_p, C.c_void_p, C.c_void_p,
-                              C.c_void_p, C.c_void_p]
+                              C.c_void_p, C.c_void_p, C.c_void_p]
         L.orc_plan.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int, C.c_int, C.c_double,
                                C.c_int, C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p,
                                C.c_void_p]
@@ -150,17 +150,19 @@ class RunResult:
     losses: np.ndarray
     makespan: float
     bubble: float
+    max_live: np.ndarray = None  # [n_stages] widest weight-version window held (pin P10)
 
 
 def run(layers, stage_last, replicas, B, M, params=None, data=None, optimizer=0, lr=0.05,
         beta1=0.9, beta2=0.999, eps=1e-8, depth=0, math=True, stash=True,
-        fwd_time=None, bwd_time=None) -> RunResult:
-    """Simulate PipeDream training.  ``params`` is a list of per-layer flat arrays."""
+        fwd_time=None, bwd_time=None, vertical_sync=False) -> RunResult:
+    """Simulate PipeDream training.  ``params`` is a list of per-layer flat arrays.
+    ``vertical_sync``: every stage uses the version the input stage tagged t with (§3.3)."""
     n = len(stage_last)
     lay = _layers(layers)
     sl = np.ascontiguousarray(stage_last, np.int32)
     rp = np.ascontiguousarray(replicas, np.int32)
-    mode = (1 if math else 0) | (0 if stash else 2)
+    mode = (1 if math else 0) | (0 if stash else 2) | (4 if vertical_sync else 0)
     inputs = tokens = labels = None
     n_data = 1
     if data is not None:
@@ -177,13 +179,15 @@ def run(layers, stage_last, replicas, B, M, params=None, data=None, optimizer=0,
     nev = C.c_int(0)
     vmap = np.full((n, M), -1, np.int32)
     losses = np.zeros(M, np.float32)
+    max_live = np.zeros(n, np.int32)
     mk = C.c_double(0)
     bub = C.c_double(0)
     ft = None if fwd_time is None else np.ascontiguousarray(fwd_time, np.float64)
     bt = None if bwd_time is None else np.ascontiguousarray(bwd_time, np.float64)
     rc = lib().orc_run(lay, len(layers), _ptr(sl), _ptr(rp), n, depth, B, M, optimizer, lr, beta1, beta2,
                        eps, mode, _ptr(inputs), _ptr(tokens), _ptr(labels), n_data, _ptr(flat), _ptr(ft),
-                       _ptr(bt), ev, cap, C.byref(nev), _ptr(vmap), _ptr(losses), C.byref(mk), C.byref(bub))
+                       _ptr(bt), ev, cap, C.byref(nev), _ptr(vmap), _ptr(losses), C.byref(mk), C.byref(bub),
+                       _ptr(max_live))
     if rc == -2:
         raise RuntimeError("oracle: deadlock")
     if rc != 0:
@@ -198,7 +202,7 @@ def run(layers, stage_last, replicas, B, M, params=None, data=None, optimizer=0,
             k = np.asarray(p).size
             out_params.append(flat[off:off + k].copy())
             off += k
-    return RunResult(evs, times, vmap, out_params, losses, mk.value, bub.value)
+    return RunResult(evs, times, vmap, out_params, losses, mk.value, bub.value, max_live)
 
 
 @dataclass

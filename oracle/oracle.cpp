@@ -443,6 +443,9 @@ struct Worker {
     int b_done = 0;                /* backward passes completed (replicated: round count) */
     double free_at = 0.0;
     int seq = 0;
+    int f_done = 0;                /* forwards completed                                     */
+    int last_tag = 0;              /* version used by the latest forward (vertical sync)     */
+    int max_live = 1;              /* widest version window held (pin P10)                   */
 };
 
 struct Sim {
@@ -453,6 +456,8 @@ struct Sim {
     long ptotal = 0;
     OptCfg opt;
     bool math, stash;
+    bool vsync;             /* vertical sync (§3.3): every stage uses the tag version */
+    std::map<std::pair<int, int>, int> act_tag; /* (stage, t) -> version tag travelling with the activation */
     const float *inputs; const int *tokens, *labels; int n_data;
     const double *ftime, *btime;
     std::vector<Worker> W;
@@ -529,8 +534,17 @@ void exec(Sim &S, Worker &w, const Op &op) {
     int s = w.stage, t = op.t;
     long np = S.stage_params(s);
     if (op.kind == 'F') {
-        /* F(s,t): latest version, stash it (L1145-1161) */
+        /* F(s,t): latest version, stash it (L1145-1161).  Vertical sync: the input stage tags
+         * t with its latest version and every later stage uses its own stashed weights of
+         * that version -- the tag travels with the activation (L1180-1186) */
         int v = w.version;
+        if (S.vsync) {
+            if (s > 0) v = S.act_tag[{s, t}];
+            if (s + 1 < S.n_stages) S.act_tag[{s + 1, t}] = v;
+            if (s > 0) S.act_tag.erase({s, t});
+        }
+        w.f_done++;
+        w.last_tag = v;
         double st = w.free_at;
         if (s > 0) st = st > S.act_t[{s, t}] ? st : S.act_t[{s, t}];
         double en = st + (S.ftime ? S.ftime[s] : 0.0);
@@ -654,16 +668,26 @@ void exec(Sim &S, Worker &w, const Op &op) {
     }
     w.version = vin + 1;
     emit(S, w, 'U', ev_t, vin, vin + 1, st, st);
+
     /* the stashed version of the backward just applied is released; a version is discarded
      * once no pending backward references it and it is not the latest (L1349-1353) */
     int vb = w.fwd_version[t];
     w.refcount[vb]--;
     w.fwd_version.erase(t);
+    /* vertical sync: a minibatch not yet forwarded here carries a tag >= the tag of the
+     * last one forwarded here (the input stage's version only grows and it forwards in t
+     * order; straight pipelines), so versions from that tag on are kept */
+    int keep_from = 1 << 30;
+    if (S.vsync && w.f_done < S.M) keep_from = w.last_tag;
     for (auto it = w.versions.begin(); it != w.versions.end();) {
         int ver = it->first;
-        if (ver != w.version && w.refcount[ver] <= 0) it = w.versions.erase(it);
+        if (ver != w.version && w.refcount[ver] <= 0 && ver < keep_from) it = w.versions.erase(it);
         else ++it;
     }
+    /* window of versions held after the update: a ring indexed by version mod depth needs
+     * depth >= this span (the consumed version's storage receives the new one) */
+    int span = w.versions.rbegin()->first - w.versions.begin()->first + 1;
+    if (span > w.max_live) w.max_live = span;
     if (S.R[s] > 1) {
         /* free round buffers once every replica has applied it */
         bool all = true;
@@ -731,21 +755,24 @@ int orc_inflight(const int *R, int n, int depth, int *k_out) {
  *   depth          : 0 => default in-flight counts (NOAM), else the R19 override
  *   mode bit0      : 1 = do the math, 0 = schedule only
  *   mode bit1      : 1 = disable weight stashing (negative control; backward uses latest)
+ *   mode bit2      : 1 = vertical sync (§3.3; straight pipelines only)
  *   inputs/tokens/labels: n_data minibatches, minibatch t uses data t mod n_data
  *   params         : in = initial flat params (layer order), out = final latest params
  *                    (replica 0 of every stage; replicas are identical by construction)
  *   fwd/bwd_time   : per-stage durations for the timeline (may be NULL => 0)
+ *   max_live       : per stage, the widest window (newest - oldest + 1) of weight versions a
+ *                    worker held after an update (may be NULL)
  * Returns 0, or -1 invalid, -2 deadlock, -3 event buffer too small.
  */
 int orc_run(const orc_layer *layers, int n_layers, const int *stage_last, const int *replicas, int n_stages,
             int depth, int B, int M, int opt_kind, float lr, float b1, float b2, float eps, int mode,
             const float *inputs, const int *tokens, const int *labels, int n_data, float *params,
             const double *fwd_time, const double *bwd_time, orc_event *events, int events_cap, int *n_events,
-            int *version_map, float *losses, double *makespan, double *bubble) {
+            int *version_map, float *losses, double *makespan, double *bubble, int *max_live) {
     Sim S;
     S.layers = layers; S.n_layers = n_layers; S.n_stages = n_stages; S.B = B; S.M = M; S.depth = depth;
     S.opt = OptCfg{opt_kind, lr, b1, b2, eps};
-    S.math = (mode & 1) != 0; S.stash = (mode & 2) == 0;
+    S.math = (mode & 1) != 0; S.stash = (mode & 2) == 0; S.vsync = (mode & 4) != 0;
     S.inputs = inputs; S.tokens = tokens; S.labels = labels; S.n_data = n_data > 0 ? n_data : 1;
     S.ftime = fwd_time; S.btime = bwd_time;
     if (n_stages < 1 || stage_last[n_stages - 1] != n_layers - 1) return -1;
@@ -755,6 +782,10 @@ int orc_run(const orc_layer *layers, int n_layers, const int *stage_last, const 
         if (S.last[s] < S.first[s] || replicas[s] < 1) return -1;
         if (M % replicas[s] != 0) return -1;
         S.R.push_back(replicas[s]);
+    }
+    if (S.vsync) {
+        if (!S.stash) return -1;
+        for (int s = 0; s < n_stages; s++) if (S.R[s] != 1) return -1; /* straight pipelines only */
     }
     S.k.assign(n_stages, 0);
     if (orc_inflight(replicas, n_stages, depth, S.k.data()) != 0) return -1;
@@ -810,6 +841,12 @@ int orc_run(const orc_layer *layers, int n_layers, const int *stage_last, const 
         if (e.end > mk) mk = e.end;
         busy += e.end - e.start;
     }
+    if (max_live)
+        for (int s = 0; s < n_stages; s++) {
+            int m = 0;
+            for (int r = 0; r < S.R[s]; r++) m = m > S.W[S.wbase[s] + r].max_live ? m : S.W[S.wbase[s] + r].max_live;
+            max_live[s] = m;
+        }
     if (makespan) *makespan = mk;
     if (bubble) *bubble = mk > 0 ? 1.0 - busy / ((double)S.W.size() * mk) : 0.0;
     if (S.math && params)
