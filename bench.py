@@ -145,6 +145,11 @@ def gemm_flops(L, B):
     return 2.0 * B * L.in_ * L.out
 
 
+def pass_flops(L, B):
+    """FLOPs of ONE GEMM pass (forward, dX or dW: 2 per MAC) of layer L for one minibatch."""
+    return layer_flops(L, B) / 3.0
+
+
 # ----------------------------------------------------------------------------- reference arm
 
 def run_reference(args):
@@ -211,6 +216,11 @@ def main():
     ap.add_argument("--cpu-batch", type=int, default=8)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--plan", default="pipeline", choices=["pipeline", "dp"],
+                    help="pipeline: pd_plan straight pipeline (VGG: (N-1)-1); dp: one stage x N replicas "
+                         "(pure data parallelism, SURVEY §8(f) NEXT #1)")
+    ap.add_argument("--sync", default="stash", choices=["stash", "vertical"],
+                    help="weight stashing (default) or vertical sync (§3.3; straight plans)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -253,8 +263,8 @@ def main():
     peaks = load_peaks()
     wl = synth.workload(args.config)
     layers, B = wl.layers, wl.batch
-    if N == 1:
-        plan = pd.Plan.manual([len(layers) - 1], [1])
+    if N == 1 or args.plan == "dp":
+        plan = pd.Plan.manual([len(layers) - 1], [N])
     elif args.config == "vgg16":
         # VGG-16 as (N-1)-1 -- conv stage replicated, FC stage alone
         conv_last = max(i for i, L in enumerate(layers) if L.kind == synth.MAXPOOL2)
@@ -264,12 +274,13 @@ def main():
         plan = pd.pd_plan(T, a, w, N, max_replicas=1)
     n = len(plan.stages)
     R0 = plan.stages[0][2]
-    M = args.minibatches or (8 if n == 1 else 16 * n)
+    M = args.minibatches or (8 * R0 if n == 1 else 16 * n)
     M = -(-M // R0) * R0  # a multiple of every replica count
     p0 = synth.init_params(layers) if True else None
     n_data = 8
     data = synth.make_data(wl, n_data)
-    P = Pipeline(plan, layers, p0, dtype=pd.PD_BF16, optimizer=wl.optimizer, lr=wl.lr, minibatch=B,
+    sync = pd.PD_SYNC_VERTICAL if args.sync == "vertical" else pd.PD_SYNC_STASH
+    P = Pipeline(plan, layers, p0, dtype=pd.PD_BF16, optimizer=wl.optimizer, lr=wl.lr, minibatch=B, sync_mode=sync,
                  record_trace=int(os.environ.get("PD_BENCH_TRACE", "2")), device_of=lambda g: g if world > 1 else local_rank,
                  local=(lambda wid: wid == rank) if world > 1 else None,
                  allgather=torch_allgather() if world > 1 else None)
@@ -317,19 +328,42 @@ def main():
         prof_cnt += np.array(st["kern_count"])
     P.set_timing(2, 0)
 
-    # ---- roofline of the dominant kernel (the dW GEMM + fused SGD update), this rank's stage
+    # ---- roofline of the dominant kernel, this rank's stage
     s_mine = [s for s, st in enumerate(plan.stages) if st[3] <= rank < st[3] + st[2]][0]
-    my_layers = [layers[l] for l in range(plan.stages[s_mine][0], plan.stages[s_mine][1] + 1)]
+    first_l = plan.stages[s_mine][0]
+    my_layers = [layers[l] for l in range(first_l, plan.stages[s_mine][1] + 1)]
     lin = [L for L in my_layers if L.kind == synth.LINEAR] or my_layers
-    dw_bytes = float(np.mean([dw_update_bytes(L, B) for L in lin]))
     stage_flops = sum(layer_flops(L, B) for L in my_layers)
+    # per-class GEMM FLOPs of the profile pass (2 runs x this replica's minibatches); dX of
+    # the model's first layer is skipped (stage 0)
+    mb_mine = 2 * M // plan.stages[s_mine][2]
+    fwd_fl = sum(pass_flops(L, B) for L in my_layers) * mb_mine
+    dx_fl = sum(pass_flops(L, B) for i, L in enumerate(my_layers) if first_l + i > 0) * mb_mine
+    dw_fl = fwd_fl
+    cls_s = prof_kern[:3] / 1e3
+    fw_tflops = fwd_fl / cls_s[0] / 1e12 if cls_s[0] > 0 else 0.0
+    dx_tflops = dx_fl / cls_s[1] / 1e12 if cls_s[1] > 0 else 0.0
+    dw_tflops = dw_fl / cls_s[2] / 1e12 if cls_s[2] > 0 else 0.0
     dw_avg_s = prof_kern[2] / max(prof_cnt[2], 1) / 1e3
-    achieved = dw_bytes / dw_avg_s / 1e9 if dw_avg_s > 0 else 0.0
-    fw_flops = float(np.mean([gemm_flops(L, B) for L in lin]))
-    fw_avg_s = prof_kern[0] / max(prof_cnt[0], 1) / 1e3
-    fw_tflops = fw_flops / fw_avg_s / 1e12 if fw_avg_s > 0 else 0.0
-    dx_avg_s = prof_kern[1] / max(prof_cnt[1], 1) / 1e3
-    dx_tflops = fw_flops / dx_avg_s / 1e12 if dx_avg_s > 0 else 0.0
+    if args.config == "mlp4096":
+        # HBM-bound: dW GEMM with the fused SGD update (K = 256), bytes per launch
+        dw_bytes = float(np.mean([dw_update_bytes(L, B) for L in lin]))
+        achieved = dw_bytes / dw_avg_s / 1e9 if dw_avg_s > 0 else 0.0
+        roof = {"bound": "hbm", "kernel": "dW GEMM + fused SGD update (tcgen05, EPI_SGD)",
+                "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / peaks["hbm_gbs"], "traffic": None,
+                "bytes_per_launch": dw_bytes, "avg_launch_us": dw_avg_s * 1e6,
+                "peak_source": peaks["source"] + " hbm_gbs (copy)"}
+    else:
+        # tensor-bound stages (convolutions / LSTM / classifier GEMMs): the dominant GEMM class
+        names = ["forward GEMMs", "dX GEMMs", "dW GEMMs (+update)"]
+        tfl = [fw_tflops, dx_tflops, dw_tflops]
+        d = int(np.argmax(cls_s))
+        roof = {"bound": "tensor", "kernel": f"{names[d]} of the stage (tcgen05), class total",
+                "achieved": tfl[d], "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
+                "frac": tfl[d] / peaks["bf16_tflops_sustained"], "traffic": None,
+                "flops_per_minibatch": [fwd_fl / mb_mine, dx_fl / mb_mine, dw_fl / mb_mine][d],
+                "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"}
     step_share = {cls: float(prof_kern[i] / max(prof_ms, 1e-9)) for i, cls in enumerate(["fwd_gemm", "dx_gemm",
                                                                                            "dw_update_gemm", "other"])}
     step_share["note"] = "profile pass (2 steps, every kernel class event-timed); dW and dX overlap on two streams"
@@ -373,24 +407,24 @@ def main():
                        "plan": "-".join(str(s[2]) for s in plan.stages) + f" ({n} stage{'s' if n > 1 else ''} "
                                f"of {[s[1] - s[0] + 1 for s in plan.stages]} layers)",
                        "global_batch": B, "minibatches_per_step": M, "noam": plan.noam,
-                       "parallelism": f"pipeline{n}" if n > 1 else "single-stage",
+                       "parallelism": (f"pipeline{n}" if n > 1 else
+                                       (f"dp{N}" if N > 1 else "single-stage")),
+                       "sync": args.sync,
                        "l2": "working set > L2: every minibatch streams 0.54 GB bf16 weights + 1.07 GB fp32 "
                              "master per 16 layers (126 MB L2), no flush needed"},
             "bubble_pct": 100.0 * bubble,
             "wall_s": wall,
             "gpu_launches": launches,
             "clocks": clk,
-            "roofline": {"bound": "hbm", "kernel": "dW GEMM + fused SGD update (tcgen05, EPI_SGD)",
-                         "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                         "frac": achieved / peaks["hbm_gbs"], "traffic": None,
-                         "bytes_per_launch": dw_bytes, "avg_launch_us": dw_avg_s * 1e6,
-                         "peak_source": peaks["source"] + " hbm_gbs (copy)",
-                         "timing": "CUDA events around every dW launch on its stream, instrumented profile pass "
-                                   "(2 steps) right after the timed region; dW overlaps the next layer's dX"},
-            "tensor_pipe": {"fwd_gemm_tflops": fw_tflops, "dx_gemm_tflops": dx_tflops,
+            "roofline": dict(roof, timing="CUDA events around every launch of the class on its stream, "
+                                          "instrumented profile pass (2 steps) right after the timed region; "
+                                          "dW overlaps the next layer's dX"),
+            "tensor_pipe": {"fwd_gemm_tflops": fw_tflops, "dx_gemm_tflops": dx_tflops, "dw_gemm_tflops": dw_tflops,
                             "peak_tflops": peaks["bf16_tflops_sustained"],
                             "fwd_frac": fw_tflops / peaks["bf16_tflops_sustained"],
                             "dx_frac": dx_tflops / peaks["bf16_tflops_sustained"],
+                            "dw_frac": dw_tflops / peaks["bf16_tflops_sustained"],
+                            "note": "class FLOPs / class device time (dW time includes the fused update)",
                             "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"},
             "step_share": step_share,
             "stage_tflops": stage_flops * args.steps * M / plan.stages[s_mine][2] / (total_ms / 1e3) / 1e12,

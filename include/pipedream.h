@@ -115,6 +115,14 @@ typedef struct {
 
 typedef enum { PD_FP32 = 0, PD_BF16 = 1 } pd_dtype;
 typedef enum { PD_SGD = 0, PD_ADAM = 1 } pd_optimizer;
+/* Weight-version semantics across stages (§3.3):
+ *   PD_SYNC_STASH     weight stashing: F(s,t) uses stage s's latest version, B(s,t) the
+ *                     version its F used (the default; w_s^(t-n+s) in L1237-1241);
+ *   PD_SYNC_VERTICAL  vertical sync: the input stage tags minibatch t with its latest
+ *                     version v and EVERY stage runs F(s,t) and B(s,t) with its own stashed
+ *                     version v (L1175-1186; update rule L1247-1253).  Straight plans only
+ *                     (every R_s = 1, else PD_EUNSUPPORTED); every stage keeps k_0 versions. */
+typedef enum { PD_SYNC_STASH = 0, PD_SYNC_VERTICAL = 1 } pd_sync_mode;
 
 typedef struct {
     int dtype;        /* PD_FP32: fp32 SIMT parity path (no tensor cores, tf32 off);
@@ -124,6 +132,7 @@ typedef struct {
     int minibatch;    /* B, samples per minibatch                                         */
     int record_trace; /* 0 = off, 1 = event trace + version map, 2 = also per-op device times */
     int max_depth;    /* largest pd_run depth override that will be requested (0 = NOAM)   */
+    int sync_mode;    /* pd_sync_mode (0 = weight stashing)                                */
 } pd_train_cfg;
 
 typedef struct pd_ctx pd_ctx;

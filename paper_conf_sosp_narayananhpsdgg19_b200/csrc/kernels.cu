@@ -373,6 +373,24 @@ cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f
     return cudaGetLastError();
 }
 
+namespace {
+__global__ void regions_bf16_to_f32_kernel(const __nv_bfloat16 *__restrict__ src, float *__restrict__ dst,
+                                           const long *__restrict__ off, const int *__restrict__ cnt) {
+    const long o = off[blockIdx.y];
+    const int n = cnt[blockIdx.y];
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+        dst[o + i] = __bfloat162float(src[o + i]);
+}
+}  // namespace
+
+cudaError_t regions_bf16_to_f32(const __nv_bfloat16 *src, float *dst, const long *off, const int *cnt, int n,
+                                cudaStream_t s) {
+    if (n <= 0) return cudaSuccess;
+    regions_bf16_to_f32_kernel<<<dim3(8, n), 256, 0, s>>>(src, dst, off, cnt);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
 cudaError_t f32_to_bf16(const float *in, __nv_bfloat16 *out, long n, cudaStream_t s) {
     f32_to_bf16_kernel<<<grid_for(n), 256, 0, s>>>(in, out, n);
     ++tl_launches;

@@ -133,6 +133,9 @@ cudaError_t adam_f32(const float *in, const float *g, float *out, float *m, floa
 cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f32, const float *const *grads,
                           int R, long goff, long n, int opt, float *m, float *v, float lr, float b1, float b2,
                           float eps, int step, cudaStream_t s);
+// dst[off[r] + i] = float(src[off[r] + i]) for i < cnt[r], r < n (off, cnt device arrays)
+cudaError_t regions_bf16_to_f32(const __nv_bfloat16 *src, float *dst, const long *off, const int *cnt, int n,
+                                cudaStream_t s);
 cudaError_t f32_to_bf16(const float *in, __nv_bfloat16 *out, long n, cudaStream_t s);
 cudaError_t bf16_to_f32(const __nv_bfloat16 *in, float *out, long n, cudaStream_t s);
 cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s);

@@ -243,6 +243,12 @@ struct Worker {
     // weights
     std::vector<void *> wslot;  // k versions (path dtype)
     float *master = nullptr;    // bf16 path
+    // vertical sync, bf16 path: fp32 biases of the version a forward uses (from its bf16
+    // slot), bias regions (offset, count) of the stage's layers on the device
+    float *fbias = nullptr;
+    long *breg_off = nullptr;
+    int *breg_cnt = nullptr;
+    int n_breg = 0;
     float *adam_m = nullptr, *adam_v = nullptr;
     float *gbuf = nullptr;      // fp32 gradient (unreplicated fp32 path / biases)
     float *ws = nullptr;        // split-K partials of the bf16 GEMMs
@@ -280,6 +286,7 @@ struct Worker {
     uint32_t *flags = nullptr;
     // bookkeeping
     int version = 0;
+    int run_base = 0;  // version at the start of the current pd_run (equal on every stage)
     std::map<int, int> fwd_version;  // local index -> version used by its forward
     std::vector<pd_event> events;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> op_ev;  // record_trace 2
@@ -303,7 +310,7 @@ Worker::~Worker() {
     void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da};
     for (void *p : lb)
         if (p) cudaFree(p);
-    void *bufs[] = {master, adam_m, adam_v, gbuf, ws, (void *)split_counters, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
+    void *bufs[] = {master, fbias, (void *)breg_off, (void *)breg_cnt, adam_m, adam_v, gbuf, ws, (void *)split_counters, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
     for (void *p : bufs)
         if (p) cudaFree(p);
@@ -475,8 +482,14 @@ struct Exec {
     const float *bias_f32(int l, int slot) const {
         const pd_layer_desc &d = layer(l);
         const long off = c->poff[l] + (long)d.out * d.in;
-        if (bf16) return w->master + off;  // master holds the latest version
-        return static_cast<const float *>(w->wslot[slot]) + off;
+        return fwd_f32(off, slot);
+    }
+    // fp32 view of forward parameters at offset `off` of version slot `slot`: the slot itself
+    // (fp32 path); on the bf16 path the fp32 master (= latest, weight stashing) or the
+    // slot's biases widened to fp32 (vertical sync, where F may use an older version)
+    const float *fwd_f32(long off, int slot) const {
+        if (!bf16) return static_cast<const float *>(w->wslot[slot]) + off;
+        return (w->fbias ? w->fbias : w->master) + off;
     }
 
     // input of layer l for local index j
@@ -544,7 +557,13 @@ struct Exec {
             // message index on this link: minibatches from p to this replica before t
             link_wait(c, L, w->stream, act_msg_index(s - 1, t));
         }
-        const int v = w->version;
+        // weight stashing: the latest version.  Vertical sync: the tag the input stage gave t,
+        // its latest version at F(0,t) = base + max(0, t - k_0 + 1) on the static schedule
+        // (L1180-1186; base = the version every stage had when this pd_run started)
+        const bool vsync = c->cfg.sync_mode == PD_SYNC_VERTICAL;
+        const int v = vsync ? w->run_base + std::max(0, t - k[0] + 1) : w->version;
+        if (v > w->version || v <= w->version - w->k)
+            throw CudaFail{cudaErrorInvalidValue, "vertical sync: tagged version not in the stash ring"};
         const int slot = v % w->k;
         w->fwd_version[j] = v;
         if (c->cfg.record_trace) c->vmap[(long)s * M + t] = v;
@@ -562,6 +581,9 @@ struct Exec {
         const long lrows = rows_of(layer(w->last), B());
         const int32_t *labels = (s + 1 == n()) ? w->labels + (long)(t % c->n_data) * lrows : nullptr;
         auto body = [&](float *loss_dst) {
+        if (w->fbias && w->n_breg)  // vertical sync, bf16: fp32 biases of the stashed version `slot`
+            CK(regions_bf16_to_f32(static_cast<const __nv_bfloat16 *>(w->wslot[slot]), w->fbias, w->breg_off,
+                                   w->breg_cnt, w->n_breg, w->stream));
         for (int l = w->first; l <= w->last; ++l) {
             const pd_layer_desc &d = layer(l);
             const void *x = layer_input(l, t, j);
@@ -734,10 +756,7 @@ struct Exec {
         const long o[4] = {0, 4 * H * I, 4 * H * I + 4 * H * H, 4 * H * I + 4 * H * H + 4 * H};
         return c->poff[l] + o[which];
     }
-    const float *param_f32(long off, int slot) const {
-        if (bf16) return w->master + off;
-        return static_cast<const float *>(w->wslot[slot]) + off;
-    }
+    const float *param_f32(long off, int slot) const { return fwd_f32(off, slot); }
 
     // Run `body` (a sequence of launches on w->stream) through a cached CUDA graph.
     template <typename F>
@@ -972,7 +991,7 @@ struct Exec {
             g.epi = EPI_STORE;
             g.out = y;
             g.ldo = Co;
-            g.bias = w->master + boff;
+            g.bias = fwd_f32(boff, slot);
             g.relu = d.act == PD_ACT_RELU;
             CK(run_gemm(1, g, w->stream));
             return;
@@ -991,7 +1010,7 @@ struct Exec {
         g.epi = EPI_STORE;
         g.out = y;
         g.ldo = Co;
-        g.bias = w->master + boff;  // latest version (forward)
+        g.bias = fwd_f32(boff, slot);
         g.relu = d.act == PD_ACT_RELU;
         CK(run_gemm(1, g, w->stream));
     }
@@ -1367,6 +1386,7 @@ struct Exec {
     void run_ops() {
         const int Rs = c->plan.stage[w->stage].replicas;
         std::vector<Op> ops = worker_ops(Rs, w->replica, k[w->stage], M);
+        w->run_base = w->version;
         for (const Op &op : ops) {
             if (c->abort) throw Abort{};
             if (op.kind == 'F') forward(op.t, op.j);
@@ -1469,6 +1489,10 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
         if (inflight_counts(*plan, cfg->max_depth, kmax) != PD_OK) return PD_EINVAL;
         for (int s = 0; s < n; ++s) kmax[s] = std::max(kmax[s], kdef[s]);
     }
+    if (cfg->sync_mode != PD_SYNC_STASH && cfg->sync_mode != PD_SYNC_VERTICAL) return PD_EINVAL;
+    if (cfg->sync_mode == PD_SYNC_VERTICAL)
+        for (int s = 0; s < n; ++s)
+            if (plan->stage[s].replicas != 1) return PD_EUNSUPPORTED;  // straight pipelines (§3.3)
     pd_ctx *c = new pd_ctx;
     c->plan = *plan;
     c->layers.assign(layers, layers + num_layers);
@@ -1487,6 +1511,10 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
     c->Galloc.assign(n, 0);
     for (int s = 1; s < n; ++s) c->Dalloc[s] = recv_ring_depth(*plan, kmax, s);
     for (int s = 0; s + 1 < n; ++s) c->Galloc[s] = kmax[s];
+    // vertical sync: stage s holds every version from the oldest tag still in flight to its
+    // latest -- a window of k_0 versions at every stage (R25); rings sized as usual
+    if (cfg->sync_mode == PD_SYNC_VERTICAL)
+        for (int s = 0; s < n; ++s) c->kalloc[s] = kmax[0];
     c->poff.assign(num_layers, 0);
     c->pcount.assign(num_layers, 0);
     c->hcount.assign(num_layers, 0);
@@ -1567,6 +1595,29 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         }
         if (bf16) w->master = stage_f32;
         else cudaFree(stage_f32);
+        if (bf16 && c->cfg.sync_mode == PD_SYNC_VERTICAL) {
+            std::vector<long> offs;
+            std::vector<int> cnts;
+            for (int l = w->first; l <= w->last; ++l) {
+                const pd_layer_desc &d = c->layers[l];
+                long o = -1, nb = 0;
+                if (d.kind == PD_LINEAR) o = c->poff[l] + (long)d.out * d.in, nb = d.out;
+                else if (d.kind == PD_CONV3X3) o = c->poff[l] + (long)d.out * 9 * cpad8(d.in), nb = d.out;
+                else if (d.kind == PD_LSTM) o = c->poff[l] + 4L * d.out * d.in + 4L * d.out * d.out, nb = 8L * d.out;
+                if (o >= 0) {
+                    offs.push_back(o);
+                    cnts.push_back((int)nb);
+                }
+            }
+            w->n_breg = (int)offs.size();
+            w->fbias = dalloc<float>(P * 4);
+            if (w->n_breg) {
+                w->breg_off = dalloc<long>(offs.size() * sizeof(long));
+                w->breg_cnt = dalloc<int>(cnts.size() * sizeof(int));
+                CK(cudaMemcpy(w->breg_off, offs.data(), offs.size() * sizeof(long), cudaMemcpyHostToDevice));
+                CK(cudaMemcpy(w->breg_cnt, cnts.data(), cnts.size() * sizeof(int), cudaMemcpyHostToDevice));
+            }
+        }
         if (c->cfg.optimizer == PD_ADAM) {
             w->adam_m = dalloc<float>(P * 4);
             w->adam_v = dalloc<float>(P * 4);

@@ -25,14 +25,14 @@ def workers_of(plan: Plan):
 class Pipeline:
     def __init__(self, plan: Plan, layers, params: Sequence[np.ndarray], *, dtype=PD_BF16, optimizer=PD_SGD,
                  lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8, minibatch=1, record_trace=1, max_depth=0,
-                 device_of: Optional[Callable[[int], int]] = None, local: Optional[Callable[[int], bool]] = None,
+                 sync_mode=0, device_of: Optional[Callable[[int], int]] = None, local: Optional[Callable[[int], bool]] = None,
                  allgather: Optional[Callable[[list], list]] = None):
         """device_of(worker_gpu) -> CUDA ordinal (default: everything on device 0, i.e. virtual
         workers); local(worker_id) -> whether this process owns the worker (default all);
         allgather(list_of_bytes) -> list over processes of lists (needed when not all local)."""
         self.plan, self.layers = plan, list(layers)
         self.ctx = pd_create(plan, self.layers, dtype, optimizer, lr, beta1, beta2, eps, minibatch, record_trace,
-                             max_depth)
+                             max_depth, sync_mode)
         device_of = device_of or (lambda g: 0)
         local = local or (lambda w: True)
         self.workers = workers_of(plan)

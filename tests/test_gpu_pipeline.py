@@ -192,3 +192,83 @@ def test_vgg_wider_bf16_two_blocks():
     assert_schedule_exact(res)
     perr, derr = param_errors(res)
     assert perr < BF16_TOL, (perr, derr)
+
+
+# ---------------------------------------------------------------- vertical sync (§3.3, NEXT #2)
+VS = pd.PD_SYNC_VERTICAL
+
+
+@pytest.mark.parametrize("last", [[7, 15], [3, 7, 11, 15], [0, 1, 2, 15], [15]])
+def test_vertical_sync_mlp_fp32(last):
+    wl = synth.workload("mlp4096", reduced=True)
+    M = 4 * len(last) + 3
+    res = run_both(wl, last, [1] * len(last), M, pd.PD_FP32, sync_mode=VS)
+    assert_schedule_exact(res)
+    k0 = len(last)
+    assert (res["vmap"] == np.array([[max(0, t - k0 + 1) for t in range(M)]] * len(last))).all()
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+@pytest.mark.parametrize("depth", [2, 6])
+def test_vertical_sync_depth_override_fp32(depth):
+    wl = synth.workload("mlp4096", reduced=True)
+    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 14, pd.PD_FP32, noam=depth, sync_mode=VS)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+def test_vertical_sync_gnmt_fp32():
+    wl = synth.workload("gnmt8", reduced=True)
+    res = run_both(wl, [2, 5, 8, 9], [1] * 4, 12, pd.PD_FP32, sync_mode=VS)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+def test_vertical_sync_vgg_fp32():
+    wl = synth.workload("vgg16", reduced=True)
+    res = run_both(wl, [2, 5], [1, 1], 9, pd.PD_FP32, sync_mode=VS)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < FP32_TOL and derr < 1e-3, (perr, derr)
+
+
+def test_vertical_sync_bf16():
+    # bf16: older versions' biases come from their bf16 stash slot (widened to fp32)
+    wl = synth.workload("mlp4096", reduced=True)
+    res = run_both(wl, [3, 7, 11, 15], [1] * 4, 16, pd.PD_BF16, lr=BF16_LR, sync_mode=VS)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
+    g = synth.workload("gnmt8", reduced=True)
+    res = run_both(g, [4, 9], [1, 1], 8, pd.PD_BF16, lr=3e-4, sync_mode=VS)
+    assert_schedule_exact(res)
+    assert param_errors(res)[0] < BF16_TOL
+    v = _vgg_bf16_workload()
+    res = run_both(v, [2, 5], [1, 1], 9, pd.PD_BF16, sync_mode=VS)
+    assert_schedule_exact(res)
+    assert param_errors(res)[0] < BF16_TOL
+
+
+def test_vertical_sync_second_run_fp32():
+    # a pd_run drains the pipeline; the next one tags relative to the versions it starts from
+    wl = synth.workload("mlp4096", reduced=True)
+    p0 = synth.init_params(wl.layers)
+    data = synth.make_data(wl, 5)
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline
+    import oracle
+    import torchref
+    last = [3, 7, 11, 15]
+    with Pipeline(pd.Plan.manual(last, [1] * 4), wl.layers, p0, dtype=pd.PD_FP32, lr=wl.lr, minibatch=wl.batch,
+                  sync_mode=VS) as P:
+        P.set_data(*data, 5)
+        P.run(9)
+        P.run(9)
+        vm = P.version_map(9)
+        got = P.params([synth.param_count(L) for L in wl.layers])
+    assert (vm == np.array([[9 + max(0, t - 3) for t in range(9)]] * 4)).all()
+    r1 = oracle.run(wl.layers, last, [1] * 4, wl.batch, 9, p0, data, lr=wl.lr, vertical_sync=True)
+    r2 = oracle.run(wl.layers, last, [1] * 4, wl.batch, 9, r1.params, data, lr=wl.lr, vertical_sync=True)
+    assert torchref.max_rel_err([got[l] for l in range(len(wl.layers))], r2.params) < FP32_TOL

@@ -103,6 +103,21 @@ def test_create_validation():
         pd.pd_create(good, wl.layers, pd.PD_FP32, minibatch=0)
 
 
+def test_create_sync_mode_validation():
+    wl = synth.workload("mlp_small")
+    ctx = pd.pd_create(pd.Plan.manual([1, 2], [1, 1]), wl.layers, pd.PD_FP32, minibatch=16,
+                       sync_mode=pd.PD_SYNC_VERTICAL)
+    pd.pd_destroy(ctx)
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_create(pd.Plan.manual([1, 2], [1, 1]), wl.layers, pd.PD_FP32, minibatch=16, sync_mode=7)
+    assert ei.value.status == pd.PD_EINVAL
+    # vertical sync is defined for straight pipelines (§3.3); replicated plans are rejected
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_create(pd.Plan.manual([1, 2], [2, 1]), wl.layers, pd.PD_FP32, minibatch=16,
+                     sync_mode=pd.PD_SYNC_VERTICAL)
+    assert ei.value.status == pd.PD_EUNSUPPORTED
+
+
 @pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU failure mode")
 def test_device_calls_fail_loudly_without_gpu():
     wl = synth.workload("mlp_small")
