@@ -24,6 +24,8 @@
 #include <cstdio>
 #include <cstdlib>
 #include <unordered_map>
+#include <vector>
+#include <algorithm>
 
 #include "pd_internal.h"
 
@@ -35,14 +37,22 @@ constexpr int BK = 64;  // 64 bf16 = 128 B = one swizzle row
 constexpr int UMMA_K = 16;
 constexpr int NUM_THREADS = 256;
 
-template <int BN>
+enum { EPI_STORE_ = 0, EPI_MASK_ = 1, EPI_F32_ = 2 };  // (mirror of pd_internal.h's EPI_* for constexprs)
+template <int BN, int EPI = 0>
 struct Cfg {
     static constexpr int A_BYTES = BM * BK * 2;
     static constexpr int B_BYTES = BN * BK * 2;
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-    static constexpr int STAGES = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
+    // epilogue staging per epilogue warp (TMA-store epilogue): two 32 x 32 output tiles (fp32
+    // 4 KB or bf16 2 KB each, swizzled) + two bf16 mask tiles (EPI_MASK)
+    static constexpr int OUT_TILE = EPI == EPI_F32_ ? 4096 : 2048;
+    static constexpr int WARP_STG = EPI > EPI_F32_ ? 0 : 2 * OUT_TILE + (EPI == EPI_MASK_ ? 2 * 2048 : 0);
+    static constexpr int EPI_STG = 4 * WARP_STG;
+    static constexpr int STAGES_MAX = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
+    static constexpr int STAGES_FIT = (232448 - 1024 - 256 - EPI_STG) / STAGE_BYTES;
+    static constexpr int STAGES = STAGES_FIT < STAGES_MAX ? STAGES_FIT : STAGES_MAX;
     static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
-    static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_STG + 1024 /*align*/ + 256 /*barriers*/;
 };
 
 struct EpiArgs {
@@ -53,6 +63,8 @@ struct EpiArgs {
     ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
     int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
     int l2_prefetch;    // producer L2-prefetch distance in K-blocks (0 = off; measured no gain so far)
+    int dbg;                    // tools only (PD_EPI_DEBUG): bit 0 skip epilogue global stores, bit 1 skip transpose
+    unsigned long long *probe;  // tools only (PD_GEMM_PROBE): per-CTA %globaltimer phase stamps [grid][8]
     // in-kernel split-K: each (tile, split) writes its fp32 partial to ws[split]; the last CTA
     // to finish a tile (per-tile counter) sums the partials in split order and applies the
     // final epilogue (final_epi = EPI_STORE or EPI_MASK) -- no separate reduction launch
@@ -158,6 +170,19 @@ __device__ __forceinline__ void tc_commit_cg(uint32_t bar) {
             "h"(mask)
             : "memory");
     }
+}
+__device__ __forceinline__ void tmem_ld32_nowait(uint32_t taddr, float (&v)[32]) {
+    uint32_t r[32];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+          "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+          "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+          "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float (&v)[32]) {
     uint32_t r[32];
@@ -342,6 +367,98 @@ __device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32],
     }
 }
 
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t src, int c0, int c1) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(map), "r"(src),
+                 "r"(c0), "r"(c1)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap *map, uint32_t src, int c0, int c1) {
+    asm volatile("cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group [%0, {%2, %3}], [%1];" ::"l"(map),
+                 "r"(src), "r"(c0), "r"(c1)
+                 : "memory");
+}
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap *map, uint32_t src, int c0, int c1, int c2) {
+    asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(map),
+                 "r"(src), "r"(c0), "r"(c1), "r"(c2)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+
+// TMA-store epilogue (STORE / MASK / F32).  Each epilogue warp owns 32 accumulator rows; a
+// 32 x 32 chunk (lane = row) gets its elementwise op in registers, is written to a swizzled
+// shared tile (16-byte stores, conflict-free) and leaves with ONE bulk tensor store (or an
+// L2-side fp32 reduce-add for split-K / per-tap partial sums), double-buffered so the next
+// chunk's TMEM load overlaps the store.  Plain st.global from 4 warps per SM sustained only
+// ~13 B/clk (latency bound); the TMA engine keeps many stores in flight.
+__device__ __forceinline__ uint32_t stg_off_f32(int r, int j) { return r * 128 + ((j ^ (r & 7)) << 4); }
+__device__ __forceinline__ uint32_t stg_off_bf16(int r, int j) { return r * 64 + ((j ^ ((r >> 1) & 3)) << 4); }
+
+template <int EPI>
+__device__ __forceinline__ void epi_math(const EpiArgs &e, float (&v)[32], int row, int col, int N,
+                                         const uint8_t *mask_tile, int lane) {
+    bool border = false;
+    if (e.conv.Hp) {
+        const int wp = row % e.conv.Wp, hp = (row / e.conv.Wp) % e.conv.Hp;
+        border = hp == 0 || hp == e.conv.Hp - 1 || wp == 0 || wp == e.conv.Wp - 1;
+    }
+    if constexpr (EPI == EPI_STORE) {
+        if (e.bias) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] += (col + i < N) ? __ldg(e.bias + col + i) : 0.f;
+        }
+        if (e.relu) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
+        }
+    } else if constexpr (EPI == EPI_MASK) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const uint4 raw = *reinterpret_cast<const uint4 *>(mask_tile + stg_off_bf16(lane, j));
+            const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) v[j * 8 + i] = (__bfloat162float(h[i]) > 0.f) ? v[j * 8 + i] : 0.f;
+        }
+    }
+    if (EPI != EPI_F32 && border) {
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = 0.f;
+    }
+}
+
+template <int EPI>
+__device__ __forceinline__ void epi_stage(uint8_t *tile, const float (&v)[32], int lane) {
+    if constexpr (EPI == EPI_F32) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+            *reinterpret_cast<float4 *>(tile + stg_off_f32(lane, j)) =
+                make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+    } else {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            uint4 w;
+            w.x = pack_bf16(v[8 * j + 0], v[8 * j + 1]);
+            w.y = pack_bf16(v[8 * j + 2], v[8 * j + 3]);
+            w.z = pack_bf16(v[8 * j + 4], v[8 * j + 5]);
+            w.w = pack_bf16(v[8 * j + 6], v[8 * j + 7]);
+            *reinterpret_cast<uint4 *>(tile + stg_off_bf16(lane, j)) = w;
+        }
+    }
+}
+
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+#define PROBE(i)                                                   \
+    do {                                                           \
+        if (e.probe) e.probe[blockIdx.x * 16 + (i)] = gtimer();    \
+    } while (0)
+
 // ---------------------------------------------------------------- the kernel
 // CG = 1: one CTA per 128 x BN tile.  CG = 2: a CTA pair (cluster of 2 on one TPC) per
 // 256 x BN tile with tcgen05.mma.cta_group::2 -- each CTA stages its 128 rows of A and half
@@ -350,17 +467,21 @@ __device__ __forceinline__ void epilogue_chunk(const EpiArgs &e, float (&v)[32],
 // FLOP, the lever that matters when the L2->SM fill (~80 GB/s per SM) is the limit.
 template <int BN, int AMAJ, int BMAJ, int EPI, int CG>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
-    tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, EpiArgs e,
+    tc_gemm_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                   const __grid_constant__ CUtensorMap tmO, const __grid_constant__ CUtensorMap tmK, EpiArgs e,
                    int M, int N, int K) {
-    using C = Cfg<BN / CG>;  // shared-memory ring holds this CTA's A rows and B columns
+    using C = Cfg<BN / CG, EPI>;  // shared-memory ring holds this CTA's A rows and B columns
     constexpr int BNC = BN / CG;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + C::STAGES * C::STAGE_BYTES);
+    uint8_t *epi_stg = smem + C::STAGES * C::STAGE_BYTES;  // 1024-aligned (ring stages are)
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + C::STAGES * C::STAGE_BYTES + C::EPI_STG);
     uint64_t *full = bars, *empty = bars + C::STAGES, *tfull = bars + 2 * C::STAGES, *tempty = tfull + 2;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(tempty + 2);
+    uint64_t *mbar = tempty + 2;  // [4 warps][2] mask-tile barriers (EPI_MASK)
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(mbar + 8);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) PROBE(0);
     uint32_t rank = 0;
     if (CG == 2) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
     const int pair = blockIdx.x / CG, npairs = gridDim.x / CG;
@@ -381,6 +502,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int a = 0; a < 2; ++a) {
             mbar_init(smem_u32(&tfull[a]), 1);
             mbar_init(smem_u32(&tempty[a]), 4 * CG);  // one arrival per epilogue warp of the pair
+        }
+        for (int a = 0; a < 8; ++a) mbar_init(smem_u32(&mbar[a]), 1);
+        if (EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) {
+            asm volatile("prefetch.tensormap [%0];" ::"l"(&tmO) : "memory");
+            if (EPI == EPI_MASK) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmK) : "memory");
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -414,6 +540,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    if (threadIdx.x == 0) PROBE(1);
 
     if (warp == 0) {
         // ===== TMA producer =====
@@ -453,6 +580,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kb = kb0; kb < kb1; ++kb) {
                     if (PF && kb + PF < kb1) prefetch(kb + PF);
                     mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                    if (kb == kb0 && unit == pair) PROBE(2);
                     // CG = 2: both CTAs' bytes land on the LEADER's full barrier (peer bit cleared)
                     const uint32_t fb = smem_u32(&full[stage]) & (CG == 2 ? 0xFEFFFFFFu : 0xFFFFFFFFu);
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
@@ -525,6 +653,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kb = kb0; kb < kb1; ++kb) {
                     mbar_wait(smem_u32(&full[stage]), phase);
                     tc_fence_after();
+                    if (kb == kb0 && unit == pair) PROBE(3);
+                    if (kb == kb0 + 1 && unit == pair) PROBE(7);
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
                     const uint32_t sb = sa + C::A_BYTES;
                     if (CG == 1 && e.conv.c8 == 1) {
@@ -563,6 +693,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     tc_commit_cg<CG>(smem_u32(&empty[stage]));  // frees the slot (both CTAs) when done
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
                 }
+                PROBE(4);
                 tc_commit_cg<CG>(smem_u32(&tfull[acc]));  // accumulator ready for both epilogues
                 if (++acc == 2) { acc = 0; acc_phase ^= 1; }
             }
@@ -572,16 +703,75 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         const int q = warp & 3;  // TMEM lane quarter this warp may access
         int acc = 0;
         uint32_t acc_phase = 0;
+        uint32_t ocnt = 0, mcnt = 0, mph = 0;  // staging-buffer / mask-buffer counters and phases
         for (int unit = pair; unit < units; unit += npairs) {
             const int tile = unit % tiles, split = unit / tiles;
             const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM, n0 = (tile / m_blocks) * BN;
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
             tc_fence_after();
+            if (warp == 4 && lane == 0) PROBE(5);
             const int row = m0 + q * 32 + lane;
             EpiArgs es = e;
             if (EPI == EPI_F32) es.out = static_cast<float *>(e.out) + (long)split * e.split_stride;
             const bool empty_range = split * kper >= kblocks;  // (host avoids it; be safe)
             const bool reduce = EPI == EPI_F32 && e.counters != nullptr;  // in-kernel split-K
+            if ((EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) && !(e.dbg & 32)) {
+                // ---- TMA-store epilogue: rows m0+32q.., one 32 x 32 chunk at a time
+                uint8_t *wst = epi_stg + q * C::WARP_STG;
+                const int r0 = m0 + q * 32;
+                const int nch = min(BN / 32, (N - n0 + 31) / 32);
+                if (EPI == EPI_MASK && lane == 0 && nch > 0) {
+                    uint8_t *mt = wst + 2 * C::OUT_TILE + (mcnt & 1) * 2048;
+                    mbar_expect_tx(smem_u32(&mbar[q * 2 + (mcnt & 1)]), 2048);
+                    tma_load_2d(smem_u32(mt), &tmK, smem_u32(&mbar[q * 2 + (mcnt & 1)]), n0, r0);
+                }
+#pragma unroll 1
+                for (int c = 0; c < nch; ++c) {
+                    if (EPI == EPI_MASK && lane == 0 && c + 1 < nch) {
+                        // prefetch the next chunk's mask tile into the other buffer
+                        const uint32_t nb = (mcnt + 1) & 1;
+                        mbar_expect_tx(smem_u32(&mbar[q * 2 + nb]), 2048);
+                        tma_load_2d(smem_u32(wst + 2 * C::OUT_TILE + nb * 2048), &tmK, smem_u32(&mbar[q * 2 + nb]),
+                                    n0 + (c + 1) * 32, r0);
+                    }
+                    float v[32];
+                    tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, v);
+                    if (warp == 4 && lane == 0 && c == 0) PROBE(8);
+                    if (empty_range && e.atomic_out) continue;
+                    if (empty_range) {
+#pragma unroll
+                        for (int i = 0; i < 32; ++i) v[i] = 0.f;
+                    }
+                    const uint8_t *mt = nullptr;
+                    if constexpr (EPI == EPI_MASK) {
+                        const uint32_t b = mcnt & 1;
+                        mbar_wait(smem_u32(&mbar[q * 2 + b]), (mph >> b) & 1);
+                        mph ^= 1u << b;
+                        mt = wst + 2 * C::OUT_TILE + b * 2048;
+                    }
+                    epi_math<EPI>(es, v, row, n0 + c * 32, N, mt, lane);
+                    if constexpr (EPI == EPI_MASK) {
+                        __syncwarp();  // every lane has read this mask buffer before it is refilled
+                        ++mcnt;
+                    }
+                    // the store issued two chunks ago has finished reading this staging buffer
+                    if (lane == 0) bulk_wait_read1();
+                    __syncwarp();
+                    uint8_t *ot = wst + (ocnt & 1) * C::OUT_TILE;
+                    epi_stage<EPI>(ot, v, lane);
+                    fence_proxy_async();
+                    __syncwarp();
+                    if (lane == 0) {
+                        if (EPI == EPI_F32 && e.atomic_out) tma_reduce_add_2d(&tmO, smem_u32(ot), n0 + c * 32, r0);
+                        else if (EPI == EPI_F32 && e.split_stride) tma_store_3d(&tmO, smem_u32(ot), n0 + c * 32, r0, split);
+                        else tma_store_2d(&tmO, smem_u32(ot), n0 + c * 32, r0);
+                        bulk_commit();
+                    }
+                    ++ocnt;
+                    if (warp == 4 && lane == 0 && c < 2) PROBE(9 + c);
+                }
+                if (reduce && lane == 0) bulk_wait0();  // partials visible before the split counter
+            } else {
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
                 float v[32];
@@ -593,6 +783,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 }
                 if (n0 + c * 32 < N) epilogue_chunk<EPI>(es, v, row, n0 + c * 32, M, N);
             }
+            }
+            if (warp == 4 && lane == 0) PROBE(11);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) {
@@ -648,6 +840,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 }
             }
         }
+        if (EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) {
+            if (lane == 0) bulk_wait0();  // every bulk store complete before the CTA retires
+        }
+        if (warp == 4 && lane == 0) PROBE(6);
     }
     tc_fence_before();
     if (CG == 2) {
@@ -675,15 +871,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 // conflict-free thanks to the swizzle) and one thread writes the tiles back with TMA bulk
 // stores.  Everything moves as full lines with the TMA engine's queue depth instead of
 // per-thread 16-byte accesses.
-__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t src, int c0, int c1) {
-    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(map), "r"(src),
-                 "r"(c0), "r"(c1)
-                 : "memory");
-}
-__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 
 template <int BN, bool ADAM>
@@ -931,15 +1118,16 @@ struct MapKey {
     const void *base;
     long inner, outer, ld;
     int bi, bo, f32, sw;
+    long planes = 0;  // 3-D maps: number of [outer][inner] planes (plane stride outer*ld)
     bool operator==(const MapKey &o) const {
         return base == o.base && inner == o.inner && outer == o.outer && ld == o.ld && bi == o.bi && bo == o.bo &&
-               f32 == o.f32 && sw == o.sw;
+               f32 == o.f32 && sw == o.sw && planes == o.planes;
     }
 };
 struct MapKeyHash {
     size_t operator()(const MapKey &k) const {
         size_t h = std::hash<const void *>()(k.base);
-        for (long v : {k.inner, k.outer, k.ld, (long)k.bi, (long)k.bo, (long)(k.f32 * 1024 + k.sw)})
+        for (long v : {k.inner, k.outer, k.ld, (long)k.bi, (long)k.bo, (long)(k.f32 * 1024 + k.sw), k.planes})
             h = h * 1000003u ^ std::hash<long>()(v);
         return h;
     }
@@ -947,6 +1135,8 @@ struct MapKeyHash {
 
 bool encode_map(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner,
                 int box_outer, bool f32, int swizzle_bytes);
+bool make_map3_f32(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, long planes,
+                   int box_inner, int box_outer, int swizzle_bytes);
 
 // Tensor maps are encoded once per (buffer, shape, box) and reused: encoding costs a driver
 // call on every launch otherwise, and the runtime's buffers are stable for a context's life.
@@ -960,6 +1150,34 @@ bool make_map(CUtensorMap *map, const void *base, long inner, long outer, long l
         return true;
     }
     if (!encode_map(map, base, inner, outer, ld_elems, box_inner, box_outer, f32, swizzle_bytes)) return false;
+    if (cache.size() > 65536) cache.clear();
+    cache.emplace(key, *map);
+    return true;
+}
+
+// 3-D fp32 map over `planes` stacked [outer][inner] matrices (split-K partials: one plane per
+// split, so a tile's out-of-range rows are clipped at its own split's M, not the next split's)
+bool make_map3_f32(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, long planes,
+                   int box_inner, int box_outer, int swizzle_bytes) {
+    thread_local std::unordered_map<MapKey, CUtensorMap, MapKeyHash> cache;
+    MapKey key{base, inner, outer, ld_elems, box_inner, box_outer, 1, swizzle_bytes};
+    key.planes = planes;
+    auto it = cache.find(key);
+    if (it != cache.end()) {
+        *map = it->second;
+        return true;
+    }
+    const Driver *d = driver();
+    if (!d) return false;
+    cuuint64_t dims[3] = {(cuuint64_t)inner, (cuuint64_t)outer, (cuuint64_t)planes};
+    cuuint64_t strides[2] = {(cuuint64_t)ld_elems * 4, (cuuint64_t)ld_elems * 4 * outer};
+    cuuint32_t box[3] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer, 1};
+    cuuint32_t estr[3] = {1, 1, 1};
+    CUresult r = d->tensorMapEncodeTiled(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<void *>(base), dims,
+                                         strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                         swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return false;
     if (cache.size() > 65536) cache.clear();
     cache.emplace(key, *map);
     return true;
@@ -995,9 +1213,49 @@ int num_sms() {
     return n;
 }
 
+// tools only: PD_GEMM_PROBE=<file> appends one line per launch with each CTA's phase stamps
+// (ns since the earliest kernel-entry stamp): entry, setup done, first TMA issued, first stage
+// full, second stage full, last MMA issued, accumulator ready, epilogue done
+static unsigned long long *probe_buf() {
+    static unsigned long long *p = nullptr;
+    static bool init = false;
+    if (!init) {
+        init = true;
+        if (getenv("PD_GEMM_PROBE") && cudaMalloc(&p, 1024 * 16 * sizeof(unsigned long long)) != cudaSuccess) p = nullptr;
+        if (p) cudaMemset(p, 0, 1024 * 16 * sizeof(unsigned long long));
+    }
+    return p;
+}
+static void probe_dump(int grid, const Gemm &g, int bn, int cg, int ksplit) {
+    unsigned long long *p = probe_buf();
+    if (!p) return;
+    std::vector<unsigned long long> h((size_t)grid * 16);
+    cudaDeviceSynchronize();
+    cudaMemcpy(h.data(), p, h.size() * 8, cudaMemcpyDeviceToHost);
+    unsigned long long t0 = ~0ull;
+    for (int b = 0; b < grid; ++b) t0 = std::min(t0, h[b * 16]);
+    FILE *f = fopen(getenv("PD_GEMM_PROBE"), "a");
+    if (!f) return;
+    fprintf(f, "M=%d N=%d K=%d BN=%d CG=%d S=%d grid=%d", g.M, g.N, g.K, bn, cg, ksplit, grid);
+    const int order[12] = {0, 1, 2, 3, 7, 4, 5, 8, 9, 10, 11, 6};
+    for (int b = 0; b < grid; ++b) {
+        fprintf(f, " |");
+        for (int i : order) fprintf(f, " %lld", h[b * 16 + i] ? (long long)(h[b * 16 + i] - t0) : -1LL);
+    }
+    fprintf(f, "\n");
+    fclose(f);
+    cudaMemset(p, 0, 1024 * 16 * sizeof(unsigned long long));
+}
+
 template <int BN, int AMAJ, int BMAJ, int EPI, int CG>
-cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e, cudaStream_t s) {
-    using C = Cfg<BN / CG>;
+cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, const EpiArgs &e0, cudaStream_t s) {
+    using C = Cfg<BN / CG, EPI>;
+    EpiArgs e = e0;
+    e.probe = probe_buf();
+    {
+        static const int dbg = getenv("PD_EPI_DEBUG") ? atoi(getenv("PD_EPI_DEBUG")) : 0;
+        e.dbg = dbg;
+    }
     auto kern = tc_gemm_kernel<BN, AMAJ, BMAJ, EPI, CG>;
     static bool attr_set = false;  // per instantiation; benign race (idempotent)
     if (!attr_set) {
@@ -1005,11 +1263,27 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         if (err != cudaSuccess) return err;
         attr_set = true;
     }
+    // epilogue tensor maps: output tile {32 cols, 32 rows} (bf16 64B-swizzled / fp32 128B-swizzled;
+    // split-K partials stacked as [S*M][N]) and the ReLU-mask tile
+    CUtensorMap mo = ma, mk = ma;
+    if (EPI == EPI_STORE || EPI == EPI_MASK) {
+        if (!make_map(&mo, e.out, g.N, g.M, e.ldo, 32, 32, false, 64)) return cudaErrorInvalidValue;
+        if (EPI == EPI_MASK && !make_map(&mk, e.mask, g.N, g.M, e.ldm, 32, 32, false, 64))
+            return cudaErrorInvalidValue;
+    } else if (EPI == EPI_F32) {
+        if (!e.atomic_out && e.split_stride) {
+            if (e.split_stride != (long)g.M * e.ldo ||
+                !make_map3_f32(&mo, e.out, g.N, g.M, e.ldo, e.ksplit, 32, 32, 128))
+                return cudaErrorInvalidValue;
+        } else if (!make_map(&mo, e.out, g.N, g.M, e.ldo, 32, 32, true, 128)) {
+            return cudaErrorInvalidValue;
+        }
+    }
     const int units = ((g.M + BM * CG - 1) / (BM * CG)) * ((g.N + BN - 1) / BN) * e.ksplit;
     const int slots = num_sms() / CG;
     const int grid = CG * (units < slots ? units : slots);
     if (CG == 1) {
-        kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, e, g.M, g.N, g.K);
+        kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, mo, mk, e, g.M, g.N, g.K);
     } else {
         cudaLaunchConfig_t cfg{};
         cfg.gridDim = dim3(grid);
@@ -1023,9 +1297,10 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         attr[0].val.clusterDim.z = 1;
         cfg.attrs = attr;
         cfg.numAttrs = 1;
-        cudaError_t err = cudaLaunchKernelEx(&cfg, kern, ma, mb, e, g.M, g.N, g.K);
+        cudaError_t err = cudaLaunchKernelEx(&cfg, kern, ma, mb, mo, mk, e, g.M, g.N, g.K);
         if (err != cudaSuccess) return err;
     }
+    if (e.probe) probe_dump(grid, g, BN, CG, e.ksplit);
     ++tl_launches;
     return cudaGetLastError();
 }

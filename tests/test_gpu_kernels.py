@@ -49,7 +49,10 @@ def test_tc_gemm_f32_out(M, N, K, amn, bmn):
 
 
 @pytest.mark.parametrize("split", [False, True])
-@pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES[:4])
+@pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES[:4] + [
+    (32, 4096, 4096, 0, 0),    # small-M split-K: 8 splits of a 128-row tile holding 32 rows
+    (40, 4096, 2048, 0, 1),    # ragged rows inside an epilogue warp's 32-row slab
+])
 def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split):
     A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16, seed=1)
     bias = torch.randn(N, device="cuda")
@@ -64,8 +67,8 @@ def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split):
 
 
 @pytest.mark.parametrize("split", [False, True])
-def test_tc_gemm_mask_epilogue(split):
-    M, N, K = 256, 1024, 4096
+@pytest.mark.parametrize("M,N,K", [(256, 1024, 4096), (40, 4096, 4096)])
+def test_tc_gemm_mask_epilogue(split, M, N, K):
     A, B, As, Bs = _operands(M, N, K, 0, 1, torch.bfloat16, seed=2)
     mask = torch.relu(torch.randn(M, N, device="cuda")).to(torch.bfloat16)
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
