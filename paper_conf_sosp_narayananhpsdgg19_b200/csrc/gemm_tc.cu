@@ -46,7 +46,8 @@ struct Cfg {
     // epilogue staging per epilogue warp (TMA-store epilogue): two 32 x 32 output tiles (fp32
     // 4 KB or bf16 2 KB each, swizzled) + two bf16 mask tiles (EPI_MASK)
     static constexpr int OUT_TILE = EPI == EPI_F32_ ? 4096 : 2048;
-    static constexpr int WARP_STG = EPI > EPI_F32_ ? 0 : 2 * OUT_TILE + (EPI == EPI_MASK_ ? 2 * 2048 : 0);
+    // (STORE / MASK also host the cluster split-K output slice: up to 4 x [128][32] bf16 = 32 KB)
+    static constexpr int WARP_STG = EPI > EPI_F32_ ? 0 : (EPI == EPI_F32_ ? 2 * OUT_TILE : 8192);
     static constexpr int EPI_STG = 4 * WARP_STG;
     static constexpr int STAGES_MAX = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
     static constexpr int STAGES_FIT = (232448 - 1024 - 256 - EPI_STG) / STAGE_BYTES;
@@ -63,7 +64,12 @@ struct EpiArgs {
     ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
     int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
     int l2_prefetch;    // producer L2-prefetch distance in K-blocks (0 = off; measured no gain so far)
-    int dbg;                    // tools only (PD_EPI_DEBUG): bit 0 skip epilogue global stores, bit 1 skip transpose
+    int dbg;                    // tools only (PD_EPI_DEBUG): bit 5 = old per-row epilogue
+    // cluster split-K (csplit > 1): the csplit K-ranges of one output tile run as one thread-block
+    // cluster (CG * csplit CTAs); partial accumulators are summed through distributed shared
+    // memory (each CTA reduces a 64-column slice, in split order) and the final bf16 epilogue is
+    // applied in the same kernel -- no fp32 partials in HBM, no second launch
+    int csplit;
     unsigned long long *probe;  // tools only (PD_GEMM_PROBE): per-CTA %globaltimer phase stamps [grid][8]
     // in-kernel split-K: each (tile, split) writes its fp32 partial to ws[split]; the last CTA
     // to finish a tile (per-tile counter) sums the partials in split order and applies the
@@ -159,11 +165,11 @@ __device__ __forceinline__ void tc_mma_cg(uint32_t d_tmem, uint64_t adesc, uint6
     }
 }
 template <int CG>
-__device__ __forceinline__ void tc_commit_cg(uint32_t bar) {
+__device__ __forceinline__ void tc_commit_cg(uint32_t bar, uint16_t mask = 0x3) {
     if (CG == 1) {
         tc_commit(bar);
     } else {
-        const uint16_t mask = 0x3;  // arrive on the barrier at this offset in both CTAs of the pair
+        // arrive on the barrier at this offset in both CTAs of the pair (mask = the pair's ranks)
         asm volatile(
             "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
                 bar),
@@ -386,6 +392,30 @@ __device__ __forceinline__ void tma_store_3d(const CUtensorMap *map, uint32_t sr
                  "r"(src), "r"(c0), "r"(c1), "r"(c2)
                  : "memory");
 }
+__device__ __forceinline__ void st_shared_v4(uint32_t addr, float a, float b, float c, float d) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "f"(a), "f"(b), "f"(c), "f"(d) : "memory");
+}
+__device__ __forceinline__ void st_shared_v4u(uint32_t addr, uint4 v) {
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                 : "memory");
+}
+__device__ __forceinline__ uint32_t mapa_cluster(uint32_t addr, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ float4 ld_dsmem_v4(uint32_t addr) {
+    float4 v;
+    asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+                 : "r"(addr)
+                 : "memory");
+    return v;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
 __device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
 
 // TMA-store epilogue (STORE / MASK / F32).  Each epilogue warp owns 32 accumulator rows; a
@@ -482,14 +512,21 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) PROBE(0);
-    uint32_t rank = 0;
-    if (CG == 2) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    uint32_t crank = 0;  // rank in the cluster (pair, or pair x cluster split)
+    if (CG == 2 || e.csplit > 1) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+    const uint32_t rank = CG == 2 ? (crank & 1u) : 0u;                  // rank in the CTA pair
+    const uint16_t pmask = (uint16_t)(3u << (crank & ~1u));              // the pair's CTAs
     const int pair = blockIdx.x / CG, npairs = gridDim.x / CG;
     const int m_blocks = (M + BM * CG - 1) / (BM * CG), n_blocks = (N + BN - 1) / BN;
     const int tiles = m_blocks * n_blocks;
     const int kblocks = (K + BK - 1) / BK;
     const int units = tiles * e.ksplit;
     const int kper = (kblocks + e.ksplit - 1) / e.ksplit;
+    // persistent loop over units (tile, split); cluster split-K: exactly one unit per CTA
+    const int csplit = e.csplit > 1 ? e.csplit : 1;
+    const int my_split = (int)(crank / CG) % csplit;
+    const int u0 = csplit > 1 ? my_split * tiles + (int)(blockIdx.x / (CG * csplit)) : pair;
+    const int ustep = csplit > 1 ? units : npairs;
     constexpr uint32_t TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
 
     if (warp == 0 && lane == 0) {
@@ -547,7 +584,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            for (int unit = pair; unit < units; unit += npairs) {
+            for (int unit = u0; unit < units; unit += ustep) {
                 const int tile = unit % tiles, split = unit / tiles;
                 const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM;
                 const int n0 = (tile / m_blocks) * BN + (int)rank * BNC;
@@ -580,7 +617,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kb = kb0; kb < kb1; ++kb) {
                     if (PF && kb + PF < kb1) prefetch(kb + PF);
                     mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-                    if (kb == kb0 && unit == pair) PROBE(2);
+                    if (kb == kb0 && unit == u0) PROBE(2);
                     // CG = 2: both CTAs' bytes land on the LEADER's full barrier (peer bit cleared)
                     const uint32_t fb = smem_u32(&full[stage]) & (CG == 2 ? 0xFEFFFFFFu : 0xFFFFFFFFu);
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
@@ -644,7 +681,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             uint32_t phase = 0;
             int acc = 0;
             uint32_t acc_phase = 0;
-            for (int unit = pair; unit < units; unit += npairs) {
+            for (int unit = u0; unit < units; unit += ustep) {
                 const int split = unit / tiles;
                 const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
                 mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
@@ -653,8 +690,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 for (int kb = kb0; kb < kb1; ++kb) {
                     mbar_wait(smem_u32(&full[stage]), phase);
                     tc_fence_after();
-                    if (kb == kb0 && unit == pair) PROBE(3);
-                    if (kb == kb0 + 1 && unit == pair) PROBE(7);
+                    if (kb == kb0 && unit == u0) PROBE(3);
+                    if (kb == kb0 + 1 && unit == u0) PROBE(7);
                     const uint32_t sa = smem_u32(smem + stage * C::STAGE_BYTES);
                     const uint32_t sb = sa + C::A_BYTES;
                     if (CG == 1 && e.conv.c8 == 1) {
@@ -690,11 +727,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                                                          : smem_desc(sb + k * 2048, BK * 128, 1024);
                         tc_mma_cg<CG>(d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
                     }
-                    tc_commit_cg<CG>(smem_u32(&empty[stage]));  // frees the slot (both CTAs) when done
+                    tc_commit_cg<CG>(smem_u32(&empty[stage]), pmask);  // frees the slot (both CTAs) when done
                     if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
                 }
                 PROBE(4);
-                tc_commit_cg<CG>(smem_u32(&tfull[acc]));  // accumulator ready for both epilogues
+                tc_commit_cg<CG>(smem_u32(&tfull[acc]), pmask);  // accumulator ready for both epilogues
                 if (++acc == 2) { acc = 0; acc_phase ^= 1; }
             }
         }
@@ -704,7 +741,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         int acc = 0;
         uint32_t acc_phase = 0;
         uint32_t ocnt = 0, mcnt = 0, mph = 0;  // staging-buffer / mask-buffer counters and phases
-        for (int unit = pair; unit < units; unit += npairs) {
+        for (int unit = u0; unit < units; unit += ustep) {
             const int tile = unit % tiles, split = unit / tiles;
             const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM, n0 = (tile / m_blocks) * BN;
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
@@ -715,7 +752,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (EPI == EPI_F32) es.out = static_cast<float *>(e.out) + (long)split * e.split_stride;
             const bool empty_range = split * kper >= kblocks;  // (host avoids it; be safe)
             const bool reduce = EPI == EPI_F32 && e.counters != nullptr;  // in-kernel split-K
-            if ((EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) && !(e.dbg & 32)) {
+            if (csplit > 1) {
+                // ---- cluster split-K: this split's partial accumulator -> own shared memory
+                // (the operand ring is idle now), row-major [128][BN + 4] fp32
+                const uint32_t pbase = smem_u32(smem) + (uint32_t)((q * 32 + lane) * (BN + 4) * 4);
+#pragma unroll 1
+                for (int c = 0; c < BN / 32; ++c) {
+                    float v[32];
+                    tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, v);
+                    if (empty_range) {
+#pragma unroll
+                        for (int i = 0; i < 32; ++i) v[i] = 0.f;
+                    }
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        st_shared_v4(pbase + (uint32_t)((c * 32 + 4 * j) * 4), v[4 * j], v[4 * j + 1], v[4 * j + 2],
+                                     v[4 * j + 3]);
+                }
+            } else if ((EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) && !(e.dbg & 32)) {
                 // ---- TMA-store epilogue: rows m0+32q.., one 32 x 32 chunk at a time
                 uint8_t *wst = epi_stg + q * C::WARP_STG;
                 const int r0 = m0 + q * 32;
@@ -844,6 +898,71 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (lane == 0) bulk_wait0();  // every bulk store complete before the CTA retires
         }
         if (warp == 4 && lane == 0) PROBE(6);
+    }
+    if (csplit > 1) {
+        // ---- cluster split-K reduction: every split's partial is in its CTA's shared memory;
+        // split s sums columns [64 s, 64 s + 64) of its pair-rank's 128 rows over all splits
+        // (in split order: deterministic), applies the epilogue and stores that bf16 slice
+        cluster_sync_all();
+        if ((EPI == EPI_STORE || EPI == EPI_MASK) && warp >= 4) {
+            const int t = threadIdx.x - 128;
+            const int tile = blockIdx.x / (CG * csplit);
+            const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM, n0 = (tile / m_blocks) * BN;
+            // this split's columns: 32-column chunks [ch0, ch1) of the BN-wide tile
+            const int nb = BN / 32, ch0 = my_split * nb / csplit, ch1 = (my_split + 1) * nb / csplit;
+            const int c_lo = ch0 * 32, groups = (ch1 - ch0) * 4;  // 8-column groups
+            const uint32_t part = smem_u32(smem), ost = smem_u32(epi_stg);
+#pragma unroll 1
+            for (int item = t; item < 128 * groups; item += 128) {
+                const int r = item / groups, g = item % groups, col = c_lo + g * 8;
+                float x[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+                const uint32_t la = part + (uint32_t)((r * (BN + 4) + col) * 4);
+                for (int sp = 0; sp < csplit; ++sp) {
+                    const uint32_t ra = mapa_cluster(la, (uint32_t)(sp * CG) + rank);
+                    const float4 a = ld_dsmem_v4(ra), b = ld_dsmem_v4(ra + 16);
+                    x[0] += a.x; x[1] += a.y; x[2] += a.z; x[3] += a.w;
+                    x[4] += b.x; x[5] += b.y; x[6] += b.z; x[7] += b.w;
+                }
+                const int grow = m0 + r, gcol = n0 + col;
+                if constexpr (EPI == EPI_STORE) {
+                    if (e.bias) {
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) x[j] += (gcol + j < N) ? __ldg(e.bias + gcol + j) : 0.f;
+                    }
+                    if (e.relu) {
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) x[j] = fmaxf(x[j], 0.f);
+                    }
+                } else if constexpr (EPI == EPI_MASK) {
+                    if (grow < M && gcol + 8 <= N) {
+                        const uint4 raw = __ldg(reinterpret_cast<const uint4 *>(e.mask + (long)grow * e.ldm + gcol));
+                        const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw);
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) x[j] = (__bfloat162float(h[j]) > 0.f) ? x[j] : 0.f;
+                    } else {
+                        for (int j = 0; j < 8; ++j)
+                            x[j] = (grow < M && gcol + j < N && __bfloat162float(e.mask[(long)grow * e.ldm + gcol + j]) > 0.f)
+                                       ? x[j] : 0.f;
+                    }
+                }
+                uint4 w;
+                w.x = pack_bf16(x[0], x[1]);
+                w.y = pack_bf16(x[2], x[3]);
+                w.z = pack_bf16(x[4], x[5]);
+                w.w = pack_bf16(x[6], x[7]);
+                // staging: one 64B-swizzled [128 rows][32 cols] bf16 box per 32-column chunk
+                const int cb = g >> 2, j = g & 3;
+                st_shared_v4u(ost + (uint32_t)(cb * 8192 + r * 64 + ((j ^ ((r >> 1) & 3)) << 4)), w);
+            }
+            fence_proxy_async();
+            asm volatile("bar.sync 1, 128;" ::: "memory");
+            if (t == 0) {
+                for (int cb = 0; cb < ch1 - ch0; ++cb) tma_store_2d(&tmO, ost + cb * 8192, n0 + c_lo + 32 * cb, m0);
+                bulk_commit();
+                bulk_wait0();
+            }
+        }
+        cluster_sync_all();  // no CTA leaves while a peer may still read its partial
     }
     tc_fence_before();
     if (CG == 2) {
@@ -1266,7 +1385,11 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
     // epilogue tensor maps: output tile {32 cols, 32 rows} (bf16 64B-swizzled / fp32 128B-swizzled;
     // split-K partials stacked as [S*M][N]) and the ReLU-mask tile
     CUtensorMap mo = ma, mk = ma;
-    if (EPI == EPI_STORE || EPI == EPI_MASK) {
+    if (e.csplit > 1) {
+        // cluster split-K: each CTA stores a [128 rows][64 cols] bf16 slice
+        if (!(EPI == EPI_STORE || EPI == EPI_MASK) || !make_map(&mo, e.out, g.N, g.M, e.ldo, 32, 128, false, 64))
+            return cudaErrorInvalidValue;
+    } else if (EPI == EPI_STORE || EPI == EPI_MASK) {
         if (!make_map(&mo, e.out, g.N, g.M, e.ldo, 32, 32, false, 64)) return cudaErrorInvalidValue;
         if (EPI == EPI_MASK && !make_map(&mk, e.mask, g.N, g.M, e.ldm, 32, 32, false, 64))
             return cudaErrorInvalidValue;
@@ -1281,8 +1404,9 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
     }
     const int units = ((g.M + BM * CG - 1) / (BM * CG)) * ((g.N + BN - 1) / BN) * e.ksplit;
     const int slots = num_sms() / CG;
-    const int grid = CG * (units < slots ? units : slots);
-    if (CG == 1) {
+    const int grid = e.csplit > 1 ? CG * units : CG * (units < slots ? units : slots);
+    const int cluster = e.csplit > 1 ? CG * e.csplit : CG;
+    if (cluster == 1) {
         kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, mo, mk, e, g.M, g.N, g.K);
     } else {
         cudaLaunchConfig_t cfg{};
@@ -1292,7 +1416,7 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         cfg.stream = s;
         cudaLaunchAttribute attr[1];
         attr[0].id = cudaLaunchAttributeClusterDimension;
-        attr[0].val.clusterDim.x = 2;
+        attr[0].val.clusterDim.x = cluster;
         attr[0].val.clusterDim.y = 1;
         attr[0].val.clusterDim.z = 1;
         cfg.attrs = attr;
@@ -1434,6 +1558,44 @@ static int use_pairs(const Gemm &g) {
     return (g.M >= 256 && g.N > 64 && (g.epi == EPI_STORE || g.epi == EPI_MASK || g.epi == EPI_F32)) ? 2 : 1;
 }
 
+// thread-block clusters of `csize` CTAs that can be resident at once (GPC-limited: 15 of 8
+// CTAs on a 148-SM B200), for the ~1-CTA-per-SM GEMM kernels; cached per (CG, size)
+static int max_active_clusters(int cg, int csize) {
+    static int cache[3][9] = {};
+    if (csize < 1 || csize > 8) return 0;
+    int &c = cache[cg][csize];
+    if (c) return c;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(csize * 64);
+    cfg.blockDim = dim3(NUM_THREADS);
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = csize;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    int n = 0;
+    cudaError_t err;
+    if (cg == 2) {
+        auto k = tc_gemm_kernel<256, KMAJ, KMAJ, EPI_STORE, 2>;
+        cfg.dynamicSmemBytes = Cfg<128, EPI_STORE>::SMEM;
+        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cfg.dynamicSmemBytes);
+        err = cudaOccupancyMaxActiveClusters(&n, k, &cfg);
+    } else {
+        auto k = tc_gemm_kernel<256, KMAJ, KMAJ, EPI_STORE, 1>;
+        cfg.dynamicSmemBytes = Cfg<256, EPI_STORE>::SMEM;
+        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cfg.dynamicSmemBytes);
+        err = cudaOccupancyMaxActiveClusters(&n, k, &cfg);
+    }
+    if (err != cudaSuccess) {
+        cudaGetLastError();
+        n = 0;
+    }
+    c = n > 0 ? n : -1;
+    return c;
+}
+
 static int choose_ksplit(const Gemm &g, int sms) {
     if (!(g.epi == EPI_STORE || g.epi == EPI_MASK) || !g.workspace || g.N % 4 || g.ldo != g.N || g.conv.taps)
         return 1;
@@ -1494,6 +1656,43 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
     {
         const int S = choose_ksplit(g, num_sms());
+        const int cg0 = use_pairs(g);
+        const long ctiles = (long)((g.M + BM * cg0 - 1) / (BM * cg0)) * ((g.N + 255) / 256);
+        int CS = 0;  // cluster split count: the largest of 4, 3, 2 whose clusters all fit in one wave
+        const int csenv = env_int("PD_GEMM_CSPLIT", 1);
+        // bit 0: forward (EPI_STORE) GEMMs, bit 1: dX (EPI_MASK) GEMMs.  Clusters need CG*CS free SMs
+        // in one GPC at launch: the dX GEMMs overlap the side stream's dW kernels, which keep SMs
+        // busy; measured in the MLP step: forward only -6 %, both -13 % -> off by default (kept for
+        // standalone GEMMs: PD_GEMM_CSPLIT_EPI=3)
+        const int csepi = env_int("PD_GEMM_CSPLIT_EPI", 0);
+        const bool epi_ok = (g.epi == EPI_STORE && (csepi & 1)) || (g.epi == EPI_MASK && (csepi & 2));
+        if (S >= 3 && csenv && epi_ok && g.N % 8 == 0)
+            for (int cs = csenv > 1 ? csenv : 4; cs >= 2 && !CS; --cs)
+                if ((g.K + BK - 1) / BK >= cs && ctiles <= max_active_clusters(cg0, cg0 * cs)) CS = cs;
+        if (getenv("PD_GEMM_CSPLIT_DEBUG"))
+            fprintf(stderr, "csplit: tiles %ld S %d maxclusters(%d)=%d (%d)=%d (%d)=%d -> CS %d\n", ctiles, S, cg0 * 4,
+                    max_active_clusters(cg0, cg0 * 4), cg0 * 3, max_active_clusters(cg0, cg0 * 3), cg0 * 2,
+                    max_active_clusters(cg0, cg0 * 2), CS);
+        if (CS) {
+            // cluster split-K: CS K-ranges of a 256-wide tile reduced through DSMEM, one launch
+            CUtensorMap ma, mbm;
+            const int cg = cg0;
+            const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
+                                            : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
+            const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, 256 / cg)
+                                            : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
+            if (!okA || !okB) return cudaErrorInvalidValue;
+            EpiArgs e{};
+            e.out = g.out;
+            e.ldo = g.ldo;
+            e.ksplit = CS;
+            e.csplit = CS;
+            e.bias = g.epi == EPI_STORE ? g.bias : nullptr;
+            e.relu = g.epi == EPI_STORE ? g.relu : 0;
+            e.mask = g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr;
+            e.ldm = g.ldm;
+            return cg == 2 ? dispatch_major<256, 2>(g, ma, mbm, e, s) : dispatch_major<256>(g, ma, mbm, e, s);
+        }
         if (S > 1) {
             CUtensorMap ma, mbm;
             const int cg = use_pairs(g);
