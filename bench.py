@@ -141,6 +141,48 @@ def dw_update_bytes(L, B):
     return B * L.out * 2 + B * L.in_ * 2 + L.out * L.in_ * (4 + 4 + 2)
 
 
+def stage_roofline(layers, plan, B, peaks, optimizer, nvlink_gbs=900.0):
+    """north_star / SURVEY §8(d) per-stage roofline:
+        samples/s = B * min_s R_s / max(F_s / P_tensor, H_s / BW_HBM, N_s / BW_NVL)
+    F_s = GEMM FLOPs per minibatch (6 per MAC; the model's first layer has no dX);
+    H_s = algorithmic HBM bytes per minibatch: bf16 weight reads fwd + bwd (4 B/param),
+          the update (fp32 master r+w 8 B + new bf16 version 2 B; Adam m, v r+w +16 B),
+          activation stash write + read of every layer input, logits write + read for CE;
+    N_s = NVLink bytes: activation out + gradient out (+ ring allreduce 2(R-1)/R grad bytes).
+    Peaks: sustained bf16 tensor (a step is a long run) and the measured HBM copy bandwidth."""
+    import synth
+    per = []
+    for s, (first, last, R, _g) in enumerate(plan.stages):
+        F = H = Nb = 0.0
+        P = 0
+        for l in range(first, last + 1):
+            L = layers[l]
+            f = layer_flops(L, B)
+            if l == 0:
+                f *= 2.0 / 3.0
+            F += f
+            p = synth.param_count(L)
+            P += p
+            H += p * (4 + 10 + (16 if optimizer == synth.ADAM else 0))
+            in_bytes = layer_out_bytes(layers[l - 1], B) if l > 0 else 0
+            H += 2 * in_bytes
+        if last == len(layers) - 1:
+            H += 2 * layer_out_bytes(layers[-1], B)
+        if last < len(layers) - 1:
+            Nb += layer_out_bytes(layers[last], B)
+        if first > 0:
+            Nb += layer_out_bytes(layers[first - 1], B)
+        if R > 1:
+            Nb += 2.0 * (R - 1) / R * 4 * P
+        t = max(F / (peaks["bf16_tflops_sustained"] * 1e12), H / (peaks["hbm_gbs"] * 1e9), Nb / (nvlink_gbs * 1e9))
+        bound = ["tensor", "hbm", "nvlink"][int(np.argmax([F / (peaks["bf16_tflops_sustained"] * 1e12),
+                                                            H / (peaks["hbm_gbs"] * 1e9), Nb / (nvlink_gbs * 1e9)]))]
+        per.append({"stage": s, "gflop": F / 1e9, "hbm_gb": H / 1e9, "nvlink_mb": Nb / 1e6, "bound": bound,
+                    "samples_per_s": B * R / t})
+    slow = min(range(len(per)), key=lambda i: per[i]["samples_per_s"])
+    return per[slow]["samples_per_s"], slow, per
+
+
 def gemm_flops(L, B):
     return 2.0 * B * L.in_ * L.out
 
@@ -213,7 +255,8 @@ def main():
     ap.add_argument("--config", default="mlp4096", choices=["mlp4096", "gnmt8", "gnmt16", "vgg16"])
     ap.add_argument("--minibatches", type=int, default=0, help="minibatches per step (default 8, 16n for n>1)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--cpu-batch", type=int, default=8)
+    ap.add_argument("--cpu-batch", type=int, default=0,
+                    help="samples in the oracle's bounded sample (default: 8 for mlp4096, 1 otherwise -- ~10-60 s)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--plan", default="pipeline", choices=["pipeline", "dp"],
@@ -222,6 +265,8 @@ def main():
     ap.add_argument("--sync", default="stash", choices=["stash", "vertical"],
                     help="weight stashing (default) or vertical sync (§3.3; straight plans)")
     args = ap.parse_args()
+    if args.cpu_batch <= 0:
+        args.cpu_batch = 8 if args.config == "mlp4096" else 1
     if args.impl == "reference":
         return run_reference(args)
 
@@ -392,6 +437,7 @@ def main():
                "d2h_bytes_per_step": int(M * 4),
                "note": "wall clock around set_data(pinned host) + pd_run + pd_get_losses, max over ranks"}
 
+    roof_sps, roof_slow, roof_stages = stage_roofline(layers, plan, B, peaks, wl.optimizer)
     cpu = None
     if rank == 0 and N == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args, layers, wl)
@@ -428,6 +474,10 @@ def main():
                             "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"},
             "step_share": step_share,
             "stage_tflops": stage_flops * args.steps * M / plan.stages[s_mine][2] / (total_ms / 1e3) / 1e12,
+            "pipeline_roofline": {"samples_per_s": roof_sps, "frac": value / roof_sps, "slowest_stage": roof_slow,
+                                  "stages": roof_stages,
+                                  "definition": "B * min_s R_s / max(F_s/P_tensor_sustained, H_s/BW_HBM, "
+                                                "N_s/900 GB/s) (north_star; bench.stage_roofline)"},
             "e2e": e2e,
             "cpu_baseline": cpu,
         }

@@ -61,6 +61,36 @@ PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *g, void *stream);
 PD_API pd_status pd_kernel_softmax_ce(int dtype, const void *logits, const int32_t *labels, long rows, int C,
                                       void *dlogits, float *loss, void *stream);
 
+/* The recurrent half of one LSTM layer (bf16 path, R22: PyTorch form, gates i, f, g,
+ * o; h0 = c0 = 0), all T steps in ONE persistent launch (csrc/lstm_rec.cu): W_hh stays in
+ * shared memory, step t waits only for the K-blocks of h[t-1] (da[t+1]) it multiplies.
+ *   direction 0 (forward):  a = gx[t] + b_ih + b_hh + h[t-1] W_hh^T  (gx = X W_ih^T, fp32
+ *       [T][B][4H]) -> gates fp32 [T][B][4H] (sigmoid/tanh activations i, f, g, o),
+ *       c fp32 [T][B][H], h bf16 [T][B][H]        (LSTM-gate layers)
+ *   direction 1 (backward through time): dh = dy[t] + da[t+1] W_hh; cell backward with the
+ *       saved gates / c -> da bf16 [T][B][4H] (pre-activation gate gradients; dc carried on
+ *       chip)                                       (row a7)
+ * w_hh: bf16 [4H][H] (the weight version the op uses).  counters: device uint32 scratch of at
+ * least 4H/64 entries, zeroed by this call on `stream`.  probe: optional device uint64
+ * [grid][T][8] %globaltimer phase stamps (tools/lstm_probe.py), NULL = off.
+ * All pointers are DEVICE pointers owned by the caller; asynchronous on `stream`.
+ * Errors: PD_EUNSUPPORTED (H % 256 != 0, H > 1024, B > 64, or the clustered grid cannot be
+ * co-resident on this GPU), PD_EINVAL (null pointer / bad direction), PD_ECUDA. */
+typedef struct {
+    int direction;
+    int T, B, H;
+    const float *gx, *b_ih, *b_hh;
+    const void *w_hh;
+    float *gates, *c;
+    void *h;
+    const void *dy;
+    void *da;
+    unsigned *counters;
+    unsigned long long *probe;
+} pd_lstm_rec_desc;
+
+PD_API pd_status pd_kernel_lstm_rec(const pd_lstm_rec_desc *d, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

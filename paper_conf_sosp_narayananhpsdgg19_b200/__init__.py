@@ -80,6 +80,13 @@ class Stats(C.Structure):
                 ("kern_ms", C.c_double * 4), ("kern_count", C.c_uint64 * 4)]
 
 
+class LstmRecDesc(C.Structure):
+    _fields_ = [("direction", C.c_int), ("T", C.c_int), ("B", C.c_int), ("H", C.c_int), ("gx", C.c_void_p),
+                ("b_ih", C.c_void_p), ("b_hh", C.c_void_p), ("w_hh", C.c_void_p), ("gates", C.c_void_p),
+                ("c", C.c_void_p), ("h", C.c_void_p), ("dy", C.c_void_p), ("da", C.c_void_p),
+                ("counters", C.c_void_p), ("probe", C.c_void_p)]
+
+
 class GemmDesc(C.Structure):
     _fields_ = [("dtype", C.c_int), ("M", C.c_int), ("N", C.c_int), ("K", C.c_int), ("A", C.c_void_p),
                 ("lda", C.c_long), ("a_mn_major", C.c_int), ("B", C.c_void_p), ("ldb", C.c_long),
@@ -112,6 +119,7 @@ def _load():
         "pd_set_timing": [vp, i, i],
         "pd_kernel_gemm": [vp, vp],
         "pd_kernel_softmax_ce": [i, vp, vp, C.c_long, i, vp, vp, vp],
+        "pd_kernel_lstm_rec": [vp, vp],
     }
     for name, args in sigs.items():
         f = getattr(L, name)
@@ -131,6 +139,7 @@ lib = _load()
 EXPORTED = ["pd_plan", "pd_create", "pd_stage_init", "pd_export_worker", "pd_import_worker", "pd_set_data", "pd_run",
             "pd_get_params", "pd_get_trace", "pd_get_version_map", "pd_get_losses", "pd_get_stats", "pd_destroy",
             "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce",
+            "pd_kernel_lstm_rec",
             "pd_set_timing"]
 
 
@@ -334,3 +343,10 @@ def pd_kernel_gemm(dtype, M, N, K, A, lda, B, ldb, out=None, ldo=0, a_mn_major=0
 
 def pd_kernel_softmax_ce(dtype, logits, labels, rows, Cn, dlogits, loss, stream=None):
     _check(lib.pd_kernel_softmax_ce(dtype, logits, labels, rows, Cn, dlogits, loss, stream))
+
+
+def pd_kernel_lstm_rec(direction, T, B, H, w_hh, gates, c, counters, gx=None, b_ih=None, b_hh=None, h=None,
+                       dy=None, da=None, probe=None, stream=None):
+    """One LSTM layer's recurrence in one persistent launch (device addresses as ints)."""
+    d = LstmRecDesc(direction, T, B, H, gx, b_ih, b_hh, w_hh, gates, c, h, dy, da, counters, probe)
+    _check(lib.pd_kernel_lstm_rec(C.byref(d), stream))

@@ -109,6 +109,10 @@ struct Gemm {
     int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
 };
 
+// cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}
+bool tma_map_bf16(CUtensorMap *map, const void *base, long inner, long outer, long ld_elems, int box_inner,
+                  int box_outer);
+
 // fp32 SIMT GEMM (parity path; no tensor cores, no TF32).  EPI_STORE/MASK/F32 only.
 cudaError_t gemm_f32(const Gemm &g, cudaStream_t s);
 // bf16 tcgen05/TMEM/TMA GEMM, fp32 accumulation.  All epilogues.
@@ -144,6 +148,20 @@ cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s);
 cudaError_t lstm_cell_fwd(int bf16, const float *gx, const float *gh, const float *b_ih, const float *b_hh,
                           const float *c_prev, float *gates, float *c_out, void *h_out, void *y_out, int B, int H,
                           cudaStream_t s);
+// Persistent weight-stationary LSTM recurrences (lstm_rec.cu, bf16 path): all T steps of one
+// layer in ONE launch; W_hh slices stay in shared memory, the step-to-step dependency is a
+// per-K-block counter in `cnt` (>= 4H/64 uints, zeroed by the caller before each launch).
+//   fwd: gates/c/h[t] from gx[t] (= X W_ih^T, [T][B][4H] fp32) + h[t-1] W_hh^T + b_ih + b_hh
+//   bwd: da[t] from dy[t] + da[t+1] W_hh and the saved gates / c (dc carried on chip)
+// lstm_rec_supported: shape (H % 256 == 0, H <= 1024, 1 <= B <= 64) and co-residency of the
+// clustered grid on this device; callers fall back to the per-step path otherwise.
+bool lstm_rec_supported(int B, int H);
+cudaError_t lstm_rec_fwd(const float *gx, const float *b_ih, const float *b_hh, const __nv_bfloat16 *Whh,
+                         float *gates, float *c, __nv_bfloat16 *h, unsigned *cnt, int T, int B, int H, cudaStream_t s,
+                         unsigned long long *probe = nullptr);
+cudaError_t lstm_rec_bwd(const __nv_bfloat16 *dy, const float *gates, const float *c, const __nv_bfloat16 *Whh,
+                         __nv_bfloat16 *da, unsigned *cnt, int T, int B, int H, cudaStream_t s,
+                         unsigned long long *probe = nullptr);
 cudaError_t lstm_cell_bwd(int bf16, const void *dy, const float *dh_rec, const float *gates, const float *c,
                           const float *c_prev, float *dc, void *da, int B, int H, cudaStream_t s);
 cudaError_t embedding_fwd(int bf16, const int32_t *tok, const void *E, void *y, long rows, int H, cudaStream_t s);

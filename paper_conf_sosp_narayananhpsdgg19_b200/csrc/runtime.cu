@@ -272,6 +272,8 @@ struct Worker {
     std::vector<long> aux_bytes;
     float *lstm_gx = nullptr, *lstm_gh = nullptr, *lstm_dh = nullptr, *lstm_dc = nullptr;
     void *lstm_da = nullptr;
+    unsigned *lstm_cnt = nullptr;  // step counters of the persistent recurrence kernels
+    int lstm_rec = -1;             // persistent recurrences usable (-1 = not decided yet)
     // CUDA graphs of the LSTM recurrences (T steps of small GEMM + cell kernels), keyed by
     // (layer, direction, saved-state slot, weight slot, dY pointer): replayed instead of
     // re-issuing ~3T launches per layer
@@ -307,7 +309,7 @@ Worker::~Worker() {
     for (void *p : act) cudaFree(p);
     for (void *p : aux)
         if (p) cudaFree(p);
-    void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da};
+    void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da, lstm_cnt};
     for (void *p : lb)
         if (p) cudaFree(p);
     void *bufs[] = {master, fbias, (void *)breg_off, (void *)breg_cnt, adam_m, adam_v, gbuf, ws, (void *)split_counters, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
@@ -835,6 +837,27 @@ struct Exec {
         return true;
     }
 
+    // Persistent recurrences (lstm_rec.cu): bf16 path, supported shape, co-resident grid, and
+    // no other LSTM-bearing worker on this GPU (two spinning grids could each hold half the
+    // SMs the other needs).  PD_LSTM_REC=0 forces the per-step path.
+    bool use_lstm_rec(const pd_layer_desc &d, int Bn) {
+        if (!bf16) return false;
+        if (w->lstm_rec < 0) {
+            const char *env = getenv("PD_LSTM_REC");
+            int others = 0;
+            for (auto &o : c->W) {
+                if (!o || o.get() == w || o->device != w->device) continue;
+                for (int l = o->first; l <= o->last; ++l)
+                    if (c->layers[l].kind == PD_LSTM) {
+                        ++others;
+                        break;
+                    }
+            }
+            w->lstm_rec = (env && env[0] == '0') || others ? 0 : 1;
+        }
+        return w->lstm_rec && lstm_rec_supported(Bn, d.out);
+    }
+
     void lstm_forward(int l, int j, int slot, const void *x, void *y) {
         const pd_layer_desc &d = layer(l);
         const int T = d.seq_len, Bn = B(), H = d.out, I = d.in;
@@ -854,6 +877,15 @@ struct Exec {
         g.ldo = 4 * H;
         CK(run_gemm(bf16, g, w->stream));
         const float *bih = param_f32(lstm_off(l, 2), slot), *bhh = param_f32(lstm_off(l, 3), slot);
+        if (use_lstm_rec(d, Bn)) {
+            // all T steps in one persistent launch (lstm_rec.cu)
+            CK(cudaMemsetAsync(w->lstm_cnt, 0, 1024 * sizeof(unsigned), w->stream));
+            CK(lstm_rec_fwd(w->lstm_gx, bih, bhh,
+                            static_cast<const __nv_bfloat16 *>(elem_ptr(w->wslot[slot], lstm_off(l, 1), esz)),
+                            st.gates, st.c, static_cast<__nv_bfloat16 *>(st.h), w->lstm_cnt, T, Bn, H, w->stream));
+            CK(cudaMemcpyAsync(y, st.h, (size_t)TB * H * esz, cudaMemcpyDeviceToDevice, w->stream));
+            return;
+        }
         // the recurrence writes h into the saved state only; one copy forwards it to y
         // (possibly another GPU's receive ring) so the captured graph is independent of y
         graph_run(std::make_tuple(l, 0, j % w->k, slot, (const void *)nullptr), [&] {
@@ -894,6 +926,12 @@ struct Exec {
         const void *Wih = elem_ptr(w->wslot[bc.sslot], lstm_off(l, 0), esz);
         const void *Whh = elem_ptr(w->wslot[bc.sslot], lstm_off(l, 1), esz);
         cudaEvent_t k0 = kstart(1);
+        if (use_lstm_rec(d, Bn)) {
+            CK(cudaMemsetAsync(w->lstm_cnt, 0, 1024 * sizeof(unsigned), w->stream));
+            CK(lstm_rec_bwd(static_cast<const __nv_bfloat16 *>(G), st.gates, st.c,
+                            static_cast<const __nv_bfloat16 *>(Whh), static_cast<__nv_bfloat16 *>(w->lstm_da),
+                            w->lstm_cnt, T, Bn, H, w->stream));
+        } else
         graph_run(std::make_tuple(l, 1, j % w->k, bc.sslot, G), [&] {
         CK(cudaMemsetAsync(w->lstm_dc, 0, (size_t)Bn * H * 4, w->stream));
         for (int t = T - 1; t >= 0; --t) {
@@ -1667,6 +1705,7 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             w->lstm_gh = dalloc<float>(4 * bh_elems * 4);
             w->lstm_dh = dalloc<float>(bh_elems * 4);
             w->lstm_dc = dalloc<float>(bh_elems * 4);
+            w->lstm_cnt = dalloc<unsigned>(1024 * sizeof(unsigned));
         }
         if (bf16) {
             w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
@@ -2163,5 +2202,24 @@ extern "C" PD_API pd_status pd_kernel_softmax_ce(int dtype, const void *logits, 
     if (!logits || !labels || !dlogits || !loss || rows < 1 || C < 1) return PD_EINVAL;
     cudaError_t e = softmax_ce(logits, dtype == PD_BF16, labels, rows, C, dlogits, loss,
                                static_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? PD_OK : PD_ECUDA;
+}
+
+extern "C" PD_API pd_status pd_kernel_lstm_rec(const pd_lstm_rec_desc *d, void *stream) {
+    if (!d || d->T < 1 || !d->w_hh || !d->counters || !d->gates || !d->c) return PD_EINVAL;
+    if (d->direction != 0 && d->direction != 1) return PD_EINVAL;
+    if (d->direction == 0 && (!d->gx || !d->b_ih || !d->b_hh || !d->h)) return PD_EINVAL;
+    if (d->direction == 1 && (!d->dy || !d->da)) return PD_EINVAL;
+    if (!lstm_rec_supported(d->B, d->H)) return PD_EUNSUPPORTED;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    if (cudaMemsetAsync(d->counters, 0, (size_t)(4 * d->H / 64) * sizeof(unsigned), s) != cudaSuccess)
+        return PD_ECUDA;
+    const __nv_bfloat16 *W = static_cast<const __nv_bfloat16 *>(d->w_hh);
+    cudaError_t e =
+        d->direction == 0
+            ? lstm_rec_fwd(d->gx, d->b_ih, d->b_hh, W, d->gates, d->c, static_cast<__nv_bfloat16 *>(d->h),
+                           d->counters, d->T, d->B, d->H, s, d->probe)
+            : lstm_rec_bwd(static_cast<const __nv_bfloat16 *>(d->dy), d->gates, d->c, W,
+                           static_cast<__nv_bfloat16 *>(d->da), d->counters, d->T, d->B, d->H, s, d->probe);
     return e == cudaSuccess ? PD_OK : PD_ECUDA;
 }

@@ -1,0 +1,70 @@
+"""Persistent LSTM recurrence kernels (csrc/lstm_rec.cu) against the oracle.
+
+The reduced GNMT configs (H = 32) run the per-step path; these GNMT-shaped stacks have
+H % 256 == 0, so the bf16 path runs each layer's whole recurrence (forward and
+backward-through-time) as one persistent launch.  SGD makes the parameter deltas a direct
+image of the gradients, so a wrong step, a wrong K-range or a mis-ordered partial shows up in
+the delta error; losses check the forward pass minibatch by minibatch.  The same run with
+PD_LSTM_REC=0 (per-step GEMM + cell kernels) must agree with it closely."""
+import os
+
+import numpy as np
+import pytest
+
+import synth
+import torchref
+import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+from gpu_helpers import run_both, assert_schedule_exact, param_errors, BF16_TOL
+
+pytestmark = pytest.mark.gpu
+
+# (layers, H, B, T): ragged batch (N = 48 > B = 40), full GNMT width with one and two layers
+SHAPES = [(2, 256, 16, 6), (1, 512, 40, 5), (1, 1024, 64, 4), (2, 1024, 64, 3)]
+
+
+def _workload(n, H, B, T):
+    return synth.Workload(f"lstm{n}x{H}", synth.gnmt(n, H, 512, T, B), B, synth.SGD, 0.05)
+
+
+def _run(wl, last, M, rec):
+    old = os.environ.get("PD_LSTM_REC")
+    os.environ["PD_LSTM_REC"] = "1" if rec else "0"
+    try:
+        return run_both(wl, last, [1] * len(last), M, pd.PD_BF16, n_data=3)
+    finally:
+        if old is None:
+            del os.environ["PD_LSTM_REC"]
+        else:
+            os.environ["PD_LSTM_REC"] = old
+
+
+@pytest.mark.parametrize("n,H,B,T", SHAPES)
+def test_persistent_recurrence_matches_oracle(n, H, B, T):
+    wl = _workload(n, H, B, T)
+    M = 3
+    res = _run(wl, [len(wl.layers) - 1], M, rec=True)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, perr
+    assert derr < 5e-2, derr
+    np.testing.assert_allclose(res["losses"], res["ref"].losses, rtol=1e-2)
+
+
+@pytest.mark.parametrize("n,H,B,T", SHAPES[:3])
+def test_persistent_equals_per_step_path(n, H, B, T):
+    wl = _workload(n, H, B, T)
+    a = _run(wl, [len(wl.layers) - 1], 2, rec=True)
+    b = _run(wl, [len(wl.layers) - 1], 2, rec=False)
+    # same bf16 operands and roundings except the fp32 summation order of the recurrent GEMM
+    d = torchref.delta_err(a["got"], b["got"], a["p0"])
+    assert d < 2e-2, d
+    np.testing.assert_allclose(a["losses"], b["losses"], rtol=2e-3)
+
+
+def test_persistent_two_stage_pipeline_only_first_worker_lstm():
+    # stage 0 = Emb + LSTM (persistent: the only LSTM worker on the GPU), stage 1 = classifier
+    wl = _workload(1, 256, 16, 5)
+    res = _run(wl, [1, 2], 8, rec=True)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL and derr < 5e-2, (perr, derr)
