@@ -26,6 +26,7 @@
 #include <cuda_bf16.h>
 
 #include <cstdio>
+#include <cstdlib>
 
 #include "pd_internal.h"
 #include "tc_ptx.h"
@@ -35,10 +36,9 @@ namespace {
 using namespace tcx;
 
 constexpr int RT = 128;           // 4 warps = the 4 TMEM lane quadrants
-constexpr int STG_LD = 68;        // staging row stride (floats): conflict-free float4 writes
 constexpr int TILE_W = 128 * 128;  // one [128 rows][64 K] bf16 SW128 tile (bytes)
 constexpr int TILE_X = 64 * 128;   // one [<=64 rows][64 K] bf16 SW128 tile (bytes)
-constexpr int STG_BYTES = 128 * STG_LD * 4;
+constexpr int RECV_BYTES = 128 * 64 * 4;  // partials pushed to this CTA: [src][rows it owns][64 b]
 
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
 
@@ -68,11 +68,24 @@ __device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence
 // split cluster barrier: arrive after the DSMEM reads of a step, wait before this CTA next
 // overwrites what its peers read (its staging buffer / the tiles the staging aliases)
 __device__ __forceinline__ void cl_arrive() { asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory"); }
+__device__ __forceinline__ void cl_sync(int dbg) {
+    if (!(dbg & 2)) {
+        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+    }
+}
 __device__ __forceinline__ void cl_wait() { asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory"); }
-__device__ __forceinline__ float ld_dsmem_f32(uint32_t addr) {
-    float v;
-    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
-    return v;
+__device__ __forceinline__ void st_dsmem_v4(uint32_t addr, float a, float b, float c, float d) {
+    asm volatile("st.shared::cluster.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "f"(a), "f"(b), "f"(c), "f"(d)
+                 : "memory");
+}
+__device__ __forceinline__ void red_relaxed_add(unsigned *p, unsigned v) {
+    asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// publish one step: release-add (orders this CTA's earlier stores, seen through bar.sync)
+__device__ __forceinline__ void red_release_add(unsigned *p, unsigned v) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 __device__ __forceinline__ uint32_t cluster_rank() {
     uint32_t r;
@@ -103,6 +116,8 @@ struct RecArgs {
     const __nv_bfloat16 *dy;
     const float *gates_in, *c_in;
     __nv_bfloat16 *da;
+    int dbg;                    // tools only (PD_LSTM_DBG): 1 no dependency waits, 2 no cluster barriers,
+                                // 4 relaxed publish (no release), 8 no MMA -- timing experiments, wrong results
     unsigned long long *probe;  // tools: [grid][T][8] %globaltimer stamps by thread 0 (nullptr = off)
 };
 
@@ -110,31 +125,43 @@ __device__ __forceinline__ void stamp(const RecArgs &a, int step, int k) {
     if (a.probe && threadIdx.x == 0) a.probe[((long)blockIdx.x * a.T + step) * 8 + k] = gtime();
 }
 
-// shared state of both kernels: after the MMAs of a step, every CTA stages its fp32 partial
-// [128 rows][N] (TMEM lane = row) into shared memory for the cluster's DSMEM reduction
-__device__ __forceinline__ void stage_partial(uint32_t tmem, float *stg, int warp, int lane) {
-    const int row = warp * 32 + lane;
+// After the MMAs of a step every CTA holds an fp32 partial D[128 rows][N] (TMEM lane = row).
+// Thread `row` pushes its 64 batch columns into the receive buffer of the CTA that owns the
+// row with st.async (16 x 16 B into distributed shared memory), each completing its bytes on
+// the owner's receive mbarrier -- a point-to-point handoff, no cluster-wide barrier.
+// dst_off = byte offset of this row's 64 floats in the owner's buffer.
+__device__ __forceinline__ void push_partial(uint32_t tmem, int warp, uint32_t recv_s, uint32_t rbar, int owner,
+                                             uint32_t dst_off) {
+    const uint32_t base = mapa_cluster(recv_s + dst_off, owner);
+    const uint32_t bar = mapa_cluster(rbar, owner);
 #pragma unroll
     for (int ch = 0; ch < 2; ++ch) {
         float v[32];
         tmem_ld32(tmem + ((uint32_t)(warp * 32) << 16) + ch * 32, v);
 #pragma unroll
         for (int q = 0; q < 8; ++q)
-            *reinterpret_cast<float4 *>(stg + row * STG_LD + ch * 32 + q * 4) =
-                make_float4(v[q * 4], v[q * 4 + 1], v[q * 4 + 2], v[q * 4 + 3]);
+            asm volatile(
+                "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+                    base + (ch * 32 + q * 4) * 4),
+                "f"(v[q * 4]), "f"(v[q * 4 + 1]), "f"(v[q * 4 + 2]), "f"(v[q * 4 + 3]), "r"(bar)
+                : "memory");
     }
 }
 
 // MMA issue for one step: KB K-blocks of 64, D[128][N] (+)= A_kb[128][64] . B_kb[N][64]^T
+// A_kb is K-major ([128 rows][64 K], forward) or MN-major (two [64 K][64 rows] chunks 8 KB
+// apart, backward: W_hh tiles loaded untransposed)
+template <int AMN>
 __device__ __forceinline__ void issue_mmas(uint32_t tmem, uint32_t a_base, uint32_t b_base, uint32_t full0,
                                            uint32_t mma_bar, int KB, int N, uint32_t parity) {
-    const uint32_t idesc = make_idesc(128, N, 0, 0);
+    const uint32_t idesc = make_idesc(128, N, AMN, 0);
     for (int kb = 0; kb < KB; ++kb) {
         mbar_wait(full0 + kb * 8, parity);
         tc_fence_after();
 #pragma unroll
         for (int kk = 0; kk < 4; ++kk) {
-            const uint64_t ad = smem_desc(a_base + kb * TILE_W + kk * 32, 16, 1024);
+            const uint64_t ad = AMN ? smem_desc(a_base + kb * TILE_W + kk * 2048, 8192, 1024)
+                                    : smem_desc(a_base + kb * TILE_W + kk * 32, 16, 1024);
             const uint64_t bd = smem_desc(b_base + kb * TILE_X + kk * 32, 16, 1024);
             tc_mma(tmem, ad, bd, idesc, (kb | kk) != 0);
         }
@@ -144,15 +171,15 @@ __device__ __forceinline__ void issue_mmas(uint32_t tmem, uint32_t a_base, uint3
 
 // ------------------------------------------------------------------------------ forward
 __global__ void __launch_bounds__(RT, 1)
-    lstm_rec_fwd_kernel(const __grid_constant__ CUtensorMap tmH, RecArgs a) {
+    lstm_rec_fwd_kernel(const __grid_constant__ CUtensorMap tmH, const __grid_constant__ CUtensorMap tmW, RecArgs a) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *sm = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const int H = a.H, B = a.B, T = a.T, N = a.N;
     const int KB = H / 4 / 64;  // K-blocks per CTA
     uint8_t *sW = sm;                       // KB x [128][64] weight tiles
     uint8_t *sX = sW + KB * TILE_W;         // KB x [N][64] h tiles
-    float *stg = reinterpret_cast<float *>(sX + KB * TILE_X);
-    uint64_t *bars = reinterpret_cast<uint64_t *>(reinterpret_cast<uint8_t *>(stg) + STG_BYTES);
+    float *recv = reinterpret_cast<float *>(sX + KB * TILE_X);  // [src 4][g 4][u 8][b 64]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(reinterpret_cast<uint8_t *>(recv) + RECV_BYTES);
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 16);
     const uint32_t full0 = smem_u32(bars), mma_bar = smem_u32(bars + 8);
 
@@ -164,17 +191,18 @@ __global__ void __launch_bounds__(RT, 1)
     const int U0 = U0c + 8 * cr;        // this CTA's 8 units
     const int k0 = cr * (H / 4);        // this CTA's K-range of h
 
-    // weights: tile kb row m = g*32 + ul  <-  W_hh[g*H + U0c + ul][k0 + kb*64 .. +64]
-    for (int i = tid; i < KB * 128 * 8; i += RT) {
-        const int q = i & 7, m = (i >> 3) & 127, kb = i >> 10;
-        const int g = m >> 5, ul = m & 31;
-        const uint4 v = *reinterpret_cast<const uint4 *>(a.W + (long)(g * H + U0c + ul) * H + k0 + kb * 64 + q * 8);
-        *reinterpret_cast<uint4 *>(sW + kb * TILE_W + sw128(m, q * 8)) = v;
-    }
+    // weights by TMA: tile kb rows g*32 .. g*32+31 <- W_hh[g*H + U0c .. +32][k0 + kb*64 .. +64]
+    const uint32_t wbar = smem_u32(bars + 9), rbar = smem_u32(bars + 10);
     if (tid == 0) {
         for (int kb = 0; kb < KB; ++kb) mbar_init(full0 + kb * 8, 1);
         mbar_init(mma_bar, 1);
+        mbar_init(wbar, 1);
+        mbar_init(rbar, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        mbar_expect_tx(wbar, (uint32_t)KB * TILE_W);
+        for (int kb = 0; kb < KB; ++kb)
+            for (int g = 0; g < 4; ++g)
+                tma_load_2d(smem_u32(sW + kb * TILE_W + g * 4096), &tmW, wbar, k0 + kb * 64, g * H + U0c);
     }
     if (warp == 0) tmem_alloc(smem_u32(tmem_slot), 64);
     fence_proxy_async();
@@ -182,6 +210,8 @@ __global__ void __launch_bounds__(RT, 1)
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    cluster_sync_all();  // every peer's receive mbarrier is initialised before the first push
+    mbar_wait(wbar, 0);
     if (a.probe && tid == 0) {
         a.probe[(long)blockIdx.x * a.T * 8 + 6] = t_entry;
         a.probe[(long)blockIdx.x * a.T * 8 + 7] = gtime();
@@ -201,7 +231,9 @@ __global__ void __launch_bounds__(RT, 1)
         bs[g][2] = x.z + y.z;
         bs[g][3] = x.w + y.w;
     }
-    const uint32_t stg_s = smem_u32(stg);
+    const uint32_t recv_s = smem_u32(recv);
+    // push role: partial row m = warp*32 + lane = gate `warp`, cluster unit `lane` -> owner lane/8
+    const uint32_t push_off = (uint32_t)(((cr * 4 + warp) * 8 + (lane & 7)) * 64 * 4);
 
     for (int t = 0; t < T; ++t) {
         stamp(a, t, 0);
@@ -219,46 +251,43 @@ __global__ void __launch_bounds__(RT, 1)
         float acc[4][4] = {};
         if (t > 0) {
             const uint32_t par = (uint32_t)(t - 1) & 1;
-            if (t > 1) cl_wait();  // peers finished reading the previous step's staging
+            if (t > 1 && !(a.dbg & 2)) cl_wait();  // every owner finished reading the previous step's partials
             if (tid == 0) {
-                fence_proxy_async();
+                // 64 units of h = 8 producer CTAs per K-block
+                if (!(a.dbg & 1))
+                    for (int kb = 0; kb < KB; ++kb) wait_count(a.cnt + (k0 >> 6) + kb, 8u * t);
+                fence_proxy_async_global();
                 for (int kb = 0; kb < KB; ++kb) {
-                    const int gkb = (k0 >> 6) + kb;    // 64 units of h = 8 producer CTAs
-                    wait_count(a.cnt + gkb, 8u * t);
-                    fence_proxy_async_global();
                     mbar_expect_tx(full0 + kb * 8, (uint32_t)N * 128);
                     tma_load_2d(smem_u32(sX + kb * TILE_X), &tmH, full0 + kb * 8, k0 + kb * 64, (t - 1) * B);
                 }
                 stamp(a, t, 1);
             } else if (tid == 32) {
-                issue_mmas(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
+                if (a.dbg & 8) tc_commit(mma_bar);
+                else issue_mmas<0>(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
             }
             __syncwarp();
             mbar_wait(mma_bar, par);
             stamp(a, t, 2);
             tc_fence_after();
-            stage_partial(tmem, stg, warp, lane);
+            if (tid == 0) mbar_expect_tx(rbar, 4u * 32 * 64 * 4);  // 4 sources x 32 rows x 64 b
+            push_partial(tmem, warp, recv_s, rbar, lane >> 3, push_off);
             tc_fence_before();
-            cluster_sync_all();
+            mbar_wait(rbar, par);
             stamp(a, t, 3);
             if (act) {
 #pragma unroll
-                for (int src = 0; src < 4; ++src) {
-                    const uint32_t base = mapa_cluster(stg_s, src);
+                for (int src = 0; src < 4; ++src)
 #pragma unroll
                     for (int g = 0; g < 4; ++g)
 #pragma unroll
-                        for (int u = 0; u < 4; ++u) {
-                            const int row = g * 32 + 8 * cr + u4 + u;
-                            acc[g][u] += ld_dsmem_f32(base + (uint32_t)(row * STG_LD + b) * 4);
-                        }
-                }
+                        for (int u = 0; u < 4; ++u) acc[g][u] += recv[((src * 4 + g) * 8 + u4 + u) * 64 + b];
             }
-            cl_arrive();
+            if (!(a.dbg & 2)) cl_arrive();
             stamp(a, t, 4);
         }
+        float ig[4], fg[4], gg[4], og[4], cc[4], hh[4];
         if (act) {
-            float ig[4], fg[4], gg[4], og[4], cc[4], hh[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
                 ig[u] = sigm(acc[0][u] + gxv[0][u] + bs[0][u]);
@@ -269,13 +298,8 @@ __global__ void __launch_bounds__(RT, 1)
                 hh[u] = og[u] * tanhf(cc[u]);
                 cst[u] = cc[u];
             }
-            const long r4 = ((long)t * B + b) * 4 * H + j;
-            *reinterpret_cast<float4 *>(a.gates + r4) = make_float4(ig[0], ig[1], ig[2], ig[3]);
-            *reinterpret_cast<float4 *>(a.gates + r4 + H) = make_float4(fg[0], fg[1], fg[2], fg[3]);
-            *reinterpret_cast<float4 *>(a.gates + r4 + 2 * H) = make_float4(gg[0], gg[1], gg[2], gg[3]);
-            *reinterpret_cast<float4 *>(a.gates + r4 + 3 * H) = make_float4(og[0], og[1], og[2], og[3]);
+            // h first: it is what the next step waits for
             const long r1 = ((long)t * B + b) * H + j;
-            *reinterpret_cast<float4 *>(a.c + r1) = make_float4(cc[0], cc[1], cc[2], cc[3]);
             uint2 p;
             p.x = pack_bf16(hh[0], hh[1]);
             p.y = pack_bf16(hh[2], hh[3]);
@@ -283,29 +307,35 @@ __global__ void __launch_bounds__(RT, 1)
         }
         __syncthreads();
         if (tid == 0 && t + 1 < T) {
-            fence_proxy_async_global();
-            __threadfence();
-            atomicAdd(a.cnt + (U0 >> 6), 1u);
+            if (a.dbg & 4) atomicAdd(a.cnt + (U0 >> 6), 1u);
+            else red_release_add(a.cnt + (U0 >> 6), 1u);
+        }
+        if (act) {
+            const long r4 = ((long)t * B + b) * 4 * H + j;
+            *reinterpret_cast<float4 *>(a.gates + r4) = make_float4(ig[0], ig[1], ig[2], ig[3]);
+            *reinterpret_cast<float4 *>(a.gates + r4 + H) = make_float4(fg[0], fg[1], fg[2], fg[3]);
+            *reinterpret_cast<float4 *>(a.gates + r4 + 2 * H) = make_float4(gg[0], gg[1], gg[2], gg[3]);
+            *reinterpret_cast<float4 *>(a.gates + r4 + 3 * H) = make_float4(og[0], og[1], og[2], og[3]);
+            *reinterpret_cast<float4 *>(a.c + ((long)t * B + b) * H + j) = make_float4(cc[0], cc[1], cc[2], cc[3]);
         }
         stamp(a, t, 5);
     }
     tc_fence_before();
-    if (T > 1) cl_wait();  // peers may still read this CTA's staging buffer
+    if (T > 1 && !(a.dbg & 2)) cl_wait();  // no peer may push into / read from an exited CTA
     if (warp == 0) tmem_free(tmem, 64);
 }
 
 // ------------------------------------------------------------------------------ backward
 __global__ void __launch_bounds__(RT, 1)
-    lstm_rec_bwd_kernel(const __grid_constant__ CUtensorMap tmA, RecArgs a) {
+    lstm_rec_bwd_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW, RecArgs a) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *sm = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const int H = a.H, B = a.B, T = a.T, N = a.N;
     const int KB = H / 2 / 64;  // K-blocks of da per CTA
     uint8_t *sW = sm;                  // KB x [128 units][64 gate rows] = W_hh^T tiles
-    uint8_t *sX = sW + KB * TILE_W;    // KB x [N][64] da tiles; reused as the staging buffer
-    float *stg = reinterpret_cast<float *>(sX);
-    const int xbytes = KB * TILE_X > STG_BYTES ? KB * TILE_X : STG_BYTES;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(sX + xbytes);
+    uint8_t *sX = sW + KB * TILE_W;    // KB x [N][64] da tiles
+    float *recv = reinterpret_cast<float *>(sX + KB * TILE_X);  // [src 8][u 16][b 64]
+    uint64_t *bars = reinterpret_cast<uint64_t *>(reinterpret_cast<uint8_t *>(recv) + RECV_BYTES);
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 16);
     const uint32_t full0 = smem_u32(bars), mma_bar = smem_u32(bars + 8);
 
@@ -317,23 +347,19 @@ __global__ void __launch_bounds__(RT, 1)
     const int U0 = U0c + 16 * cr;    // this CTA's 16 units
     const int k0 = cr * (H / 2);     // this CTA's range of gate rows r
 
-    // W_hh^T tiles: tile kb row m (unit U0c + m), column kin (gate row k0 + kb*64 + kin)
-    for (int i = tid; i < KB * 8 * 128; i += RT) {
-        const int m = i & 127, q = (i >> 7) & 7, kb = i >> 10;
-        const long r = k0 + kb * 64 + q * 8;
-        uint32_t w[4];
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-            const __nv_bfloat16 lo = a.W[(r + 2 * e) * H + U0c + m];
-            const __nv_bfloat16 hi = a.W[(r + 2 * e + 1) * H + U0c + m];
-            w[e] = (uint32_t)__bfloat16_as_ushort(lo) | ((uint32_t)__bfloat16_as_ushort(hi) << 16);
-        }
-        *reinterpret_cast<uint4 *>(sW + kb * TILE_W + sw128(m, q * 8)) = make_uint4(w[0], w[1], w[2], w[3]);
-    }
+    // W_hh tiles by TMA, untransposed (MN-major A operand): tile kb = two [64 gate rows][64
+    // units] chunks <- W_hh[k0 + kb*64 .. +64][U0c + 64 j .. +64]
+    const uint32_t wbar = smem_u32(bars + 9), rbar = smem_u32(bars + 10);
     if (tid == 0) {
         for (int kb = 0; kb < KB; ++kb) mbar_init(full0 + kb * 8, 1);
         mbar_init(mma_bar, 1);
+        mbar_init(wbar, 1);
+        mbar_init(rbar, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        mbar_expect_tx(wbar, (uint32_t)KB * TILE_W);
+        for (int kb = 0; kb < KB; ++kb)
+            for (int jj = 0; jj < 2; ++jj)
+                tma_load_2d(smem_u32(sW + kb * TILE_W + jj * 8192), &tmW, wbar, U0c + 64 * jj, k0 + kb * 64);
     }
     if (warp == 0) tmem_alloc(smem_u32(tmem_slot), 64);
     fence_proxy_async();
@@ -341,6 +367,8 @@ __global__ void __launch_bounds__(RT, 1)
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    cluster_sync_all();  // every peer's receive mbarrier is initialised before the first push
+    mbar_wait(wbar, 0);
     if (a.probe && tid == 0) {
         a.probe[(long)blockIdx.x * a.T * 8 + 6] = t_entry;
         a.probe[(long)blockIdx.x * a.T * 8 + 7] = gtime();
@@ -351,10 +379,14 @@ __global__ void __launch_bounds__(RT, 1)
     const int j = U0 + u8;
     const bool act = b < B;
     float dc[8] = {};
-    const uint32_t stg_s = smem_u32(stg);
+    const uint32_t recv_s = smem_u32(recv);
+    // push role: partial row m = warp*32 + lane = cluster unit m -> owner m/16
+    const int m = warp * 32 + lane;
+    const uint32_t push_off = (uint32_t)((cr * 16 + (m & 15)) * 64 * 4);
 
     for (int s = 0; s < T; ++s) {
         const int t = T - 1 - s;
+        stamp(a, s, 0);
         float dh[8], gi[8], gf[8], gg[8], go[8], ct[8], cp[8];
         if (act) {
             const long r1 = ((long)t * B + b) * H + j;
@@ -387,42 +419,40 @@ __global__ void __launch_bounds__(RT, 1)
         }
         if (s > 0) {
             const uint32_t par = (uint32_t)(s - 1) & 1;
-            if (s > 1) cl_wait();  // peers finished reading the staging that aliases the da tiles
+            if (s > 1 && !(a.dbg & 2)) cl_wait();  // every owner finished reading the previous step's partials
             if (tid == 0) {
-                fence_proxy_async();  // the staging writes of the last step aliased these tiles
+                // 64 gate rows of da = 4 producer CTAs per K-block
+                if (!(a.dbg & 1))
+                    for (int kb = 0; kb < KB; ++kb) wait_count(a.cnt + (k0 >> 6) + kb, 4u * s);
+                fence_proxy_async_global();
                 for (int kb = 0; kb < KB; ++kb) {
-                    const int gkb = (k0 >> 6) + kb;   // 64 gate rows = 4 producer CTAs
-                    wait_count(a.cnt + gkb, 4u * s);
-                    fence_proxy_async_global();
                     mbar_expect_tx(full0 + kb * 8, (uint32_t)N * 128);
                     tma_load_2d(smem_u32(sX + kb * TILE_X), &tmA, full0 + kb * 8, k0 + kb * 64, (t + 1) * B);
                 }
                 stamp(a, s, 1);
             } else if (tid == 32) {
-                issue_mmas(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
+                if (a.dbg & 8) tc_commit(mma_bar);
+                else issue_mmas<1>(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
             }
             __syncwarp();
             mbar_wait(mma_bar, par);
             stamp(a, s, 2);
             tc_fence_after();
-            stage_partial(tmem, stg, warp, lane);
+            if (tid == 0) mbar_expect_tx(rbar, 8u * 16 * 64 * 4);  // 8 sources x 16 rows x 64 b
+            push_partial(tmem, warp, recv_s, rbar, m >> 4, push_off);
             tc_fence_before();
-            cluster_sync_all();
+            mbar_wait(rbar, par);
             stamp(a, s, 3);
             if (act) {
                 float rec[8] = {};
 #pragma unroll
-                for (int src = 0; src < 8; ++src) {
-                    const uint32_t base = mapa_cluster(stg_s, src);
+                for (int src = 0; src < 8; ++src)
 #pragma unroll
-                    for (int u = 0; u < 8; ++u)
-                        rec[u] += ld_dsmem_f32(base + (uint32_t)((16 * cr + u8 + u) * STG_LD + b) * 4);
-                }
+                    for (int u = 0; u < 8; ++u) rec[u] += recv[((src * 16 + u8 + u) * 64) + b];
 #pragma unroll
                 for (int u = 0; u < 8; ++u) dh[u] += rec[u];
             }
-            fence_proxy_async();  // generic staging writes before the next step's TMA overwrite
-            cl_arrive();
+            if (!(a.dbg & 2)) cl_arrive();
             stamp(a, s, 4);
         }
         if (act) {
@@ -451,27 +481,23 @@ __global__ void __launch_bounds__(RT, 1)
         }
         __syncthreads();
         if (tid == 0 && s + 1 < T) {
-            fence_proxy_async_global();
-            __threadfence();
+            fence_acq_rel_gpu();
 #pragma unroll
-            for (int g = 0; g < 4; ++g) atomicAdd(a.cnt + ((g * H + U0) >> 6), 1u);
+            for (int g = 0; g < 4; ++g) red_relaxed_add(a.cnt + ((g * H + U0) >> 6), 1u);
         }
         stamp(a, s, 5);
     }
     tc_fence_before();
-    if (T > 1) cl_wait();
+    if (T > 1 && !(a.dbg & 2)) cl_wait();
     if (warp == 0) tmem_free(tmem, 64);
 }
 
-int fwd_smem(int H) { return (H / 256) * (TILE_W + TILE_X) + STG_BYTES + 256 + 1024; }
-int bwd_smem(int H) {
-    const int KB = H / 128;
-    return KB * TILE_W + (KB * TILE_X > STG_BYTES ? KB * TILE_X : STG_BYTES) + 256 + 1024;
-}
+int fwd_smem(int H) { return (H / 256) * (TILE_W + TILE_X) + RECV_BYTES + 256 + 1024; }
+int bwd_smem(int H) { return (H / 128) * (TILE_W + TILE_X) + RECV_BYTES + 256 + 1024; }
 
 template <typename K>
-cudaError_t launch_clustered(K kern, int grid, int csize, int smem, const CUtensorMap &map, const RecArgs &a,
-                             cudaStream_t s) {
+cudaError_t launch_clustered(K kern, int grid, int csize, int smem, const CUtensorMap &map, const CUtensorMap &wmap,
+                             const RecArgs &a, cudaStream_t s) {
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(RT);
@@ -484,7 +510,7 @@ cudaError_t launch_clustered(K kern, int grid, int csize, int smem, const CUtens
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, kern, map, a);
+    return cudaLaunchKernelEx(&cfg, kern, map, wmap, a);
 }
 
 // can `grid` CTAs in clusters of `csize` (smem bytes each) all be resident at once?
@@ -534,10 +560,13 @@ cudaError_t lstm_rec_fwd(const float *gx, const float *b_ih, const float *b_hh, 
     a.T = T, a.B = B, a.H = H, a.N = (B + 15) / 16 * 16;
     a.cnt = cnt, a.W = Whh, a.gx = gx, a.b_ih = b_ih, a.b_hh = b_hh, a.gates = gates, a.c = c, a.h = h;
     a.probe = probe;
+    if (const char *e = getenv("PD_LSTM_DBG")) a.dbg = atoi(e);
     CUtensorMap map;
-    if (!tma_map_bf16(&map, h, H, (long)T * B, H, 64, a.N)) return cudaErrorInvalidValue;
+    CUtensorMap wmap;
+    if (!tma_map_bf16(&map, h, H, (long)T * B, H, 64, a.N) || !tma_map_bf16(&wmap, Whh, H, 4L * H, H, 64, 32))
+        return cudaErrorInvalidValue;
     ++tl_launches;
-    return launch_clustered(lstm_rec_fwd_kernel, H / 8, 4, fwd_smem(H), map, a, s);
+    return launch_clustered(lstm_rec_fwd_kernel, H / 8, 4, fwd_smem(H), map, wmap, a, s);
 }
 
 cudaError_t lstm_rec_bwd(const __nv_bfloat16 *dy, const float *gates, const float *c, const __nv_bfloat16 *Whh,
@@ -548,10 +577,13 @@ cudaError_t lstm_rec_bwd(const __nv_bfloat16 *dy, const float *gates, const floa
     a.T = T, a.B = B, a.H = H, a.N = (B + 15) / 16 * 16;
     a.cnt = cnt, a.W = Whh, a.dy = dy, a.gates_in = gates, a.c_in = c, a.da = da;
     a.probe = probe;
+    if (const char *e = getenv("PD_LSTM_DBG")) a.dbg = atoi(e);
     CUtensorMap map;
-    if (!tma_map_bf16(&map, da, 4L * H, (long)T * B, 4L * H, 64, a.N)) return cudaErrorInvalidValue;
+    CUtensorMap wmap;
+    if (!tma_map_bf16(&map, da, 4L * H, (long)T * B, 4L * H, 64, a.N) || !tma_map_bf16(&wmap, Whh, H, 4L * H, H, 64, 64))
+        return cudaErrorInvalidValue;
     ++tl_launches;
-    return launch_clustered(lstm_rec_bwd_kernel, H / 16, 8, bwd_smem(H), map, a, s);
+    return launch_clustered(lstm_rec_bwd_kernel, H / 16, 8, bwd_smem(H), map, wmap, a, s);
 }
 
 }  // namespace pd

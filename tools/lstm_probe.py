@@ -62,6 +62,14 @@ def main():
                               gx=gx.data_ptr(), b_ih=bih.data_ptr(), b_hh=bhh.data_ptr(), h=h.data_ptr(),
                               dy=dy.data_ptr(), da=da.data_ptr(), probe=probe, stream=st)
 
+    # bring the SM clock up before timing (an idle B200 sits at ~120 MHz) with the kernel
+    # itself: a matmul warm-up hits the power cap and leaves the clock low
+    for _ in range(400):
+        call(0)
+    torch.cuda.synchronize()
+    import subprocess
+    print(subprocess.run(["nvidia-smi", "--query-gpu=clocks.sm,clocks.max.sm", "--format=csv,noheader"],
+                         capture_output=True, text=True).stdout.strip())
     for direction, name in ((0, "forward"), (1, "backward")):
         for _ in range(3):
             call(direction)
