@@ -137,6 +137,21 @@ typedef struct {
 
 typedef struct pd_ctx pd_ctx;
 
+/* Self-profiler (L841-847 "Profiler"), B200-native: measures the planner's profile on THIS
+ * GPU.  Runs the whole model as one stage (plain SGD/Adam) on `cuda_device` for 2 warm-up
+ * and `num_minibatches` timed minibatches of synthetic inputs, with CUDA events around each
+ * layer's share of every forward (the loss counts to the last layer) and backward (dX, dW
+ * and the fused weight update), serialised on one stream.
+ *   out[l].compute_s   = mean forward + backward device seconds of layer l per minibatch (T_l)
+ *   out[l].act_bytes   = bytes of layer l's output activation in cfg->dtype (a_l)
+ *   out[l].param_bytes = 4 * parameters of layer l: the fp32 gradient bytes a replicated
+ *                        stage exchanges per round (w_l)
+ * cfg: dtype, optimizer, lr/betas/eps and minibatch are used; the rest is ignored.
+ * Errors: PD_EINVAL (bad arguments or layer shapes), PD_EUNSUPPORTED, PD_ENOMEM, PD_ECUDA. */
+PD_API pd_status pd_profile(const pd_layer_desc *layers, int num_layers, const pd_train_cfg *cfg,
+                            int cuda_device, int num_minibatches, pd_layer_profile *out);
+
+
 /* Creates a context for the whole plan.  Nothing touches a device until pd_stage_init.
  * Validation (PD_EINVAL): stages contiguous and covering layers 0..num_layers-1, each
  * R_s >= 1, layer shapes consistent (out of layer l == in of layer l+1 etc.), minibatch
@@ -239,6 +254,15 @@ PD_API pd_status pd_get_stats(pd_ctx *ctx, pd_stats *out);
  * (0 forward GEMMs, 1 dX GEMMs, 2 dW GEMMs incl. the fused update, 3 bias / other); each timed
  * launch costs two event records, so time only what is needed inside a timed region. */
 PD_API pd_status pd_set_timing(pd_ctx *ctx, int record_trace, int kernel_timing_mask);
+
+/* Layer profiling of later pd_run calls (the self-profiler's mechanism, usable on any plan):
+ * on = 1 records CUDA events around each layer's share of every F and B op; those ops then
+ * run serialised on the worker's stream (no side stream, no CUDA-graph replay), so
+ * throughput drops.  pd_get_layer_times returns, for the last run, the mean device seconds
+ * per minibatch of each layer's forward / backward over the local workers that ran it
+ * (0 for layers without a local worker); count must equal num_layers. */
+PD_API pd_status pd_set_layer_profiling(pd_ctx *ctx, int on);
+PD_API pd_status pd_get_layer_times(pd_ctx *ctx, double *fwd_s, double *bwd_s, size_t count);
 
 /* Releases everything the context owns.  Safe on NULL. */
 PD_API void pd_destroy(pd_ctx *ctx);

@@ -120,6 +120,9 @@ def _load():
         "pd_kernel_gemm": [vp, vp],
         "pd_kernel_softmax_ce": [i, vp, vp, C.c_long, i, vp, vp, vp],
         "pd_kernel_lstm_rec": [vp, vp],
+        "pd_profile": [vp, i, vp, i, i, vp],
+        "pd_set_layer_profiling": [vp, i],
+        "pd_get_layer_times": [vp, vp, vp, st],
     }
     for name, args in sigs.items():
         f = getattr(L, name)
@@ -139,7 +142,7 @@ lib = _load()
 EXPORTED = ["pd_plan", "pd_create", "pd_stage_init", "pd_export_worker", "pd_import_worker", "pd_set_data", "pd_run",
             "pd_get_params", "pd_get_trace", "pd_get_version_map", "pd_get_losses", "pd_get_stats", "pd_destroy",
             "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce",
-            "pd_kernel_lstm_rec",
+            "pd_kernel_lstm_rec", "pd_profile", "pd_set_layer_profiling", "pd_get_layer_times",
             "pd_set_timing"]
 
 
@@ -207,6 +210,18 @@ def pd_plan(compute_s, act_bytes, param_bytes, num_gpus, bandwidth_Bps=0.0, max_
     out = PlanT()
     _check(lib.pd_plan(prof, n, num_gpus, C.byref(opts), C.byref(out)))
     return Plan.from_c(out)
+
+
+def pd_profile(layers, dtype=PD_BF16, optimizer=PD_SGD, lr=0.01, minibatch=1, device=0, num_minibatches=8,
+               beta1=0.9, beta2=0.999, eps=1e-8):
+    """The B200 self-profiler (L841-847): (T_l seconds, a_l bytes, w_l bytes) per layer,
+    measured on `device` by the library."""
+    n = len(layers)
+    out = (LayerProfile * n)()
+    cfg = TrainCfg(dtype, optimizer, lr, beta1, beta2, eps, minibatch, 0, 0, 0)
+    _check(lib.pd_profile(_layer_descs(layers), n, C.byref(cfg), device, num_minibatches, out))
+    return ([out[k].compute_s for k in range(n)], [int(out[k].act_bytes) for k in range(n)],
+            [int(out[k].param_bytes) for k in range(n)])
 
 
 def pd_inflight(plan: Plan, noam: int = 0) -> List[int]:
@@ -315,6 +330,18 @@ def pd_get_stats(ctx) -> dict:
 
 def pd_set_timing(ctx, record_trace: int, kernel_timing_mask: int = 0xF):
     _check(lib.pd_set_timing(ctx, record_trace, kernel_timing_mask), ctx)
+
+
+def pd_set_layer_profiling(ctx, on: bool):
+    _check(lib.pd_set_layer_profiling(ctx, int(bool(on))), ctx)
+
+
+def pd_get_layer_times(ctx, num_layers: int):
+    """(forward seconds, backward seconds) per layer, mean per minibatch of the last run."""
+    f = np.zeros(num_layers, np.float64)
+    b = np.zeros(num_layers, np.float64)
+    _check(lib.pd_get_layer_times(ctx, _ptr(f), _ptr(b), num_layers), ctx)
+    return f, b
 
 
 def pd_destroy(ctx):

@@ -201,6 +201,7 @@ struct pd_ctx {
     std::vector<int32_t> vmap;
     double host_ms = 0;
     int ktime_mask = 0xF;            // kernel classes timed when record_trace >= 2
+    int layer_prof = 0;              // per-layer F / B device times (pd_set_layer_profiling)
     std::atomic<bool> abort{false};
     std::mutex err_mu;
     pd_status sticky = PD_OK;
@@ -295,6 +296,12 @@ struct Worker {
     std::vector<cudaEvent_t> ev_pool;
     cudaEvent_t run_ev[2] = {nullptr, nullptr};  // start / end of this worker's part of a run
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev[4];  // per kernel class (record_trace 2)
+    struct LayerEv {
+        int layer;
+        char dir;  // 'F' or 'B'
+        cudaEvent_t a, b;
+    };
+    std::vector<LayerEv> lev;  // layer profiling: one per layer per F / B op
     uint64_t launches = 0;
     uint64_t bytes_sent = 0;
     int updates_total = 0;  // Adam step counter base (persists across runs)
@@ -522,6 +529,20 @@ struct Exec {
         CK(cudaEventRecord(b, w->stream));
         w->kev[cls].push_back({a, b});
     }
+    // layer profiling (the self-profiler's T_l, L841-843): events around each layer's share of
+    // an F or B op; the op then runs serialised on the worker's stream (no side stream, no graphs)
+    cudaEvent_t lstart() {
+        if (!c->layer_prof || capturing) return nullptr;
+        cudaEvent_t a = w->ev_pool[ev_used++];
+        CK(cudaEventRecord(a, w->stream));
+        return a;
+    }
+    void lend(int l, char dir, cudaEvent_t a) {
+        if (!a) return;
+        cudaEvent_t b = w->ev_pool[ev_used++];
+        CK(cudaEventRecord(b, w->stream));
+        w->lev.push_back({l, dir, a, b});
+    }
     void record_start() {
         if (!timing) return;
         cudaEvent_t a = w->ev_pool[ev_used++];
@@ -582,6 +603,7 @@ struct Exec {
         }
         const long lrows = rows_of(layer(w->last), B());
         const int32_t *labels = (s + 1 == n()) ? w->labels + (long)(t % c->n_data) * lrows : nullptr;
+        cudaEvent_t last_l0 = nullptr;
         auto body = [&](float *loss_dst) {
         if (w->fbias && w->n_breg)  // vertical sync, bf16: fp32 biases of the stashed version `slot`
             CK(regions_bf16_to_f32(static_cast<const __nv_bfloat16 *>(w->wslot[slot]), w->fbias, w->breg_off,
@@ -592,6 +614,7 @@ struct Exec {
             void *y = l < w->last ? elem_ptr(w->act[l + 1 - w->first],
                                              (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz)
                                   : y_last;
+            cudaEvent_t l0 = lstart();
             cudaEvent_t k0 = kstart(0);
             if (d.kind == PD_LINEAR) {
                 LayerCtx lc{c, w, bf16};
@@ -610,10 +633,13 @@ struct Exec {
                 throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
             }
             kend(0, k0);
+            if (l < w->last || s + 1 < n()) lend(l, 'F', l0);
+            else last_l0 = l0;  // the loss belongs to the model's last layer
         }
         if (s + 1 == n()) {
             if (loss_dst == w->loss_scratch) CK(cudaMemsetAsync(loss_dst, 0, 4, w->stream));
             CK(softmax_ce(w->logits, bf16, labels, lrows, layer(w->last).out, w->dlogits, loss_dst, w->stream));
+            lend(w->last, 'F', last_l0);
         }
         };
         if (op_graphs_ok()) {
@@ -829,7 +855,7 @@ struct Exec {
             const char *e = getenv("PD_OP_GRAPHS");
             return e ? atoi(e) : 1;
         }();
-        if (!env || !bf16 || c->cfg.optimizer != PD_SGD) return false;
+        if (!env || !bf16 || c->cfg.optimizer != PD_SGD || c->layer_prof) return false;
         if (c->plan.stage[w->stage].replicas != 1) return false;
         if (timing && c->ktime_mask) return false;
         for (int l = w->first; l <= w->last; ++l)
@@ -1306,7 +1332,7 @@ struct Exec {
         BwdCtx bc{fused, gdst, nslot, sslot};
         bool all_linear = true;
         for (int l = w->first; l <= w->last; ++l) all_linear = all_linear && layer(l).kind == PD_LINEAR;
-        if (fused && all_linear && concurrent_dw()) {
+        if (fused && all_linear && concurrent_dw() && !c->layer_prof) {
             const void *dx_first = nullptr;
             if (!(s == 0 && w->first == 0)) {
                 const int Rp = c->plan.stage[s - 1].replicas;
@@ -1340,6 +1366,7 @@ struct Exec {
                     dx = w->scratch[cur ^ 1];
                 }
             }
+            cudaEvent_t l0 = lstart();
             if (d.kind == PD_LINEAR) linear_backward(l, x, G, dx, bc);
             else if (d.kind == PD_LSTM) lstm_backward(l, j, x, G, dx, bc);
             else if (d.kind == PD_EMBEDDING) embedding_backward(l, x, G, bc);
@@ -1353,6 +1380,7 @@ struct Exec {
                     kend(1, k0);
                 }
             } else throw CudaFail{cudaErrorNotSupported, "layer kind not implemented"};
+            lend(l, 'B', l0);
             G = dx;
             cur ^= 1;
         }
@@ -1981,7 +2009,9 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
             for (auto &e : w->run_ev)
                 if (!e) CK(cudaEventCreate(&e));
             const int nl = w->last - w->first + 1;
-            const size_t need = c->cfg.record_trace >= 2 ? (size_t)(6 + 8 * nl) * M + 16 : 0;
+            w->lev.clear();
+            const size_t need = (c->cfg.record_trace >= 2 ? (size_t)(6 + 8 * nl) * M + 16 : 0) +
+                                (c->layer_prof ? (size_t)4 * nl * M + 16 : 0);
             while (w->ev_pool.size() < need) {
                 cudaEvent_t e;
                 CK(cudaEventCreate(&e));
@@ -2141,6 +2171,95 @@ pd_status pd_set_timing(pd_ctx *c, int record_trace, int mask) {
     c->cfg.record_trace = record_trace;
     c->ktime_mask = mask & 0xF;
     return PD_OK;
+}
+
+pd_status pd_set_layer_profiling(pd_ctx *c, int on) {
+    CHECK_CTX(c);
+    c->layer_prof = on ? 1 : 0;
+    return PD_OK;
+}
+
+pd_status pd_get_layer_times(pd_ctx *c, double *fwd_s, double *bwd_s, size_t count) {
+    CHECK_CTX(c);
+    if (!fwd_s || !bwd_s || count != c->layers.size()) return PD_EINVAL;
+    std::vector<double> f(count, 0.0), b(count, 0.0);
+    std::vector<int> nf(count, 0), nb(count, 0);
+    for (auto &wp : c->W) {
+        Worker *w = wp.get();
+        if (!w) continue;
+        if (cudaSetDevice(w->device) != cudaSuccess) return PD_ECUDA;
+        for (auto &e : w->lev) {
+            float ms = 0.f;
+            if (cudaEventElapsedTime(&ms, e.a, e.b) != cudaSuccess) {
+                c->fail(PD_ECUDA, "pd_get_layer_times: event elapsed time");
+                return PD_ECUDA;
+            }
+            if (e.dir == 'F') f[e.layer] += ms * 1e-3, ++nf[e.layer];
+            else b[e.layer] += ms * 1e-3, ++nb[e.layer];
+        }
+    }
+    for (size_t l = 0; l < count; ++l) {
+        fwd_s[l] = nf[l] ? f[l] / nf[l] : 0.0;
+        bwd_s[l] = nb[l] ? b[l] / nb[l] : 0.0;
+    }
+    return PD_OK;
+}
+
+// The self-profiler: one single-stage (plain SGD/Adam, k = 1) pipeline of the whole model on
+// `cuda_device`, synthetic inputs, per-layer events around every layer's forward (+ loss on
+// the last layer) and backward (+ its fused weight update).
+pd_status pd_profile(const pd_layer_desc *layers, int num_layers, const pd_train_cfg *cfg_in, int cuda_device,
+                     int num_minibatches, pd_layer_profile *out) {
+    if (!layers || num_layers < 1 || !cfg_in || !out || num_minibatches < 1 || cuda_device < 0) return PD_EINVAL;
+    pd_plan_t plan{};
+    plan.num_stages = 1;
+    plan.stage[0] = {0, num_layers - 1, 1, 0};
+    plan.noam = 1;
+    pd_train_cfg cfg = *cfg_in;
+    cfg.record_trace = 0;
+    cfg.max_depth = 0;
+    cfg.sync_mode = PD_SYNC_STASH;
+    pd_ctx *c = nullptr;
+    pd_status st = pd_create(&c, &plan, layers, num_layers, &cfg);
+    if (st != PD_OK) return st;
+    // deterministic small parameters / inputs (a counter hash; values only need to be finite)
+    auto val = [](uint64_t i, float scale) {
+        uint64_t x = i * 0x9E3779B97F4A7C15ull;
+        x ^= x >> 29;
+        return scale * ((float)(x % 2001) / 1000.f - 1.f);
+    };
+    std::vector<std::vector<float>> p(num_layers);
+    std::vector<const float *> pp(num_layers, nullptr);
+    for (int l = 0; l < num_layers; ++l) {
+        const pd_layer_desc &d = layers[l];
+        const int fan = d.kind == PD_LSTM ? d.out : d.kind == PD_CONV3X3 ? 9 * d.in : d.in;
+        p[l].resize((size_t)c->hcount[l]);
+        for (size_t i = 0; i < p[l].size(); ++i) p[l][i] = val(i + 7919ull * l, 1.f / std::sqrt((float)std::max(fan, 1)));
+        pp[l] = p[l].empty() ? nullptr : p[l].data();
+    }
+    const int B = cfg.minibatch, nd = 2;
+    const long in_n = in_elems(layers[0], B), rows = rows_of(layers[num_layers - 1], B);
+    std::vector<float> x((size_t)nd * in_n);
+    std::vector<int32_t> tok((size_t)nd * in_n), lab((size_t)nd * rows);
+    for (size_t i = 0; i < x.size(); ++i) x[i] = val(i, 1.f);
+    for (size_t i = 0; i < tok.size(); ++i) tok[i] = (int32_t)(i % (size_t)std::max(layers[0].in, 1));
+    for (size_t i = 0; i < lab.size(); ++i) lab[i] = (int32_t)(i % (size_t)std::max(layers[num_layers - 1].out, 1));
+    const bool emb = layers[0].kind == PD_EMBEDDING;
+    std::vector<double> f(num_layers), b(num_layers);
+    if ((st = pd_stage_init(c, 0, 0, cuda_device, pp.data())) == PD_OK &&
+        (st = pd_set_data(c, emb ? nullptr : x.data(), emb ? tok.data() : nullptr, lab.data(), nd)) == PD_OK &&
+        (st = pd_run(c, 2, 0)) == PD_OK &&  // warm-up: allocations, tensor maps, graphs
+        (st = pd_set_layer_profiling(c, 1)) == PD_OK && (st = pd_run(c, num_minibatches, 0)) == PD_OK &&
+        (st = pd_get_layer_times(c, f.data(), b.data(), num_layers)) == PD_OK) {
+        const uint64_t esz = cfg.dtype == PD_BF16 ? 2 : 4;
+        for (int l = 0; l < num_layers; ++l) {
+            out[l].compute_s = f[l] + b[l];
+            out[l].act_bytes = (uint64_t)out_elems(layers[l], B) * esz;
+            out[l].param_bytes = (uint64_t)numel_params(layers[l]) * 4;  // fp32 gradients of the replica sync
+        }
+    }
+    pd_destroy(c);
+    return st;
 }
 
 void pd_destroy(pd_ctx *c) {

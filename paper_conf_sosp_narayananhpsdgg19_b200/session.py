@@ -7,9 +7,9 @@ from typing import Callable, Dict, List, Optional, Sequence
 
 import numpy as np
 
-from . import (PD_BF16, PD_SGD, Plan, pd_create, pd_destroy, pd_export_worker, pd_get_losses, pd_get_params,
-               pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data, pd_set_timing,
-               pd_stage_init, pd_run)
+from . import (PD_BF16, PD_SGD, Plan, pd_create, pd_destroy, pd_export_worker, pd_get_layer_times, pd_get_losses,
+               pd_get_params, pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data,
+               pd_set_layer_profiling, pd_set_timing, pd_stage_init, pd_run)
 
 
 def workers_of(plan: Plan):
@@ -78,6 +78,13 @@ class Pipeline:
 
     def set_timing(self, record_trace, kernel_timing_mask=0xF):
         pd_set_timing(self.ctx, record_trace, kernel_timing_mask)
+
+    def set_layer_profiling(self, on: bool):
+        pd_set_layer_profiling(self.ctx, on)
+
+    def layer_times(self):
+        """(forward s, backward s) per layer, mean per minibatch of the last run."""
+        return pd_get_layer_times(self.ctx, len(self.layers))
 
     def close(self):
         if self.ctx is not None:
