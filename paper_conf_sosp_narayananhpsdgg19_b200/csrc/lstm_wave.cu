@@ -1,0 +1,437 @@
+// lstm_wave.cu -- a stage's stack of LSTM layers as ONE wavefront kernel (bf16 path).
+//
+// Layer l's step t needs only layer l-1's step t (its input) and its own step t-1, so the
+// L layers of a stage can run as a wavefront: at wave w every layer l with t = w - l in
+// [0, T) advances one step, T + L - 1 waves instead of L * T dependent steps.  The per-step
+// work is the gate GEMM with the input projection folded in,
+//     forward   a[t] = [x_t | h_{t-1}] . [W_ih | W_hh]^T + b_ih + b_hh        (K = 2H)
+//     backward dh[t] = dy[t] + da[t+1] W_hh + da^{l+1}[t] W_ih^{l+1}          (K = 8H)
+// (dy of the stage's top layer comes from the stage's output gradient), which makes the
+// recurrence a weight-streaming problem -- all L layers' weights pass through the SMs once
+// per wave -- instead of a chain of latency-bound small GEMMs.
+//
+// Persistent, warp-specialised, one CTA per SM; every CTA owns a fixed list of work items
+// (layer, tile of hidden units) and walks the waves in order:
+//   warp 0  weight producer: TMA of the A tiles (weight rows) into an S-stage ring; runs ahead
+//           of the dependencies (weights never wait);
+//   warp 1  activation producer: waits for the item's inputs (per-layer step counters,
+//           acquire) and TMAs the B tiles (x_t / h_{t-1} or da) into the same ring stages;
+//   warp 2  MMA: tcgen05.mma M = 128, N = B rounded up to 16, into a double-buffered TMEM
+//           accumulator;
+//   warp 3  TMEM allocator;
+//   warps 4-7 epilogue: the LSTM cell (forward) or cell backward, stores, then publish the
+//           item (release) so dependent items of the next wave can start.
+// forward tile = 32 units (128 gate rows, gate-major: row = g*32 + u, K-major weights);
+// backward tile = 128 units (row = unit; W^T read untransposed as an MN-major operand).
+// All dependencies point to an earlier wave, and every CTA processes its items in wave
+// order, so the spin-waits cannot deadlock once the grid is resident.
+#include <cuda_bf16.h>
+
+#include <cstdio>
+#include <cstring>
+
+#include "pd_internal.h"
+#include "tc_ptx.h"
+
+namespace pd {
+namespace {
+using namespace tcx;
+
+constexpr int NT = 256;
+constexpr int ATILE = 128 * 128;         // [128 rows][64 K] bf16 (or 2 x [64 K][64 rows] MN-major)
+constexpr int BTILE = 64 * 128;          // [<= 64 rows][64 K] bf16
+constexpr int STAGE = ATILE + BTILE;
+constexpr int STG_LD = 68;               // forward epilogue staging row stride (floats)
+constexpr int STG_BYTES = 128 * STG_LD * 4;
+
+__device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long gtime() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ void wait_count(const unsigned *p, unsigned target) {
+    if (ld_acquire(p) >= target) return;
+    const unsigned long long t0 = gtime();
+    while (ld_acquire(p) < target) {
+        if (gtime() - t0 > 4000000000ull) {
+            printf("lstm_wave: dependency timeout (counter %u < %u)\n", ld_acquire(p), target);
+            __trap();
+        }
+    }
+}
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
+__device__ __forceinline__ void epi_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+struct WaveLayer {
+    const float *b_ih, *b_hh;  // forward
+    float *gates, *c;          // saved state [T][B][4H], [T][B][H] (written fwd, read bwd)
+    __nv_bfloat16 *h;          // forward output [T][B][H]
+    __nv_bfloat16 *da;         // backward output [T][B][4H]
+    float *dc;                 // backward carry [B][H] (scratch)
+};
+
+struct WaveMaps {
+    CUtensorMap w_ih[LSTM_WAVE_MAX_L], w_hh[LSTM_WAVE_MAX_L];
+    CUtensorMap act[LSTM_WAVE_MAX_L + 1];  // fwd: act[0] = stage input, act[l+1] = h of l; bwd: act[l] = da of l
+};
+
+struct WaveArgs {
+    int L, T, B, H, N, tiles;  // tiles per layer
+    WaveLayer layer[LSTM_WAVE_MAX_L];
+    const __nv_bfloat16 *dy_top;  // backward: gradient w.r.t. the top layer's output [T][B][H]
+    unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
+};
+
+// the item sequence of this CTA: items i = blockIdx.x + k * gridDim.x (i = l * tiles + tile),
+// visited wave by wave; returns false when done
+struct ItemIter {
+    int wave = 0, k = -1;
+    __device__ bool next(const WaveArgs &a, bool bwd, int &l, int &tile, int &t) {
+        const int items = a.L * a.tiles, waves = a.T + a.L - 1;
+        while (wave < waves) {
+            ++k;
+            const int i = blockIdx.x + k * gridDim.x;
+            if (i >= items) {
+                k = -1;
+                ++wave;
+                continue;
+            }
+            l = i / a.tiles;
+            tile = i % a.tiles;
+            t = bwd ? a.T - 1 - (wave - (a.L - 1 - l)) : wave - l;
+            if (t >= 0 && t < a.T) return true;
+        }
+        return false;
+    }
+};
+
+// K-blocks of an item: forward [x part (H/64) | h part (t > 0 ? H/64 : 0)];
+// backward [da[t+1] part (t < T-1 ? 4H/64 : 0) | da^{l+1}[t] part (l < L-1 ? 4H/64 : 0)]
+__device__ __forceinline__ void item_kbs(const WaveArgs &a, bool bwd, int l, int t, int &n0, int &n1) {
+    if (!bwd) {
+        n0 = a.H / 64;
+        n1 = t > 0 ? a.H / 64 : 0;
+    } else {
+        n0 = t < a.T - 1 ? 4 * a.H / 64 : 0;
+        n1 = l < a.L - 1 ? 4 * a.H / 64 : 0;
+    }
+}
+
+template <bool BWD>
+__global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *sm = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    constexpr int S = BWD ? 8 : 7;
+    float *stg = reinterpret_cast<float *>(sm + S * STAGE);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * STAGE + (BWD ? 0 : STG_BYTES));
+    // bars: full_w[S], full_x[S], empty[S], acc_full[2], acc_empty[2]
+    const uint32_t fw0 = smem_u32(bars), fx0 = smem_u32(bars + S), em0 = smem_u32(bars + 2 * S);
+    const uint32_t af0 = smem_u32(bars + 3 * S), ae0 = smem_u32(bars + 3 * S + 2);
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * S + 4);
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int H = a.H, B = a.B, N = a.N;
+
+    if (tid == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(fw0 + 8 * s, 1);
+            mbar_init(fx0 + 8 * s, 1);
+            mbar_init(em0 + 8 * s, 1);
+        }
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(af0 + 8 * b, 1);
+            mbar_init(ae0 + 8 * b, 128);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 3) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" ::"r"(smem_u32(tmem_slot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0 && lane == 0) {
+        // ---------------- weight producer
+        ItemIter it;
+        int l, tile, t, s = 0;
+        uint32_t ph = 0;
+        while (it.next(a, BWD, l, tile, t)) {
+            int n0, n1;
+            item_kbs(a, BWD, l, t, n0, n1);
+            for (int kb = 0; kb < n0 + n1; ++kb) {
+                mbar_wait(em0 + 8 * s, ph ^ 1);
+                const uint32_t dst = smem_u32(sm + s * STAGE);
+                mbar_expect_tx(fw0 + 8 * s, ATILE);
+                if (!BWD) {
+                    const CUtensorMap *w = kb < n0 ? &m.w_ih[l] : &m.w_hh[l];
+                    const int k = (kb < n0 ? kb : kb - n0) * 64;
+                    for (int g = 0; g < 4; ++g) tma_load_2d(dst + g * 4096, w, fw0 + 8 * s, k, g * H + tile * 32);
+                } else {
+                    const CUtensorMap *w = kb < n0 ? &m.w_hh[l] : &m.w_ih[l + 1];
+                    const int r = (kb < n0 ? kb : kb - n0) * 64;
+                    for (int jj = 0; jj < 2; ++jj) tma_load_2d(dst + jj * 8192, w, fw0 + 8 * s, tile * 128 + 64 * jj, r);
+                }
+                if (++s == S) s = 0, ph ^= 1;
+            }
+        }
+    } else if (warp == 1 && lane == 0) {
+        // ---------------- activation producer (waits for the item's inputs)
+        ItemIter it;
+        int l, tile, t, s = 0;
+        uint32_t ph = 0;
+        while (it.next(a, BWD, l, tile, t)) {
+            int n0, n1;
+            item_kbs(a, BWD, l, t, n0, n1);
+            if (n0 + n1 == 0) continue;
+            if (!BWD) {
+                if (l > 0) wait_count(a.cnt + l - 1, (unsigned)(t + 1) * a.tiles);  // x_t = h^{l-1}[t]
+                if (n1) wait_count(a.cnt + l, (unsigned)t * a.tiles);                // h^l[t-1]
+            } else {
+                if (n0) wait_count(a.cnt + l, (unsigned)(a.T - 1 - t) * a.tiles);    // da^l[t+1]
+                if (n1) wait_count(a.cnt + l + 1, (unsigned)(a.T - t) * a.tiles);    // da^{l+1}[t]
+            }
+            fence_proxy_async_global();
+            for (int kb = 0; kb < n0 + n1; ++kb) {
+                mbar_wait(em0 + 8 * s, ph ^ 1);
+                const uint32_t dst = smem_u32(sm + s * STAGE + ATILE);
+                mbar_expect_tx(fx0 + 8 * s, (uint32_t)N * 128);
+                if (!BWD) {
+                    if (kb < n0) tma_load_2d(dst, &m.act[l], fx0 + 8 * s, kb * 64, t * B);
+                    else tma_load_2d(dst, &m.act[l + 1], fx0 + 8 * s, (kb - n0) * 64, (t - 1) * B);
+                } else {
+                    if (kb < n0) tma_load_2d(dst, &m.act[l], fx0 + 8 * s, kb * 64, (t + 1) * B);
+                    else tma_load_2d(dst, &m.act[l + 1], fx0 + 8 * s, (kb - n0) * 64, t * B);
+                }
+                if (++s == S) s = 0, ph ^= 1;
+            }
+        }
+    } else if (warp == 2 && lane == 0) {
+        // ---------------- MMA issuer
+        const uint32_t idesc = make_idesc(128, N, BWD ? 1 : 0, 0);
+        ItemIter it;
+        int l, tile, t, s = 0, acc = 0;
+        uint32_t ph = 0, aph[2] = {0, 0};
+        while (it.next(a, BWD, l, tile, t)) {
+            int n0, n1;
+            item_kbs(a, BWD, l, t, n0, n1);
+            mbar_wait(ae0 + 8 * acc, aph[acc] ^ 1);  // epilogue drained this accumulator
+            tc_fence_after();
+            const uint32_t d = tmem + acc * 64;
+            for (int kb = 0; kb < n0 + n1; ++kb) {
+                mbar_wait(fw0 + 8 * s, ph);
+                mbar_wait(fx0 + 8 * s, ph);
+                tc_fence_after();
+                const uint32_t sa = smem_u32(sm + s * STAGE), sb = sa + ATILE;
+#pragma unroll
+                for (int kk = 0; kk < 4; ++kk) {
+                    const uint64_t ad = BWD ? smem_desc(sa + kk * 2048, 8192, 1024) : smem_desc(sa + kk * 32, 16, 1024);
+                    const uint64_t bd = smem_desc(sb + kk * 32, 16, 1024);
+                    tc_mma(d, ad, bd, idesc, (kb | kk) != 0);
+                }
+                tc_commit(em0 + 8 * s);
+                if (++s == S) s = 0, ph ^= 1;
+            }
+            if (n0 + n1) tc_commit(af0 + 8 * acc);
+            else mbar_arrive(af0 + 8 * acc);  // nothing to multiply: the epilogue uses 0
+            aph[acc] ^= 1;
+            acc ^= 1;
+        }
+    } else if (warp >= 4) {
+        // ---------------- epilogue
+        const int q = warp - 4;  // TMEM lane quadrant
+        const int et = tid - 128;
+        ItemIter it;
+        int l, tile, t, acc = 0;
+        uint32_t aph[2] = {0, 0};
+        while (it.next(a, BWD, l, tile, t)) {
+            int n0, n1;
+            item_kbs(a, BWD, l, t, n0, n1);
+            const bool mm = n0 + n1 > 0;
+            mbar_wait(af0 + 8 * acc, aph[acc]);
+            aph[acc] ^= 1;
+            tc_fence_after();
+            const uint32_t d = tmem + acc * 64 + ((uint32_t)(q * 32) << 16);
+            const WaveLayer &Ly = a.layer[l];
+            if (!BWD) {
+                // stage D[row = g*32 + u][b] so one thread sees all four gates of (u, b)
+                const int row = q * 32 + lane;
+#pragma unroll
+                for (int ch = 0; ch < 2; ++ch) {
+                    float v[32];
+                    tmem_ld32(d + ch * 32, v);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i)
+                        *reinterpret_cast<float4 *>(stg + row * STG_LD + ch * 32 + i * 4) =
+                            make_float4(v[i * 4], v[i * 4 + 1], v[i * 4 + 2], v[i * 4 + 3]);
+                }
+                tc_fence_before();
+                mbar_arrive(ae0 + 8 * acc);
+                epi_sync();
+                const int b = et & 63, u0 = (et >> 6) * 16, j0 = tile * 32 + u0;
+                if (b < B) {
+                    const long r1 = ((long)t * B + b) * H, r4 = ((long)t * B + b) * 4 * H;
+#pragma unroll
+                    for (int u4 = 0; u4 < 16; u4 += 4) {
+                        const int j = j0 + u4;
+                        float gv[4][4];
+#pragma unroll
+                        for (int g = 0; g < 4; ++g) {
+                            const float4 bi = *reinterpret_cast<const float4 *>(Ly.b_ih + g * H + j);
+                            const float4 bh = *reinterpret_cast<const float4 *>(Ly.b_hh + g * H + j);
+                            const float bb[4] = {bi.x + bh.x, bi.y + bh.y, bi.z + bh.z, bi.w + bh.w};
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) gv[g][e] = stg[(g * 32 + u0 + u4 + e) * STG_LD + b] + bb[e];
+                        }
+                        float cp[4] = {0.f, 0.f, 0.f, 0.f};
+                        if (t > 0) {
+                            const float4 c4 = *reinterpret_cast<const float4 *>(Ly.c + r1 - (long)B * H + j);
+                            cp[0] = c4.x, cp[1] = c4.y, cp[2] = c4.z, cp[3] = c4.w;
+                        }
+                        float ig[4], fg[4], gg[4], og[4], cc[4], hh[4];
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            ig[e] = sigm(gv[0][e]);
+                            fg[e] = sigm(gv[1][e]);
+                            gg[e] = tanhf(gv[2][e]);
+                            og[e] = sigm(gv[3][e]);
+                            cc[e] = fg[e] * cp[e] + ig[e] * gg[e];
+                            hh[e] = og[e] * tanhf(cc[e]);
+                        }
+                        uint2 p;
+                        p.x = pack_bf16(hh[0], hh[1]);
+                        p.y = pack_bf16(hh[2], hh[3]);
+                        *reinterpret_cast<uint2 *>(Ly.h + r1 + j) = p;
+                        *reinterpret_cast<float4 *>(Ly.c + r1 + j) = make_float4(cc[0], cc[1], cc[2], cc[3]);
+                        *reinterpret_cast<float4 *>(Ly.gates + r4 + j) = make_float4(ig[0], ig[1], ig[2], ig[3]);
+                        *reinterpret_cast<float4 *>(Ly.gates + r4 + H + j) = make_float4(fg[0], fg[1], fg[2], fg[3]);
+                        *reinterpret_cast<float4 *>(Ly.gates + r4 + 2 * H + j) = make_float4(gg[0], gg[1], gg[2], gg[3]);
+                        *reinterpret_cast<float4 *>(Ly.gates + r4 + 3 * H + j) = make_float4(og[0], og[1], og[2], og[3]);
+                    }
+                }
+            } else {
+                // thread = hidden unit j (TMEM lane), loops over the batch (TMEM column b)
+                const int j = tile * 128 + q * 32 + lane;
+                const bool top = l == a.L - 1;
+#pragma unroll
+                for (int ch = 0; ch < 2; ++ch) {
+                    float v[32];
+                    if (mm) {
+                        tmem_ld32(d + ch * 32, v);
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < 32; ++i) v[i] = 0.f;
+                    }
+                    if (ch == 1) {
+                        tc_fence_before();
+                        mbar_arrive(ae0 + 8 * acc);
+                    }
+#pragma unroll 8
+                    for (int i = 0; i < 32; ++i) {
+                        const int b = ch * 32 + i;
+                        if (b >= B) break;
+                        const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
+                        float dh = v[i];
+                        if (top) dh += __bfloat162float(a.dy_top[r1]);
+                        const float ig = Ly.gates[r4], fg = Ly.gates[r4 + H], gg = Ly.gates[r4 + 2 * H],
+                                    og = Ly.gates[r4 + 3 * H];
+                        const float ct = Ly.c[r1], cp = t > 0 ? Ly.c[r1 - (long)B * H] : 0.f;
+                        const float dcn = t < a.T - 1 ? Ly.dc[(long)b * H + j] : 0.f;
+                        const float tc = tanhf(ct);
+                        const float dct = dh * og * (1.f - tc * tc) + dcn;
+                        Ly.dc[(long)b * H + j] = dct * fg;
+                        Ly.da[r4] = __float2bfloat16_rn(dct * gg * ig * (1.f - ig));
+                        Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp * fg * (1.f - fg));
+                        Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig * (1.f - gg * gg));
+                        Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og * (1.f - og));
+                    }
+                }
+            }
+            epi_sync();
+            if (et == 0) {
+                asm volatile("fence.acq_rel.gpu;" ::: "memory");
+                asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(a.cnt + l) : "memory");
+            }
+            acc ^= 1;
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 3) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
+}
+
+int wave_smem(bool bwd) { return (bwd ? 8 * STAGE : 7 * STAGE + STG_BYTES) + 256 + 1024; }
+
+}  // namespace
+
+int lstm_wave_grid(int L, int H, bool bwd) {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    const int items = L * (bwd ? H / 128 : H / 32);
+    return items < sms ? items : sms;
+}
+
+bool lstm_wave_supported(int L, int B, int H, int I) {
+    if (L < 1 || L > LSTM_WAVE_MAX_L || B < 1 || B > 64 || H < 128 || H % 128 || I != H) return false;
+    static int ok[2] = {0, 0};
+    for (int bwd = 0; bwd < 2; ++bwd) {
+        if (ok[bwd]) continue;
+        const void *k = bwd ? (const void *)lstm_wave_kernel<true> : (const void *)lstm_wave_kernel<false>;
+        int n = 0;
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, wave_smem(bwd)) != cudaSuccess ||
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k, NT, wave_smem(bwd)) != cudaSuccess || n < 1) {
+            cudaGetLastError();
+            ok[bwd] = -1;
+        } else {
+            ok[bwd] = 1;
+        }
+    }
+    return ok[0] > 0 && ok[1] > 0;
+}
+
+cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
+    const int L = w.L, H = w.H, T = w.T, B = w.B;
+    if (!lstm_wave_supported(L, B, H, H)) return cudaErrorNotSupported;
+    WaveArgs a{};
+    a.L = L, a.T = T, a.B = B, a.H = H, a.N = (B + 15) / 16 * 16;
+    a.tiles = w.bwd ? H / 128 : H / 32;
+    a.dy_top = w.dy_top;
+    a.cnt = w.cnt;
+    WaveMaps m;
+    std::memset(&m, 0, sizeof(m));
+    const long TB = (long)T * B;
+    for (int l = 0; l < L; ++l) {
+        a.layer[l] = {w.b_ih[l], w.b_hh[l], w.gates[l], w.c[l], w.h[l], w.da[l], w.dc[l]};
+        const int rows = w.bwd ? 64 : 32, cols = 64;
+        if (!tma_map_bf16(&m.w_ih[l], w.W_ih[l], H, 4L * H, H, cols, rows) ||
+            !tma_map_bf16(&m.w_hh[l], w.W_hh[l], H, 4L * H, H, cols, rows))
+            return cudaErrorInvalidValue;
+        if (!w.bwd) {
+            if (!tma_map_bf16(&m.act[l + 1], w.h[l], H, TB, H, 64, a.N)) return cudaErrorInvalidValue;
+        } else if (!tma_map_bf16(&m.act[l], w.da[l], 4L * H, TB, 4L * H, 64, a.N)) {
+            return cudaErrorInvalidValue;
+        }
+    }
+    if (!w.bwd && !tma_map_bf16(&m.act[0], w.x, H, TB, H, 64, a.N)) return cudaErrorInvalidValue;
+    cudaError_t e = cudaMemsetAsync(w.cnt, 0, sizeof(unsigned) * L, s);
+    if (e != cudaSuccess) return e;
+    const int grid = lstm_wave_grid(L, H, w.bwd);
+    ++tl_launches;
+    if (w.bwd) lstm_wave_kernel<true><<<grid, NT, wave_smem(true), s>>>(m, a);
+    else lstm_wave_kernel<false><<<grid, NT, wave_smem(false), s>>>(m, a);
+    return cudaGetLastError();
+}
+
+}  // namespace pd

@@ -162,6 +162,23 @@ cudaError_t lstm_rec_fwd(const float *gx, const float *b_ih, const float *b_hh, 
 cudaError_t lstm_rec_bwd(const __nv_bfloat16 *dy, const float *gates, const float *c, const __nv_bfloat16 *Whh,
                          __nv_bfloat16 *da, unsigned *cnt, int T, int B, int H, cudaStream_t s,
                          unsigned long long *probe = nullptr);
+// A stage's stack of L LSTM layers (H = in = out, bf16) as ONE wavefront kernel per direction
+// (lstm_wave.cu): the input projection is folded into the per-step GEMM and every layer
+// advances one step per wave.  Per layer: weights of the version used, saved state
+// (gates / c / h as the per-layer path lays them out), da output, dc scratch [B][H].
+constexpr int LSTM_WAVE_MAX_L = 16;
+struct LstmWaveDesc {
+    int bwd = 0, L = 0, T = 0, B = 0, H = 0;
+    const __nv_bfloat16 *x = nullptr;       // forward: input of the bottom layer [T][B][H]
+    const __nv_bfloat16 *dy_top = nullptr;  // backward: gradient of the top layer's output
+    const __nv_bfloat16 *W_ih[LSTM_WAVE_MAX_L] = {}, *W_hh[LSTM_WAVE_MAX_L] = {};
+    const float *b_ih[LSTM_WAVE_MAX_L] = {}, *b_hh[LSTM_WAVE_MAX_L] = {};
+    float *gates[LSTM_WAVE_MAX_L] = {}, *c[LSTM_WAVE_MAX_L] = {}, *dc[LSTM_WAVE_MAX_L] = {};
+    __nv_bfloat16 *h[LSTM_WAVE_MAX_L] = {}, *da[LSTM_WAVE_MAX_L] = {};
+    unsigned *cnt = nullptr;  // >= L uints (zeroed by lstm_wave on the stream)
+};
+bool lstm_wave_supported(int L, int B, int H, int I);
+cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s);
 cudaError_t lstm_cell_bwd(int bf16, const void *dy, const float *dh_rec, const float *gates, const float *c,
                           const float *c_prev, float *dc, void *da, int B, int H, cudaStream_t s);
 cudaError_t embedding_fwd(int bf16, const int32_t *tok, const void *E, void *y, long rows, int H, cudaStream_t s);

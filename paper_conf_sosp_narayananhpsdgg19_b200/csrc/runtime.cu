@@ -274,6 +274,8 @@ struct Worker {
     float *lstm_gx = nullptr, *lstm_gh = nullptr, *lstm_dh = nullptr, *lstm_dc = nullptr;
     void *lstm_da = nullptr;
     unsigned *lstm_cnt = nullptr;  // step counters of the persistent recurrence kernels
+    void *lstm_wda = nullptr;      // wavefront backward: da of every layer of an LSTM run
+    float *lstm_wdc = nullptr;     // ... and their dc carries
     int lstm_rec = -1;             // persistent recurrences usable (-1 = not decided yet)
     // CUDA graphs of the LSTM recurrences (T steps of small GEMM + cell kernels), keyed by
     // (layer, direction, saved-state slot, weight slot, dY pointer): replayed instead of
@@ -316,7 +318,7 @@ Worker::~Worker() {
     for (void *p : act) cudaFree(p);
     for (void *p : aux)
         if (p) cudaFree(p);
-    void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da, lstm_cnt};
+    void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da, lstm_cnt, lstm_wda, lstm_wdc};
     for (void *p : lb)
         if (p) cudaFree(p);
     void *bufs[] = {master, fbias, (void *)breg_off, (void *)breg_cnt, adam_m, adam_v, gbuf, ws, (void *)split_counters, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
@@ -614,6 +616,13 @@ struct Exec {
             void *y = l < w->last ? elem_ptr(w->act[l + 1 - w->first],
                                              (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz)
                                   : y_last;
+            if (const int run = lstm_wave_run(l)) {
+                cudaEvent_t k0 = kstart(0);
+                lstm_wave_forward(l, run, t, j, slot, y_last);
+                kend(0, k0);
+                l += run - 1;
+                continue;
+            }
             cudaEvent_t l0 = lstart();
             cudaEvent_t k0 = kstart(0);
             if (d.kind == PD_LINEAR) {
@@ -866,7 +875,8 @@ struct Exec {
     // Persistent recurrences (lstm_rec.cu): bf16 path, supported shape, co-resident grid, and
     // no other LSTM-bearing worker on this GPU (two spinning grids could each hold half the
     // SMs the other needs).  PD_LSTM_REC=0 forces the per-step path.
-    bool use_lstm_rec(const pd_layer_desc &d, int Bn) {
+    bool use_lstm_rec(const pd_layer_desc &d, int Bn) { return lstm_rec_allowed() && lstm_rec_supported(Bn, d.out); }
+    bool lstm_rec_allowed() {
         if (!bf16) return false;
         if (w->lstm_rec < 0) {
             const char *env = getenv("PD_LSTM_REC");
@@ -881,7 +891,100 @@ struct Exec {
             }
             w->lstm_rec = (env && env[0] == '0') || others ? 0 : 1;
         }
-        return w->lstm_rec && lstm_rec_supported(Bn, d.out);
+        return w->lstm_rec != 0;
+    }
+
+    // ---------------- wavefront over a run of LSTM layers (lstm_wave.cu)
+    // Length of the run of LSTM layers starting at l that runs as one wavefront (>= 2 equal
+    // layers, H = in = out, same T; bf16; the co-residency rule of use_lstm_rec), else 0.
+    int lstm_wave_run(int l) {
+        const char *env = getenv("PD_LSTM_WAVE");  // 0 = per-layer recurrences (tools / tests)
+        if ((env && env[0] == '0') || !bf16 || c->layer_prof) return 0;
+        const pd_layer_desc &d = layer(l);
+        if (d.kind != PD_LSTM || d.in != d.out || !lstm_rec_allowed()) return 0;
+        int n = 1;
+        while (n < LSTM_WAVE_MAX_L && lstm_chain(l + n - 1)) ++n;
+        if (n < 2 || !lstm_wave_supported(n, B(), d.out, d.in)) return 0;
+        if (l > w->first && lstm_chain(l - 1)) return 0;  // not the start of its run
+        return n;
+    }
+    // layers a and a+1 are equal square LSTMs (a wavefront run continues through them)
+    bool lstm_chain(int a) const {
+        if (a + 1 > w->last) return false;
+        const pd_layer_desc &p = layer(a), &q = layer(a + 1);
+        return p.kind == PD_LSTM && q.kind == PD_LSTM && p.in == p.out && q.in == p.out && q.out == p.out &&
+               q.seq_len == p.seq_len;
+    }
+
+    void lstm_wave_forward(int l0, int L, int t, int j, int slot, void *y_last) {
+        const pd_layer_desc &d = layer(l0);
+        const int T = d.seq_len, Bn = B(), H = d.out;
+        const long TB = (long)T * Bn;
+        LstmWaveDesc wd;
+        wd.bwd = 0, wd.L = L, wd.T = T, wd.B = Bn, wd.H = H;
+        wd.x = static_cast<const __nv_bfloat16 *>(layer_input(l0, t, j));
+        wd.cnt = w->lstm_cnt;
+        for (int i = 0; i < L; ++i) {
+            const int l = l0 + i;
+            LstmState st = lstm_state(l, j);
+            wd.W_ih[i] = static_cast<const __nv_bfloat16 *>(elem_ptr(w->wslot[slot], lstm_off(l, 0), esz));
+            wd.W_hh[i] = static_cast<const __nv_bfloat16 *>(elem_ptr(w->wslot[slot], lstm_off(l, 1), esz));
+            wd.b_ih[i] = param_f32(lstm_off(l, 2), slot);
+            wd.b_hh[i] = param_f32(lstm_off(l, 3), slot);
+            wd.gates[i] = st.gates, wd.c[i] = st.c, wd.h[i] = static_cast<__nv_bfloat16 *>(st.h);
+        }
+        CK(lstm_wave(wd, w->stream));
+        // each layer's output to the next layer's input stash (its backward reads it) / the
+        // stage output
+        for (int i = 0; i < L; ++i) {
+            const int l = l0 + i;
+            void *y = l < w->last ? elem_ptr(w->act[l + 1 - w->first],
+                                             (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz)
+                                  : y_last;
+            CK(cudaMemcpyAsync(y, lstm_state(l, j).h, (size_t)TB * H * esz, cudaMemcpyDeviceToDevice, w->stream));
+        }
+    }
+
+    void lstm_wave_backward(int l0, int L, int t, int j, const void *G, void *dx, const BwdCtx &bc) {
+        const pd_layer_desc &d = layer(l0);
+        const int T = d.seq_len, Bn = B(), H = d.out;
+        const long TB = (long)T * Bn;
+        if (!w->lstm_wda) {
+            w->lstm_wda = dalloc<void>((size_t)LSTM_WAVE_MAX_L * TB * 4 * H * esz);
+            w->lstm_wdc = dalloc<float>((size_t)LSTM_WAVE_MAX_L * Bn * H * 4);
+        }
+        LstmWaveDesc wd;
+        wd.bwd = 1, wd.L = L, wd.T = T, wd.B = Bn, wd.H = H;
+        wd.dy_top = static_cast<const __nv_bfloat16 *>(G);
+        wd.cnt = w->lstm_cnt;
+        for (int i = 0; i < L; ++i) {
+            const int l = l0 + i;
+            LstmState st = lstm_state(l, j);
+            wd.W_ih[i] = static_cast<const __nv_bfloat16 *>(elem_ptr(w->wslot[bc.sslot], lstm_off(l, 0), esz));
+            wd.W_hh[i] = static_cast<const __nv_bfloat16 *>(elem_ptr(w->wslot[bc.sslot], lstm_off(l, 1), esz));
+            wd.gates[i] = st.gates, wd.c[i] = st.c;
+            wd.da[i] = static_cast<__nv_bfloat16 *>(elem_ptr(w->lstm_wda, (long)i * TB * 4 * H, esz));
+            wd.dc[i] = w->lstm_wdc + (long)i * Bn * H;
+        }
+        cudaEvent_t k0 = kstart(1);
+        CK(lstm_wave(wd, w->stream));
+        // the bottom layer's input gradient (inner layers' are folded into the wavefront)
+        if (dx) gemm_dx(l0, (int)TB, H, 4 * H, wd.da[0], 4 * H, wd.W_ih[0], H, layer_input(l0, t, j), dx);
+        kend(1, k0);
+        k0 = kstart(2);
+        for (int i = L - 1; i >= 0; --i) {
+            const int l = l0 + i;
+            gemm_dw(bc, lstm_off(l, 0), 4 * H, H, (int)TB, wd.da[i], 4 * H, layer_input(l, t, j), H);
+            gemm_dw(bc, lstm_off(l, 1), 4 * H, H, (int)((T - 1) * (long)Bn), elem_ptr(wd.da[i], (long)Bn * 4 * H, esz),
+                    4 * H, lstm_state(l, j).h, H);
+        }
+        kend(2, k0);
+        k0 = kstart(3);
+        for (int i = L - 1; i >= 0; --i) {
+            bias_update(bc, lstm_off(l0 + i, 2), wd.da[i], TB, 4 * H);
+            bias_update(bc, lstm_off(l0 + i, 3), wd.da[i], TB, 4 * H);
+        }
+        kend(3, k0);
     }
 
     void lstm_forward(int l, int j, int slot, const void *x, void *y) {
@@ -1351,6 +1454,12 @@ struct Exec {
             }
         } else
         for (int l = w->last; l >= w->first; --l) {
+            // top layer of a wavefront run: the whole run's backward in one go
+            int run_first = l;
+            while (run_first > w->first && lstm_chain(run_first - 1)) --run_first;
+            const int run = lstm_wave_run(run_first);
+            const bool wave = run > 0 && run_first + run - 1 == l;
+            if (wave) l = run_first;  // dX below is the run's bottom layer's
             const pd_layer_desc &d = layer(l);
             const void *x = layer_input(l, t, j);
             const bool need_dx = !(s == 0 && l == 0) && d.kind != PD_EMBEDDING;
@@ -1367,7 +1476,8 @@ struct Exec {
                 }
             }
             cudaEvent_t l0 = lstart();
-            if (d.kind == PD_LINEAR) linear_backward(l, x, G, dx, bc);
+            if (wave) lstm_wave_backward(l, lstm_wave_run(l), t, j, G, dx, bc);
+            else if (d.kind == PD_LINEAR) linear_backward(l, x, G, dx, bc);
             else if (d.kind == PD_LSTM) lstm_backward(l, j, x, G, dx, bc);
             else if (d.kind == PD_EMBEDDING) embedding_backward(l, x, G, bc);
             else if (d.kind == PD_CONV3X3) conv_backward(l, x, G, dx, bc);

@@ -18,24 +18,29 @@ from gpu_helpers import run_both, assert_schedule_exact, param_errors, BF16_TOL
 
 pytestmark = pytest.mark.gpu
 
-# (layers, H, B, T): ragged batch (N = 48 > B = 40), full GNMT width with one and two layers
+# (layers, H, B, T): ragged batch (N = 48 > B = 40), full GNMT width with one and two layers.
+# One layer runs the persistent per-layer kernels; runs of >= 2 layers the wavefront kernel
+# (lstm_wave.cu) unless PD_LSTM_WAVE=0.
 SHAPES = [(2, 256, 16, 6), (1, 512, 40, 5), (1, 1024, 64, 4), (2, 1024, 64, 3)]
+WAVE_SHAPES = [(4, 256, 16, 6), (3, 512, 40, 5), (8, 128, 8, 4), (4, 1024, 64, 3)]
 
 
 def _workload(n, H, B, T):
     return synth.Workload(f"lstm{n}x{H}", synth.gnmt(n, H, 512, T, B), B, synth.SGD, 0.05)
 
 
-def _run(wl, last, M, rec):
-    old = os.environ.get("PD_LSTM_REC")
+def _run(wl, last, M, rec, wave=True):
+    old = {k: os.environ.get(k) for k in ("PD_LSTM_REC", "PD_LSTM_WAVE")}
     os.environ["PD_LSTM_REC"] = "1" if rec else "0"
+    os.environ["PD_LSTM_WAVE"] = "1" if wave else "0"
     try:
         return run_both(wl, last, [1] * len(last), M, pd.PD_BF16, n_data=3)
     finally:
-        if old is None:
-            del os.environ["PD_LSTM_REC"]
-        else:
-            os.environ["PD_LSTM_REC"] = old
+        for k, v in old.items():
+            if v is None:
+                del os.environ[k]
+            else:
+                os.environ[k] = v
 
 
 @pytest.mark.parametrize("n,H,B,T", SHAPES)
@@ -65,6 +70,37 @@ def test_persistent_two_stage_pipeline_only_first_worker_lstm():
     # stage 0 = Emb + LSTM (persistent: the only LSTM worker on the GPU), stage 1 = classifier
     wl = _workload(1, 256, 16, 5)
     res = _run(wl, [1, 2], 8, rec=True)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL and derr < 5e-2, (perr, derr)
+
+
+@pytest.mark.parametrize("n,H,B,T", WAVE_SHAPES)
+def test_wavefront_matches_oracle(n, H, B, T):
+    wl = _workload(n, H, B, T)
+    res = _run(wl, [len(wl.layers) - 1], 3, rec=True)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, perr
+    assert derr < 5e-2, derr
+    np.testing.assert_allclose(res["losses"], res["ref"].losses, rtol=1e-2)
+
+
+@pytest.mark.parametrize("n,H,B,T", WAVE_SHAPES[:2])
+def test_wavefront_equals_per_layer_kernels(n, H, B, T):
+    wl = _workload(n, H, B, T)
+    a = _run(wl, [len(wl.layers) - 1], 2, rec=True, wave=True)
+    b = _run(wl, [len(wl.layers) - 1], 2, rec=True, wave=False)
+    d = torchref.delta_err(a["got"], b["got"], a["p0"])
+    assert d < 2e-2, d
+    np.testing.assert_allclose(a["losses"], b["losses"], rtol=2e-3)
+
+
+def test_wavefront_inside_a_pipeline_stage():
+    # stage 0 = Emb + 3 LSTMs (one wavefront run, dX of the bottom layer into the embedding),
+    # stage 1 = classifier: startup / steady state / drain with stashed versions
+    wl = _workload(3, 256, 16, 5)
+    res = _run(wl, [3, 4], 8, rec=True)
     assert_schedule_exact(res)
     perr, derr = param_errors(res)
     assert perr < BF16_TOL and derr < 5e-2, (perr, derr)

@@ -129,3 +129,26 @@ def test_device_calls_fail_loudly_without_gpu():
     with pytest.raises(pd.PDError):
         pd.pd_run(ctx, 4)
     pd.pd_destroy(ctx)
+
+
+@pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU failure mode")
+def test_profiler_fails_loudly_without_gpu():
+    wl = synth.workload("mlp_small")
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_profile(wl.layers, pd.PD_FP32, minibatch=16)
+    assert ei.value.status in (pd.PD_ECUDA, pd.PD_EUNSUPPORTED)
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_profile([], pd.PD_FP32, minibatch=16)
+    assert ei.value.status == pd.PD_EINVAL
+
+
+def test_layer_time_queries_validate_arguments():
+    wl = synth.workload("mlp_small")
+    ctx = pd.pd_create(pd.Plan.manual([2], [1]), wl.layers, pd.PD_FP32, minibatch=16)
+    pd.pd_set_layer_profiling(ctx, True)
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_get_layer_times(ctx, len(wl.layers) + 1)
+    assert ei.value.status == pd.PD_EINVAL
+    f, b = pd.pd_get_layer_times(ctx, len(wl.layers))  # no run yet: zeros
+    assert not f.any() and not b.any()
+    pd.pd_destroy(ctx)
