@@ -514,8 +514,10 @@ cudaError_t launch_clustered(K kern, int grid, int csize, int smem, const CUtens
 }
 
 // can `grid` CTAs in clusters of `csize` (smem bytes each) all be resident at once?
-bool coresident(const void *kern, int grid, int csize, int smem) {
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) {
+// (the attribute is set to the largest size any supported H launches with, so launches of
+// different H, from several host threads, never race on it)
+bool coresident(const void *kern, int grid, int csize, int smem, int smem_max) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
@@ -545,8 +547,8 @@ bool lstm_rec_supported(int B, int H) {
     static int cache[5] = {};  // per H / 256
     int &c = cache[H / 256];
     if (!c) {
-        const bool ok = coresident((const void *)lstm_rec_fwd_kernel, H / 8, 4, fwd_smem(H)) &&
-                        coresident((const void *)lstm_rec_bwd_kernel, H / 16, 8, bwd_smem(H));
+        const bool ok = coresident((const void *)lstm_rec_fwd_kernel, H / 8, 4, fwd_smem(H), fwd_smem(1024)) &&
+                        coresident((const void *)lstm_rec_bwd_kernel, H / 16, 8, bwd_smem(H), bwd_smem(1024));
         c = ok ? 1 : -1;
     }
     return c > 0;
