@@ -43,6 +43,7 @@ constexpr int BTILE = 64 * 128;          // [<= 64 rows][64 K] bf16
 constexpr int STAGE = ATILE + BTILE;
 constexpr int STG_LD = 68;               // forward epilogue staging row stride (floats)
 constexpr int STG_BYTES = 128 * STG_LD * 4;
+constexpr int RECV_BYTES = 128 * 32 * 4;  // backward: the peer's partial for this CTA's batch half
 
 __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
     unsigned v;
@@ -88,15 +89,16 @@ struct WaveArgs {
     unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
 };
 
-// the item sequence of this CTA: items i = blockIdx.x + k * gridDim.x (i = l * tiles + tile),
-// visited wave by wave; returns false when done
+// the item sequence of this CTA (pair): items i = c + k * C (c = cluster index, C = clusters,
+// i = l * tiles + tile), visited wave by wave; returns false when done
+template <int CL>
 struct ItemIter {
     int wave = 0, k = -1;
     __device__ bool next(const WaveArgs &a, bool bwd, int &l, int &tile, int &t) {
         const int items = a.L * a.tiles, waves = a.T + a.L - 1;
         while (wave < waves) {
             ++k;
-            const int i = blockIdx.x + k * gridDim.x;
+            const int i = (int)(blockIdx.x / CL) + k * (int)(gridDim.x / CL);
             if (i >= items) {
                 k = -1;
                 ++wave;
@@ -113,29 +115,47 @@ struct ItemIter {
 
 // K-blocks of an item: forward [x part (H/64) | h part (t > 0 ? H/64 : 0)];
 // backward [da[t+1] part (t < T-1 ? 4H/64 : 0) | da^{l+1}[t] part (l < L-1 ? 4H/64 : 0)]
-__device__ __forceinline__ void item_kbs(const WaveArgs &a, bool bwd, int l, int t, int &n0, int &n1) {
+// The CTAs of a cluster split an item's K-blocks: this CTA (rank of csize) takes the global
+// K-block indices [lo, hi); index kb < n0 is part 0, else part 1 (kb - n0).
+struct ItemK {
+    int n0, n1, lo, hi;
+};
+__device__ __forceinline__ ItemK item_k(const WaveArgs &a, bool bwd, int l, int t, int rank, int csize) {
+    ItemK r;
     if (!bwd) {
-        n0 = a.H / 64;
-        n1 = t > 0 ? a.H / 64 : 0;
+        r.n0 = a.H / 64;
+        r.n1 = t > 0 ? a.H / 64 : 0;
     } else {
-        n0 = t < a.T - 1 ? 4 * a.H / 64 : 0;
-        n1 = l < a.L - 1 ? 4 * a.H / 64 : 0;
+        r.n0 = t < a.T - 1 ? 4 * a.H / 64 : 0;
+        r.n1 = l < a.L - 1 ? 4 * a.H / 64 : 0;
     }
+    const int tot = r.n0 + r.n1;
+    r.lo = tot * rank / csize;
+    r.hi = tot * (rank + 1) / csize;
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
 }
 
 template <bool BWD>
 __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *sm = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    constexpr int S = BWD ? 8 : 7;
-    float *stg = reinterpret_cast<float *>(sm + S * STAGE);
-    uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * STAGE + (BWD ? 0 : STG_BYTES));
-    // bars: full_w[S], full_x[S], empty[S], acc_full[2], acc_empty[2]
+    // backward: a cluster of 2 CTAs splits every item's K-blocks; each finishes half the batch
+    constexpr int S = BWD ? 8 : 7, CL = BWD ? 2 : 1;
+    float *stg = reinterpret_cast<float *>(sm + S * STAGE);  // fwd staging / bwd receive buffer
+    uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * STAGE + (BWD ? RECV_BYTES : STG_BYTES));
+    // bars: full_w[S], full_x[S], empty[S], acc_full[2], acc_empty[2], recv_full, recv_empty
     const uint32_t fw0 = smem_u32(bars), fx0 = smem_u32(bars + S), em0 = smem_u32(bars + 2 * S);
     const uint32_t af0 = smem_u32(bars + 3 * S), ae0 = smem_u32(bars + 3 * S + 2);
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * S + 4);
+    const uint32_t rfull = smem_u32(bars + 3 * S + 4), rempty = smem_u32(bars + 3 * S + 5);
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * S + 6);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int H = a.H, B = a.B, N = a.N;
+    const int rank = BWD ? (int)cluster_rank() : 0;
 
     if (tid == 0) {
         for (int s = 0; s < S; ++s) {
@@ -147,6 +167,8 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
             mbar_init(af0 + 8 * b, 1);
             mbar_init(ae0 + 8 * b, 128);
         }
+        mbar_init(rfull, 1);
+        mbar_init(rempty, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 3) {
@@ -155,60 +177,64 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
     }
     tc_fence_before();
     __syncthreads();
+    if (BWD) cluster_sync_all();  // the peer's barriers exist before any remote arrive / st.async
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    // published (step, tile, CTA) items of a layer per completed step
+    const unsigned per_step = (unsigned)a.tiles * CL;
 
     if (warp == 0 && lane == 0) {
         // ---------------- weight producer
-        ItemIter it;
+        ItemIter<CL> it;
         int l, tile, t, s = 0;
         uint32_t ph = 0;
         while (it.next(a, BWD, l, tile, t)) {
-            int n0, n1;
-            item_kbs(a, BWD, l, t, n0, n1);
-            for (int kb = 0; kb < n0 + n1; ++kb) {
+            const ItemK ik = item_k(a, BWD, l, t, rank, CL);
+            for (int kb = ik.lo; kb < ik.hi; ++kb) {
                 mbar_wait(em0 + 8 * s, ph ^ 1);
                 const uint32_t dst = smem_u32(sm + s * STAGE);
                 mbar_expect_tx(fw0 + 8 * s, ATILE);
+                const bool p1 = kb >= ik.n0;
+                const int k = (p1 ? kb - ik.n0 : kb) * 64;
                 if (!BWD) {
-                    const CUtensorMap *w = kb < n0 ? &m.w_ih[l] : &m.w_hh[l];
-                    const int k = (kb < n0 ? kb : kb - n0) * 64;
+                    const CUtensorMap *w = p1 ? &m.w_hh[l] : &m.w_ih[l];
                     for (int g = 0; g < 4; ++g) tma_load_2d(dst + g * 4096, w, fw0 + 8 * s, k, g * H + tile * 32);
                 } else {
-                    const CUtensorMap *w = kb < n0 ? &m.w_hh[l] : &m.w_ih[l + 1];
-                    const int r = (kb < n0 ? kb : kb - n0) * 64;
-                    for (int jj = 0; jj < 2; ++jj) tma_load_2d(dst + jj * 8192, w, fw0 + 8 * s, tile * 128 + 64 * jj, r);
+                    const CUtensorMap *w = p1 ? &m.w_ih[l + 1] : &m.w_hh[l];
+                    for (int jj = 0; jj < 2; ++jj) tma_load_2d(dst + jj * 8192, w, fw0 + 8 * s, tile * 128 + 64 * jj, k);
                 }
                 if (++s == S) s = 0, ph ^= 1;
             }
         }
     } else if (warp == 1 && lane == 0) {
         // ---------------- activation producer (waits for the item's inputs)
-        ItemIter it;
+        ItemIter<CL> it;
         int l, tile, t, s = 0;
         uint32_t ph = 0;
         while (it.next(a, BWD, l, tile, t)) {
-            int n0, n1;
-            item_kbs(a, BWD, l, t, n0, n1);
-            if (n0 + n1 == 0) continue;
+            const ItemK ik = item_k(a, BWD, l, t, rank, CL);
+            if (ik.lo == ik.hi) continue;
+            const bool need0 = ik.lo < ik.n0, need1 = ik.hi > ik.n0;
             if (!BWD) {
-                if (l > 0) wait_count(a.cnt + l - 1, (unsigned)(t + 1) * a.tiles);  // x_t = h^{l-1}[t]
-                if (n1) wait_count(a.cnt + l, (unsigned)t * a.tiles);                // h^l[t-1]
+                if (l > 0) wait_count(a.cnt + l - 1, (unsigned)(t + 1) * per_step);  // x_t = h^{l-1}[t]
+                if (need1) wait_count(a.cnt + l, (unsigned)t * per_step);            // h^l[t-1]
             } else {
-                if (n0) wait_count(a.cnt + l, (unsigned)(a.T - 1 - t) * a.tiles);    // da^l[t+1]
-                if (n1) wait_count(a.cnt + l + 1, (unsigned)(a.T - t) * a.tiles);    // da^{l+1}[t]
+                if (need0) wait_count(a.cnt + l, (unsigned)(a.T - 1 - t) * per_step);  // da^l[t+1]
+                if (need1) wait_count(a.cnt + l + 1, (unsigned)(a.T - t) * per_step);  // da^{l+1}[t]
             }
             fence_proxy_async_global();
-            for (int kb = 0; kb < n0 + n1; ++kb) {
+            for (int kb = ik.lo; kb < ik.hi; ++kb) {
                 mbar_wait(em0 + 8 * s, ph ^ 1);
                 const uint32_t dst = smem_u32(sm + s * STAGE + ATILE);
                 mbar_expect_tx(fx0 + 8 * s, (uint32_t)N * 128);
+                const bool p1 = kb >= ik.n0;
+                const int k = (p1 ? kb - ik.n0 : kb) * 64;
                 if (!BWD) {
-                    if (kb < n0) tma_load_2d(dst, &m.act[l], fx0 + 8 * s, kb * 64, t * B);
-                    else tma_load_2d(dst, &m.act[l + 1], fx0 + 8 * s, (kb - n0) * 64, (t - 1) * B);
+                    if (!p1) tma_load_2d(dst, &m.act[l], fx0 + 8 * s, k, t * B);
+                    else tma_load_2d(dst, &m.act[l + 1], fx0 + 8 * s, k, (t - 1) * B);
                 } else {
-                    if (kb < n0) tma_load_2d(dst, &m.act[l], fx0 + 8 * s, kb * 64, (t + 1) * B);
-                    else tma_load_2d(dst, &m.act[l + 1], fx0 + 8 * s, (kb - n0) * 64, t * B);
+                    if (!p1) tma_load_2d(dst, &m.act[l], fx0 + 8 * s, k, (t + 1) * B);
+                    else tma_load_2d(dst, &m.act[l + 1], fx0 + 8 * s, k, t * B);
                 }
                 if (++s == S) s = 0, ph ^= 1;
             }
@@ -216,16 +242,15 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
     } else if (warp == 2 && lane == 0) {
         // ---------------- MMA issuer
         const uint32_t idesc = make_idesc(128, N, BWD ? 1 : 0, 0);
-        ItemIter it;
+        ItemIter<CL> it;
         int l, tile, t, s = 0, acc = 0;
         uint32_t ph = 0, aph[2] = {0, 0};
         while (it.next(a, BWD, l, tile, t)) {
-            int n0, n1;
-            item_kbs(a, BWD, l, t, n0, n1);
+            const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             mbar_wait(ae0 + 8 * acc, aph[acc] ^ 1);  // epilogue drained this accumulator
             tc_fence_after();
             const uint32_t d = tmem + acc * 64;
-            for (int kb = 0; kb < n0 + n1; ++kb) {
+            for (int kb = ik.lo; kb < ik.hi; ++kb) {
                 mbar_wait(fw0 + 8 * s, ph);
                 mbar_wait(fx0 + 8 * s, ph);
                 tc_fence_after();
@@ -234,12 +259,12 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 for (int kk = 0; kk < 4; ++kk) {
                     const uint64_t ad = BWD ? smem_desc(sa + kk * 2048, 8192, 1024) : smem_desc(sa + kk * 32, 16, 1024);
                     const uint64_t bd = smem_desc(sb + kk * 32, 16, 1024);
-                    tc_mma(d, ad, bd, idesc, (kb | kk) != 0);
+                    tc_mma(d, ad, bd, idesc, (kb > ik.lo || kk) ? 1u : 0u);
                 }
                 tc_commit(em0 + 8 * s);
                 if (++s == S) s = 0, ph ^= 1;
             }
-            if (n0 + n1) tc_commit(af0 + 8 * acc);
+            if (ik.hi > ik.lo) tc_commit(af0 + 8 * acc);
             else mbar_arrive(af0 + 8 * acc);  // nothing to multiply: the epilogue uses 0
             aph[acc] ^= 1;
             acc ^= 1;
@@ -248,13 +273,12 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         // ---------------- epilogue
         const int q = warp - 4;  // TMEM lane quadrant
         const int et = tid - 128;
-        ItemIter it;
+        ItemIter<CL> it;
         int l, tile, t, acc = 0;
-        uint32_t aph[2] = {0, 0};
+        uint32_t aph[2] = {0, 0}, rph = 0, eph = 0;
         while (it.next(a, BWD, l, tile, t)) {
-            int n0, n1;
-            item_kbs(a, BWD, l, t, n0, n1);
-            const bool mm = n0 + n1 > 0;
+            const ItemK ik = item_k(a, BWD, l, t, rank, CL);
+            const bool mm = ik.hi > ik.lo;
             mbar_wait(af0 + 8 * acc, aph[acc]);
             aph[acc] ^= 1;
             tc_fence_after();
@@ -317,41 +341,63 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                     }
                 }
             } else {
-                // thread = hidden unit j (TMEM lane), loops over the batch (TMEM column b)
-                const int j = tile * 128 + q * 32 + lane;
+                // thread = hidden unit (TMEM lane m); this CTA finishes batch rows [hb, hb + 32)
+                // and swaps the other half of its K-partial with the peer CTA
+                const int mrow = q * 32 + lane, j = tile * 128 + mrow, hb = rank * 32;
+                float mine[32], other[32];
+                if (mm) {
+                    tmem_ld32(d + hb, mine);
+                    tmem_ld32(d + (32 - hb), other);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < 32; ++i) mine[i] = other[i] = 0.f;
+                }
+                tc_fence_before();
+                mbar_arrive(ae0 + 8 * acc);
+                if (ik.n0 + ik.n1 > 0) {
+                    const int peer = rank ^ 1;
+                    mbar_wait(rempty, eph ^ 1);  // the peer consumed the previous exchange
+                    eph ^= 1;
+                    const uint32_t dst = mapa_cluster(smem_u32(stg) + mrow * 32 * 4, peer);
+                    const uint32_t pbar = mapa_cluster(rfull, peer);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i)
+                        asm volatile(
+                            "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+                                dst + i * 16),
+                            "f"(other[i * 4]), "f"(other[i * 4 + 1]), "f"(other[i * 4 + 2]), "f"(other[i * 4 + 3]),
+                            "r"(pbar)
+                            : "memory");
+                    if (et == 0) mbar_expect_tx(rfull, 128 * 32 * 4);
+                    mbar_wait(rfull, rph);
+                    rph ^= 1;
+#pragma unroll
+                    for (int i = 0; i < 32; ++i) mine[i] += stg[mrow * 32 + i];
+                    epi_sync();  // every thread read its row: hand the buffer back to the peer
+                    if (et == 0)
+                        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
+                                         mapa_cluster(rempty, peer))
+                                     : "memory");
+                }
                 const bool top = l == a.L - 1;
-#pragma unroll
-                for (int ch = 0; ch < 2; ++ch) {
-                    float v[32];
-                    if (mm) {
-                        tmem_ld32(d + ch * 32, v);
-                    } else {
-#pragma unroll
-                        for (int i = 0; i < 32; ++i) v[i] = 0.f;
-                    }
-                    if (ch == 1) {
-                        tc_fence_before();
-                        mbar_arrive(ae0 + 8 * acc);
-                    }
 #pragma unroll 8
-                    for (int i = 0; i < 32; ++i) {
-                        const int b = ch * 32 + i;
-                        if (b >= B) break;
-                        const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
-                        float dh = v[i];
-                        if (top) dh += __bfloat162float(a.dy_top[r1]);
-                        const float ig = Ly.gates[r4], fg = Ly.gates[r4 + H], gg = Ly.gates[r4 + 2 * H],
-                                    og = Ly.gates[r4 + 3 * H];
-                        const float ct = Ly.c[r1], cp = t > 0 ? Ly.c[r1 - (long)B * H] : 0.f;
-                        const float dcn = t < a.T - 1 ? Ly.dc[(long)b * H + j] : 0.f;
-                        const float tc = tanhf(ct);
-                        const float dct = dh * og * (1.f - tc * tc) + dcn;
-                        Ly.dc[(long)b * H + j] = dct * fg;
-                        Ly.da[r4] = __float2bfloat16_rn(dct * gg * ig * (1.f - ig));
-                        Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp * fg * (1.f - fg));
-                        Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig * (1.f - gg * gg));
-                        Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og * (1.f - og));
-                    }
+                for (int i = 0; i < 32; ++i) {
+                    const int b = hb + i;
+                    if (b >= B) break;
+                    const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
+                    float dh = mine[i];
+                    if (top) dh += __bfloat162float(a.dy_top[r1]);
+                    const float ig = Ly.gates[r4], fg = Ly.gates[r4 + H], gg = Ly.gates[r4 + 2 * H],
+                                og = Ly.gates[r4 + 3 * H];
+                    const float ct = Ly.c[r1], cp = t > 0 ? Ly.c[r1 - (long)B * H] : 0.f;
+                    const float dcn = t < a.T - 1 ? Ly.dc[(long)b * H + j] : 0.f;
+                    const float tc = tanhf(ct);
+                    const float dct = dh * og * (1.f - tc * tc) + dcn;
+                    Ly.dc[(long)b * H + j] = dct * fg;
+                    Ly.da[r4] = __float2bfloat16_rn(dct * gg * ig * (1.f - ig));
+                    Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp * fg * (1.f - fg));
+                    Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig * (1.f - gg * gg));
+                    Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og * (1.f - og));
                 }
             }
             epi_sync();
@@ -364,14 +410,14 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
     }
     tc_fence_before();
     __syncthreads();
+    if (BWD) cluster_sync_all();  // no peer st.async / arrive may target an exited CTA
     if (warp == 3) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
 }
 
-int wave_smem(bool bwd) { return (bwd ? 8 * STAGE : 7 * STAGE + STG_BYTES) + 256 + 1024; }
+int wave_smem(bool bwd) { return (bwd ? 8 * STAGE + RECV_BYTES : 7 * STAGE + STG_BYTES) + 256 + 1024; }
 
-}  // namespace
 
-int lstm_wave_grid(int L, int H, bool bwd) {
+int num_sm() {
     static int sms = 0;
     if (!sms) {
         int dev = 0;
@@ -379,26 +425,68 @@ int lstm_wave_grid(int L, int H, bool bwd) {
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (sms <= 0) sms = 148;
     }
-    const int items = L * (bwd ? H / 128 : H / 32);
-    return items < sms ? items : sms;
+    return sms;
 }
+
+// forward: one CTA per item up to one per SM; backward: a CTA pair per item up to one pair
+// per two SMs (and no more pairs than can be resident at once)
+int wave_grid(int L, int H, bool bwd, int max_pairs) {
+    const int items = L * (bwd ? H / 128 : H / 32);
+    if (!bwd) return items < num_sm() ? items : num_sm();
+    const int pairs = items < max_pairs ? items : max_pairs;
+    return 2 * pairs;
+}
+
+cudaLaunchConfig_t wave_cfg(bool bwd, int grid, cudaStream_t s, cudaLaunchAttribute *attr) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(NT);
+    cfg.dynamicSmemBytes = wave_smem(bwd);
+    cfg.stream = s;
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = bwd ? 2 : 1;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cfg;
+}
+
+int max_pairs_resident() {
+    static int n = -1;
+    if (n < 0) {
+        cudaLaunchAttribute attr[1];
+        cudaLaunchConfig_t cfg = wave_cfg(true, 2 * 64, nullptr, attr);
+        int c = 0;
+        if (cudaOccupancyMaxActiveClusters(&c, lstm_wave_kernel<true>, &cfg) != cudaSuccess) {
+            cudaGetLastError();
+            c = 0;
+        }
+        n = c;
+    }
+    return n;
+}
+
+}  // namespace
 
 bool lstm_wave_supported(int L, int B, int H, int I) {
     if (L < 1 || L > LSTM_WAVE_MAX_L || B < 1 || B > 64 || H < 128 || H % 128 || I != H) return false;
-    static int ok[2] = {0, 0};
-    for (int bwd = 0; bwd < 2; ++bwd) {
-        if (ok[bwd]) continue;
-        const void *k = bwd ? (const void *)lstm_wave_kernel<true> : (const void *)lstm_wave_kernel<false>;
+    static int ok = 0;
+    if (!ok) {
         int n = 0;
-        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, wave_smem(bwd)) != cudaSuccess ||
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k, NT, wave_smem(bwd)) != cudaSuccess || n < 1) {
+        ok = 1;
+        if (cudaFuncSetAttribute(lstm_wave_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 wave_smem(false)) != cudaSuccess ||
+            cudaFuncSetAttribute(lstm_wave_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 wave_smem(true)) != cudaSuccess ||
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lstm_wave_kernel<false>, NT, wave_smem(false)) !=
+                cudaSuccess ||
+            n < 1 || max_pairs_resident() < 1) {
             cudaGetLastError();
-            ok[bwd] = -1;
-        } else {
-            ok[bwd] = 1;
+            ok = -1;
         }
     }
-    return ok[0] > 0 && ok[1] > 0;
+    return ok > 0;
 }
 
 cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
@@ -427,11 +515,12 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     if (!w.bwd && !tma_map_bf16(&m.act[0], w.x, H, TB, H, 64, a.N)) return cudaErrorInvalidValue;
     cudaError_t e = cudaMemsetAsync(w.cnt, 0, sizeof(unsigned) * L, s);
     if (e != cudaSuccess) return e;
-    const int grid = lstm_wave_grid(L, H, w.bwd);
+    const int grid = wave_grid(L, H, w.bwd, max_pairs_resident());
+    cudaLaunchAttribute attr[1];
+    cudaLaunchConfig_t cfg = wave_cfg(w.bwd, grid, s, attr);
     ++tl_launches;
-    if (w.bwd) lstm_wave_kernel<true><<<grid, NT, wave_smem(true), s>>>(m, a);
-    else lstm_wave_kernel<false><<<grid, NT, wave_smem(false), s>>>(m, a);
-    return cudaGetLastError();
+    return w.bwd ? cudaLaunchKernelEx(&cfg, lstm_wave_kernel<true>, m, a)
+                 : cudaLaunchKernelEx(&cfg, lstm_wave_kernel<false>, m, a);
 }
 
 }  // namespace pd
