@@ -902,11 +902,35 @@ struct Exec {
         if ((env && env[0] == '0') || !bf16 || c->layer_prof) return 0;
         const pd_layer_desc &d = layer(l);
         if (d.kind != PD_LSTM || d.in != d.out || !lstm_rec_allowed()) return 0;
+        // a chain of equal LSTMs is cut into runs of at most G layers: G * 16 MB of bf16
+        // weights stream through the SMs every wave, so runs that fit the 126 MB L2 are
+        // read from L2 instead of HBM (PD_LSTM_WAVE_L overrides G)
+        const char *ge = getenv("PD_LSTM_WAVE_L");
+        const long wbytes = 8L * d.out * d.out * esz;  // W_ih + W_hh of one layer
+        int G = ge ? atoi(ge) : (int)std::max(2L, std::min((long)LSTM_WAVE_MAX_L, (64L << 20) / wbytes));
+        G = std::max(2, std::min(G, LSTM_WAVE_MAX_L));
+        int cs = l;
+        while (cs > w->first && lstm_chain(cs - 1)) --cs;
+        if ((l - cs) % G) return 0;  // not the start of a run
         int n = 1;
-        while (n < LSTM_WAVE_MAX_L && lstm_chain(l + n - 1)) ++n;
+        while (n < G && lstm_chain(l + n - 1)) ++n;
         if (n < 2 || !lstm_wave_supported(n, B(), d.out, d.in)) return 0;
-        if (l > w->first && lstm_chain(l - 1)) return 0;  // not the start of its run
         return n;
+    }
+    // the run (start, length) containing layer l, or length 0
+    int lstm_wave_run_of(int l, int &start) {
+        int cs = l;
+        while (cs > w->first && lstm_chain(cs - 1)) --cs;
+        for (int s0 = cs; s0 <= l;) {
+            const int n = lstm_wave_run(s0);
+            if (n == 0) return 0;
+            if (l < s0 + n) {
+                start = s0;
+                return n;
+            }
+            s0 += n;
+        }
+        return 0;
     }
     // layers a and a+1 are equal square LSTMs (a wavefront run continues through them)
     bool lstm_chain(int a) const {
@@ -1456,8 +1480,7 @@ struct Exec {
         for (int l = w->last; l >= w->first; --l) {
             // top layer of a wavefront run: the whole run's backward in one go
             int run_first = l;
-            while (run_first > w->first && lstm_chain(run_first - 1)) --run_first;
-            const int run = lstm_wave_run(run_first);
+            const int run = lstm_wave_run_of(l, run_first);
             const bool wave = run > 0 && run_first + run - 1 == l;
             if (wave) l = run_first;  // dX below is the run's bottom layer's
             const pd_layer_desc &d = layer(l);
