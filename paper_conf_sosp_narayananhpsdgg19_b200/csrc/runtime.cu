@@ -902,12 +902,13 @@ struct Exec {
         if ((env && env[0] == '0') || !bf16 || c->layer_prof) return 0;
         const pd_layer_desc &d = layer(l);
         if (d.kind != PD_LSTM || d.in != d.out || !lstm_rec_allowed()) return 0;
-        // a chain of equal LSTMs is cut into runs of at most G layers: G * 16 MB of bf16
-        // weights stream through the SMs every wave, so runs that fit the 126 MB L2 are
-        // read from L2 instead of HBM (PD_LSTM_WAVE_L overrides G)
+        // a chain of equal LSTMs is cut into runs of at most G layers (PD_LSTM_WAVE_L; default
+        // the kernel's maximum).  Measured on GNMT-8 / -16: the wave time is set by
+        // per-wave latency, not by the weight bytes, so fewer, longer runs win (G = 2: 3.8k /
+        // 2.0k samples/s, G = 8: 8.1k / 4.7k, G = 16: - / 5.3k) even though 4 layers' weights
+        // would stay L2-resident
         const char *ge = getenv("PD_LSTM_WAVE_L");
-        const long wbytes = 8L * d.out * d.out * esz;  // W_ih + W_hh of one layer
-        int G = ge ? atoi(ge) : (int)std::max(2L, std::min((long)LSTM_WAVE_MAX_L, (64L << 20) / wbytes));
+        int G = ge ? atoi(ge) : LSTM_WAVE_MAX_L;
         G = std::max(2, std::min(G, LSTM_WAVE_MAX_L));
         int cs = l;
         while (cs > w->first && lstm_chain(cs - 1)) --cs;
