@@ -1287,8 +1287,12 @@ cudaError_t update_major(const Gemm &g, const CUtensorMap &ma, const CUtensorMap
 // rows 16-byte aligned (N % 8 == 0 for bf16, % 4 for fp32).
 cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
     const bool adam = g.epi == EPI_ADAM;
-    constexpr int BN_SGD = 128, BN_ADAM = 64;
-    const int BN = adam ? BN_ADAM : BN_SGD;
+    // tile width: the update streams master (+ Adam m, v) per output element, the GEMM streams
+    // (128 + BN) x 64 operand elements per K-block into the SM; wider tiles raise the FLOPs per
+    // ingested byte (the per-SM TMA ingest, ~60 GB/s, bounds these tiles -- tools/tma_bw.cu)
+    static const int bn_adam = getenv("PD_UPD_BN_ADAM") ? atoi(getenv("PD_UPD_BN_ADAM")) : 128;
+    constexpr int BN_SGD = 128;
+    const int BN = adam ? bn_adam : BN_SGD;
     CUtensorMap ma, mbm, mw, mm, mv, ms;
     const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
@@ -1302,7 +1306,8 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
     else mm = mv = mw;
     if (!ok) return cudaErrorInvalidValue;
     UpdArgs u{g.lr, g.b1, g.b2, g.eps, 1.f - powf(g.b1, (float)g.step), 1.f - powf(g.b2, (float)g.step)};
-    if (adam) return update_major<BN_ADAM, true>(g, ma, mbm, mw, mm, mv, ms, u, s);
+    if (adam) return BN == 64 ? update_major<64, true>(g, ma, mbm, mw, mm, mv, ms, u, s)
+                              : update_major<128, true>(g, ma, mbm, mw, mm, mv, ms, u, s);
     return update_major<BN_SGD, false>(g, ma, mbm, mw, mm, mv, ms, u, s);
 }
 
