@@ -135,6 +135,21 @@ def model_profile(layers, B, peaks):
     return T, a, w
 
 
+def choose_plan(config, plan_mode, N, layers, B, peaks):
+    """The plan every rank computes independently (deterministic, no exchange): one stage x N
+    replicas for N = 1 or --plan dp; VGG-16 as (N-1)-1; otherwise pd_plan(max_replicas=1)."""
+    import synth
+    import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+    if N == 1 or plan_mode == "dp":
+        return pd.Plan.manual([len(layers) - 1], [N])
+    if config == "vgg16":
+        # SURVEY §8(d): VGG-16 as (N-1)-1 -- conv stage replicated, FC stage alone
+        conv_last = max(i for i, L in enumerate(layers) if L.kind == synth.MAXPOOL2)
+        return pd.Plan.manual([conv_last, len(layers) - 1], [N - 1, 1])
+    T, a, w = model_profile(layers, B, peaks)
+    return pd.pd_plan(T, a, w, N, max_replicas=1)
+
+
 def dw_update_bytes(L, B):
     """Algorithmic HBM bytes of one dW GEMM with the fused SGD update:
     read G [B][out] and X [B][in] (bf16), read+write the fp32 master, write the bf16 version."""
@@ -274,7 +289,7 @@ def main():
     import torch.distributed as dist
     import synth
     import paper_conf_sosp_narayananhpsdgg19_b200 as pd
-    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline, torch_allgather
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline, stage_of_rank, torch_allgather
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -308,15 +323,7 @@ def main():
     peaks = load_peaks()
     wl = synth.workload(args.config)
     layers, B = wl.layers, wl.batch
-    if N == 1 or args.plan == "dp":
-        plan = pd.Plan.manual([len(layers) - 1], [N])
-    elif args.config == "vgg16":
-        # VGG-16 as (N-1)-1 -- conv stage replicated, FC stage alone
-        conv_last = max(i for i, L in enumerate(layers) if L.kind == synth.MAXPOOL2)
-        plan = pd.Plan.manual([conv_last, len(layers) - 1], [N - 1, 1])
-    else:
-        T, a, w = model_profile(layers, B, peaks)
-        plan = pd.pd_plan(T, a, w, N, max_replicas=1)
+    plan = choose_plan(args.config, args.plan, N, layers, B, peaks)
     n = len(plan.stages)
     R0 = plan.stages[0][2]
     M = args.minibatches or (8 * R0 if n == 1 else 16 * n)
@@ -374,7 +381,7 @@ def main():
     P.set_timing(2, 0)
 
     # ---- roofline of the dominant kernel, this rank's stage
-    s_mine = [s for s, st in enumerate(plan.stages) if st[3] <= rank < st[3] + st[2]][0]
+    s_mine = stage_of_rank(plan, rank)
     first_l = plan.stages[s_mine][0]
     my_layers = [layers[l] for l in range(first_l, plan.stages[s_mine][1] + 1)]
     lin = [L for L in my_layers if L.kind == synth.LINEAR] or my_layers

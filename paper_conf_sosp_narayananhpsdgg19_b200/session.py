@@ -22,6 +22,14 @@ def workers_of(plan: Plan):
     return out
 
 
+def stage_of_rank(plan: Plan, rank: int) -> int:
+    """Stage whose replica runs on process `rank` (one process per GPU, R18 placement)."""
+    for s, (first, last, reps, gpu0) in enumerate(plan.stages):
+        if gpu0 <= rank < gpu0 + reps:
+            return s
+    raise ValueError(f"rank {rank} is outside the plan's {sum(st[2] for st in plan.stages)} GPUs")
+
+
 class Pipeline:
     def __init__(self, plan: Plan, layers, params: Sequence[np.ndarray], *, dtype=PD_BF16, optimizer=PD_SGD,
                  lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8, minibatch=1, record_trace=1, max_depth=0,
