@@ -83,6 +83,8 @@ struct EpiArgs {
     int relu;
     const __nv_bfloat16 *mask;
     long ldm;
+    const void *l2_next;  // L2 prefetch of the next layer's operand (warp 3), nullptr = off
+    long l2_next_bytes;
     float *master;
     __nv_bfloat16 *slot;
     float *adam_m, *adam_v;
@@ -381,6 +383,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const uint32_t tmem_base = *tmem_slot;
     if (threadIdx.x == 0) PROBE(1);
 
+    if (warp == 3 && lane == 0 && e.l2_next) {
+        // next layer's weights -> L2 while this GEMM streams its own: this CTA's contiguous
+        // share, 32 KB bulk prefetches (no smem, no completion to wait for)
+        const long share = ((e.l2_next_bytes + gridDim.x - 1) / gridDim.x + 15) & ~15L;
+        const long b0 = (long)blockIdx.x * share, b1 = min(e.l2_next_bytes, b0 + share);
+        for (long off = b0; off < b1; off += 32768) {
+            const uint32_t sz = (uint32_t)min(32768L, b1 - off) & ~15u;
+            if (sz)
+                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(
+                                 static_cast<const char *>(e.l2_next) + off),
+                             "r"(sz)
+                             : "memory");
+        }
+    }
     if (warp == 0) {
         // ===== TMA producer =====
         if (lane == 0) {
@@ -1499,6 +1515,8 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             e.ldo = g.ldo;
             e.ksplit = CS;
             e.csplit = CS;
+            e.l2_next = g.l2_next;
+            e.l2_next_bytes = g.l2_next_bytes;
             e.bias = g.epi == EPI_STORE ? g.bias : nullptr;
             e.relu = g.epi == EPI_STORE ? g.relu : 0;
             e.mask = g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr;
@@ -1519,6 +1537,8 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             e.ldo = g.N;
             e.ksplit = S;
             e.split_stride = (long)g.M * g.N;
+            e.l2_next = g.l2_next;
+            e.l2_next_bytes = g.l2_next_bytes;
             const bool inkernel = g.split_counters != nullptr && env_int("PD_SPLIT_INKERNEL", 0);
             if (inkernel) {
                 e.counters = g.split_counters;
@@ -1597,6 +1617,8 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         e.ksplit = (kb + kper - 1) / kper;
     }
     e.split_stride = 0;
+    e.l2_next = g.l2_next;
+    e.l2_next_bytes = g.l2_next_bytes;
     e.bias = g.bias;
     e.relu = g.relu;
     e.mask = static_cast<const __nv_bfloat16 *>(g.mask);

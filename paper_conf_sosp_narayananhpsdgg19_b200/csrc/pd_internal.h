@@ -107,6 +107,10 @@ struct Gemm {
     int max_ctas = 0;     // cap on resident CTAs (0 = every SM): leaves SMs to a concurrent kernel
     int *split_counters = nullptr;  // >= 8192 zeroed ints: split-K tiles reduce in-kernel (last CTA)
     int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
+    // optional: bytes [l2_next, l2_next + l2_next_bytes) are prefetched into L2 by an idle warp
+    // while this GEMM runs (the next layer's weights on the forward / dX chains)
+    const void *l2_next = nullptr;
+    long l2_next_bytes = 0;
 };
 
 // cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}

@@ -444,8 +444,17 @@ void *elem_ptr(void *base, long idx, int esz) { return static_cast<char *>(base)
 cudaError_t run_gemm(int bf16, const Gemm &g, cudaStream_t s) { return bf16 ? gemm_bf16(g, s) : gemm_f32(g, s); }
 
 // y = act(x W^T + b)
+// PD_L2_PF bit 0: forward GEMMs prefetch the next layer's weights into L2; bit 1: dX GEMMs
+int l2_pf_mask() {
+    static const int v = [] {
+        const char *e = getenv("PD_L2_PF");
+        return e ? atoi(e) : 0;
+    }();
+    return v;
+}
+
 void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, const float *bias_f32, const void *x,
-                    void *y, float *ws, long ws_bytes) {
+                    void *y, float *ws, long ws_bytes, const void *next_w = nullptr, long next_bytes = 0) {
     const int B = L.c->cfg.minibatch;
     Gemm g;
     g.M = (int)rows_of(d, B);
@@ -465,6 +474,8 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.workspace = ws;
     g.workspace_bytes = ws_bytes;
     g.split_counters = L.w->split_counters;
+    g.l2_next = next_w;
+    g.l2_next_bytes = next_bytes;
     CK(run_gemm(L.bf16, g, L.w->stream));
 }
 
@@ -627,7 +638,9 @@ struct Exec {
             cudaEvent_t k0 = kstart(0);
             if (d.kind == PD_LINEAR) {
                 LayerCtx lc{c, w, bf16};
-                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes);
+                const bool pf = bf16 && (l2_pf_mask() & 1) && l < w->last && layer(l + 1).kind == PD_LINEAR;
+                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes,
+                               pf ? Wl(l + 1, slot) : nullptr, pf ? (long)layer(l + 1).in * layer(l + 1).out * esz : 0);
             } else if (d.kind == PD_LSTM) {
                 lstm_forward(l, j, slot, x, y);
             } else if (d.kind == PD_EMBEDDING) {
@@ -687,7 +700,8 @@ struct Exec {
     };
 
     // dX = G W (B(n,k) given by the caller) fused with the previous layer's ReLU derivative
-    void gemm_dx(int l, int M, int N, int K, const void *G, long ldg, const void *W, long ldw, const void *x, void *dx) {
+    void gemm_dx(int l, int M, int N, int K, const void *G, long ldg, const void *W, long ldw, const void *x, void *dx,
+                 const void *next_w = nullptr, long next_bytes = 0) {
         const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
         Gemm g;
         g.M = M;
@@ -707,6 +721,8 @@ struct Exec {
         g.workspace = w->ws;
         g.workspace_bytes = w->ws_bytes;
         g.split_counters = w->split_counters;
+        g.l2_next = next_w;
+        g.l2_next_bytes = next_bytes;
         CK(run_gemm(bf16, g, w->stream));
     }
 
@@ -1380,7 +1396,9 @@ struct Exec {
                     if (l + 2 <= last) CK(cudaStreamWaitEvent(w->stream, w->ev_dw[l + 2 - first], 0));
                 }
                 cudaEvent_t k0 = kstart(1);
-                gemm_dx(l, (int)rows, d.in, d.out, Gl, d.out, Wl(l, bc.sslot), d.in, x, dx);
+                const bool pf = (l2_pf_mask() & 2) && l - 1 >= first && !(s == 0 && l - 1 == 0);
+                gemm_dx(l, (int)rows, d.in, d.out, Gl, d.out, Wl(l, bc.sslot), d.in, x, dx,
+                        pf ? Wl(l - 1, bc.sslot) : nullptr, pf ? (long)layer(l - 1).in * layer(l - 1).out * esz : 0);
                 kend(1, k0);
                 CK(cudaEventRecord(w->ev_dx[l - first], w->stream));
                 CK(cudaStreamWaitEvent(w->side, w->ev_dx[l - first], 0));
