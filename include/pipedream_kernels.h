@@ -52,6 +52,11 @@ typedef struct {
     float *workspace;      /* optional fp32 scratch (device) for split-K partial sums of small-M
                               STORE/MASK GEMMs (bf16); NULL disables split-K           */
     long workspace_bytes;
+    int workspace_zeroed;  /* 1: the caller guarantees `workspace` is all-zero on entry; split-K
+                              partials are then summed by TMA reduce-add (fp32, in L2) into ONE
+                              M x N set, and the workspace is all-zero again when the GEMM's
+                              last kernel completes (the summation order of the splits is not
+                              fixed).  0: partials stored per split, summed in split order */
 } pd_gemm_desc;
 
 PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *g, void *stream);

@@ -94,7 +94,8 @@ class GemmDesc(C.Structure):
                 ("bias", C.c_void_p), ("relu", C.c_int), ("mask", C.c_void_p), ("ldm", C.c_long),
                 ("master", C.c_void_p), ("slot", C.c_void_p), ("adam_m", C.c_void_p), ("adam_v", C.c_void_p),
                 ("lr", C.c_float), ("beta1", C.c_float), ("beta2", C.c_float), ("eps", C.c_float),
-                ("step", C.c_int), ("workspace", C.c_void_p), ("workspace_bytes", C.c_long)]
+                ("step", C.c_int), ("workspace", C.c_void_p), ("workspace_bytes", C.c_long),
+                ("workspace_zeroed", C.c_int)]
 
 
 def _load():
@@ -361,10 +362,11 @@ def pd_last_error(ctx) -> str:
 def pd_kernel_gemm(dtype, M, N, K, A, lda, B, ldb, out=None, ldo=0, a_mn_major=0, b_mn_major=0,
                    epilogue=PD_EPI_STORE, bias=None, relu=0, mask=None, ldm=0, master=None, slot=None,
                    adam_m=None, adam_v=None, lr=0.0, beta1=0.9, beta2=0.999, eps=1e-8, step=1, stream=None,
-                   workspace=None, workspace_bytes=0):
+                   workspace=None, workspace_bytes=0, workspace_zeroed=0):
     """All array arguments are device addresses (ints), e.g. torch ``tensor.data_ptr()``."""
     d = GemmDesc(dtype, M, N, K, A, lda, a_mn_major, B, ldb, b_mn_major, epilogue, out, ldo, bias, relu, mask, ldm,
-                 master, slot, adam_m, adam_v, lr, beta1, beta2, eps, step, workspace, workspace_bytes)
+                 master, slot, adam_m, adam_v, lr, beta1, beta2, eps, step, workspace, workspace_bytes,
+                 workspace_zeroed)
     _check(lib.pd_kernel_gemm(C.byref(d), stream))
 
 

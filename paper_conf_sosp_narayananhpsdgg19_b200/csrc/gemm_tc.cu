@@ -1329,14 +1329,16 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
 
 // out = act(sum_s ws[s] + bias) or (sum_s ws[s]) * (mask > 0), bf16; partials summed in
 // split order (deterministic).  4 columns per thread, 16-byte loads.
-__global__ void splitk_epilogue_kernel(const float *__restrict__ ws, int S, long split_stride, int M, int N,
+__global__ void splitk_epilogue_kernel(const float *ws, int S, long split_stride, int M, int N,
                                        const float *__restrict__ bias, int relu, const __nv_bfloat16 *__restrict__ mask,
-                                       long ldm, __nv_bfloat16 *__restrict__ out, long ldo) {
+                                       long ldm, __nv_bfloat16 *__restrict__ out, long ldo,
+                                       float *__restrict__ zero_ws) {
     const long n4 = N / 4;
     const long total = (long)M * n4;
     for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long)gridDim.x * blockDim.x) {
         const long m = i / n4, c = (i % n4) * 4;
         float4 a = *reinterpret_cast<const float4 *>(ws + m * N + c);
+        if (zero_ws) *reinterpret_cast<float4 *>(zero_ws + m * N + c) = make_float4(0.f, 0.f, 0.f, 0.f);
         for (int sp = 1; sp < S; ++sp) {
             const float4 b = *reinterpret_cast<const float4 *>(ws + sp * split_stride + m * N + c);
             a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
@@ -1550,6 +1552,16 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
                 e.mask = g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr;
                 e.ldm = g.ldm;
             }
+            // zeroed workspace: every split reduce-adds (TMA, in L2) into one fp32 partial set, the
+            // reduction kernel reads M*N instead of S*M*N floats and re-zeroes them.  Measured
+            // (MLP-4096 M = 256 GEMMs): 27.6 -> 29.7 us isolated, -1 % in the step -> off unless
+            // PD_SPLIT_ATOMIC=1
+            static const int split_atomic = env_int("PD_SPLIT_ATOMIC", 0);
+            const bool atomic = g.ws_zeroed && split_atomic && !inkernel;
+            if (atomic) {
+                e.atomic_out = 1;
+                e.split_stride = 0;
+            }
             Gemm gf = g;
             gf.epi = EPI_F32;
             cudaError_t err = cg == 2 ? dispatch_major<256, 2>(gf, ma, mbm, e, s) : dispatch_major<256>(gf, ma, mbm, e, s);
@@ -1558,9 +1570,9 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             long blocks = (total + 255) / 256;
             if (blocks > 148L * 8) blocks = 148L * 8;
             splitk_epilogue_kernel<<<(unsigned)blocks, 256, 0, s>>>(
-                g.workspace, S, (long)g.M * g.N, g.M, g.N, g.epi == EPI_STORE ? g.bias : nullptr,
+                g.workspace, atomic ? 1 : S, (long)g.M * g.N, g.M, g.N, g.epi == EPI_STORE ? g.bias : nullptr,
                 g.epi == EPI_STORE ? g.relu : 0, g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr,
-                g.ldm, static_cast<__nv_bfloat16 *>(g.out), g.ldo);
+                g.ldm, static_cast<__nv_bfloat16 *>(g.out), g.ldo, atomic ? g.workspace : nullptr);
             ++tl_launches;
             return cudaGetLastError();
         }
@@ -1576,7 +1588,15 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     if (cg == 2) {
         // pair tiles of 256 rows; BN >= 128 so each CTA holds >= 64 B columns
         const long pm = (g.M + 255) / 256;
-        if (pm * ((g.N + 255) / 256) < sms / 2 || g.N <= 128) BN = 128;
+        if (env_int("PD_GEMM_BNSEL", 1)) {
+            // operand bytes each CTA ingests per K-block (32 KB at BN 256, 24 KB at BN 128) x
+            // waves of pair tiles: the per-SM TMA ingest bounds these GEMMs (tools/tma_bw.cu)
+            const long slots = sms / 2, t256 = pm * ((g.N + 255) / 256), t128 = pm * ((g.N + 127) / 128);
+            const long c256 = (t256 + slots - 1) / slots * 32, c128 = (t128 + slots - 1) / slots * 24;
+            if (c128 < c256 || g.N <= 128) BN = 128;
+        } else if (pm * ((g.N + 255) / 256) < sms / 2 || g.N <= 128) {
+            BN = 128;
+        }
     } else {
         if ((long)mb * ((g.N + 255) / 256) < sms || g.N <= 128) BN = 128;
         if (BN == 128 && ((long)mb * ((g.N + 127) / 128) < sms || g.N <= 64)) BN = 64;

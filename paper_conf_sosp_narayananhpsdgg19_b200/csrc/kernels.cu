@@ -208,6 +208,85 @@ __global__ void __launch_bounds__(256) softmax_ce_kernel(const T *z, const int32
     if (threadIdx.x == 0) atomicAdd(loss, (m + __logf(s) - ld_as_f32(zr, lab)) * inv_rows);
 }
 
+// bf16 rows with C % 8 == 0 (16-byte aligned) and C <= 32 * blockDim.x: the row is read from
+// HBM ONCE into registers (up to 4 x 8 bf16 per thread, 16-byte loads), max / sum-of-exp are
+// block reductions over the registers, and dlogits is written with 16-byte stores -- one read
+// and one write of the logits (HBM-bound: 4 B per logit)
+__device__ __forceinline__ float block_reduce(float v, float *red, bool is_max) {
+    for (int o = 16; o; o >>= 1) {
+        const float u = __shfl_xor_sync(0xffffffffu, v, o);
+        v = is_max ? fmaxf(v, u) : v + u;
+    }
+    __syncthreads();  // red[] free (previous reduction consumed)
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+    __syncthreads();
+    const int nw = blockDim.x >> 5;
+    v = (int)(threadIdx.x & 31) < nw ? red[threadIdx.x & 31] : (is_max ? -INFINITY : 0.f);
+    for (int o = 16; o; o >>= 1) {
+        const float u = __shfl_xor_sync(0xffffffffu, v, o);
+        v = is_max ? fmaxf(v, u) : v + u;
+    }
+    return v;
+}
+
+__global__ void __launch_bounds__(1024) softmax_ce_bf16_row_kernel(const __nv_bfloat16 *__restrict__ z,
+                                                                   const int32_t *__restrict__ labels, long rows,
+                                                                   int C, __nv_bfloat16 *__restrict__ dz,
+                                                                   float *loss) {
+    constexpr int KMAX = 4;
+    const long r = blockIdx.x;
+    const uint4 *zr = reinterpret_cast<const uint4 *>(z + r * C);
+    uint4 *dr = reinterpret_cast<uint4 *>(dz + r * C);
+    const int n8 = C / 8;
+    __shared__ float red[32];
+    uint4 raw[KMAX];
+    float m = -INFINITY;
+#pragma unroll
+    for (int k = 0; k < KMAX; ++k) {
+        const int i = threadIdx.x + k * blockDim.x;
+        if (i < n8) {
+            raw[k] = zr[i];
+            const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw[k]);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) m = fmaxf(m, __bfloat162float(h[j]));
+        }
+    }
+    m = block_reduce(m, red, true);
+    float s = 0.f;
+#pragma unroll
+    for (int k = 0; k < KMAX; ++k) {
+        const int i = threadIdx.x + k * blockDim.x;
+        if (i < n8) {
+            const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw[k]);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) s += __expf(__bfloat162float(h[j]) - m);
+        }
+    }
+    s = block_reduce(s, red, false);
+    const int lab = labels[r];
+    const float inv_rows = 1.0f / (float)rows;
+    const float inv_s = 1.0f / s;
+#pragma unroll
+    for (int k = 0; k < KMAX; ++k) {
+        const int i = threadIdx.x + k * blockDim.x;
+        if (i < n8) {
+            const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw[k]);
+            uint4 o;
+            uint32_t *ow = reinterpret_cast<uint32_t *>(&o);
+#pragma unroll
+            for (int j = 0; j < 8; j += 2) {
+                const int c = i * 8 + j;
+                const float d0 = (__expf(__bfloat162float(h[j]) - m) * inv_s - (c == lab ? 1.f : 0.f)) * inv_rows;
+                const float d1 = (__expf(__bfloat162float(h[j + 1]) - m) * inv_s - (c + 1 == lab ? 1.f : 0.f)) * inv_rows;
+                __nv_bfloat162 p2 = __floats2bfloat162_rn(d0, d1);
+                ow[j / 2] = *reinterpret_cast<uint32_t *>(&p2);
+            }
+            dr[i] = o;
+        }
+    }
+    if (threadIdx.x == 0) atomicAdd(loss, (m + __logf(s) - __bfloat162float(z[r * C + lab])) * inv_rows);
+}
+
 // ------------------------------------------------------------------ optimizer updates
 __global__ void sgd_f32_kernel(const float *__restrict__ in, const float *__restrict__ g, float *__restrict__ out,
                                long n, float lr) {
@@ -266,6 +345,41 @@ __global__ void update_master_kernel(float *master, __nv_bfloat16 *slot_bf16, fl
         master[i] = w;
         if (slot_bf16) slot_bf16[i] = __float2bfloat16_rn(w);
         if (slot_f32) slot_f32[i] = w;
+    }
+}
+
+// one unreplicated gradient g (fp32, 16-byte aligned, n % 4 == 0): master -= SGD/Adam step,
+// slot = bf16(master); 4 elements per thread, 16-byte loads/stores (HBM-bound: SGD 18 B,
+// Adam 34 B per parameter)
+template <bool ADAM>
+__global__ void __launch_bounds__(256) update_vec4_kernel(float *__restrict__ master, __nv_bfloat16 *__restrict__ slot,
+                                                          const float *__restrict__ g, long n4, float *__restrict__ m,
+                                                          float *__restrict__ v, float lr, float b1, float b2,
+                                                          float eps, float bc1, float bc2) {
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
+        const float4 gg = reinterpret_cast<const float4 *>(g)[i];
+        float4 w = reinterpret_cast<const float4 *>(master)[i];
+        if constexpr (ADAM) {
+            float4 mm = reinterpret_cast<const float4 *>(m)[i], vv = reinterpret_cast<const float4 *>(v)[i];
+            w.x = adam_step(w.x, gg.x, mm.x, vv.x, lr, b1, b2, eps, bc1, bc2);
+            w.y = adam_step(w.y, gg.y, mm.y, vv.y, lr, b1, b2, eps, bc1, bc2);
+            w.z = adam_step(w.z, gg.z, mm.z, vv.z, lr, b1, b2, eps, bc1, bc2);
+            w.w = adam_step(w.w, gg.w, mm.w, vv.w, lr, b1, b2, eps, bc1, bc2);
+            reinterpret_cast<float4 *>(m)[i] = mm;
+            reinterpret_cast<float4 *>(v)[i] = vv;
+        } else {
+            w.x -= lr * gg.x;
+            w.y -= lr * gg.y;
+            w.z -= lr * gg.z;
+            w.w -= lr * gg.w;
+        }
+        reinterpret_cast<float4 *>(master)[i] = w;
+        __nv_bfloat162 lo = __floats2bfloat162_rn(w.x, w.y), hi = __floats2bfloat162_rn(w.z, w.w);
+        uint2 o;
+        o.x = *reinterpret_cast<uint32_t *>(&lo);
+        o.y = *reinterpret_cast<uint32_t *>(&hi);
+        reinterpret_cast<uint2 *>(slot)[i] = o;
     }
 }
 
@@ -339,7 +453,14 @@ cudaError_t bias_grad(const void *G, int bf16, long rows, long cols, float *grad
 
 cudaError_t softmax_ce(const void *logits, int bf16, const int32_t *labels, long rows, int C, void *dlogits,
                        float *loss_out, cudaStream_t s) {
-    if (bf16)
+    if (bf16 && C % 8 == 0 && C <= 32 * 1024 && ((uintptr_t)logits & 15) == 0 && ((uintptr_t)dlogits & 15) == 0) {
+        const int n8 = C / 8;
+        int threads = ((n8 + 3) / 4 + 31) / 32 * 32;  // <= 4 chunks of 8 per thread
+        if (threads < 64) threads = 64;
+        softmax_ce_bf16_row_kernel<<<(unsigned)rows, threads, 0, s>>>(static_cast<const __nv_bfloat16 *>(logits),
+                                                                      labels, rows, C,
+                                                                      static_cast<__nv_bfloat16 *>(dlogits), loss_out);
+    } else if (bf16)
         softmax_ce_kernel<<<(unsigned)rows, 256, 0, s>>>(static_cast<const __nv_bfloat16 *>(logits), labels, rows, C,
                                                          static_cast<__nv_bfloat16 *>(dlogits), loss_out);
     else
@@ -369,6 +490,21 @@ cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f
     const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
     update_master_kernel<<<grid_for(n), 256, 0, s>>>(master, slot_bf16, slot_f32, grads, R, goff, n, opt, m, v, lr,
                                                      b1, b2, eps, bc1, bc2);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
+cudaError_t update_from_grad(float *master, __nv_bfloat16 *slot, const float *g, long n, int opt, float *m, float *v,
+                             float lr, float b1, float b2, float eps, int step, cudaStream_t s) {
+    if ((n & 3) || ((uintptr_t)master & 15) || ((uintptr_t)g & 15) || ((uintptr_t)slot & 7) ||
+        (opt == PD_ADAM && (((uintptr_t)m & 15) || ((uintptr_t)v & 15))))
+        return cudaErrorInvalidValue;
+    const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
+    const long n4 = n / 4;
+    if (opt == PD_ADAM)
+        update_vec4_kernel<true><<<grid_for(n4), 256, 0, s>>>(master, slot, g, n4, m, v, lr, b1, b2, eps, bc1, bc2);
+    else
+        update_vec4_kernel<false><<<grid_for(n4), 256, 0, s>>>(master, slot, g, n4, m, v, lr, b1, b2, eps, bc1, bc2);
     ++tl_launches;
     return cudaGetLastError();
 }

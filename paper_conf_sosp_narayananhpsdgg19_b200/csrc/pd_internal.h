@@ -102,6 +102,9 @@ struct Gemm {
     // optional fp32 scratch for split-K partials (bf16 EPI_STORE / EPI_MASK); nullptr = off
     float *workspace = nullptr;
     long workspace_bytes = 0;
+    // the caller keeps `workspace` all-zero between GEMMs: split-K partials are then summed by
+    // TMA reduce-add into ONE fp32 tile set (and the reduction kernel re-zeroes what it read)
+    int ws_zeroed = 0;
     ConvGeom conv;        // implicit-GEMM convolution (bf16 path only)
     int ksplit = 1;       // explicit split-K (EPI_F32 with atomic_out)
     int max_ctas = 0;     // cap on resident CTAs (0 = every SM): leaves SMs to a concurrent kernel
@@ -141,6 +144,10 @@ cudaError_t adam_f32(const float *in, const float *g, float *out, float *m, floa
 cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f32, const float *const *grads,
                           int R, long goff, long n, int opt, float *m, float *v, float lr, float b1, float b2,
                           float eps, int step, cudaStream_t s);
+// bf16 path, one unreplicated fp32 gradient: master -= SGD/Adam step of g, slot = bf16(master);
+// vectorised (n % 4 == 0, 16-byte aligned arrays; else cudaErrorInvalidValue)
+cudaError_t update_from_grad(float *master, __nv_bfloat16 *slot, const float *g, long n, int opt, float *m, float *v,
+                             float lr, float b1, float b2, float eps, int step, cudaStream_t s);
 // dst[off[r] + i] = float(src[off[r] + i]) for i < cnt[r], r < n (off, cnt device arrays)
 cudaError_t regions_bf16_to_f32(const __nv_bfloat16 *src, float *dst, const long *off, const int *cnt, int n,
                                 cudaStream_t s);

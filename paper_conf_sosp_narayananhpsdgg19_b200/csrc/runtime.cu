@@ -473,6 +473,7 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.relu = d.act == PD_ACT_RELU;
     g.workspace = ws;
     g.workspace_bytes = ws_bytes;
+    g.ws_zeroed = 1;  // w->ws is zero-filled at allocation and re-zeroed by every split-K use
     g.split_counters = L.w->split_counters;
     g.l2_next = next_w;
     g.l2_next_bytes = next_bytes;
@@ -720,10 +721,21 @@ struct Exec {
         g.ldm = N;
         g.workspace = w->ws;
         g.workspace_bytes = w->ws_bytes;
+        g.ws_zeroed = 1;
         g.split_counters = w->split_counters;
         g.l2_next = next_w;
         g.l2_next_bytes = next_bytes;
         CK(run_gemm(bf16, g, w->stream));
+    }
+
+    // PD_DW_SPLIT_K: fused-path weight gradients with K >= this many rows (and M, N >= 256) run
+    // as GEMM -> fp32 gradient -> update kernel instead of the fused-epilogue GEMM (0 = never).
+    // Default 1024: GNMT-8 at N = 1 8.68k -> 9.74k samples/s (the LSTM W_ih / W_hh and
+    // classifier gradients, K = T*B = 3200); the MLP's K = 256 dW stays fused
+    bool split_dw(int M, int N, int K) const {
+        const char *e = getenv("PD_DW_SPLIT_K");  // read per call (tests toggle it)
+        const int kmin = e ? atoi(e) : 1024;
+        return bf16 && kmin > 0 && K >= kmin && M >= 256 && N >= 256 && (long)M * N % 4 == 0;
     }
 
     // dW (M x N, row-major at parameter offset woff) = A^T B over K rows, either fused with
@@ -740,6 +752,20 @@ struct Exec {
         g.ldb = ldb;
         g.bmaj = MNMAJ;
         g.ldo = N;
+        if (bc.fused && split_dw(M, N, K)) {
+            // long-K weight gradients (LSTM W_ih / W_hh over T*B rows, classifier): the plain
+            // 2-CTA GEMM into an fp32 gradient, then one vectorised update pass.  The fused
+            // epilogue's single-CTA 128-wide tiles ingest 2x the operand bytes per FLOP
+            const bool adam = c->cfg.optimizer == PD_ADAM;
+            g.epi = EPI_F32;
+            g.out = w->gbuf + woff;
+            CK(run_gemm(bf16, g, w->stream));
+            CK(update_from_grad(w->master + woff, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], woff, esz)),
+                                w->gbuf + woff, (long)M * N, c->cfg.optimizer, adam ? w->adam_m + woff : nullptr,
+                                adam ? w->adam_v + woff : nullptr, c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps,
+                                w->updates_total + 1, w->stream));
+            return;
+        }
         if (bc.fused) {
             const bool adam = c->cfg.optimizer == PD_ADAM;
             g.epi = adam ? EPI_ADAM : EPI_SGD;
@@ -1347,11 +1373,20 @@ struct Exec {
         cudaEvent_t k0 = kstart(2);
         CK(cudaMemsetAsync(gE, 0, (size_t)n * 4, w->stream));
         CK(embedding_bwd(bf16, static_cast<const int32_t *>(tok), G, gE, rows_of(d, B()), d.out, w->stream));
-        if (bc.fused)
-            CK(update_master(w->master + off, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], off, esz)),
-                             nullptr, w->self_grad_ptr, 1, off, n, c->cfg.optimizer,
-                             w->adam_m ? w->adam_m + off : nullptr, w->adam_v ? w->adam_v + off : nullptr, c->cfg.lr,
-                             c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+        if (bc.fused) {
+            // vectorised update (16-byte accesses); the generic replica kernel if unaligned
+            const cudaError_t e = update_from_grad(
+                w->master + off, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], off, esz)), gE, n,
+                c->cfg.optimizer, w->adam_m ? w->adam_m + off : nullptr, w->adam_v ? w->adam_v + off : nullptr,
+                c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream);
+            if (e == cudaErrorInvalidValue)
+                CK(update_master(w->master + off, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], off, esz)),
+                                 nullptr, w->self_grad_ptr, 1, off, n, c->cfg.optimizer,
+                                 w->adam_m ? w->adam_m + off : nullptr, w->adam_v ? w->adam_v + off : nullptr,
+                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+            else
+                CK(e);
+        }
         kend(2, k0);
     }
 
@@ -2455,6 +2490,7 @@ extern "C" PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *d, void *stream) 
     g.master = d->master; g.slot = d->slot; g.adam_m = d->adam_m; g.adam_v = d->adam_v;
     g.lr = d->lr; g.b1 = d->beta1; g.b2 = d->beta2; g.eps = d->eps; g.step = d->step;
     g.workspace = d->workspace; g.workspace_bytes = d->workspace_bytes;
+    g.ws_zeroed = d->workspace_zeroed;
     static int *counters = nullptr;  // kernel-level API: one zeroed counter array per process
     if (d->dtype == PD_BF16 && d->workspace && !counters) {
         if (cudaMalloc(&counters, 8192 * sizeof(int)) != cudaSuccess || cudaMemset(counters, 0, 8192 * sizeof(int)) != cudaSuccess ||

@@ -48,35 +48,46 @@ def test_tc_gemm_f32_out(M, N, K, amn, bmn):
     assert _rel(out, ref) < 1e-5
 
 
-@pytest.mark.parametrize("split", [False, True])
+def _ws(split, M, N):
+    """split: 0 = none, 1 = per-split partials, 2 = zeroed workspace (TMA reduce-add partials)"""
+    if not split:
+        return None, {}
+    ws = torch.zeros(8 * M * N, device="cuda") if split == 2 else torch.empty(8 * M * N, device="cuda")
+    return ws, dict(workspace=ws.data_ptr(), workspace_bytes=ws.numel() * 4, workspace_zeroed=int(split == 2))
+
+
+@pytest.mark.parametrize("split", [0, 1, 2])
 @pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES[:4] + [
     (32, 4096, 4096, 0, 0),    # small-M split-K: 8 splits of a 128-row tile holding 32 rows
     (40, 4096, 2048, 0, 1),    # ragged rows inside an epilogue warp's 32-row slab
+    (256, 4096, 4096, 0, 0),   # the MLP-4096 forward shape (2-CTA, 4 splits)
 ])
 def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split):
     A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16, seed=1)
     bias = torch.randn(N, device="cuda")
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
-    ws = torch.empty(8 * M * N, device="cuda") if split else None
+    ws, kw = _ws(split, M, N)
     pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], out.data_ptr(),
-                      N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1,
-                      workspace=ws.data_ptr() if split else None, workspace_bytes=ws.numel() * 4 if split else 0)
+                      N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1, **kw)
     torch.cuda.synchronize()
     ref = torch.relu(A.float() @ B.float().t() + bias)
     assert _rel(out, ref) < 1e-2
+    if split == 2:  # the contract: the workspace is all-zero again afterwards
+        assert int(torch.count_nonzero(ws)) == 0
 
 
-@pytest.mark.parametrize("split", [False, True])
-@pytest.mark.parametrize("M,N,K", [(256, 1024, 4096), (40, 4096, 4096)])
+@pytest.mark.parametrize("split", [0, 1, 2])
+@pytest.mark.parametrize("M,N,K", [(256, 1024, 4096), (40, 4096, 4096), (256, 4096, 4096)])
 def test_tc_gemm_mask_epilogue(split, M, N, K):
     A, B, As, Bs = _operands(M, N, K, 0, 1, torch.bfloat16, seed=2)
     mask = torch.relu(torch.randn(M, N, device="cuda")).to(torch.bfloat16)
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
-    ws = torch.empty(8 * M * N, device="cuda") if split else None
+    ws, kw = _ws(split, M, N)
     pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), K, Bs.data_ptr(), N, out.data_ptr(), N, 0, 1,
-                      pd.PD_EPI_MASK, mask=mask.data_ptr(), ldm=N,
-                      workspace=ws.data_ptr() if split else None, workspace_bytes=ws.numel() * 4 if split else 0)
+                      pd.PD_EPI_MASK, mask=mask.data_ptr(), ldm=N, **kw)
     torch.cuda.synchronize()
+    if split == 2:
+        assert int(torch.count_nonzero(ws)) == 0
     ref = (A.float() @ B.float().t()) * (mask.float() > 0)
     assert _rel(out, ref) < 1e-2
     assert bool(((out.float() == 0) | (mask.float() > 0)).all())
@@ -122,11 +133,16 @@ def test_simt_fp32_gemm(M, N, K, amn, bmn):
     assert _rel(out, ref) < 1e-5
 
 
-@pytest.mark.parametrize("dtype", [pd.PD_FP32, pd.PD_BF16])
-def test_softmax_ce_kernel_vs_oracle(dtype):
+@pytest.mark.parametrize("dtype,Cn", [(pd.PD_FP32, 1000), (pd.PD_BF16, 1000),
+                                      # bf16 register-resident row kernel (C % 8 == 0, C <= 32768)
+                                      # incl. GNMT's vocabulary, the 4-chunk limit, a 1-chunk row;
+                                      # C % 8 != 0 and C > 32768 take the 3-pass kernel
+                                      (pd.PD_BF16, 32000), (pd.PD_BF16, 32768), (pd.PD_BF16, 8),
+                                      (pd.PD_BF16, 4096), (pd.PD_BF16, 10), (pd.PD_BF16, 40000)])
+def test_softmax_ce_kernel_vs_oracle(dtype, Cn):
     import oracle
     rng = np.random.default_rng(5)
-    R, Cn = 48, 1000
+    R = 48
     z = (rng.standard_normal((R, Cn)) * 3).astype(np.float32)
     lab = rng.integers(0, Cn, R).astype(np.int32)
     tdt = torch.bfloat16 if dtype == pd.PD_BF16 else torch.float32

@@ -104,3 +104,39 @@ def test_wavefront_inside_a_pipeline_stage():
     assert_schedule_exact(res)
     perr, derr = param_errors(res)
     assert perr < BF16_TOL and derr < 5e-2, (perr, derr)
+
+
+def _run_env(wl, last, M, env):
+    old = {k: os.environ.get(k) for k in env}
+    os.environ.update(env)
+    try:
+        return run_both(wl, last, [1] * len(last), M, pd.PD_BF16, n_data=3)
+    finally:
+        for k, v in old.items():
+            if v is None:
+                del os.environ[k]
+            else:
+                os.environ[k] = v
+
+
+@pytest.mark.parametrize("opt", [synth.SGD, synth.ADAM])
+def test_split_weight_gradient_path_matches_oracle(opt):
+    # PD_DW_SPLIT_K: the long-K weight gradients (LSTM W_ih/W_hh over T*B rows, classifier) as
+    # 2-CTA GEMM -> fp32 gradient -> vectorised update, instead of the fused-epilogue GEMM;
+    # (4, 256, 16, 6): M = 4H = 1024, N = 256, K = 96 / 80; classifier M = 512, N = 256, K = 96
+    wl = synth.Workload("lstm4x256", synth.gnmt(4, 256, 512, 6, 16), 16, opt, 0.05 if opt == synth.SGD else 3e-4)
+    last = [len(wl.layers) - 1]
+    a = _run_env(wl, last, 3, {"PD_DW_SPLIT_K": "64"})
+    assert_schedule_exact(a)
+    perr, derr = param_errors(a)
+    assert perr < BF16_TOL, perr
+    if opt == synth.SGD:
+        assert derr < 5e-2, derr
+    b = _run_env(wl, last, 3, {"PD_DW_SPLIT_K": "0"})
+    # same bf16 operands; only the GEMM tiling (fp32 summation order) and the update kernel differ
+    if opt == synth.SGD:
+        d = torchref.delta_err(a["got"], b["got"], a["p0"])
+        assert d < 2e-2, d
+    else:  # Adam moves every weight by ~lr*sign(g): compare parameters, not deltas
+        assert torchref.max_rel_err(a["got"], b["got"]) < 2e-2
+    np.testing.assert_allclose(a["losses"], b["losses"], rtol=2e-3)

@@ -14,14 +14,15 @@ def bench(M, N, K, amn, bmn, epi, split_ws, iters=20):
     master = torch.randn(M, N, device="cuda")
     slot = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
     bias = torch.zeros(N, device="cuda")
-    ws = torch.empty(8 * M * N, device="cuda")
+    ws = torch.zeros(8 * M * N, device="cuda")  # stays zero under ZEROWS=1 (workspace_zeroed contract)
     s = torch.cuda.current_stream()
     if epi == pd.PD_EPI_STORE:
         kw = dict(bias=bias.data_ptr(), relu=1)
     else:
         kw = dict(master=master.data_ptr(), slot=slot.data_ptr(), lr=1e-3)
     if split_ws:
-        kw.update(workspace=ws.data_ptr(), workspace_bytes=ws.numel() * 4)
+        kw.update(workspace=ws.data_ptr(), workspace_bytes=ws.numel() * 4,
+                  workspace_zeroed=int(bool(os.environ.get("ZEROWS"))))
     f = lambda: pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, A.data_ptr(), A.shape[1], B.data_ptr(), B.shape[1],
                                   out.data_ptr(), N, amn, bmn, epi, stream=s.cuda_stream, **kw)
     for _ in range(3):
