@@ -815,7 +815,7 @@ struct UpdCfg {
     static constexpr int A_BYTES = BM * BK * 2;
     static constexpr int B_BYTES = BN * BK * 2;
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-    static constexpr int STAGES = 3;
+    static constexpr int STAGES = BN == 256 ? 2 : 3;  // (BN 256: 2 x 48 KB operand stages fit beside the epilogue ring)
     // epilogue sub-tiles: ECOLS columns of the [128][BN] tile, double-buffered so the TMA
     // load of sub-tile k+1 and the TMA store of sub-tile k-1 overlap the update of k
     static constexpr int ECOLS = ADAM ? 32 : 64;
@@ -1307,8 +1307,9 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
     // (128 + BN) x 64 operand elements per K-block into the SM; wider tiles raise the FLOPs per
     // ingested byte (the per-SM TMA ingest, ~60 GB/s, bounds these tiles -- tools/tma_bw.cu)
     static const int bn_adam = getenv("PD_UPD_BN_ADAM") ? atoi(getenv("PD_UPD_BN_ADAM")) : 128;
-    constexpr int BN_SGD = 128;
-    const int BN = adam ? bn_adam : BN_SGD;
+    const char *bs = getenv("PD_UPD_BN_SGD");  // read per call (tests toggle it)
+    const int bn_sgd = bs && atoi(bs) == 256 ? 256 : 128;
+    const int BN = adam ? bn_adam : bn_sgd;
     CUtensorMap ma, mbm, mw, mm, mv, ms;
     const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
                                     : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
@@ -1324,7 +1325,8 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
     UpdArgs u{g.lr, g.b1, g.b2, g.eps, 1.f - powf(g.b1, (float)g.step), 1.f - powf(g.b2, (float)g.step)};
     if (adam) return BN == 64 ? update_major<64, true>(g, ma, mbm, mw, mm, mv, ms, u, s)
                               : update_major<128, true>(g, ma, mbm, mw, mm, mv, ms, u, s);
-    return update_major<BN_SGD, false>(g, ma, mbm, mw, mm, mv, ms, u, s);
+    return BN == 256 ? update_major<256, false>(g, ma, mbm, mw, mm, mv, ms, u, s)
+                     : update_major<128, false>(g, ma, mbm, mw, mm, mv, ms, u, s);
 }
 
 // out = act(sum_s ws[s] + bias) or (sum_s ws[s]) * (mask > 0), bf16; partials summed in
@@ -1553,11 +1555,8 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
                 e.ldm = g.ldm;
             }
             // zeroed workspace: every split reduce-adds (TMA, in L2) into one fp32 partial set, the
-            // reduction kernel reads M*N instead of S*M*N floats and re-zeroes them.  Measured
-            // (MLP-4096 M = 256 GEMMs): 27.6 -> 29.7 us isolated, -1 % in the step -> off unless
-            // PD_SPLIT_ATOMIC=1
-            static const int split_atomic = env_int("PD_SPLIT_ATOMIC", 0);
-            const bool atomic = g.ws_zeroed && split_atomic && !inkernel;
+            // reduction kernel reads M*N instead of S*M*N floats and re-zeroes them
+            const bool atomic = g.ws_zeroed && !inkernel;
             if (atomic) {
                 e.atomic_out = 1;
                 e.split_stride = 0;
