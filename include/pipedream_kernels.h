@@ -66,6 +66,16 @@ PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *g, void *stream);
 PD_API pd_status pd_kernel_softmax_ce(int dtype, const void *logits, const int32_t *labels, long rows, int C,
                                       void *dlogits, float *loss, void *stream);
 
+/* Bias gradient db[c] = sum_r G[r][c] over `rows` rows of a row-major [rows][cols] output
+ * gradient G (dtype of the path) -- the db = sum dY of the backward pass (PAPER.md L1145-1161,
+ * SURVEY §8(a) a7) -- either written to grad_out (device fp32 [cols]) or, when `master` is
+ * given (bf16 path), applied as the optimizer step of a10 to the latest weights: master -= SGD
+ * or Adam step (m, v fp32, bias-corrected with `step`), slot_bf16 = bf16(master).  Sums are in
+ * a fixed order (deterministic).  Device pointers; PD_EINVAL on bad sizes/pointers. */
+PD_API pd_status pd_kernel_bias_grad(int dtype, const void *G, long rows, long cols, float *grad_out, float *master,
+                                     void *slot_bf16, int optimizer, float *m, float *v, float lr, float beta1,
+                                     float beta2, float eps, int step, void *stream);
+
 /* The recurrent half of one LSTM layer (bf16 path, R22: PyTorch form, gates i, f, g,
  * o; h0 = c0 = 0), all T steps in ONE persistent launch (csrc/lstm_rec.cu): W_hh stays in
  * shared memory, step t waits only for the K-blocks of h[t-1] (da[t+1]) it multiplies.

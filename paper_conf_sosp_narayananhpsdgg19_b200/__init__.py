@@ -121,6 +121,8 @@ def _load():
         "pd_kernel_gemm": [vp, vp],
         "pd_kernel_softmax_ce": [i, vp, vp, C.c_long, i, vp, vp, vp],
         "pd_kernel_lstm_rec": [vp, vp],
+        "pd_kernel_bias_grad": [i, vp, C.c_long, C.c_long, vp, vp, vp, i, vp, vp, C.c_float, C.c_float, C.c_float,
+                                C.c_float, i, vp],
         "pd_profile": [vp, i, vp, i, i, vp],
         "pd_set_layer_profiling": [vp, i],
         "pd_get_layer_times": [vp, vp, vp, st],
@@ -144,7 +146,7 @@ EXPORTED = ["pd_plan", "pd_create", "pd_stage_init", "pd_export_worker", "pd_imp
             "pd_get_params", "pd_get_trace", "pd_get_version_map", "pd_get_losses", "pd_get_stats", "pd_destroy",
             "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce",
             "pd_kernel_lstm_rec", "pd_profile", "pd_set_layer_profiling", "pd_get_layer_times",
-            "pd_set_timing"]
+            "pd_set_timing", "pd_kernel_bias_grad"]
 
 
 def _strerror(s):
@@ -368,6 +370,13 @@ def pd_kernel_gemm(dtype, M, N, K, A, lda, B, ldb, out=None, ldo=0, a_mn_major=0
                  master, slot, adam_m, adam_v, lr, beta1, beta2, eps, step, workspace, workspace_bytes,
                  workspace_zeroed)
     _check(lib.pd_kernel_gemm(C.byref(d), stream))
+
+
+def pd_kernel_bias_grad(dtype, G, rows, cols, grad_out=None, master=None, slot=None, optimizer=PD_SGD, m=None,
+                        v=None, lr=0.0, beta1=0.9, beta2=0.999, eps=1e-8, step=1, stream=None):
+    """db = column sums of G (device addresses as ints), written or applied as the update."""
+    _check(lib.pd_kernel_bias_grad(dtype, G, rows, cols, grad_out, master, slot, optimizer, m, v, lr, beta1, beta2,
+                                   eps, step, stream))
 
 
 def pd_kernel_softmax_ce(dtype, logits, labels, rows, Cn, dlogits, loss, stream=None):

@@ -162,6 +162,84 @@ __global__ void __launch_bounds__(1024) bias_grad_kernel(const T *__restrict__ G
     }
 }
 
+// Tall G (rows >= 1024, e.g. LSTM da over T*B rows): the rows are split over a cluster of CS
+// CTAs (grid.y), so 4x more SMs stream G; each CTA reduces its rows as above, then rank 0
+// adds the CS partial sums through distributed shared memory in rank order (deterministic)
+// and applies the update.
+template <typename T, int CS>
+__global__ void __launch_bounds__(1024) bias_grad_cluster_kernel(const T *__restrict__ G, long rows, long cols,
+                                                                 float *grad_out, float *master,
+                                                                 __nv_bfloat16 *slot, int opt, float *m, float *v,
+                                                                 float lr, float b1, float b2, float eps, float bc1,
+                                                                 float bc2) {
+    __shared__ float part[32][65];
+    __shared__ float psum[64];
+    const int lane = threadIdx.x & 31, rg = threadIdx.x >> 5;
+    uint32_t crank;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+    const long r_lo = rows * (long)crank / CS, r_hi = rows * (long)(crank + 1) / CS;
+    const long c = (long)blockIdx.x * 64 + 2 * lane;
+    float a0 = 0.f, a1 = 0.f;
+    if (c + 1 < cols) {
+        long r = r_lo + rg;
+        for (; r + 7 * 32 < r_hi; r += 8 * 32) {
+            float2 x[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) x[u] = ld2_as_f32(G, (r + u * 32) * cols + c);
+#pragma unroll
+            for (int u = 0; u < 8; ++u) { a0 += x[u].x; a1 += x[u].y; }
+        }
+        for (; r < r_hi; r += 32) {
+            const float2 x = ld2_as_f32(G, r * cols + c);
+            a0 += x.x;
+            a1 += x.y;
+        }
+    } else if (c < cols) {
+        for (long r = r_lo + rg; r < r_hi; r += 32) a0 += ld_as_f32(G, r * cols + c);
+    }
+    part[rg][2 * lane] = a0;
+    part[rg][2 * lane + 1] = a1;
+    __syncthreads();
+    if (threadIdx.x < 64) {
+        float g = part[0][threadIdx.x];
+        for (int q = 1; q < 32; ++q) g += part[q][threadIdx.x];
+        psum[threadIdx.x] = g;
+    }
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (crank == 0 && threadIdx.x < 64) {
+        const long cc = (long)blockIdx.x * 64 + threadIdx.x;
+        if (cc < cols) {
+            const uint32_t local = (uint32_t)__cvta_generic_to_shared(&psum[threadIdx.x]);
+            float g = 0.f;
+#pragma unroll
+            for (int q = 0; q < CS; ++q) {
+                uint32_t ra;
+                float x;
+                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local), "r"((uint32_t)q));
+                asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(x) : "r"(ra) : "memory");
+                g += x;
+            }
+            if (grad_out) grad_out[cc] = g;
+            if (master) {
+                float w = master[cc];
+                if (opt == PD_SGD) {
+                    w = w - lr * g;
+                } else {
+                    const float mm = b1 * m[cc] + (1.f - b1) * g;
+                    const float vv = b2 * v[cc] + (1.f - b2) * g * g;
+                    m[cc] = mm;
+                    v[cc] = vv;
+                    w = w - lr * (mm / bc1) / (sqrtf(vv / bc2) + eps);
+                }
+                master[cc] = w;
+                if (slot) slot[cc] = __float2bfloat16_rn(w);
+            }
+        }
+    }
+    // no CTA may exit while rank 0 still reads its partial sums
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 // ------------------------------------------------------------------ softmax cross-entropy
 // One block per row: max, sum of exp, loss += (lse - z[label]) / rows, and
 // dlogits = (softmax - onehot) / rows written in the logits' dtype (L1217, R8).
@@ -441,6 +519,27 @@ cudaError_t bias_grad(const void *G, int bf16, long rows, long cols, float *grad
                       int step, cudaStream_t s) {
     const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
     const unsigned blocks = (unsigned)((cols + 63) / 64);
+    if (rows >= 1024) {
+        constexpr int CS = 4;
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(blocks, CS);
+        cfg.blockDim = dim3(1024);
+        cfg.stream = s;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = 1;
+        attr[0].val.clusterDim.y = CS;
+        attr[0].val.clusterDim.z = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        ++tl_launches;
+        if (bf16)
+            return cudaLaunchKernelEx(&cfg, bias_grad_cluster_kernel<__nv_bfloat16, CS>,
+                                      static_cast<const __nv_bfloat16 *>(G), rows, cols, grad_out, master, slot, opt,
+                                      m, v, lr, b1, b2, eps, bc1, bc2);
+        return cudaLaunchKernelEx(&cfg, bias_grad_cluster_kernel<float, CS>, static_cast<const float *>(G), rows, cols,
+                                  grad_out, master, slot, opt, m, v, lr, b1, b2, eps, bc1, bc2);
+    }
     if (bf16)
         bias_grad_kernel<<<blocks, 1024, 0, s>>>(static_cast<const __nv_bfloat16 *>(G), rows, cols, grad_out, master,
                                                  slot, opt, m, v, lr, b1, b2, eps, bc1, bc2);

@@ -29,6 +29,7 @@
 
 #include <cstdio>
 #include <cstring>
+#include <vector>
 
 #include "pd_internal.h"
 #include "tc_ptx.h"
@@ -87,7 +88,19 @@ struct WaveArgs {
     WaveLayer layer[LSTM_WAVE_MAX_L];
     const __nv_bfloat16 *dy_top;  // backward: gradient w.r.t. the top layer's output [T][B][H]
     unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
+    unsigned long long *probe;    // tools only (PD_WAVE_PROBE): [CTA][visit < PROBE_V][8] %globaltimer
 };
+constexpr int PROBE_V = 256;
+// probe events per item visit: 0 weight producer first K-block issued, 1 activation producer
+// dependencies satisfied, 2 MMA last K-block issued, 3 epilogue accumulator ready, 4 epilogue
+// partials exchanged / staged, 5 epilogue item published
+__device__ __forceinline__ void probe(const WaveArgs &a, int v, int ev) {
+    if (a.probe && v < PROBE_V) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        a.probe[((long)blockIdx.x * PROBE_V + v) * 8 + ev] = t;
+    }
+}
 
 // the item sequence of this CTA (pair): items i = c + k * C (c = cluster index, C = clusters,
 // i = l * tiles + tile), visited wave by wave; returns false when done
@@ -186,12 +199,13 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
     if (warp == 0 && lane == 0) {
         // ---------------- weight producer
         ItemIter<CL> it;
-        int l, tile, t, s = 0;
+        int l, tile, t, s = 0, pv = 0;
         uint32_t ph = 0;
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             for (int kb = ik.lo; kb < ik.hi; ++kb) {
                 mbar_wait(em0 + 8 * s, ph ^ 1);
+                if (kb == ik.lo) probe(a, pv, 0);
                 const uint32_t dst = smem_u32(sm + s * STAGE);
                 mbar_expect_tx(fw0 + 8 * s, ATILE);
                 const bool p1 = kb >= ik.n0;
@@ -205,14 +219,16 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 }
                 if (++s == S) s = 0, ph ^= 1;
             }
+            ++pv;
         }
     } else if (warp == 1 && lane == 0) {
         // ---------------- activation producer (waits for the item's inputs)
         ItemIter<CL> it;
-        int l, tile, t, s = 0;
+        int l, tile, t, s = 0, pv = -1;
         uint32_t ph = 0;
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
+            ++pv;
             if (ik.lo == ik.hi) continue;
             const bool need0 = ik.lo < ik.n0, need1 = ik.hi > ik.n0;
             if (!BWD) {
@@ -223,6 +239,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 if (need1) wait_count(a.cnt + l + 1, (unsigned)(a.T - t) * per_step);  // da^{l+1}[t]
             }
             fence_proxy_async_global();
+            probe(a, pv, 1);
             for (int kb = ik.lo; kb < ik.hi; ++kb) {
                 mbar_wait(em0 + 8 * s, ph ^ 1);
                 const uint32_t dst = smem_u32(sm + s * STAGE + ATILE);
@@ -243,7 +260,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         // ---------------- MMA issuer
         const uint32_t idesc = make_idesc(128, N, BWD ? 1 : 0, 0);
         ItemIter<CL> it;
-        int l, tile, t, s = 0, acc = 0;
+        int l, tile, t, s = 0, acc = 0, pv = 0;
         uint32_t ph = 0, aph[2] = {0, 0};
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
@@ -264,6 +281,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 tc_commit(em0 + 8 * s);
                 if (++s == S) s = 0, ph ^= 1;
             }
+            probe(a, pv++, 2);
             if (ik.hi > ik.lo) tc_commit(af0 + 8 * acc);
             else mbar_arrive(af0 + 8 * acc);  // nothing to multiply: the epilogue uses 0
             aph[acc] ^= 1;
@@ -274,7 +292,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         const int q = warp - 4;  // TMEM lane quadrant
         const int et = tid - 128;
         ItemIter<CL> it;
-        int l, tile, t, acc = 0;
+        int l, tile, t, acc = 0, pv = 0;
         uint32_t aph[2] = {0, 0}, rph = 0, eph = 0;
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
@@ -282,6 +300,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
             mbar_wait(af0 + 8 * acc, aph[acc]);
             aph[acc] ^= 1;
             tc_fence_after();
+            if (et == 0) probe(a, pv, 3);
             const uint32_t d = tmem + acc * 64 + ((uint32_t)(q * 32) << 16);
             const WaveLayer &Ly = a.layer[l];
             if (!BWD) {
@@ -296,29 +315,37 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                         *reinterpret_cast<float4 *>(stg + row * STG_LD + ch * 32 + i * 4) =
                             make_float4(v[i * 4], v[i * 4 + 1], v[i * 4 + 2], v[i * 4 + 3]);
                 }
+                // gate row `row` = g*32 + u: b_ih + b_hh into the staging row's spare column 64
+                // (STG_LD = 68), so the cell loop below reads biases from shared memory
+                {
+                    const int gi = row >> 5, uu = row & 31, jb = gi * H + tile * 32 + uu;
+                    stg[row * STG_LD + 64] = __ldg(Ly.b_ih + jb) + __ldg(Ly.b_hh + jb);
+                }
                 tc_fence_before();
                 mbar_arrive(ae0 + 8 * acc);
                 epi_sync();
+                if (et == 0) probe(a, pv, 4);
                 const int b = et & 63, u0 = (et >> 6) * 16, j0 = tile * 32 + u0;
                 if (b < B) {
                     const long r1 = ((long)t * B + b) * H, r4 = ((long)t * B + b) * 4 * H;
+                    // c[t-1] of all 16 units first: no load waits behind this thread's stores
+                    float4 cpv[4];
+#pragma unroll
+                    for (int q4 = 0; q4 < 4; ++q4)
+                        cpv[q4] = t > 0 ? *reinterpret_cast<const float4 *>(Ly.c + r1 - (long)B * H + j0 + 4 * q4)
+                                        : make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
                     for (int u4 = 0; u4 < 16; u4 += 4) {
                         const int j = j0 + u4;
                         float gv[4][4];
 #pragma unroll
-                        for (int g = 0; g < 4; ++g) {
-                            const float4 bi = *reinterpret_cast<const float4 *>(Ly.b_ih + g * H + j);
-                            const float4 bh = *reinterpret_cast<const float4 *>(Ly.b_hh + g * H + j);
-                            const float bb[4] = {bi.x + bh.x, bi.y + bh.y, bi.z + bh.z, bi.w + bh.w};
+                        for (int g = 0; g < 4; ++g)
 #pragma unroll
-                            for (int e = 0; e < 4; ++e) gv[g][e] = stg[(g * 32 + u0 + u4 + e) * STG_LD + b] + bb[e];
-                        }
-                        float cp[4] = {0.f, 0.f, 0.f, 0.f};
-                        if (t > 0) {
-                            const float4 c4 = *reinterpret_cast<const float4 *>(Ly.c + r1 - (long)B * H + j);
-                            cp[0] = c4.x, cp[1] = c4.y, cp[2] = c4.z, cp[3] = c4.w;
-                        }
+                            for (int e = 0; e < 4; ++e) {
+                                const int gr = g * 32 + u0 + u4 + e;
+                                gv[g][e] = stg[gr * STG_LD + b] + stg[gr * STG_LD + 64];
+                            }
+                        const float cp[4] = {cpv[u4 / 4].x, cpv[u4 / 4].y, cpv[u4 / 4].z, cpv[u4 / 4].w};
                         float ig[4], fg[4], gg[4], og[4], cc[4], hh[4];
 #pragma unroll
                         for (int e = 0; e < 4; ++e) {
@@ -374,37 +401,62 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
 #pragma unroll
                     for (int i = 0; i < 32; ++i) mine[i] += stg[mrow * 32 + i];
                     epi_sync();  // every thread read its row: hand the buffer back to the peer
+                    if (et == 0) probe(a, pv, 4);
                     if (et == 0)
                         asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
                                          mapa_cluster(rempty, peer))
                                      : "memory");
                 }
                 const bool top = l == a.L - 1;
-#pragma unroll 8
-                for (int i = 0; i < 32; ++i) {
-                    const int b = hb + i;
-                    if (b >= B) break;
-                    const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
-                    float dh = mine[i];
-                    if (top) dh += __bfloat162float(a.dy_top[r1]);
-                    const float ig = Ly.gates[r4], fg = Ly.gates[r4 + H], gg = Ly.gates[r4 + 2 * H],
-                                og = Ly.gates[r4 + 3 * H];
-                    const float ct = Ly.c[r1], cp = t > 0 ? Ly.c[r1 - (long)B * H] : 0.f;
-                    const float dcn = t < a.T - 1 ? Ly.dc[(long)b * H + j] : 0.f;
-                    const float tc = tanhf(ct);
-                    const float dct = dh * og * (1.f - tc * tc) + dcn;
-                    Ly.dc[(long)b * H + j] = dct * fg;
-                    Ly.da[r4] = __float2bfloat16_rn(dct * gg * ig * (1.f - ig));
-                    Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp * fg * (1.f - fg));
-                    Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig * (1.f - gg * gg));
-                    Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og * (1.f - og));
+                // cell backward over this CTA's 32 batch rows, 8 rows at a time: every load of a
+                // chunk is issued before any store (the stores may alias the loads as far as the
+                // compiler knows, which otherwise serialises one memory latency per row -- the
+                // probe measured 23 us of a 46 us wave); gates / c were written by the forward
+                // launch, so they take the read-only path
+                const int nb = min(32, B - hb);
+#pragma unroll
+                for (int i0 = 0; i0 < 32; i0 += 8) {  // unrolled: mine[] stays in registers
+                    if (i0 >= nb) break;
+                    float ig[8], fg[8], gg[8], og[8], ct[8], cp[8], dcn[8], dyv[8];
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) {
+                        const int b = hb + i0 + u;
+                        ig[u] = fg[u] = gg[u] = og[u] = ct[u] = cp[u] = dcn[u] = dyv[u] = 0.f;
+                        if (i0 + u < nb) {
+                            const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
+                            ig[u] = __ldg(Ly.gates + r4);
+                            fg[u] = __ldg(Ly.gates + r4 + H);
+                            gg[u] = __ldg(Ly.gates + r4 + 2 * H);
+                            og[u] = __ldg(Ly.gates + r4 + 3 * H);
+                            ct[u] = __ldg(Ly.c + r1);
+                            if (t > 0) cp[u] = __ldg(Ly.c + r1 - (long)B * H);
+                            if (t < a.T - 1) dcn[u] = Ly.dc[(long)b * H + j];
+                            if (top) dyv[u] = __bfloat162float(a.dy_top[r1]);
+                        }
+                    }
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) {
+                        if (i0 + u >= nb) break;
+                        const int b = hb + i0 + u;
+                        const long r4 = ((long)t * B + b) * 4 * H + j;
+                        const float dh = mine[i0 + u] + dyv[u];
+                        const float tc = tanhf(ct[u]);
+                        const float dct = dh * og[u] * (1.f - tc * tc) + dcn[u];
+                        Ly.dc[(long)b * H + j] = dct * fg[u];
+                        Ly.da[r4] = __float2bfloat16_rn(dct * gg[u] * ig[u] * (1.f - ig[u]));
+                        Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp[u] * fg[u] * (1.f - fg[u]));
+                        Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig[u] * (1.f - gg[u] * gg[u]));
+                        Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og[u] * (1.f - og[u]));
+                    }
                 }
             }
             epi_sync();
             if (et == 0) {
                 asm volatile("fence.acq_rel.gpu;" ::: "memory");
                 asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(a.cnt + l) : "memory");
+                probe(a, pv, 5);
             }
+            ++pv;
             acc ^= 1;
         }
     }
@@ -516,11 +568,46 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(w.cnt, 0, sizeof(unsigned) * L, s);
     if (e != cudaSuccess) return e;
     const int grid = wave_grid(L, H, w.bwd, max_pairs_resident());
+    // tools only: PD_WAVE_PROBE=<file> appends one line per launch with every CTA's per-visit
+    // phase stamps (not while the stream is being captured into a graph)
+    static unsigned long long *pbuf = nullptr;
+    const char *pfile = getenv("PD_WAVE_PROBE");
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if (pfile) cudaStreamIsCapturing(s, &cap);
+    const size_t pbytes = (size_t)grid * PROBE_V * 8 * sizeof(unsigned long long);
+    if (pfile && cap == cudaStreamCaptureStatusNone) {
+        if (!pbuf && cudaMalloc(&pbuf, (size_t)1024 * PROBE_V * 8 * sizeof(unsigned long long)) != cudaSuccess)
+            pbuf = nullptr;
+        if (pbuf && cudaMemsetAsync(pbuf, 0, pbytes, s) == cudaSuccess) a.probe = pbuf;
+    }
     cudaLaunchAttribute attr[1];
     cudaLaunchConfig_t cfg = wave_cfg(w.bwd, grid, s, attr);
     ++tl_launches;
-    return w.bwd ? cudaLaunchKernelEx(&cfg, lstm_wave_kernel<true>, m, a)
-                 : cudaLaunchKernelEx(&cfg, lstm_wave_kernel<false>, m, a);
+    e = w.bwd ? cudaLaunchKernelEx(&cfg, lstm_wave_kernel<true>, m, a)
+              : cudaLaunchKernelEx(&cfg, lstm_wave_kernel<false>, m, a);
+    if (e == cudaSuccess && a.probe) {
+        std::vector<unsigned long long> h(pbytes / 8);
+        if (cudaStreamSynchronize(s) == cudaSuccess && cudaMemcpy(h.data(), pbuf, pbytes, cudaMemcpyDeviceToHost) == cudaSuccess) {
+            unsigned long long t0 = ~0ull;
+            for (auto x : h)
+                if (x && x < t0) t0 = x;
+            if (FILE *f = fopen(pfile, "a")) {
+                fprintf(f, "%s L=%d T=%d B=%d H=%d grid=%d", w.bwd ? "bwd" : "fwd", L, T, B, H, grid);
+                for (int c = 0; c < grid; ++c) {
+                    fprintf(f, " |");
+                    for (int v = 0; v < PROBE_V; ++v) {
+                        const unsigned long long *q = &h[((size_t)c * PROBE_V + v) * 8];
+                        if (!q[3]) break;
+                        for (int ev = 0; ev < 6; ++ev) fprintf(f, " %lld", q[ev] ? (long long)(q[ev] - t0) : -1LL);
+                        fprintf(f, " ;");
+                    }
+                }
+                fprintf(f, "\n");
+                fclose(f);
+            }
+        }
+    }
+    return e;
 }
 
 }  // namespace pd

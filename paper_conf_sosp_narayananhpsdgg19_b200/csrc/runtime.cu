@@ -2515,6 +2515,17 @@ extern "C" PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *d, void *stream) 
     return e == cudaSuccess ? PD_OK : PD_ECUDA;
 }
 
+extern "C" PD_API pd_status pd_kernel_bias_grad(int dtype, const void *G, long rows, long cols, float *grad_out,
+                                                float *master, void *slot_bf16, int optimizer, float *m, float *v,
+                                                float lr, float beta1, float beta2, float eps, int step, void *stream) {
+    if (!G || rows < 1 || cols < 1 || (!grad_out && !master) || (master && dtype != PD_BF16) ||
+        (master && optimizer == PD_ADAM && (!m || !v)))
+        return PD_EINVAL;
+    cudaError_t e = bias_grad(G, dtype == PD_BF16, rows, cols, grad_out, master, static_cast<__nv_bfloat16 *>(slot_bf16),
+                              optimizer, m, v, lr, beta1, beta2, eps, step, static_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? PD_OK : PD_ECUDA;
+}
+
 extern "C" PD_API pd_status pd_kernel_softmax_ce(int dtype, const void *logits, const int32_t *labels, long rows,
                                                  int C, void *dlogits, float *loss, void *stream) {
     if (!logits || !labels || !dlogits || !loss || rows < 1 || C < 1) return PD_EINVAL;

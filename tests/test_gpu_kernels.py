@@ -159,3 +159,38 @@ def test_softmax_ce_kernel_vs_oracle(dtype, Cn):
     assert abs(loss.item() - ref_loss) < 1e-4 * max(1, abs(ref_loss))
     tol = 1e-2 if dtype == pd.PD_BF16 else 1e-5
     assert np.abs(dz.float().cpu().numpy() - ref_dz).max() / np.abs(ref_dz).max() < tol
+
+
+@pytest.mark.parametrize("rows,cols", [(256, 4096), (3200, 4096), (1025, 1000), (3200, 32000), (4096, 66)])
+@pytest.mark.parametrize("mode", ["grad", "sgd", "adam"])
+def test_bias_grad_kernel(rows, cols, mode):
+    # db = column sums of G (rows >= 1024: rows split over a 4-CTA cluster, DSMEM rank-order sum)
+    g = torch.Generator(device="cuda").manual_seed(7)
+    G = torch.randn(rows, cols, device="cuda", generator=g).to(torch.bfloat16)
+    ref = G.double().sum(0)
+    if mode == "grad":
+        out = torch.full((cols,), float("nan"), device="cuda")
+        pd.pd_kernel_bias_grad(pd.PD_BF16, G.data_ptr(), rows, cols, grad_out=out.data_ptr())
+        torch.cuda.synchronize()
+        assert float((out.double() - ref).abs().max() / ref.abs().max()) < 1e-5
+        return
+    master = torch.randn(cols, device="cuda", generator=g)
+    slot = torch.empty(cols, device="cuda", dtype=torch.bfloat16)
+    m = torch.rand(cols, device="cuda", generator=g) * 0.1
+    v = torch.rand(cols, device="cuda", generator=g) * 0.1
+    w0, m0, v0 = master.double(), m.double(), v.double()
+    lr, b1, b2, eps, step = 0.01, 0.9, 0.999, 1e-8, 3
+    adam = mode == "adam"
+    pd.pd_kernel_bias_grad(pd.PD_BF16, G.data_ptr(), rows, cols, master=master.data_ptr(), slot=slot.data_ptr(),
+                           optimizer=pd.PD_ADAM if adam else pd.PD_SGD, m=m.data_ptr(), v=v.data_ptr(), lr=lr,
+                           beta1=b1, beta2=b2, eps=eps, step=step)
+    torch.cuda.synchronize()
+    if adam:
+        mr = b1 * m0 + (1 - b1) * ref
+        vr = b2 * v0 + (1 - b2) * ref * ref
+        wr = w0 - lr * (mr / (1 - b1 ** step)) / ((vr / (1 - b2 ** step)).sqrt() + eps)
+        assert float((m.double() - mr).abs().max() / mr.abs().max()) < 1e-5
+    else:
+        wr = w0 - lr * ref
+    assert float((master.double() - wr).abs().max() / wr.abs().max()) < 1e-5
+    assert torch.equal(slot, master.to(torch.bfloat16))
