@@ -427,8 +427,8 @@ __global__ void update_master_kernel(float *master, __nv_bfloat16 *slot_bf16, fl
 }
 
 // one unreplicated gradient g (fp32, 16-byte aligned, n % 4 == 0): master -= SGD/Adam step,
-// slot = bf16(master); 4 elements per thread, 16-byte loads/stores (HBM-bound: SGD 18 B,
-// Adam 34 B per parameter)
+// slot = bf16(master); 4 elements per thread, 16-byte loads/stores (HBM-bound: SGD 14 B,
+// Adam 30 B per parameter: g 4, master 4 + 4, m and v 8 + 8, slot 2)
 template <bool ADAM>
 __global__ void __launch_bounds__(256) update_vec4_kernel(float *__restrict__ master, __nv_bfloat16 *__restrict__ slot,
                                                           const float *__restrict__ g, long n4, float *__restrict__ m,

@@ -297,6 +297,22 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             const bool mm = ik.hi > ik.lo;
+            if (BWD) {
+                // while the MMA runs: pull this item's cell-backward inputs (saved gates, c[t],
+                // c[t-1], the dc carry; written long before, mostly in HBM) into L2 -- lane i of
+                // warp q fetches the 128-byte lines of batch row hb + i for units q*32 .. q*32+31
+                const int b = rank * 32 + lane, jq = tile * 128 + q * 32;
+                if (b < B) {
+                    const WaveLayer &Lp = a.layer[l];
+                    const long r1 = ((long)t * B + b) * H + jq, r4 = ((long)t * B + b) * 4 * H + jq;
+#pragma unroll
+                    for (int g = 0; g < 4; ++g)
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.gates + r4 + (long)g * H));
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.c + r1));
+                    if (t > 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.c + r1 - (long)B * H));
+                    if (t < a.T - 1) asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.dc + (long)b * H + jq));
+                }
+            }
             mbar_wait(af0 + 8 * acc, aph[acc]);
             aph[acc] ^= 1;
             tc_fence_after();
