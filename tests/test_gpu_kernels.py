@@ -93,9 +93,11 @@ def test_tc_gemm_mask_epilogue(split, M, N, K):
     assert bool(((out.float() == 0) | (mask.float() > 0)).all())
 
 
-@pytest.mark.parametrize("adam,bn", [(False, 128), (False, 256), (True, 0)])
+@pytest.mark.parametrize("adam,bn,deep", [(False, 128, 1), (False, 128, 0), (False, 256, 1), (True, 0, 1)])
 @pytest.mark.parametrize("M,N,K", [(512, 384, 256), (4096, 4096, 256), (200, 72, 40), (1000, 4096, 64)])
-def test_tc_gemm_fused_update(adam, bn, M, N, K, monkeypatch):
+def test_tc_gemm_fused_update(adam, bn, deep, M, N, K, monkeypatch):
+    # deep: 2 operand + 3 epilogue stages (the SGD default) vs 3 + 2 (PD_UPD_DEEP, read per call)
+    monkeypatch.setenv("PD_UPD_DEEP", str(deep))
     if bn:  # SGD tile width (PD_UPD_BN_SGD, read per call)
         monkeypatch.setenv("PD_UPD_BN_SGD", str(bn))
     # dW of an N -> M layer over K rows, optimizer fused (TMA-staged epilogue)

@@ -27,4 +27,12 @@ if [[ $what == all || $what == ncu ]]; then
     -o gpurun_out/dw_update --force-overwrite \
     python bench.py --steps 1 --warmup 1 --minibatches 2 --no-cpu-baseline --no-e2e > gpurun_out/ncu_full.log 2>&1
 fi
+if [[ $what == all || $what == ncu || $what == ncu_gnmt ]]; then
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+    --log-file gpurun_out/launches_gnmt8.csv \
+    python bench.py --config gnmt8 --steps 1 --warmup 1 --minibatches 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:lstm_wave_kernel -c 2 \
+    -o gpurun_out/lstm_wave --force-overwrite \
+    python bench.py --config gnmt8 --steps 1 --warmup 1 --minibatches 1 --no-cpu-baseline --no-e2e > gpurun_out/ncu_wave.log 2>&1
+fi
 echo done > gpurun_out/round_done.txt
