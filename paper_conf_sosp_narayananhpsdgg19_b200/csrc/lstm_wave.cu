@@ -93,7 +93,8 @@ struct WaveArgs {
 constexpr int PROBE_V = 256;
 // probe events per item visit: 0 weight producer first K-block issued, 1 activation producer
 // dependencies satisfied, 2 MMA last K-block issued, 3 epilogue accumulator ready, 4 epilogue
-// partials exchanged / staged, 5 epilogue item published
+// partials exchanged / staged, 6 thread 0's cell loop done, 7 all epilogue threads done,
+// 5 epilogue item published (after the release fence)
 __device__ __forceinline__ void probe(const WaveArgs &a, int v, int ev) {
     if (a.probe && v < PROBE_V) {
         unsigned long long t;
@@ -466,8 +467,10 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                     }
                 }
             }
+            if (et == 0) probe(a, pv, 6);  // this thread's cell loop done
             epi_sync();
             if (et == 0) {
+                probe(a, pv, 7);  // all 128 epilogue threads done
                 asm volatile("fence.acq_rel.gpu;" ::: "memory");
                 asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(a.cnt + l) : "memory");
                 probe(a, pv, 5);
@@ -614,7 +617,7 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
                     for (int v = 0; v < PROBE_V; ++v) {
                         const unsigned long long *q = &h[((size_t)c * PROBE_V + v) * 8];
                         if (!q[3]) break;
-                        for (int ev = 0; ev < 6; ++ev) fprintf(f, " %lld", q[ev] ? (long long)(q[ev] - t0) : -1LL);
+                        for (int ev = 0; ev < 8; ++ev) fprintf(f, " %lld", q[ev] ? (long long)(q[ev] - t0) : -1LL);
                         fprintf(f, " ;");
                     }
                 }

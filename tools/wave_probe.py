@@ -32,6 +32,10 @@ def summarise(head, rows):
             per["mma_to_acc"].append(e[3] - e[2])
             per["exchange_or_stage"].append(e[4] - e[3])
             per["cell_publish"].append(e[5] - e[4])
+            if len(e) > 7 and e[6] > 0 and e[7] > 0:
+                per.setdefault("cell_loop_t0", []).append(e[6] - e[4])
+                per.setdefault("epi_barrier", []).append(e[7] - e[6])
+                per.setdefault("fence_publish", []).append(e[5] - e[7])
     end = max(r[-1][5] for r in rows)
     print(f"  visits/CTA {nv}, CTAs {len(rows)}, kernel span {end:.1f} us")
     for k, v in per.items():
