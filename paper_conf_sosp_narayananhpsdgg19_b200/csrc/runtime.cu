@@ -808,6 +808,29 @@ struct Exec {
                          0.f, 1, w->stream));
     }
 
+    // LSTM b_ih and b_hh receive the same gradient (sum over rows of da): on the fused path it is
+    // reduced ONCE -- written to the gradient scratch while b_ih is updated -- and b_hh is updated
+    // from the scratch by the vectorised update kernel
+    void bias_update_pair(const BwdCtx &bc, long boff_ih, long boff_hh, const void *G, long rows, int cols) {
+        if (!bc.fused) {
+            bias_update(bc, boff_ih, G, rows, cols);
+            bias_update(bc, boff_hh, G, rows, cols);
+            return;
+        }
+        const bool adam = c->cfg.optimizer == PD_ADAM;
+        CK(bias_grad(G, bf16, rows, cols, w->gbuf + boff_ih, w->master + boff_ih,
+                     static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], boff_ih, esz)), c->cfg.optimizer,
+                     adam ? w->adam_m + boff_ih : nullptr, adam ? w->adam_v + boff_ih : nullptr, c->cfg.lr,
+                     c->cfg.beta1, c->cfg.beta2, c->cfg.eps, w->updates_total + 1, w->stream));
+        const cudaError_t e = update_from_grad(
+            w->master + boff_hh, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], boff_hh, esz)),
+            w->gbuf + boff_ih, cols, c->cfg.optimizer, adam ? w->adam_m + boff_hh : nullptr,
+            adam ? w->adam_v + boff_hh : nullptr, c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps,
+            w->updates_total + 1, w->stream);
+        if (e == cudaErrorInvalidValue) bias_update(bc, boff_hh, G, rows, cols);  // unaligned: reduce again
+        else CK(e);
+    }
+
     void linear_backward(int l, const void *x, const void *G, void *dx, const BwdCtx &bc) {
         const pd_layer_desc &d = layer(l);
         const long rows = rows_of(d, B());
@@ -1059,8 +1082,7 @@ struct Exec {
         kend(2, k0);
         k0 = kstart(3);
         for (int i = L - 1; i >= 0; --i) {
-            bias_update(bc, lstm_off(l0 + i, 2), wd.da[i], TB, 4 * H);
-            bias_update(bc, lstm_off(l0 + i, 3), wd.da[i], TB, 4 * H);
+            bias_update_pair(bc, lstm_off(l0 + i, 2), lstm_off(l0 + i, 3), wd.da[i], TB, 4 * H);
         }
         kend(3, k0);
     }
@@ -1178,8 +1200,7 @@ struct Exec {
                 4 * H, st.h, H);
         kend(2, k0);
         k0 = kstart(3);
-        bias_update(bc, lstm_off(l, 2), w->lstm_da, TB, 4 * H);
-        bias_update(bc, lstm_off(l, 3), w->lstm_da, TB, 4 * H);
+        bias_update_pair(bc, lstm_off(l, 2), lstm_off(l, 3), w->lstm_da, TB, 4 * H);
         kend(3, k0);
     }
 
