@@ -397,9 +397,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                              : "memory");
         }
     }
+    // programmatic dependent launch: let the next kernel of the stream get scheduled now (its
+    // own wait holds it until this grid completes); everything above touched only on-chip state
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (warp == 0) {
         // ===== TMA producer =====
         if (lane == 0) {
+            // the previous kernel's outputs (operands, and the buffers this GEMM overwrites) are
+            // complete and visible from here on; every other role's global access is ordered
+            // after this thread's loads (mbarriers).  A no-op without the PDL launch attribute
+            asm volatile("griddepcontrol.wait;" ::: "memory");
             int stage = 0;
             uint32_t phase = 0;
             for (int unit = u0; unit < units; unit += ustep) {
@@ -1141,6 +1148,17 @@ bool encode_map(CUtensorMap *map, const void *base, long inner, long outer, long
     return r == CUDA_SUCCESS;
 }
 
+// PD_PDL=1: GEMMs and split-K reductions that the caller marks (Gemm::pdl) launch with
+// programmatic stream serialization, so a kernel's launch and prologue overlap its predecessor's
+// tail (griddepcontrol.wait in the kernels holds every dependent access)
+bool g_pdl_enabled() {
+    static const int v = [] {
+        const char *e = getenv("PD_PDL");
+        return e ? atoi(e) : 0;
+    }();
+    return v != 0;
+}
+
 int num_sms() {
     static int n = 0;
     if (!n) {
@@ -1226,7 +1244,8 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
     const int slots = num_sms() / CG;
     const int grid = e.csplit > 1 ? CG * units : CG * (units < slots ? units : slots);
     const int cluster = e.csplit > 1 ? CG * e.csplit : CG;
-    if (cluster == 1) {
+    const bool pdl = g_pdl_enabled() && g.pdl;
+    if (cluster == 1 && !pdl) {
         kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, mo, mk, e, g.M, g.N, g.K);
     } else {
         cudaLaunchConfig_t cfg{};
@@ -1234,13 +1253,22 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         cfg.blockDim = dim3(NUM_THREADS);
         cfg.dynamicSmemBytes = C::SMEM;
         cfg.stream = s;
-        cudaLaunchAttribute attr[1];
-        attr[0].id = cudaLaunchAttributeClusterDimension;
-        attr[0].val.clusterDim.x = cluster;
-        attr[0].val.clusterDim.y = 1;
-        attr[0].val.clusterDim.z = 1;
+        cudaLaunchAttribute attr[2];
+        int na = 0;
+        if (cluster > 1) {
+            attr[na].id = cudaLaunchAttributeClusterDimension;
+            attr[na].val.clusterDim.x = cluster;
+            attr[na].val.clusterDim.y = 1;
+            attr[na].val.clusterDim.z = 1;
+            ++na;
+        }
+        if (pdl) {
+            attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            attr[na].val.programmaticStreamSerializationAllowed = 1;
+            ++na;
+        }
         cfg.attrs = attr;
-        cfg.numAttrs = 1;
+        cfg.numAttrs = na;
         cudaError_t err = cudaLaunchKernelEx(&cfg, kern, ma, mb, mo, mk, e, g.M, g.N, g.K);
         if (err != cudaSuccess) return err;
     }
@@ -1342,6 +1370,8 @@ __global__ void splitk_epilogue_kernel(const float *ws, int S, long split_stride
                                        const float *__restrict__ bias, int relu, const __nv_bfloat16 *__restrict__ mask,
                                        long ldm, __nv_bfloat16 *__restrict__ out, long ldo,
                                        float *__restrict__ zero_ws) {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // the GEMM's partials (no-op without PDL)
     const long n4 = N / 4;
     const long total = (long)M * n4;
     for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long)gridDim.x * blockDim.x) {
@@ -1575,12 +1605,21 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             const long total = (long)g.M * (g.N / 4);
             long blocks = (total + 255) / 256;
             if (blocks > 148L * 8) blocks = 148L * 8;
-            splitk_epilogue_kernel<<<(unsigned)blocks, 256, 0, s>>>(
-                g.workspace, atomic ? 1 : S, (long)g.M * g.N, g.M, g.N, g.epi == EPI_STORE ? g.bias : nullptr,
-                g.epi == EPI_STORE ? g.relu : 0, g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr,
-                g.ldm, static_cast<__nv_bfloat16 *>(g.out), g.ldo, atomic ? g.workspace : nullptr);
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3((unsigned)blocks);
+            cfg.blockDim = dim3(256);
+            cfg.stream = s;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            attr[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = (g_pdl_enabled() && g.pdl) ? 1 : 0;
             ++tl_launches;
-            return cudaGetLastError();
+            return cudaLaunchKernelEx(&cfg, splitk_epilogue_kernel, (const float *)g.workspace, atomic ? 1 : S,
+                                      (long)g.M * g.N, g.M, g.N, g.epi == EPI_STORE ? g.bias : nullptr,
+                                      g.epi == EPI_STORE ? g.relu : 0,
+                                      g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr, g.ldm,
+                                      static_cast<__nv_bfloat16 *>(g.out), g.ldo, atomic ? g.workspace : nullptr);
         }
     }
     if ((g.epi == EPI_SGD || g.epi == EPI_ADAM) && g.ldo == g.N && g.N % 8 == 0) return gemm_bf16_update(g, s);

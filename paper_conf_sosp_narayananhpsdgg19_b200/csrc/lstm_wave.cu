@@ -28,6 +28,7 @@
 #include <cuda_bf16.h>
 
 #include <cstdio>
+#include <algorithm>
 #include <cstring>
 #include <vector>
 
@@ -89,6 +90,9 @@ struct WaveArgs {
     const __nv_bfloat16 *dy_top;  // backward: gradient w.r.t. the top layer's output [T][B][H]
     unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
     unsigned long long *probe;    // tools only (PD_WAVE_PROBE): [CTA][visit < PROBE_V][8] %globaltimer
+    int keep_layers;              // weights of layers < keep_layers load with L2 evict_last, the rest
+                                  // evict_first (0: no hint): a fixed subset stays L2-resident across
+                                  // waves instead of the whole run thrashing the 126 MB L2
 };
 constexpr int PROBE_V = 256;
 // probe events per item visit: 0 weight producer first K-block issued, 1 activation producer
@@ -202,6 +206,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         ItemIter<CL> it;
         int l, tile, t, s = 0, pv = 0;
         uint32_t ph = 0;
+        const uint64_t pol_last = l2_policy_evict_last(), pol_first = l2_policy_evict_first();
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             for (int kb = ik.lo; kb < ik.hi; ++kb) {
@@ -211,12 +216,21 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 mbar_expect_tx(fw0 + 8 * s, ATILE);
                 const bool p1 = kb >= ik.n0;
                 const int k = (p1 ? kb - ik.n0 : kb) * 64;
+                // the layer whose weights this K-block reads
+                const int lw = BWD && p1 ? l + 1 : l;
+                const uint64_t pol = lw < a.keep_layers ? pol_last : pol_first;
                 if (!BWD) {
                     const CUtensorMap *w = p1 ? &m.w_hh[l] : &m.w_ih[l];
-                    for (int g = 0; g < 4; ++g) tma_load_2d(dst + g * 4096, w, fw0 + 8 * s, k, g * H + tile * 32);
+                    for (int g = 0; g < 4; ++g) {
+                        if (a.keep_layers) tma_load_2d_hint(dst + g * 4096, w, fw0 + 8 * s, k, g * H + tile * 32, pol);
+                        else tma_load_2d(dst + g * 4096, w, fw0 + 8 * s, k, g * H + tile * 32);
+                    }
                 } else {
                     const CUtensorMap *w = p1 ? &m.w_ih[l + 1] : &m.w_hh[l];
-                    for (int jj = 0; jj < 2; ++jj) tma_load_2d(dst + jj * 8192, w, fw0 + 8 * s, tile * 128 + 64 * jj, k);
+                    for (int jj = 0; jj < 2; ++jj) {
+                        if (a.keep_layers) tma_load_2d_hint(dst + jj * 8192, w, fw0 + 8 * s, tile * 128 + 64 * jj, k, pol);
+                        else tma_load_2d(dst + jj * 8192, w, fw0 + 8 * s, tile * 128 + 64 * jj, k);
+                    }
                 }
                 if (++s == S) s = 0, ph ^= 1;
             }
@@ -587,6 +601,13 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(w.cnt, 0, sizeof(unsigned) * L, s);
     if (e != cudaSuccess) return e;
     const int grid = wave_grid(L, H, w.bwd, max_pairs_resident());
+    {
+        // PD_WAVE_L2_MB (default 0 = off): MB of the run's weights kept L2-resident (whole layers)
+        const char *e2 = getenv("PD_WAVE_L2_MB");
+        const long keep = e2 ? atol(e2) : 0;
+        const long per_layer = 2L * 4 * H * H * 2;  // W_ih + W_hh bf16
+        a.keep_layers = keep > 0 ? (int)std::min<long>(L, keep * 1000000L / per_layer) : 0;
+    }
     // tools only: PD_WAVE_PROBE=<file> appends one line per launch with every CTA's per-visit
     // phase stamps (not while the stream is being captured into a graph)
     static unsigned long long *pbuf = nullptr;

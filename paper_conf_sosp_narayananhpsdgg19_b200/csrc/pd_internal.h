@@ -114,6 +114,9 @@ struct Gemm {
     // while this GEMM runs (the next layer's weights on the forward / dX chains)
     const void *l2_next = nullptr;
     long l2_next_bytes = 0;
+    // programmatic dependent launch allowed for this GEMM's kernels (with PD_PDL=1): set by the
+    // runtime for the forward / dX chains, whose predecessor on the stream is another such kernel
+    int pdl = 0;
 };
 
 // cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}

@@ -488,6 +488,7 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.split_counters = L.w->split_counters;
     g.l2_next = next_w;
     g.l2_next_bytes = next_bytes;
+    g.pdl = 1;
     CK(run_gemm(L.bf16, g, L.w->stream));
 }
 
@@ -736,6 +737,7 @@ struct Exec {
         g.split_counters = w->split_counters;
         g.l2_next = next_w;
         g.l2_next_bytes = next_bytes;
+        g.pdl = 1;
         CK(run_gemm(bf16, g, w->stream));
     }
 

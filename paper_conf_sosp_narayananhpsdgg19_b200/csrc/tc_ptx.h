@@ -38,6 +38,26 @@ static __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorM
         "l"(map), "r"(bar), "r"(c0), "r"(c1)
         : "memory");
 }
+// same, with an L2 cache-policy hint (createpolicy: evict_last keeps the box's lines resident
+// across re-reads, evict_first lets a stream pass through without displacing them)
+static __device__ __forceinline__ void tma_load_2d_hint(uint32_t dst, const CUtensorMap *map, uint32_t bar, int c0,
+                                                        int c1, uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%3, "
+        "%4}], [%2], %5;" ::"r"(dst),
+        "l"(map), "r"(bar), "r"(c0), "r"(c1), "l"(policy)
+        : "memory");
+}
+static __device__ __forceinline__ uint64_t l2_policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+static __device__ __forceinline__ uint64_t l2_policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
 // L2 prefetch of a tensor-map box (no shared memory, no barrier): lets the producer run far
 // ahead of the smem ring so HBM-streamed operands (the weights of a small-M GEMM) are in
 // flight long before their stage is free
