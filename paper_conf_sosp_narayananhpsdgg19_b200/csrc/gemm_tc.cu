@@ -79,6 +79,10 @@ struct EpiArgs {
     long split_stride_out;  // its row stride
     int *counters;
     int final_epi;
+    // distributed in-kernel split-K (with counters): every split CTA of a tile, once all S
+    // partials are in L2, sums 1/S of the tile's columns and applies the final epilogue
+    // (needs all of a launch's CTAs co-resident: one unit per CTA, one such GEMM per GPU)
+    int dist;
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
@@ -671,7 +675,67 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 else mbar_arrive_cluster(smem_u32(&tempty[acc]) & 0xFEFFFFFFu);  // the leader's barrier
             }
             if (++acc == 2) { acc = 0; acc_phase ^= 1; }
-            if (reduce) {
+            if (reduce && e.dist) {
+                // publish this partial, wait for the tile's other splits, then reduce this split's
+                // share of the columns (32-column groups [g0, g1) of BN / 32) over all S partials
+                __threadfence();
+                asm volatile("bar.sync 1, 128;" ::: "memory");
+                const int cidx = tile * CG + (int)rank;
+                if (warp == 4 && lane == 0) {
+                    atomicAdd(e.counters + cidx, 1);
+                    unsigned v;
+                    do {
+                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(e.counters + cidx) : "memory");
+                    } while ((int)v < e.ksplit);
+                }
+                asm volatile("bar.sync 1, 128;" ::: "memory");
+                __threadfence();
+                const int ngr = BN / 32, g0 = split * ngr / e.ksplit, g1 = (split + 1) * ngr / e.ksplit;
+                const int nf4 = (g1 - g0) * 8;  // float4 per row of this share
+                const int et = (int)threadIdx.x - 128;
+                const float *part = static_cast<const float *>(e.out);
+                __nv_bfloat16 *dst = static_cast<__nv_bfloat16 *>(e.ws);
+#pragma unroll 2
+                for (int it = et; it < BM * nf4; it += 128) {
+                    const int r = it / nf4, f = it % nf4;
+                    const int grow = m0 + r, col = n0 + g0 * 32 + f * 4;
+                    if (grow >= M || col >= N) continue;
+                    const long off = (long)grow * e.ldo + col;
+                    float4 acc4 = __ldcg(reinterpret_cast<const float4 *>(part + off));
+                    for (int sp = 1; sp < e.ksplit; ++sp) {
+                        const float4 b4 = __ldcg(reinterpret_cast<const float4 *>(part + (long)sp * e.split_stride + off));
+                        acc4.x += b4.x; acc4.y += b4.y; acc4.z += b4.z; acc4.w += b4.w;
+                    }
+                    float v4[4] = {acc4.x, acc4.y, acc4.z, acc4.w};
+                    if (e.final_epi == EPI_STORE) {
+                        if (e.bias) {
+                            const float4 bb = *reinterpret_cast<const float4 *>(e.bias + col);
+                            v4[0] += bb.x; v4[1] += bb.y; v4[2] += bb.z; v4[3] += bb.w;
+                        }
+                        if (e.relu)
+#pragma unroll
+                            for (int i = 0; i < 4; ++i) v4[i] = fmaxf(v4[i], 0.f);
+                    } else {
+                        const uint2 mr = *reinterpret_cast<const uint2 *>(e.mask + (long)grow * e.ldm + col);
+                        const __nv_bfloat16 *mh = reinterpret_cast<const __nv_bfloat16 *>(&mr);
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) v4[i] = __bfloat162float(mh[i]) > 0.f ? v4[i] : 0.f;
+                    }
+                    uint2 o;
+                    o.x = pack_bf16(v4[0], v4[1]);
+                    o.y = pack_bf16(v4[2], v4[3]);
+                    *reinterpret_cast<uint2 *>(dst + (long)grow * e.split_stride_out + col) = o;
+                }
+                // the last split done reading resets both counters for the next launch
+                asm volatile("bar.sync 1, 128;" ::: "memory");
+                if (warp == 4 && lane == 0) {
+                    const int old = atomicAdd(e.counters + 4096 + cidx, 1);
+                    if (old == e.ksplit - 1) {
+                        e.counters[cidx] = 0;
+                        e.counters[4096 + cidx] = 0;
+                    }
+                }
+            } else if (reduce) {
                 // publish this partial; the tile's last arriving split reduces all of them
                 __threadfence();
                 asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -1580,8 +1644,13 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             e.split_stride = (long)g.M * g.N;
             e.l2_next = g.l2_next;
             e.l2_next_bytes = g.l2_next_bytes;
-            const bool inkernel = g.split_counters != nullptr && env_int("PD_SPLIT_INKERNEL", 0);
+            // in-kernel reduction: PD_SPLIT_INKERNEL=1 last CTA of a tile sums the S partials;
+            // =2 (needs Gemm::split_dist: the caller's guarantee that no other co-residency-
+            // dependent kernel shares the GPU) every split sums 1/S of the columns
+            const int ik_mode = env_int("PD_SPLIT_INKERNEL", 0);
+            const bool inkernel = g.split_counters != nullptr && (ik_mode == 1 || (ik_mode == 2 && g.split_dist));
             if (inkernel) {
+                e.dist = ik_mode == 2;
                 e.counters = g.split_counters;
                 e.ws = g.out;
                 e.split_stride_out = g.ldo;

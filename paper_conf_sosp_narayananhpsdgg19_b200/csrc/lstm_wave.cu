@@ -412,88 +412,73 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 }
                 tc_fence_before();
                 mbar_arrive(ae0 + 8 * acc);
-                const bool exch = ik.n0 + ik.n1 > 0;
-                const int peer = rank ^ 1;
-                if (exch) {
+                if (ik.n0 + ik.n1 > 0) {
+                    const int peer = rank ^ 1;
                     mbar_wait(rempty, eph ^ 1);  // the peer consumed the previous exchange
                     eph ^= 1;
-                    // the peer's half of our batch rows lands in stg as [32 rows][128 units]
-                    // (unit-contiguous: the reads below are bank-conflict-free)
-                    const uint32_t dst = mapa_cluster(smem_u32(stg) + mrow * 4, peer);
+                    const uint32_t dst = mapa_cluster(smem_u32(stg) + mrow * 32 * 4, peer);
                     const uint32_t pbar = mapa_cluster(rfull, peer);
 #pragma unroll
-                    for (int i = 0; i < 32; ++i)
-                        asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(
-                                         dst + i * 128 * 4),
-                                     "r"(__float_as_uint(other[i])), "r"(pbar)
-                                     : "memory");
+                    for (int i = 0; i < 8; ++i)
+                        asm volatile(
+                            "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+                                dst + i * 16),
+                            "f"(other[i * 4]), "f"(other[i * 4 + 1]), "f"(other[i * 4 + 2]), "f"(other[i * 4 + 3]),
+                            "r"(pbar)
+                            : "memory");
                     if (et == 0) mbar_expect_tx(rfull, 128 * 32 * 4);
                     mbar_wait(rfull, rph);
                     rph ^= 1;
-                    // dh partial sums stay in shared memory (frees mine[] for the load pipeline);
-                    // the buffer goes back to the peer after the cell loop
 #pragma unroll
-                    for (int i = 0; i < 32; ++i) stg[i * 128 + mrow] += mine[i];
+                    for (int i = 0; i < 32; ++i) mine[i] += stg[mrow * 32 + i];
+                    epi_sync();  // every thread read its row: hand the buffer back to the peer
                     if (et == 0) probe(a, pv, 4);
+                    if (et == 0)
+                        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
+                                         mapa_cluster(rempty, peer))
+                                     : "memory");
                 }
                 const bool top = l == a.L - 1;
-                // cell backward over this CTA's 32 batch rows in 8-row chunks, software-pipelined:
-                // the next chunk's loads are issued before this chunk's stores, so one memory
-                // latency is exposed per item instead of one per chunk (the probe measured the
-                // loop as latency-bound); gates / c were written by the forward launch
+                // cell backward over this CTA's 32 batch rows, 8 rows at a time: every load of a
+                // chunk is issued before any store (the stores may alias the loads as far as the
+                // compiler knows, which otherwise serialises one memory latency per row -- the
+                // probe measured 23 us of a 46 us wave); gates / c were written by the forward
+                // launch, so they take the read-only path
                 const int nb = min(32, B - hb);
-                float cur[8][7], nxt[8][7];  // [row][ig fg gg og ct cp dcn]
-                auto load_chunk = [&](int i0, float (&v)[8][7]) {
+#pragma unroll
+                for (int i0 = 0; i0 < 32; i0 += 8) {  // unrolled: mine[] stays in registers
+                    if (i0 >= nb) break;
+                    float ig[8], fg[8], gg[8], og[8], ct[8], cp[8], dcn[8], dyv[8];
 #pragma unroll
                     for (int u = 0; u < 8; ++u) {
-#pragma unroll
-                        for (int k = 0; k < 7; ++k) v[u][k] = 0.f;
+                        const int b = hb + i0 + u;
+                        ig[u] = fg[u] = gg[u] = og[u] = ct[u] = cp[u] = dcn[u] = dyv[u] = 0.f;
                         if (i0 + u < nb) {
-                            const int b = hb + i0 + u;
                             const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
-                            v[u][0] = __ldg(Ly.gates + r4);
-                            v[u][1] = __ldg(Ly.gates + r4 + H);
-                            v[u][2] = __ldg(Ly.gates + r4 + 2 * H);
-                            v[u][3] = __ldg(Ly.gates + r4 + 3 * H);
-                            v[u][4] = __ldg(Ly.c + r1);
-                            if (t > 0) v[u][5] = __ldg(Ly.c + r1 - (long)B * H);
-                            if (t < a.T - 1) v[u][6] = Ly.dc[(long)b * H + j];
+                            ig[u] = __ldg(Ly.gates + r4);
+                            fg[u] = __ldg(Ly.gates + r4 + H);
+                            gg[u] = __ldg(Ly.gates + r4 + 2 * H);
+                            og[u] = __ldg(Ly.gates + r4 + 3 * H);
+                            ct[u] = __ldg(Ly.c + r1);
+                            if (t > 0) cp[u] = __ldg(Ly.c + r1 - (long)B * H);
+                            if (t < a.T - 1) dcn[u] = Ly.dc[(long)b * H + j];
+                            if (top) dyv[u] = __bfloat162float(a.dy_top[r1]);
                         }
                     }
-                };
-                if (nb > 0) load_chunk(0, cur);
-#pragma unroll
-                for (int i0 = 0; i0 < 32; i0 += 8) {  // unrolled: the chunks stay in registers
-                    if (i0 >= nb) break;
-                    if (i0 + 8 < nb) load_chunk(i0 + 8, nxt);
 #pragma unroll
                     for (int u = 0; u < 8; ++u) {
                         if (i0 + u >= nb) break;
                         const int b = hb + i0 + u;
                         const long r4 = ((long)t * B + b) * 4 * H + j;
-                        const float ig = cur[u][0], fg = cur[u][1], gg = cur[u][2], og = cur[u][3];
-                        // (the top layer's output gradient: loaded here, one layer of L)
-                        const float dh = (exch ? stg[(i0 + u) * 128 + mrow] : 0.f) +
-                                         (top ? __bfloat162float(a.dy_top[((long)t * B + b) * H + j]) : 0.f);
-                        const float tc = tanhf(cur[u][4]);
-                        const float dct = dh * og * (1.f - tc * tc) + cur[u][6];
-                        Ly.dc[(long)b * H + j] = dct * fg;
-                        Ly.da[r4] = __float2bfloat16_rn(dct * gg * ig * (1.f - ig));
-                        Ly.da[r4 + H] = __float2bfloat16_rn(dct * cur[u][5] * fg * (1.f - fg));
-                        Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig * (1.f - gg * gg));
-                        Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og * (1.f - og));
+                        const float dh = mine[i0 + u] + dyv[u];
+                        const float tc = tanhf(ct[u]);
+                        const float dct = dh * og[u] * (1.f - tc * tc) + dcn[u];
+                        Ly.dc[(long)b * H + j] = dct * fg[u];
+                        Ly.da[r4] = __float2bfloat16_rn(dct * gg[u] * ig[u] * (1.f - ig[u]));
+                        Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp[u] * fg[u] * (1.f - fg[u]));
+                        Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig[u] * (1.f - gg[u] * gg[u]));
+                        Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og[u] * (1.f - og[u]));
                     }
-#pragma unroll
-                    for (int u = 0; u < 8; ++u)
-#pragma unroll
-                        for (int k = 0; k < 7; ++k) cur[u][k] = nxt[u][k];
-                }
-                if (exch) {
-                    epi_sync();  // every thread read its dh rows: hand the buffer back to the peer
-                    if (et == 0)
-                        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
-                                         mapa_cluster(rempty, peer))
-                                     : "memory");
                 }
             }
             if (et == 0) probe(a, pv, 6);  // this thread's cell loop done

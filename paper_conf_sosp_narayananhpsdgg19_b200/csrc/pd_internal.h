@@ -117,6 +117,9 @@ struct Gemm {
     // programmatic dependent launch allowed for this GEMM's kernels (with PD_PDL=1): set by the
     // runtime for the forward / dX chains, whose predecessor on the stream is another such kernel
     int pdl = 0;
+    // the caller guarantees this GEMM's CTAs can all be co-resident (no other worker's spin-waiting
+    // kernel on the GPU): allows the distributed in-kernel split-K reduction (PD_SPLIT_INKERNEL=2)
+    int split_dist = 0;
 };
 
 // cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}

@@ -255,6 +255,8 @@ struct Worker {
     float *ws = nullptr;        // split-K partials of the bf16 GEMMs
     long ws_bytes = 0;
     int *split_counters = nullptr;  // per-tile arrival counters of in-kernel split-K
+    bool alone = false;  // the only worker on its GPU (all workers in this process): GEMMs may rely
+                         // on co-residency of their own CTAs (Gemm::split_dist)
     float *rgrad[2] = {};       // replicated stages: gradient per round parity
     const float **rgrad_ptrs = nullptr;  // device array [2][R]: peers' rgrad for each parity
     const float **self_grad_ptr = nullptr;  // device array [1]: gbuf
@@ -486,6 +488,7 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.workspace_bytes = ws_bytes;
     g.ws_zeroed = split_atomic();  // w->ws is zero-filled at allocation and re-zeroed by every reduce-add use
     g.split_counters = L.w->split_counters;
+    g.split_dist = L.w->alone;
     g.l2_next = next_w;
     g.l2_next_bytes = next_bytes;
     g.pdl = 1;
@@ -735,6 +738,7 @@ struct Exec {
         g.workspace_bytes = w->ws_bytes;
         g.ws_zeroed = split_atomic();
         g.split_counters = w->split_counters;
+        g.split_dist = w->alone;
         g.l2_next = next_w;
         g.l2_next_bytes = next_bytes;
         g.pdl = 1;
@@ -2135,9 +2139,18 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
     if (c->n_data < 1) return PD_ESTATE;
     for (int id = 0; id < c->nw; ++id)
         if (!c->shared[id].valid) return PD_ESTATE;
-    bool any_local = false;
-    for (auto &w : c->W) any_local = any_local || (bool)w;
+    bool any_local = false, all_local = true;
+    for (auto &w : c->W) {
+        any_local = any_local || (bool)w;
+        all_local = all_local && (bool)w;
+    }
     if (!any_local) return PD_ESTATE;
+    for (auto &w : c->W) {
+        if (!w) continue;
+        int same = 0;
+        for (auto &o : c->W) same += o && o->device == w->device;
+        w->alone = all_local && same == 1;
+    }
     // with a depth override the stash ring must still hold k_s versions at every worker
     try {
         // links (created once; local when both ends are in this process)
