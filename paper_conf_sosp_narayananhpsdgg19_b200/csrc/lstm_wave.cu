@@ -69,7 +69,8 @@ __device__ __forceinline__ void wait_count(const unsigned *p, unsigned target) {
 }
 __device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
 __device__ __forceinline__ float sigm(float x) { return 1.0f / (1.0f + __expf(-x)); }
-__device__ __forceinline__ void epi_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+template <int NE>
+__device__ __forceinline__ void epi_sync_n() { asm volatile("bar.sync 1, %0;" ::"n"(NE) : "memory"); }
 
 struct WaveLayer {
     const float *b_ih, *b_hh;  // forward
@@ -158,8 +159,15 @@ __device__ __forceinline__ uint32_t cluster_rank() {
     return r;
 }
 
+// backward: 8 epilogue warps (two per TMEM lane quadrant, 16 batch rows each) -- the cell
+// backward is the latency-bound part of a wave; forward: 4
 template <bool BWD>
-__global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
+__host__ __device__ constexpr int wave_threads() { return BWD ? 384 : 256; }
+
+template <bool BWD>
+__global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
+    constexpr int NE = wave_threads<BWD>() - 128;  // epilogue threads
+    auto epi_sync = [] { epi_sync_n<NE>(); };
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *sm = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     // backward: a cluster of 2 CTAs splits every item's K-blocks; each finishes half the batch
@@ -183,7 +191,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         }
         for (int b = 0; b < 2; ++b) {
             mbar_init(af0 + 8 * b, 1);
-            mbar_init(ae0 + 8 * b, 128);
+            mbar_init(ae0 + 8 * b, NE);
         }
         mbar_init(rfull, 1);
         mbar_init(rempty, 1);
@@ -304,7 +312,8 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
         }
     } else if (warp >= 4) {
         // ---------------- epilogue
-        const int q = warp - 4;  // TMEM lane quadrant
+        const int q = (warp - 4) & 3;   // TMEM lane quadrant (warp % 4)
+        const int half = (warp - 4) >> 2;  // backward: which 16 of the 32 batch rows
         const int et = tid - 128;
         ItemIter<CL> it;
         int l, tile, t, acc = 0, pv = 0;
@@ -317,7 +326,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                 // c[t-1], the dc carry; written long before, mostly in HBM) into L2 -- lane i of
                 // warp q fetches the 128-byte lines of batch row hb + i for units q*32 .. q*32+31
                 const int b = rank * 32 + lane, jq = tile * 128 + q * 32;
-                if (b < B) {
+                if (half == 0 && b < B) {
                     const WaveLayer &Lp = a.layer[l];
                     const long r1 = ((long)t * B + b) * H + jq, r4 = ((long)t * B + b) * 4 * H + jq;
 #pragma unroll
@@ -399,16 +408,17 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                     }
                 }
             } else {
-                // thread = hidden unit (TMEM lane m); this CTA finishes batch rows [hb, hb + 32)
-                // and swaps the other half of its K-partial with the peer CTA
-                const int mrow = q * 32 + lane, j = tile * 128 + mrow, hb = rank * 32;
-                float mine[32], other[32];
+                // thread = hidden unit (TMEM lane m); this CTA finishes batch rows [hb, hb + 32),
+                // this warp rows [hb + 16 half, +16), and swaps the matching 16 columns of the
+                // peer's half of its K-partial with the peer CTA
+                const int mrow = q * 32 + lane, j = tile * 128 + mrow, hb = rank * 32, c16 = half * 16;
+                float mine[16], other[16];
                 if (mm) {
-                    tmem_ld32(d + hb, mine);
-                    tmem_ld32(d + (32 - hb), other);
+                    tmem_ld16(d + hb + c16, mine);
+                    tmem_ld16(d + (32 - hb) + c16, other);
                 } else {
 #pragma unroll
-                    for (int i = 0; i < 32; ++i) mine[i] = other[i] = 0.f;
+                    for (int i = 0; i < 16; ++i) mine[i] = other[i] = 0.f;
                 }
                 tc_fence_before();
                 mbar_arrive(ae0 + 8 * acc);
@@ -416,10 +426,10 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                     const int peer = rank ^ 1;
                     mbar_wait(rempty, eph ^ 1);  // the peer consumed the previous exchange
                     eph ^= 1;
-                    const uint32_t dst = mapa_cluster(smem_u32(stg) + mrow * 32 * 4, peer);
+                    const uint32_t dst = mapa_cluster(smem_u32(stg) + (mrow * 32 + c16) * 4, peer);
                     const uint32_t pbar = mapa_cluster(rfull, peer);
 #pragma unroll
-                    for (int i = 0; i < 8; ++i)
+                    for (int i = 0; i < 4; ++i)
                         asm volatile(
                             "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
                                 dst + i * 16),
@@ -430,7 +440,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                     mbar_wait(rfull, rph);
                     rph ^= 1;
 #pragma unroll
-                    for (int i = 0; i < 32; ++i) mine[i] += stg[mrow * 32 + i];
+                    for (int i = 0; i < 16; ++i) mine[i] += stg[mrow * 32 + c16 + i];
                     epi_sync();  // every thread read its row: hand the buffer back to the peer
                     if (et == 0) probe(a, pv, 4);
                     if (et == 0)
@@ -439,19 +449,18 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
                                      : "memory");
                 }
                 const bool top = l == a.L - 1;
-                // cell backward over this CTA's 32 batch rows, 8 rows at a time: every load of a
+                // cell backward over this warp's 16 batch rows, 8 rows at a time: every load of a
                 // chunk is issued before any store (the stores may alias the loads as far as the
-                // compiler knows, which otherwise serialises one memory latency per row -- the
-                // probe measured 23 us of a 46 us wave); gates / c were written by the forward
-                // launch, so they take the read-only path
-                const int nb = min(32, B - hb);
+                // compiler knows, which otherwise serialises one memory latency per row); gates /
+                // c were written by the forward launch, so they take the read-only path
+                const int hb2 = hb + c16, nb = min(16, B - hb2);
 #pragma unroll
-                for (int i0 = 0; i0 < 32; i0 += 8) {  // unrolled: mine[] stays in registers
+                for (int i0 = 0; i0 < 16; i0 += 8) {  // unrolled: mine[] stays in registers
                     if (i0 >= nb) break;
                     float ig[8], fg[8], gg[8], og[8], ct[8], cp[8], dcn[8], dyv[8];
 #pragma unroll
                     for (int u = 0; u < 8; ++u) {
-                        const int b = hb + i0 + u;
+                        const int b = hb2 + i0 + u;
                         ig[u] = fg[u] = gg[u] = og[u] = ct[u] = cp[u] = dcn[u] = dyv[u] = 0.f;
                         if (i0 + u < nb) {
                             const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
@@ -468,7 +477,7 @@ __global__ void __launch_bounds__(NT, 1) lstm_wave_kernel(const __grid_constant_
 #pragma unroll
                     for (int u = 0; u < 8; ++u) {
                         if (i0 + u >= nb) break;
-                        const int b = hb + i0 + u;
+                        const int b = hb2 + i0 + u;
                         const long r4 = ((long)t * B + b) * 4 * H + j;
                         const float dh = mine[i0 + u] + dyv[u];
                         const float tc = tanhf(ct[u]);
@@ -525,7 +534,7 @@ int wave_grid(int L, int H, bool bwd, int max_pairs) {
 cudaLaunchConfig_t wave_cfg(bool bwd, int grid, cudaStream_t s, cudaLaunchAttribute *attr) {
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(NT);
+    cfg.blockDim = dim3(bwd ? wave_threads<true>() : wave_threads<false>());
     cfg.dynamicSmemBytes = wave_smem(bwd);
     cfg.stream = s;
     attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -564,7 +573,7 @@ bool lstm_wave_supported(int L, int B, int H, int I) {
                                  wave_smem(false)) != cudaSuccess ||
             cudaFuncSetAttribute(lstm_wave_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  wave_smem(true)) != cudaSuccess ||
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lstm_wave_kernel<false>, NT, wave_smem(false)) !=
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lstm_wave_kernel<false>, wave_threads<false>(), wave_smem(false)) !=
                 cudaSuccess ||
             n < 1 || max_pairs_resident() < 1) {
             cudaGetLastError();
