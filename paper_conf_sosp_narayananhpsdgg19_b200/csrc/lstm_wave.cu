@@ -159,10 +159,11 @@ __device__ __forceinline__ uint32_t cluster_rank() {
     return r;
 }
 
-// backward: 8 epilogue warps (two per TMEM lane quadrant, 16 batch rows each) -- the cell
-// backward is the latency-bound part of a wave; forward: 4
+// 8 epilogue warps, two per TMEM lane quadrant: backward -- 16 batch rows each (the cell
+// backward is the latency-bound part of a wave); forward -- one 32-column accumulator chunk
+// each to stage, 8 of a thread's 16 units each in the cell
 template <bool BWD>
-__host__ __device__ constexpr int wave_threads() { return BWD ? 384 : 256; }
+__host__ __device__ constexpr int wave_threads() { return 384; }
 
 template <bool BWD>
 __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
@@ -346,8 +347,9 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
             if (!BWD) {
                 // stage D[row = g*32 + u][b] so one thread sees all four gates of (u, b)
                 const int row = q * 32 + lane;
+                constexpr int NWQ = NE / 128;  // epilogue warps per TMEM lane quadrant
 #pragma unroll
-                for (int ch = 0; ch < 2; ++ch) {
+                for (int ch = half; ch < 2; ch += NWQ) {
                     float v[32];
                     tmem_ld32(d + ch * 32, v);
 #pragma unroll
@@ -357,7 +359,7 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
                 }
                 // gate row `row` = g*32 + u: b_ih + b_hh into the staging row's spare column 64
                 // (STG_LD = 68), so the cell loop below reads biases from shared memory
-                {
+                if (half == 0) {
                     const int gi = row >> 5, uu = row & 31, jb = gi * H + tile * 32 + uu;
                     stg[row * STG_LD + 64] = __ldg(Ly.b_ih + jb) + __ldg(Ly.b_hh + jb);
                 }
@@ -365,17 +367,18 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
                 mbar_arrive(ae0 + 8 * acc);
                 epi_sync();
                 if (et == 0) probe(a, pv, 4);
-                const int b = et & 63, u0 = (et >> 6) * 16, j0 = tile * 32 + u0;
+                constexpr int UPT = 16 / NWQ;  // units per thread
+                const int b = et & 63, u0 = (et >> 6) * UPT, j0 = tile * 32 + u0;
                 if (b < B) {
                     const long r1 = ((long)t * B + b) * H, r4 = ((long)t * B + b) * 4 * H;
-                    // c[t-1] of all 16 units first: no load waits behind this thread's stores
-                    float4 cpv[4];
+                    // c[t-1] of all this thread's units first: no load waits behind its stores
+                    float4 cpv[UPT / 4];
 #pragma unroll
-                    for (int q4 = 0; q4 < 4; ++q4)
+                    for (int q4 = 0; q4 < UPT / 4; ++q4)
                         cpv[q4] = t > 0 ? *reinterpret_cast<const float4 *>(Ly.c + r1 - (long)B * H + j0 + 4 * q4)
                                         : make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-                    for (int u4 = 0; u4 < 16; u4 += 4) {
+                    for (int u4 = 0; u4 < UPT; u4 += 4) {
                         const int j = j0 + u4;
                         float gv[4][4];
 #pragma unroll

@@ -1,0 +1,11 @@
+#!/bin/bash
+mkdir -p gpurun_out
+{
+timeout 900 python -m pytest tests/test_gpu_lstm_rec.py -x -q 2>&1 | tail -2
+rm -f gpurun_out/wave_probe.txt
+PD_WAVE_PROBE=gpurun_out/wave_probe.txt timeout 300 python bench.py --config gnmt8 --steps 1 --warmup 1 --minibatches 1 --no-cpu-baseline --no-e2e > /dev/null 2>&1
+python tools/wave_probe.py gpurun_out/wave_probe.txt | head -13
+P='import sys,json; d=json.loads(sys.stdin.read()); print(round(d["value"]), d["clocks"]["sm_mhz"])'
+B="timeout 400 python bench.py --steps 20 --no-cpu-baseline --no-e2e"
+for cfg in gnmt8 gnmt16 gnmt8; do echo "--- $cfg"; $B --config $cfg | python -c "$P"; done
+} > gpurun_out/exp16.log 2>&1

@@ -1,6 +1,6 @@
 #!/bin/bash
 # L2-prefetch experiment: isolated M=256 GEMMs (L2 flushed vs warm), probe, and the MLP step with
-# PD_L2_PF = 0..3.  gpurun -- bash tools/exp_pf.sh
+# PD_L2_PF = 0..3.  gpurun -- bash tools/experiments/exp_pf.sh
 mkdir -p gpurun_out
 {
 python tools/gemm_bench.py all
