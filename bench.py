@@ -167,6 +167,16 @@ def dw_update_bytes(L, B):
     return B * L.out * 2 + B * L.in_ * 2 + L.out * L.in_ * (4 + 4 + 2)
 
 
+def l2_note(layers, optimizer):
+    """The timing rule's L2 statement, computed from the workload: bytes every minibatch streams
+    (bf16 weights, fp32 master, Adam m and v) against the 126 MB L2."""
+    import synth
+    P = sum(synth.param_count(L) for L in layers)
+    opt = f" + {8 * P / 1e9:.2f} GB Adam m, v" if optimizer == synth.ADAM else ""
+    return (f"working set > L2: every minibatch streams {2 * P / 1e9:.2f} GB bf16 weights + "
+            f"{4 * P / 1e9:.2f} GB fp32 master{opt} over {len(layers)} layers (126 MB L2), no flush needed")
+
+
 def stage_roofline(layers, plan, B, peaks, optimizer, nvlink_gbs=900.0):
     """north_star / SURVEY §8(d) per-stage roofline:
         samples/s = B * min_s R_s / max(F_s / P_tensor, H_s / BW_HBM, N_s / BW_NVL)
@@ -476,8 +486,7 @@ def main():
                        "parallelism": (f"pipeline{n}" if n > 1 else
                                        (f"dp{N}" if N > 1 else "single-stage")),
                        "sync": args.sync,
-                       "l2": "working set > L2: every minibatch streams 0.54 GB bf16 weights + 1.07 GB fp32 "
-                             "master per 16 layers (126 MB L2), no flush needed"},
+                       "l2": l2_note(layers, wl.optimizer)},
             "bubble_pct": 100.0 * bubble,
             "wall_s": wall,
             "gpu_launches": launches,
