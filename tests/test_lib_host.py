@@ -152,3 +152,21 @@ def test_layer_time_queries_validate_arguments():
     f, b = pd.pd_get_layer_times(ctx, len(wl.layers))  # no run yet: zeros
     assert not f.any() and not b.any()
     pd.pd_destroy(ctx)
+
+
+def test_bench_l2_note_per_workload():
+    """bench.py's L2 statement is computed from each workload's parameter count: the MLP-4096
+    stage (16 x 4096^2 + biases = 268.5 M params) streams 0.54 GB of bf16 weights and 1.07 GB of
+    fp32 master per minibatch; Adam workloads add m and v (8 B/param); every config exceeds L2."""
+    import os, sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    import synth
+    wl = synth.workload("mlp4096")
+    note = bench.l2_note(wl.layers, wl.optimizer)
+    assert "0.54 GB bf16 weights + 1.07 GB fp32 master over 16 layers" in note and "Adam" not in note
+    g = synth.workload("gnmt8")
+    assert "Adam m, v" in bench.l2_note(g.layers, g.optimizer)
+    for name in ("mlp4096", "gnmt8", "gnmt16", "vgg16"):
+        w = synth.workload(name)
+        assert 2 * sum(synth.param_count(L) for L in w.layers) > 126e6
