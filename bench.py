@@ -230,55 +230,170 @@ def pass_flops(L, B):
 
 # ----------------------------------------------------------------------------- reference arm
 
+def oracle_sample(config, wl, mlp_batch):
+    """A bounded sample of the workload for the single-threaded oracle (~0.4-1 GFLOP/s):
+    (layers, B, scale, text).  Samples/s of the full workload = scale * B / seconds, where
+    `scale` converts the sample's work to whole samples:
+      mlp4096   B = mlp_batch samples of the full model (scale 1);
+      gnmt*     1 sequence, 2 of its T = 50 tokens (LSTM / classifier work per token is
+                constant; scale 2/50);
+      vgg16     1 image cropped to 32 x 32 (conv work per pixel is constant; the FC stack is
+                < 1 % of VGG-16's FLOPs; scale (32/224)^2)."""
+    import synth
+    if config in ("gnmt8", "gnmt16"):
+        n = sum(1 for L in wl.layers if L.kind == synth.LSTM)
+        T = wl.layers[0].seq_len
+        return (synth.gnmt(n, 1024, 32000, 2, 1), 1, 2.0 / T,
+                f"1 sequence (B=1) of 2 of its {T} tokens through all {len(wl.layers)} layers, scaled by 2/{T}")
+    if config == "vgg16":
+        return (synth.vgg(synth.VGG16_BLOCKS, 32, 3, [4096, 4096], 1000), 1, (32.0 / 224.0) ** 2,
+                "1 image cropped to 32x32 through VGG-16 (FC6 input 1x1x512), scaled by (32/224)^2")
+    return wl.layers, mlp_batch, 1.0, f"1 minibatch of B={mlp_batch} (not {wl.batch}) of the full model"
+
+
 def run_reference(args):
     """--impl reference: the oracle (this tier's reference arm) on the host cores, on a
-    bounded sample of the same workload; one JSON line."""
+    bounded sample of the same workload (oracle_sample, a few seconds per step); one JSON line."""
     import oracle
     import synth
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     wl = synth.workload(args.config)
-    # bounded sample per step: 1 sample of the full model (mlp4096 ~3.7 s of single-thread
-    # oracle work per step), so --steps K --warmup W (every warm-up step run) ends within minutes
-    Bs = max(1, args.cpu_batch // 8)
-    layers = wl.layers
+    layers, Bs, scale, text = oracle_sample(args.config, wl, max(1, args.cpu_batch // 8))
     p0 = synth.init_params(layers)
     wl_s = synth.Workload(wl.name, layers, Bs, wl.optimizer, wl.lr)
     data = synth.make_data(wl_s, 1)
+    oracle.lib()
     times = []
-    for i in range(args.warmup + max(1, args.steps)):
-        t0 = time.perf_counter()
-        oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
-        if i >= args.warmup:
-            times.append(time.perf_counter() - t0)
+    with pinned_to_core0() as core:
+        for i in range(args.warmup + max(1, args.steps)):
+            t0 = time.perf_counter()
+            oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
+            if i >= args.warmup:
+                times.append(time.perf_counter() - t0)
     per = float(np.median(times))
-    value = Bs / per
+    value = scale * Bs / per
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": args.gpus,
             "steps": len(times), "warmup": args.warmup, "ms_per_step": per * 1e3, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": WORKLOAD_DESC.get(args.config, args.config) + " run by the CPU oracle (1 stage); "
-                                   f"bounded sample: 1 minibatch of B={Bs} per step", "global_batch": Bs},
+                                   f"bounded sample per step: {text}", "global_batch": Bs},
             "cpu_baseline": {"value": value, "unit": "samples/s", "cores": 1, "kind": "oracle",
-                             "sample": f"1 minibatch of B={Bs} through all {len(layers)} layers (fwd+bwd+SGD), "
-                                       f"single-threaded fp32 naive loops"},
+                             "cpu_model": cpu_model(), "nproc": os.cpu_count(), "pinned_core": core,
+                             "sample": f"{text}; fwd+bwd+{'Adam' if wl.optimizer else 'SGD'}, single-threaded fp32 "
+                                       f"naive loops pinned to core {core}"},
             "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+class pinned_to_core0:
+    """taskset -c 0 for the oracle timing (BASELINE.md CPU-baseline plan), restored after."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, {min(self.old)})
+        return min(self.old)
+
+    def __exit__(self, *a):
+        os.sched_setaffinity(0, self.old)
 
 
 def cpu_baseline(args, layers, wl):
     import oracle
     import synth
-    Bs = args.cpu_batch
+    layers, Bs, scale, text = oracle_sample(args.config, wl, args.cpu_batch)
     p0 = synth.init_params(layers)
     wl_s = synth.Workload(wl.name, layers, Bs, wl.optimizer, wl.lr)
     data = synth.make_data(wl_s, 1)
-    t0 = time.perf_counter()
-    oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
-    dt = time.perf_counter() - t0
-    return {"value": Bs / dt, "unit": "samples/s", "cores": 1, "kind": "oracle",
-            "sample": f"1 minibatch of B={Bs} (not 256) through all {len(layers)} layers of {args.config} "
-                      f"(fwd+bwd+SGD), single-threaded fp32 naive loops, {dt:.1f} s"}
+    oracle.lib()  # load (and if needed build) outside the timed region
+    with pinned_to_core0() as core:
+        t0 = time.perf_counter()
+        oracle.run(layers, [len(layers) - 1], [1], Bs, 1, p0, data, wl.optimizer, wl.lr)
+        dt = time.perf_counter() - t0
+    return {"value": scale * Bs / dt, "unit": "samples/s", "cores": 1, "kind": "oracle",
+            "cpu_model": cpu_model(), "nproc": os.cpu_count(), "pinned_core": core,
+            "sample": f"{text}; fwd+bwd+{'Adam' if wl.optimizer else 'SGD'}, single-threaded fp32 naive loops "
+                      f"pinned to core {core} (taskset -c {core} equivalent), {dt:.1f} s"}
+
+
+# ----------------------------------------------------------------------------- per-stage table
+
+def solo_stage(plan, s, layers, wl, p0, data, n_data, M_solo, runs=3, warm=2, profile=True):
+    """Stage s (replica 0) of `plan` alone on this GPU (pd_stage_solo: absent neighbours are
+    infinitely fast stand-ins).  Returns ms per minibatch of this replica and kernel-class
+    shares of an instrumented run."""
+    import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline, workers_of
+    wid = [w for w, st, r, g in workers_of(plan) if st == s and r == 0][0]
+    first, last, R = plan.stages[s][0], plan.stages[s][1], plan.stages[s][2]
+    P = Pipeline(plan, layers, p0, dtype=pd.PD_BF16, optimizer=wl.optimizer, lr=wl.lr, minibatch=wl.batch,
+                 record_trace=2, local=lambda w: w == wid, solo=True)
+    try:
+        P.set_data(*data, n_data)
+        P.set_timing(2, 0)
+        for _ in range(warm):
+            P.run(M_solo)
+        ms = []
+        for _ in range(runs):
+            P.run(M_solo)
+            ms.append(P.stats()["run_ms"])
+        mb = M_solo // R  # minibatches this replica processes per run
+        out = {"stage": s, "layers": [first, last], "replicas": R, "ms_per_minibatch": float(np.median(ms)) / mb}
+        if profile:
+            P.set_timing(2, 0xF)
+            P.run(M_solo)
+            st = P.stats()
+            out["class_ms_per_minibatch"] = {k: st["kern_ms"][i] / mb for i, k in
+                                             enumerate(["fwd", "dx", "dw_update", "other"])}
+            out["instrumented_ms_per_minibatch"] = st["run_ms"] / mb
+    finally:
+        P.close()
+    return out
+
+
+def stage_table(args, wl, peaks, n_plan, only=-1):
+    """Every stage of the n_plan-GPU plan bench.py would run, measured alone (solo mode); the
+    slowest stage sets the pipeline's throughput (L775-777): projected = B * min_s R_s / t_s."""
+    import synth
+    layers, B = wl.layers, wl.batch
+    plan = choose_plan(args.config, "pipeline", n_plan, layers, B, peaks)
+    p0 = synth.init_params(layers)
+    n_data = 8
+    data = synth.make_data(wl, n_data)
+    rows = []
+    for s in range(len(plan.stages)):
+        if only >= 0 and s != only:
+            continue
+        R = plan.stages[s][2]
+        M_solo = 8 * R
+        r = solo_stage(plan, s, layers, wl, p0, data, n_data, M_solo)
+        r["gflop_per_minibatch"] = sum(layer_flops(layers[l], B) * (2.0 / 3.0 if l == 0 else 1.0)
+                                       for l in range(plan.stages[s][0], plan.stages[s][1] + 1)) / 1e9
+        r["tflops"] = r["gflop_per_minibatch"] / r["ms_per_minibatch"]
+        r["frac_sustained_peak"] = r["tflops"] / peaks["bf16_tflops_sustained"]
+        rows.append(r)
+        print(json.dumps({"solo_stage": r}), file=sys.stderr, flush=True)
+    out = {"plan": [[a, b, r] for a, b, r, _g in plan.stages], "n_gpus": n_plan, "stages": rows,
+           "method": "pd_stage_solo: each stage (replica 0) alone on one GPU, neighbours replaced by "
+                     "infinitely fast stand-ins, receive rings synthetic; 3 timed runs of 8 R_s minibatches "
+                     "after 2 warm-up runs, median"}
+    if only < 0:
+        slow = max(rows, key=lambda r: r["ms_per_minibatch"] / r["replicas"])
+        proj = B * slow["replicas"] / (slow["ms_per_minibatch"] / 1e3)
+        out.update({"slowest_stage": slow["stage"], "projected_samples_per_s": proj,
+                    "projection": "B * R_s / t_s of the slowest stage (no transfer or bubble cost)"})
+    return out
 
 
 # ----------------------------------------------------------------------------- main arm
@@ -288,8 +403,15 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="mlp4096", choices=["mlp4096", "gnmt8", "gnmt16", "vgg16"])
-    ap.add_argument("--minibatches", type=int, default=0, help="minibatches per step (default 8, 16n for n>1)")
+    ap.add_argument("--config", default="gnmt16", choices=["mlp4096", "gnmt8", "gnmt16", "vgg16"])
+    ap.add_argument("--minibatches", type=int, default=0,
+                    help="minibatches per step (default 8 for one stage; 1024 for n > 1 stages: steady state, "
+                         "fill/drain bubble (n-1)/(M+n-1) < 1 %%)")
+    ap.add_argument("--stage-plan", type=int, default=8,
+                    help="per-stage table (solo mode, pd_stage_solo): each stage of the N-GPU plan measured "
+                         "alone on this GPU, projected N-GPU throughput = B min_s R_s / t_s (L775-777); 0 = off")
+    ap.add_argument("--stage", type=int, default=-1,
+                    help="measure only this stage of the --stage-plan plan in solo mode (for ncu) and exit")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-batch", type=int, default=0,
                     help="samples in the oracle's bounded sample (default: 8 for mlp4096, 1 otherwise -- ~10-60 s)")
@@ -309,6 +431,10 @@ def main():
     import torch
     import torch.distributed as dist
     import synth
+    if args.stage >= 0:  # one stage of the --stage-plan plan in solo mode (ncu captures), then exit
+        wl = synth.workload(args.config)
+        print(json.dumps(stage_table(args, wl, load_peaks(), args.stage_plan or 8, only=args.stage)), flush=True)
+        return
     import paper_conf_sosp_narayananhpsdgg19_b200 as pd
     from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline, stage_of_rank, torch_allgather
 
@@ -347,7 +473,7 @@ def main():
     plan = choose_plan(args.config, args.plan, N, layers, B, peaks)
     n = len(plan.stages)
     R0 = plan.stages[0][2]
-    M = args.minibatches or (8 * R0 if n == 1 else 16 * n)
+    M = args.minibatches or (8 * R0 if n == 1 else 1024)
     M = -(-M // R0) * R0  # a multiple of every replica count
     p0 = synth.init_params(layers) if True else None
     n_data = 8
@@ -468,10 +594,14 @@ def main():
                "note": "wall clock around set_data(pinned host) + pd_run + pd_get_losses, max over ranks"}
 
     roof_sps, roof_slow, roof_stages = stage_roofline(layers, plan, B, peaks, wl.optimizer)
+    P.close()
     cpu = None
     if rank == 0 and N == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args, layers, wl)
-    P.close()
+    solo = None
+    if rank == 0 and N == 1 and args.stage_plan > 1:
+        solo = stage_table(args, wl, peaks, args.stage_plan)
+        solo["projected_speedup_over_this_run"] = solo["projected_samples_per_s"] / value
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": N, "steps": args.steps,
@@ -509,6 +639,7 @@ def main():
                                                 "N_s/900 GB/s) (north_star; bench.stage_roofline)"},
             "e2e": e2e,
             "cpu_baseline": cpu,
+            "stage_table": solo,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -155,8 +155,9 @@ PD_API pd_status pd_profile(const pd_layer_desc *layers, int num_layers, const p
 /* Creates a context for the whole plan.  Nothing touches a device until pd_stage_init.
  * Validation (PD_EINVAL): stages contiguous and covering layers 0..num_layers-1, each
  * R_s >= 1, layer shapes consistent (out of layer l == in of layer l+1 etc.), minibatch
- * >= 1, max_depth only on straight plans.  PD_EUNSUPPORTED: layer kind / dtype combination
- * not implemented. */
+ * >= 1, max_depth only on straight plans, plan->noam either 0 or exactly ceil(W / R_0) (the
+ * value pd_plan / pd_inflight derive; anything else is rejected, not ignored).
+ * PD_EUNSUPPORTED: layer kind / dtype combination not implemented. */
 PD_API pd_status pd_create(pd_ctx **ctx, const pd_plan_t *plan, const pd_layer_desc *layers, int num_layers,
                     const pd_train_cfg *cfg);
 
@@ -176,7 +177,9 @@ PD_API pd_status pd_stage_init(pd_ctx *ctx, int stage, int replica, int cuda_dev
  * the caller's.  In a single process that owns every worker these calls are not needed.
  *   pd_export_worker : writes at most `cap` bytes to `blob`, sets *len.  PD_EINVAL if the
  *                      worker is not local or cap is too small (*len gives the size needed).
- *   pd_import_worker : PD_EINVAL on a malformed blob or a blob of a local worker. */
+ *   pd_import_worker : PD_EINVAL on a malformed blob or a blob of a local worker.
+ * A blob starts with {uint32 magic, int32 stage, int32 replica} (little-endian), so a caller can
+ * skip its own workers' blobs without importing them. */
 PD_API pd_status pd_export_worker(pd_ctx *ctx, int stage, int replica, void *blob, size_t cap, size_t *len);
 PD_API pd_status pd_import_worker(pd_ctx *ctx, const void *blob, size_t len);
 
@@ -199,9 +202,29 @@ PD_API pd_status pd_set_data(pd_ctx *ctx, const float *inputs, const int32_t *to
  *   noam : 0 => the plan's in-flight counts k_s = ceil(W_{>=s} / R_s) (NOAM = k_0, R2);
  *          D > 0 => depth override for straight plans, k_s = max(1, D - s), k_{n-1} = 1 (R19),
  *          requires D <= cfg.max_depth.
+ * Slot ownership (L1349-1353): every rewrite of a ring slot (activation / gradient receive
+ * slot, replica gradient buffer, weight-stash slot) is checked on the host to follow the
+ * completion of the op that last reads the slot's previous content, through the vector
+ * clocks the awaited messages carry (workers of this process); a violation fails the run
+ * with PD_ESTATE and a "slot ownership: ..." message in pd_last_error.
  * Errors: PD_EINVAL (num_minibatches < 1 or not a multiple of every R_s, bad noam),
- *         PD_ESTATE (workers not all initialised / imported, no data), PD_ECUDA. */
+ *         PD_ESTATE (workers not all initialised / imported, no data, slot ownership
+ *         violated), PD_ECUDA. */
 PD_API pd_status pd_run(pd_ctx *ctx, int num_minibatches, int noam);
+
+/* Solo measurement mode (SURVEY.md §8(d) per-stage table; throughput is set by the slowest
+ * stage, L775-777): measures the local workers of a multi-stage plan on their own, as if
+ * every absent neighbour were infinitely fast.  Every worker NOT initialised in this process
+ * is replaced by library-owned stand-in buffers (receive rings, gradient ring, replica
+ * buffers, flag words) on the device of the first local worker; the local workers' own
+ * receive rings are filled with synthetic values (activations U(-1, 1), gradients
+ * U(-1e-3, 1e-3)) and their incoming flag words are pre-posted, so each runs its static op
+ * list (same kernels, same k_s, same transfers into the stand-ins) without waiting.  The
+ * parameters and losses it produces are not training results.  Call after pd_stage_init of
+ * the local workers and instead of pd_import_worker; then pd_set_data / pd_run as usual.
+ * Errors: PD_ESTATE (no local worker, or a real peer was already imported), PD_ENOMEM,
+ *         PD_ECUDA. */
+PD_API pd_status pd_stage_solo(pd_ctx *ctx);
 
 /* Copies the LATEST fp32 parameters of `layer` (master weights) to host_out.  The layer's
  * stage must have a local worker (replica 0 preferred).  count must equal the layer's

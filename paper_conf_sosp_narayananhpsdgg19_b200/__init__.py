@@ -19,7 +19,9 @@ import numpy as np
 os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libpipedream.so")
+# PD_LIBRARY: the negative-control tests point a subprocess at a fault-injected build
+# (build.py FAULTS); the product path always loads the in-tree libpipedream.so
+LIB_PATH = os.environ.get("PD_LIBRARY") or os.path.join(_HERE, "libpipedream.so")
 
 PD_OK, PD_EINVAL, PD_ENOMEM, PD_ECUDA, PD_ENCCL, PD_ESTATE, PD_EUNSUPPORTED, PD_EINFEASIBLE = 0, -1, -2, -3, -4, -5, -6, -7
 PD_LINEAR, PD_LSTM, PD_CONV3X3, PD_MAXPOOL2, PD_EMBEDDING = 0, 1, 2, 3, 4
@@ -126,6 +128,7 @@ def _load():
         "pd_profile": [vp, i, vp, i, i, vp],
         "pd_set_layer_profiling": [vp, i],
         "pd_get_layer_times": [vp, vp, vp, st],
+        "pd_stage_solo": [vp],
     }
     for name, args in sigs.items():
         f = getattr(L, name)
@@ -146,7 +149,7 @@ EXPORTED = ["pd_plan", "pd_create", "pd_stage_init", "pd_export_worker", "pd_imp
             "pd_get_params", "pd_get_trace", "pd_get_version_map", "pd_get_losses", "pd_get_stats", "pd_destroy",
             "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce",
             "pd_kernel_lstm_rec", "pd_profile", "pd_set_layer_profiling", "pd_get_layer_times",
-            "pd_set_timing", "pd_kernel_bias_grad"]
+            "pd_set_timing", "pd_kernel_bias_grad", "pd_stage_solo"]
 
 
 def _strerror(s):
@@ -200,8 +203,9 @@ class Plan:
         for last, r in zip(stage_last, replicas):
             st.append((first, int(last), int(r), gpu))
             first, gpu = int(last) + 1, gpu + int(r)
-        noam = -(-gpu // int(replicas[0]))
-        return Plan(st, noam, 0.0)
+        plan = Plan(st, 0, 0.0)
+        plan.noam = pd_inflight(plan)[0]  # the library derives NOAM = k_0 (R1)
+        return plan
 
 
 def pd_plan(compute_s, act_bytes, param_bytes, num_gpus, bandwidth_Bps=0.0, max_replicas=0, comm_model=0) -> Plan:
@@ -345,6 +349,11 @@ def pd_get_layer_times(ctx, num_layers: int):
     b = np.zeros(num_layers, np.float64)
     _check(lib.pd_get_layer_times(ctx, _ptr(f), _ptr(b), num_layers), ctx)
     return f, b
+
+
+def pd_stage_solo(ctx):
+    """Solo measurement mode: absent workers become stand-ins, local receive rings synthetic."""
+    _check(lib.pd_stage_solo(ctx), ctx)
 
 
 def pd_destroy(ctx):

@@ -66,6 +66,47 @@ def build(force: bool = False, verbose: bool = False, jobs: int = 8) -> str:
     return LIB
 
 
+# Fault-injected variants of the library (tests only, never loaded by the product path):
+# runtime.cu recompiled with one PD_FAULT_* define, linked with the product's other objects
+# into build/<name>/libpipedream.so.  The negative-control tests load them through
+# PD_LIBRARY in a subprocess and require the parity / slot-ownership checks to FAIL.
+FAULTS = {
+    "fault_stash": "PD_FAULT_STASH",            # backward reads the latest weight version
+    "fault_no_dxwait": "PD_FAULT_NO_DXWAIT",    # side-stream dW + update not ordered after dX / G
+    "fault_recv_depth": "PD_FAULT_RECV_DEPTH",  # activation receive rings one slot too shallow
+}
+
+
+def fault_lib(name: str) -> str:
+    return os.path.join(HERE, "build", name, "libpipedream.so")
+
+
+def build_faults(force: bool = False) -> None:
+    build()
+    objdir = os.path.join(HERE, "build")
+    common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
+              "-I", CSRC, "-I", os.path.join(HERE, "..", "include")] + ARCH
+    rt = os.path.join(CSRC, "runtime.cu")
+    others = [os.path.join(objdir, os.path.basename(f) + ".o") for f in sources() if f != rt]
+    procs = []
+    for name, define in FAULTS.items():
+        out = fault_lib(name)
+        if not force and os.path.exists(out) and os.path.getmtime(out) >= os.path.getmtime(LIB):
+            continue
+        os.makedirs(os.path.dirname(out), exist_ok=True)
+        obj = os.path.join(os.path.dirname(out), "runtime.cu.o")
+        procs.append((out, obj, subprocess.Popen([NVCC, "-c", rt, "-o", obj, "-D" + define] + common)))
+    for out, obj, p in procs:
+        if p.wait() != 0:
+            raise RuntimeError(f"fault variant build failed: {out}")
+        tmp = out + f".tmp{os.getpid()}"
+        subprocess.check_call([NVCC, "-shared", "-o", tmp, obj] + others + ARCH +
+                              ["-cudart", "static", "-lpthread", "-ldl", "-lrt"])
+        os.replace(tmp, out)
+
+
 if __name__ == "__main__":
     build(force="--force" in sys.argv, verbose="-v" in sys.argv)
+    if "--faults" in sys.argv:
+        build_faults(force="--force" in sys.argv)
     print(LIB)

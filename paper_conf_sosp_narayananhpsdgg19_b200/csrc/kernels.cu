@@ -638,6 +638,28 @@ cudaError_t bf16_to_f32(const __nv_bfloat16 *in, float *out, long n, cudaStream_
     return cudaGetLastError();
 }
 
+// solo measurement mode: counter-hash values uniform in [-scale, scale) (content does not
+// affect the kernels' speed, but all-zero operands would understate power draw)
+__global__ void fill_uniform_kernel(void *p, long n, int bf16, float scale, uint32_t seed) {
+    for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long)gridDim.x * blockDim.x) {
+        uint32_t x = (uint32_t)i * 0x9E3779B9u ^ seed;
+        x ^= x >> 16;
+        x *= 0x7FEB352Du;
+        x ^= x >> 15;
+        x *= 0x846CA68Bu;
+        x ^= x >> 16;
+        const float v = scale * ((float)(x >> 8) * (2.f / 16777216.f) - 1.f);
+        if (bf16) static_cast<__nv_bfloat16 *>(p)[i] = __float2bfloat16(v);
+        else static_cast<float *>(p)[i] = v;
+    }
+}
+
+cudaError_t fill_uniform(void *p, long n, int bf16, float scale, uint32_t seed, cudaStream_t s) {
+    fill_uniform_kernel<<<grid_for(n), 256, 0, s>>>(p, n, bf16, scale, seed);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
 cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s) {
     signal_kernel<<<1, 1, 0, s>>>(flag, value);
     ++tl_launches;

@@ -160,6 +160,8 @@ cudaError_t regions_bf16_to_f32(const __nv_bfloat16 *src, float *dst, const long
 cudaError_t f32_to_bf16(const float *in, __nv_bfloat16 *out, long n, cudaStream_t s);
 cudaError_t bf16_to_f32(const __nv_bfloat16 *in, float *out, long n, cudaStream_t s);
 cudaError_t signal_flag(uint32_t *flag, uint32_t value, cudaStream_t s);
+// n elements (bf16 or fp32) uniform in [-scale, scale) from a counter hash of (index, seed)
+cudaError_t fill_uniform(void *p, long n, int bf16, float scale, uint32_t seed, cudaStream_t s);
 
 // LSTM / embedding (lstm.cu); `bf16` selects the path dtype of h / dy / da / y / E
 cudaError_t lstm_cell_fwd(int bf16, const float *gx, const float *gh, const float *b_ih, const float *b_hh,

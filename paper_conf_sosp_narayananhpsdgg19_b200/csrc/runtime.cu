@@ -60,6 +60,9 @@ struct CudaFail {
         if (_e != cudaSuccess) throw CudaFail{_e, #x};     \
     } while (0)
 struct Abort {};
+struct SlotViolation {
+    std::string msg;
+};
 
 long numel_params(const pd_layer_desc &d) {
     switch (d.kind) {
@@ -153,7 +156,10 @@ struct Link {
     uint32_t *remote_flag = nullptr;  // producer side, IPC-mapped
     uint32_t *local_flag = nullptr;   // consumer side
     int64_t rposted = 0;              // producer: messages posted over all runs
-    int64_t rbase = 0, rcount = 0;    // consumer: messages of earlier runs / of this run
+    int64_t rbase = 0, rcount = 0;    // consumer: messages of earlier runs / the producer posts this run
+                                      // (static: known from the schedule, not from what was awaited)
+    // slot-ownership checker (local links): the producer's vector clock at each post
+    std::vector<std::vector<int32_t>> snap;
 };
 
 // ---------------------------------------------------------------- IPC blob
@@ -172,6 +178,7 @@ struct Shared {
     float *rgrad[2] = {};      // replica gradient buffers (R_s > 1), round parity
     uint32_t *flags = nullptr; // flag words (remote links)
     bool valid = false;
+    bool standin = false;      // pd_stage_solo: local buffers standing in for an absent worker
 };
 
 struct Worker;
@@ -200,8 +207,11 @@ struct pd_ctx {
     int last_M = 0;
     std::vector<int32_t> vmap;
     double host_ms = 0;
+    // op index of F / B / U of local index j in worker w's static list of this run (checker)
+    std::vector<std::vector<int32_t>> opF, opB, opU;
     int ktime_mask = 0xF;            // kernel classes timed when record_trace >= 2
     int layer_prof = 0;              // per-layer F / B device times (pd_set_layer_profiling)
+    std::vector<void *> solo_bufs;   // pd_stage_solo stand-in buffers (owned)
     std::atomic<bool> abort{false};
     std::mutex err_mu;
     pd_status sticky = PD_OK;
@@ -241,6 +251,7 @@ struct Worker {
     cudaStream_t stream = nullptr;
     cudaStream_t side = nullptr;           // second stream: dW+update overlapping the next dX
     std::vector<cudaEvent_t> ev_dx, ev_dw; // per stage layer, reused by every backward
+    cudaEvent_t ev_fork = nullptr;         // main -> side fork at the start of an overlapped backward
     // weights
     std::vector<void *> wslot;  // k versions (path dtype)
     float *master = nullptr;    // bf16 path
@@ -309,6 +320,10 @@ struct Worker {
     uint64_t launches = 0;
     uint64_t bytes_sent = 0;
     int updates_total = 0;  // Adam step counter base (persists across runs)
+    // slot-ownership checker: vc[w] = number of ops of worker w known (through the messages
+    // this worker has awaited, transitively) to be complete before this worker's current op;
+    // vc[id] counts this worker's own ops
+    std::vector<int32_t> vc;
 
     ~Worker();
 };
@@ -335,6 +350,7 @@ Worker::~Worker() {
     if (loss_scratch) cudaFree(loss_scratch);
     for (cudaEvent_t e : ev_dx) cudaEventDestroy(e);
     for (cudaEvent_t e : ev_dw) cudaEventDestroy(e);
+    if (ev_fork) cudaEventDestroy(ev_fork);
     if (side) cudaStreamDestroy(side);
     if (stream) cudaStreamDestroy(stream);
 }
@@ -390,7 +406,8 @@ Link &get_link(pd_ctx *c, int type, int src, int dst) {
     return *it->second;
 }
 
-void link_post(pd_ctx *c, Link &L, cudaStream_t s) {
+// `vc`: the posting worker's vector clock (snapshotted with the message, local links only)
+void link_post(pd_ctx *c, Link &L, cudaStream_t s, const std::vector<int32_t> &vc) {
     if (L.remote) {
         ++L.rposted;
         CK(signal_flag(L.remote_flag, (uint32_t)L.rposted, s));
@@ -405,20 +422,25 @@ void link_post(pd_ctx *c, Link &L, cudaStream_t s) {
     CK(cudaEventRecord(L.ev[L.posted % E], s));
     {
         std::lock_guard<std::mutex> g(L.mu);
+        L.snap[L.posted % E] = vc;
         ++L.posted;
     }
     L.cv.notify_all();
 }
 
-void link_wait(pd_ctx *c, Link &L, cudaStream_t s, int64_t idx) {
+// Message idx of this run (idx < 0: the previous runs' messages -- every one of them).  The
+// waiting worker's vector clock absorbs the producer's snapshot (local links).
+void link_wait(pd_ctx *c, Link &L, cudaStream_t s, int64_t idx, std::vector<int32_t> &vc) {
     if (L.remote) {
         // flags are never reset: run r's message idx is value rbase + idx + 1
-        if (L.rcount < idx + 1) L.rcount = idx + 1;
-        CUresult r = driver()->streamWaitValue32(s, (CUdeviceptr)L.local_flag, (cuuint32_t)(L.rbase + idx + 1),
+        const int64_t want = idx < 0 ? L.rbase : L.rbase + idx + 1;
+        if (want <= 0) return;
+        CUresult r = driver()->streamWaitValue32(s, (CUdeviceptr)L.local_flag, (cuuint32_t)want,
                                                  CU_STREAM_WAIT_VALUE_GEQ);
         if (r != CUDA_SUCCESS) throw CudaFail{cudaErrorUnknown, "cuStreamWaitValue32"};
         return;
     }
+    if (idx < 0) return;  // same process: the previous pd_run joined every worker's stream
     const int E = (int)L.ev.size();
     {
         std::unique_lock<std::mutex> g(L.mu);
@@ -428,6 +450,8 @@ void link_wait(pd_ctx *c, Link &L, cudaStream_t s, int64_t idx) {
     CK(cudaStreamWaitEvent(s, L.ev[idx % E], 0));
     {
         std::lock_guard<std::mutex> g(L.mu);
+        const std::vector<int32_t> &sn = L.snap[idx % E];
+        for (size_t i = 0; i < sn.size() && i < vc.size(); ++i) vc[i] = std::max(vc[i], sn[i]);
         if (L.waited < idx + 1) L.waited = idx + 1;
     }
     L.cv.notify_all();
@@ -599,6 +623,36 @@ struct Exec {
         w->events.push_back(e);
     }
 
+    // ---------------- slot ownership (L1349-1353)
+    // A ring slot may be rewritten only once the op that last reads its previous content is
+    // known to be complete: `other`'s op (F/B/U list `opl`, local index jo) must be in this
+    // worker's vector clock, i.e. some message this worker awaited was posted after it (every
+    // post is the last action of an op, stream-ordered after all of the op's kernels).  A
+    // violation is a schedule / ring-depth bug: the run fails with PD_ESTATE.  Only workers of
+    // this process are checked (remote clocks do not travel with the flag words).
+    void hb_require(int other, const std::vector<std::vector<int32_t>> &opl, int jo, const char *what, int t) {
+        if (jo < 0 || other == w->id || !c->W[other] || jo >= (int)opl[other].size()) return;
+        const int op = opl[other][jo];
+        if (w->vc[other] > op) return;
+        char buf[320];
+        snprintf(buf, sizeof buf,
+                 "slot ownership: worker %d, minibatch %d: %s (op %d of worker %d is not known to be complete)",
+                 w->id, t, what, op, other);
+        throw SlotViolation{buf};
+    }
+    // the weight slot a backward's update writes holds no version a pending backward still uses
+    void check_weight_slot(int nslot, int j, int t) {
+        for (const auto &kv : w->fwd_version)
+            if (kv.first != j && kv.second % w->k == nslot) {
+                char buf[256];
+                snprintf(buf, sizeof buf,
+                         "slot ownership: worker %d, minibatch %d: update would overwrite version %d (slot %d) "
+                         "still stashed for local minibatch %d",
+                         w->id, t, kv.second, nslot, kv.first);
+                throw SlotViolation{buf};
+            }
+    }
+
     // ---------------- F(s, t)
     void forward(int t, int j) {
         const int s = w->stage;
@@ -607,7 +661,8 @@ struct Exec {
             const int src = c->worker_id(s - 1, p);
             Link &L = get_link(c, L_ACT, src, w->id);
             // message index on this link: minibatches from p to this replica before t
-            link_wait(c, L, w->stream, act_msg_index(s - 1, t));
+            link_wait(c, L, w->stream, act_msg_index(s - 1, t), w->vc);
+            hb_require(src, c->opF, t / c->plan.stage[s - 1].replicas, "activation used before its forward", t);
         }
         // weight stashing: the latest version.  Vertical sync: the tag the input stage gave t,
         // its latest version at F(0,t) = base + max(0, t - k_0 + 1) on the static schedule
@@ -626,6 +681,8 @@ struct Exec {
             const int Rn = c->plan.stage[s + 1].replicas;
             const int cw = c->worker_id(s + 1, t % Rn);
             const int jc = t / Rn;
+            hb_require(cw, c->opB, jc - c->Dalloc[s + 1],
+                       "activation receive slot rewritten before the backward that reads it", t);
             y_last = elem_ptr(c->shared[cw].recv, (long)(jc % c->Dalloc[s + 1]) * dev_out_elems(c->layers, w->last, B()),
                               esz);
             w->bytes_sent += (uint64_t)dev_out_elems(c->layers, w->last, B()) * esz;
@@ -694,7 +751,7 @@ struct Exec {
         } else {
             const int Rn = c->plan.stage[s + 1].replicas;
             Link &L = get_link(c, L_ACT, w->id, c->worker_id(s + 1, t % Rn));
-            link_post(c, L, w->stream);
+            link_post(c, L, w->stream, w->vc);
         }
         record_end();
     }
@@ -1454,6 +1511,12 @@ struct Exec {
         auto Gof = [&](int l) -> const void * {
             return l == last ? G_ext : w->scratch[(last - l - 1) % 3];
         };
+#ifndef PD_FAULT_NO_DXWAIT
+        // fork: the side stream's first dW reads G_ext (the gradient the main stream waited
+        // for, or dlogits written by this worker's forward) -- also when no dX precedes it
+        CK(cudaEventRecord(w->ev_fork, w->stream));
+        CK(cudaStreamWaitEvent(w->side, w->ev_fork, 0));
+#endif
         for (int l = last; l >= first; --l) {
             const pd_layer_desc &d = layer(l);
             const void *x = layer_input(l, t, j);
@@ -1473,8 +1536,11 @@ struct Exec {
                 gemm_dx(l, (int)rows, d.in, d.out, Gl, d.out, Wl(l, bc.sslot), d.in, x, dx,
                         pf ? Wl(l - 1, bc.sslot) : nullptr, pf ? (long)layer(l - 1).in * layer(l - 1).out * esz : 0);
                 kend(1, k0);
+#ifndef PD_FAULT_NO_DXWAIT
+                // dW_l + update rewrites W_l in place when k_s = 1: after dX_l has read it
                 CK(cudaEventRecord(w->ev_dx[l - first], w->stream));
                 CK(cudaStreamWaitEvent(w->side, w->ev_dx[l - first], 0));
+#endif
             }
             // side stream: dW_l + fused update, bias
             cudaStream_t main = w->stream;
@@ -1525,19 +1591,32 @@ struct Exec {
         if (s + 1 < n()) {
             const int Rn = c->plan.stage[s + 1].replicas;
             Link &L = get_link(c, L_GRAD, c->worker_id(s + 1, t % Rn), w->id);
-            link_wait(c, L, w->stream, act_msg_index(s, t));
+            link_wait(c, L, w->stream, act_msg_index(s, t), w->vc);
+            hb_require(c->worker_id(s + 1, t % Rn), c->opB, t / Rn, "gradient used before its backward", t);
         }
         const int vst = w->fwd_version[j];
+#ifdef PD_FAULT_STASH
+        const int sslot = w->version % w->k;  // fault injection (tests): the latest, not the stashed, version
+#else
         const int sslot = vst % w->k;  // stashed version (L1157-1161)
+#endif
+        if (s > 0) {
+            const int Rp = c->plan.stage[s - 1].replicas;
+            hb_require(c->worker_id(s - 1, t % Rp), c->opB, t / Rp - c->Galloc[s - 1],
+                       "gradient receive slot rewritten before the backward that reads it", t);
+        }
         trace('B', t, vst, vst);
         record_start();
         const int jr = j;  // round index on a replicated stage
-        if (Rs > 1 && jr >= 2) {
-            // gradient buffer parity jr%2 was last read by every replica in round jr-2
+        if (Rs > 1) {
+            // gradient buffer parity jr%2 was last read by every replica in round jr-2 (rounds 0
+            // and 1 of a run: by the previous run's last rounds -- wait for all of its messages)
             for (int r = 0; r < Rs; ++r) {
                 if (r == w->replica) continue;
                 Link &L = get_link(c, L_DONE, c->worker_id(s, r), w->id);
-                link_wait(c, L, w->stream, jr - 2);
+                link_wait(c, L, w->stream, jr >= 2 ? jr - 2 : -1, w->vc);
+                hb_require(c->worker_id(s, r), c->opU, jr - 2,
+                           "replica gradient buffer rewritten before the round that reads it", t);
             }
         }
         // gradient w.r.t. the stage output (pre-activation of the last layer)
@@ -1548,6 +1627,7 @@ struct Exec {
         float *gdst = Rs > 1 ? w->rgrad[jr & 1] : w->gbuf;
         const int next_version = w->version + 1;
         const int nslot = next_version % w->k;
+        check_weight_slot(nslot, j, t);
         BwdCtx bc{fused, gdst, nslot, sslot};
         bool all_linear = true;
         for (int l = w->first; l <= w->last; ++l) all_linear = all_linear && layer(l).kind == PD_LINEAR;
@@ -1612,13 +1692,13 @@ struct Exec {
         if (s > 0) {
             const int Rp = c->plan.stage[s - 1].replicas;
             Link &L = get_link(c, L_GRAD, w->id, c->worker_id(s - 1, t % Rp));
-            link_post(c, L, w->stream);
+            link_post(c, L, w->stream, w->vc);
         }
         if (Rs > 1) {
             for (int r = 0; r < Rs; ++r) {
                 if (r == w->replica) continue;
                 Link &L = get_link(c, L_READY, w->id, c->worker_id(s, r));
-                link_post(c, L, w->stream);
+                link_post(c, L, w->stream, w->vc);
             }
         }
         record_end();
@@ -1638,7 +1718,8 @@ struct Exec {
             for (int r = 0; r < Rs; ++r) {
                 if (r == w->replica) continue;
                 Link &L = get_link(c, L_READY, c->worker_id(s, r), w->id);
-                link_wait(c, L, w->stream, j);
+                link_wait(c, L, w->stream, j, w->vc);
+                hb_require(c->worker_id(s, r), c->opB, j, "replica gradient reduced before its backward", t);
             }
             if (bf16) {
                 CK(update_master(w->master, static_cast<__nv_bfloat16 *>(w->wslot[nslot]), nullptr,
@@ -1657,7 +1738,7 @@ struct Exec {
             for (int r = 0; r < Rs; ++r) {
                 if (r == w->replica) continue;
                 Link &L = get_link(c, L_DONE, w->id, c->worker_id(s, r));
-                link_post(c, L, w->stream);
+                link_post(c, L, w->stream, w->vc);
             }
         } else if (!bf16) {
             const float *latest = static_cast<const float *>(w->wslot[vin % w->k]);
@@ -1678,8 +1759,11 @@ struct Exec {
         const int Rs = c->plan.stage[w->stage].replicas;
         std::vector<Op> ops = worker_ops(Rs, w->replica, k[w->stage], M);
         w->run_base = w->version;
-        for (const Op &op : ops) {
+        w->vc.assign(c->nw, 0);
+        for (size_t i = 0; i < ops.size(); ++i) {
+            const Op &op = ops[i];
             if (c->abort) throw Abort{};
+            w->vc[w->id] = (int32_t)i + 1;  // a post during op i claims ops 0..i complete
             if (op.kind == 'F') forward(op.t, op.j);
             else if (op.kind == 'B') backward(op.t, op.j);
             else update(op.t, op.j);
@@ -1700,6 +1784,9 @@ void worker_thread(pd_ctx *c, Worker *w, int M, std::vector<int> k) {
         char buf[256];
         snprintf(buf, sizeof buf, "worker %d: %s failed: %s", w->id, f.what, cudaGetErrorString(f.e));
         c->fail(f.e == cudaErrorNotSupported ? PD_EUNSUPPORTED : PD_ECUDA, buf);
+    } catch (const SlotViolation &v) {
+        c->fail(PD_ESTATE, v.msg);
+        if (w->stream) cudaStreamSynchronize(w->stream);
     } catch (const Abort &) {
         if (w->stream) cudaStreamSynchronize(w->stream);
     }
@@ -1780,6 +1867,8 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
         if (inflight_counts(*plan, cfg->max_depth, kmax) != PD_OK) return PD_EINVAL;
         for (int s = 0; s < n; ++s) kmax[s] = std::max(kmax[s], kdef[s]);
     }
+    // plan.noam is derived, not chosen: 0, or exactly k_0 = ceil(W / R_0) (L1021, R1)
+    if (plan->noam != 0 && plan->noam != kdef[0]) return PD_EINVAL;
     if (cfg->sync_mode != PD_SYNC_STASH && cfg->sync_mode != PD_SYNC_VERTICAL) return PD_EINVAL;
     if (cfg->sync_mode == PD_SYNC_VERTICAL)
         for (int s = 0; s < n; ++s)
@@ -1801,6 +1890,9 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
     c->Dalloc.assign(n, 0);
     c->Galloc.assign(n, 0);
     for (int s = 1; s < n; ++s) c->Dalloc[s] = recv_ring_depth(*plan, kmax, s);
+#ifdef PD_FAULT_RECV_DEPTH
+    for (int s = 1; s < n; ++s) c->Dalloc[s] = std::max(1, c->Dalloc[s] - 1);  // fault injection (tests)
+#endif
     for (int s = 0; s + 1 < n; ++s) c->Galloc[s] = kmax[s];
     // vertical sync: stage s holds every version from the oldest tag still in flight to its
     // latest -- a window of k_0 versions at every stage (R25); rings sized as usual
@@ -1939,6 +2031,7 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         w->ev_dw.resize(w->last - w->first + 1);
         for (auto &e : w->ev_dx) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         for (auto &e : w->ev_dw) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&w->ev_fork, cudaEventDisableTiming));
         w->aux.assign(w->last - w->first + 1, nullptr);
         w->aux_bytes.assign(w->last - w->first + 1, 0);
         long gx_elems = 0, bh_elems = 0;
@@ -2165,6 +2258,7 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
                 CK(cudaSetDevice(ws->device));
                 const int E = 2 * std::max(8, std::max(c->Dalloc[wd->stage], c->kalloc[ws->stage])) + 4;
                 L->ev.resize(E);
+                L->snap.resize(E);
                 for (auto &e : L->ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
                 if (ws->device != wd->device) {
                     int can = 0;
@@ -2213,12 +2307,42 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
             }
         }
         // reset the host-side counters of local links; remote flags are monotonic across
-        // runs (no reset, so no cross-process barrier is needed before a run)
+        // runs (no reset, so no cross-process barrier is needed before a run): the consumer's
+        // base advances by what the producer posted in the previous run, which the static
+        // schedule fixes -- activations / gradients: the minibatches routed from the source
+        // replica to the destination replica; READY / DONE: one per round (M / R_s)
         for (auto &kv : c->links) {
             Link &L = *kv.second;
             L.posted = L.waited = 0;
+            const int type = std::get<0>(kv.first), src = std::get<1>(kv.first), dst = std::get<2>(kv.first);
+            const int ss = c->stage_of(src), ds = c->stage_of(dst);
+            const int sr = src - c->wbase[ss], dr = dst - c->wbase[ds];
+            int64_t msgs = 0;
+            if (type == L_READY || type == L_DONE) {
+                msgs = M / c->plan.stage[ss].replicas;
+            } else {
+                const int Rs = c->plan.stage[ss].replicas, Rd = c->plan.stage[ds].replicas;
+                for (int t = 0; t < M; ++t) msgs += (t % Rs == sr && t % Rd == dr);
+            }
             L.rbase += L.rcount;
-            L.rcount = 0;
+            L.rcount = msgs;
+        }
+        // op indices of every worker's static list (slot-ownership checker)
+        c->opF.assign(c->nw, {});
+        c->opB.assign(c->nw, {});
+        c->opU.assign(c->nw, {});
+        for (int s = 0; s < c->n; ++s) {
+            const int Rs = c->plan.stage[s].replicas;
+            for (int r = 0; r < Rs; ++r) {
+                const int id = c->worker_id(s, r);
+                const std::vector<Op> ops = worker_ops(Rs, r, k[s], M);
+                const int Mr = (int)(ops.size() / 3);
+                c->opF[id].assign(Mr, -1);
+                c->opB[id].assign(Mr, -1);
+                c->opU[id].assign(Mr, -1);
+                for (size_t i = 0; i < ops.size(); ++i)
+                    (ops[i].kind == 'F' ? c->opF : ops[i].kind == 'B' ? c->opB : c->opU)[id][ops[i].j] = (int32_t)i;
+            }
         }
         for (auto &wp : c->W) {
             Worker *w = wp.get();
@@ -2267,6 +2391,62 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
     for (auto &t : th) t.join();
     c->host_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     if (c->sticky != PD_OK) return c->sticky;
+    return PD_OK;
+}
+
+pd_status pd_stage_solo(pd_ctx *c) {
+    CHECK_CTX(c);
+    Worker *w0 = nullptr;
+    for (auto &w : c->W)
+        if (w) {
+            w0 = w.get();
+            break;
+        }
+    if (!w0) return PD_ESTATE;
+    for (int id = 0; id < c->nw; ++id)
+        if (!c->W[id] && c->shared[id].valid && !c->shared[id].standin) return PD_ESTATE;  // real peer imported
+    const int B = c->cfg.minibatch, esz = c->esz;
+    try {
+        CK(cudaSetDevice(w0->device));
+        auto own = [&](size_t bytes) {
+            void *p = dalloc<void>(bytes);
+            c->solo_bufs.push_back(p);
+            return p;
+        };
+        for (int id = 0; id < c->nw; ++id) {
+            if (c->W[id] || c->shared[id].valid) continue;
+            const int s = c->stage_of(id);
+            const int first = c->plan.stage[s].first_layer, last = c->plan.stage[s].last_layer;
+            Shared sh;
+            if (s > 0) sh.recv = own((size_t)c->Dalloc[s] * dev_in_elems(c->layers, first, B) * esz);
+            if (s + 1 < c->n) sh.grad = own((size_t)c->Galloc[s] * dev_out_elems(c->layers, last, B) * esz);
+            if (c->plan.stage[s].replicas > 1) {
+                const long P = c->poff[last] + (long)align_up(c->pcount[last], 64);
+                sh.rgrad[0] = static_cast<float *>(own((size_t)P * 4));
+                sh.rgrad[1] = static_cast<float *>(own((size_t)P * 4));
+            }
+            sh.flags = static_cast<uint32_t *>(own(sizeof(uint32_t) * std::max(1, c->flag_count(s))));
+            sh.valid = sh.standin = true;
+            c->shared[id] = sh;
+        }
+        // local workers: synthetic receive-ring contents, incoming flag words pre-posted
+        for (auto &wp : c->W) {
+            Worker *w = wp.get();
+            if (!w) continue;
+            CK(cudaSetDevice(w->device));
+            if (w->recv)
+                CK(fill_uniform(w->recv, (long)w->D * dev_in_elems(c->layers, w->first, B), esz == 2, 1.f,
+                                0x5EED0000u + w->id, w->stream));
+            if (w->gring)
+                CK(fill_uniform(w->gring, (long)w->G * dev_out_elems(c->layers, w->last, B), esz == 2, 1e-3f,
+                                0x5EED1000u + w->id, w->stream));
+            CK(cudaMemsetAsync(w->flags, 0x7F, sizeof(uint32_t) * std::max(1, c->flag_count(w->stage)), w->stream));
+            CK(cudaStreamSynchronize(w->stream));
+        }
+    } catch (const CudaFail &f) {
+        c->fail(PD_ECUDA, std::string("pd_stage_solo: ") + f.what + ": " + cudaGetErrorString(f.e));
+        return f.e == cudaErrorMemoryAllocation ? PD_ENOMEM : PD_ECUDA;
+    }
     return PD_OK;
 }
 
@@ -2506,8 +2686,9 @@ void pd_destroy(pd_ctx *c) {
     for (auto &kv : c->links)
         for (auto e : kv.second->ev) cudaEventDestroy(e);
     c->links.clear();
+    for (void *p : c->solo_bufs) cudaFree(p);
     for (int id = 0; id < c->nw; ++id) {
-        if (c->W[id] || !c->shared[id].valid) continue;
+        if (c->W[id] || !c->shared[id].valid || c->shared[id].standin) continue;
         Shared &sh = c->shared[id];
         void *ps[] = {sh.recv, sh.grad, sh.rgrad[0], sh.rgrad[1], sh.flags};
         for (void *p : ps)

@@ -3,13 +3,14 @@ several "virtual" workers may share a GPU) or one process per GPU (torch.distrib
 exchanges the CUDA-IPC blobs; plumbing only, no data-path collective)."""
 from __future__ import annotations
 
+import struct
 from typing import Callable, Dict, List, Optional, Sequence
 
 import numpy as np
 
 from . import (PD_BF16, PD_SGD, Plan, pd_create, pd_destroy, pd_export_worker, pd_get_layer_times, pd_get_losses,
                pd_get_params, pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data,
-               pd_set_layer_profiling, pd_set_timing, pd_stage_init, pd_run)
+               pd_set_layer_profiling, pd_set_timing, pd_stage_init, pd_stage_solo, pd_run)
 
 
 def workers_of(plan: Plan):
@@ -20,6 +21,12 @@ def workers_of(plan: Plan):
             out.append((wid, s, r, gpu0 + r))
             wid += 1
     return out
+
+
+def blob_worker(blob: bytes):
+    """(stage, replica) a pd_export_worker blob describes."""
+    _magic, stage, replica = struct.unpack_from("<Iii", blob, 0)
+    return stage, replica
 
 
 def stage_of_rank(plan: Plan, rank: int) -> int:
@@ -34,10 +41,11 @@ class Pipeline:
     def __init__(self, plan: Plan, layers, params: Sequence[np.ndarray], *, dtype=PD_BF16, optimizer=PD_SGD,
                  lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8, minibatch=1, record_trace=1, max_depth=0,
                  sync_mode=0, device_of: Optional[Callable[[int], int]] = None, local: Optional[Callable[[int], bool]] = None,
-                 allgather: Optional[Callable[[list], list]] = None):
+                 allgather: Optional[Callable[[list], list]] = None, solo: bool = False):
         """device_of(worker_gpu) -> CUDA ordinal (default: everything on device 0, i.e. virtual
         workers); local(worker_id) -> whether this process owns the worker (default all);
-        allgather(list_of_bytes) -> list over processes of lists (needed when not all local)."""
+        allgather(list_of_bytes) -> list over processes of lists (needed when not all local);
+        solo: measure the local workers alone (pd_stage_solo) instead of importing peers."""
         self.plan, self.layers = plan, list(layers)
         self.ctx = pd_create(plan, self.layers, dtype, optimizer, lr, beta1, beta2, eps, minibatch, record_trace,
                              max_depth, sync_mode)
@@ -50,17 +58,21 @@ class Pipeline:
                 continue
             first, last = plan.stages[s][0], plan.stages[s][1]
             pd_stage_init(self.ctx, s, r, device_of(g), [params[l] for l in range(first, last + 1)])
-        if len(self.local_ids) < len(self.workers):
+        if solo:
+            pd_stage_solo(self.ctx)
+        elif len(self.local_ids) < len(self.workers):
             if allgather is None:
                 raise ValueError("remote workers need an allgather for the IPC blobs")
             mine = [pd_export_worker(self.ctx, s, r) for wid, s, r, g in self.workers if local(wid)]
+            local_sr = {(s, r) for wid, s, r, g in self.workers if local(wid)}
             for blobs in allgather(mine):
                 for b in blobs:
-                    try:
-                        pd_import_worker(self.ctx, b)
-                    except Exception:
-                        # our own blobs come back too; the library rejects local workers
-                        pass
+                    # our own blobs come back too: skip them by (stage, replica) (blob header
+                    # {u32 magic, i32 stage, i32 replica, ...}, include/pipedream.h); every other
+                    # import error is real and propagates
+                    if blob_worker(b) in local_sr:
+                        continue
+                    pd_import_worker(self.ctx, b)
 
     def set_data(self, inputs, tokens, labels, n):
         pd_set_data(self.ctx, inputs, tokens, labels, n)

@@ -112,12 +112,17 @@ def test_tc_gemm_fused_update(adam, bn, deep, M, N, K, monkeypatch):
                       pd.PD_EPI_ADAM if adam else pd.PD_EPI_SGD, master=master.data_ptr(), slot=slot.data_ptr(),
                       adam_m=m.data_ptr(), adam_v=v.data_ptr(), lr=lr, beta1=b1, beta2=b2, eps=eps, step=step)
     torch.cuda.synchronize()
-    g = A.float() @ B.float().t()
+    # reference in fp64 from the exact (bf16 x bf16) products: the kernel's only rounding is
+    # its fp32 accumulation and the fp32 optimizer arithmetic (~1e-7 relative)
+    g = A.double() @ B.double().t()
+    ref_w, ref_m, ref_v = ref_w.double(), ref_m.double(), ref_v.double()
     if adam:
         ref_m = b1 * ref_m + (1 - b1) * g
         ref_v = b2 * ref_v + (1 - b2) * g * g
         ref_w = ref_w - lr * (ref_m / (1 - b1 ** step)) / ((ref_v / (1 - b2 ** step)).sqrt() + eps)
-        assert _rel(m, ref_m) < 1e-5 and _rel(v, ref_v) < 1e-4
+        em, ev = _rel(m, ref_m), _rel(v, ref_v)
+        print("adam m / v relative error", em, ev)
+        assert em < 1e-5 and ev < 1e-5, (em, ev)
     else:
         ref_w = ref_w - lr * g
     assert float((master - ref_w).abs().max()) < 1e-4

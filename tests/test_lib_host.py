@@ -170,3 +170,36 @@ def test_bench_l2_note_per_workload():
     for name in ("mlp4096", "gnmt8", "gnmt16", "vgg16"):
         w = synth.workload(name)
         assert 2 * sum(synth.param_count(L) for L in w.layers) > 126e6
+
+
+def test_create_validates_noam():
+    """plan.noam is derived (R1: ceil(W / R_0)): 0 or that value is accepted, anything else is
+    rejected instead of silently ignored (VERDICT r1 hygiene)."""
+    wl = synth.workload("mlp_small")
+    plan = pd.Plan.manual([1, 2], [2, 1])
+    assert plan.noam == pd.pd_inflight(plan)[0] == 2
+    pd.pd_destroy(pd.pd_create(plan, wl.layers, pd.PD_FP32, minibatch=16))
+    plan.noam = 0
+    pd.pd_destroy(pd.pd_create(plan, wl.layers, pd.PD_FP32, minibatch=16))
+    plan.noam = 3
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_create(plan, wl.layers, pd.PD_FP32, minibatch=16)
+    assert ei.value.status == pd.PD_EINVAL
+
+
+def test_blob_header_names_its_worker():
+    """session.Pipeline skips its own workers' blobs by the header (stage, replica) instead of
+    swallowing import errors."""
+    import struct
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import blob_worker
+    blob = struct.pack("<Iiii", 0x50443031, 3, 1, 0) + bytes(64)
+    assert blob_worker(blob) == (3, 1)
+
+
+def test_stage_solo_needs_a_local_worker():
+    wl = synth.workload("mlp_small")
+    ctx = pd.pd_create(pd.Plan.manual([1, 2], [1, 1]), wl.layers, pd.PD_FP32, minibatch=16)
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_stage_solo(ctx)
+    assert ei.value.status == pd.PD_ESTATE
+    pd.pd_destroy(ctx)
