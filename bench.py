@@ -219,6 +219,40 @@ def stage_roofline(layers, plan, B, peaks, optimizer, nvlink_gbs=900.0):
     return per[slow]["samples_per_s"], slow, per
 
 
+def class_flops(layers, first, last, B):
+    """Algorithmic FLOPs per minibatch of one stage [first, last] split by the runtime's kernel
+    classes (pd.KERNEL_CLASSES): 0 forward GEMMs, 1 dX GEMMs, 2 dW GEMMs, 4 / 5 the LSTM
+    wavefront kernels (runs of >= 2 equal LSTMs: forward with the input projection folded in,
+    backward dh over W_hh plus the inner layers' input gradients), 2 per MAC."""
+    import synth
+    fl = [0.0] * 8
+    l = first
+    while l <= last:
+        L = layers[l]
+        run = 1
+        if L.kind == synth.LSTM:
+            while (l + run <= last and layers[l + run].kind == synth.LSTM and run < 16 and
+                   layers[l + run].in_ == L.out == layers[l + run].out and L.in_ == L.out):
+                run += 1
+        need_dx = l > 0
+        if L.kind == synth.LSTM and run >= 2:
+            H, T = L.out, L.seq_len
+            fl[4] += run * 2.0 * B * T * 4 * H * 2 * H
+            fl[5] += run * 2.0 * B * T * 4 * H * H + (run - 1) * 2.0 * B * T * 4 * H * H
+            if need_dx:
+                fl[1] += 2.0 * B * T * 4 * H * H
+            fl[2] += run * (2.0 * B * T * 4 * H * H + 2.0 * B * (T - 1) * 4 * H * H)
+            l += run
+            continue
+        f = layer_flops(L, B) / 3.0
+        fl[0] += f
+        fl[2] += f
+        if need_dx:
+            fl[1] += f
+        l += 1
+    return fl
+
+
 def gemm_flops(L, B):
     return 2.0 * B * L.in_ * L.out
 
@@ -351,11 +385,10 @@ def solo_stage(plan, s, layers, wl, p0, data, n_data, M_solo, runs=3, warm=2, pr
         mb = M_solo // R  # minibatches this replica processes per run
         out = {"stage": s, "layers": [first, last], "replicas": R, "ms_per_minibatch": float(np.median(ms)) / mb}
         if profile:
-            P.set_timing(2, 0xF)
+            P.set_timing(2, 0xFF)
             P.run(M_solo)
             st = P.stats()
-            out["class_ms_per_minibatch"] = {k: st["kern_ms"][i] / mb for i, k in
-                                             enumerate(["fwd", "dx", "dw_update", "other"])}
+            out["class_ms_per_minibatch"] = {k: st["kern_ms"][i] / mb for i, k in enumerate(pd.KERNEL_CLASSES)}
             out["instrumented_ms_per_minibatch"] = st["run_ms"] / mb
     finally:
         P.close()
@@ -495,7 +528,7 @@ def main():
     for _ in range(args.warmup):
         P.run(M)
     barrier()
-    step_ms, launches, kern_ms, kern_cnt, bubbles = [], 0, np.zeros(4), np.zeros(4), []
+    step_ms, launches, kern_ms, kern_cnt, bubbles = [], 0, np.zeros(8), np.zeros(8), []
     barrier()
     t_wall0 = time.perf_counter()
     for _ in range(args.steps):
@@ -516,9 +549,9 @@ def main():
     bubble = allmax(float(np.mean(bubbles)))
 
     # ---- profile pass (not part of `value`): every kernel class timed, for step shares
-    P.set_timing(2, 0xF)
-    prof_ms, prof_kern = 0.0, np.zeros(4)
-    prof_cnt = np.zeros(4)
+    P.set_timing(2, 0xFF)
+    prof_ms, prof_kern = 0.0, np.zeros(8)
+    prof_cnt = np.zeros(8)
     for _ in range(2):
         P.run(M)
         st = P.stats()
@@ -529,23 +562,18 @@ def main():
 
     # ---- roofline of the dominant kernel, this rank's stage
     s_mine = stage_of_rank(plan, rank)
-    first_l = plan.stages[s_mine][0]
-    my_layers = [layers[l] for l in range(first_l, plan.stages[s_mine][1] + 1)]
+    first_l, last_l = plan.stages[s_mine][0], plan.stages[s_mine][1]
+    my_layers = [layers[l] for l in range(first_l, last_l + 1)]
     lin = [L for L in my_layers if L.kind == synth.LINEAR] or my_layers
     stage_flops = sum(layer_flops(L, B) for L in my_layers)
-    # per-class GEMM FLOPs of the profile pass (2 runs x this replica's minibatches); dX of
-    # the model's first layer is skipped (stage 0)
-    mb_mine = 2 * M // plan.stages[s_mine][2]
-    fwd_fl = sum(pass_flops(L, B) for L in my_layers) * mb_mine
-    dx_fl = sum(pass_flops(L, B) for i, L in enumerate(my_layers) if first_l + i > 0) * mb_mine
-    dw_fl = fwd_fl
-    cls_s = prof_kern[:3] / 1e3
-    fw_tflops = fwd_fl / cls_s[0] / 1e12 if cls_s[0] > 0 else 0.0
-    dx_tflops = dx_fl / cls_s[1] / 1e12 if cls_s[1] > 0 else 0.0
-    dw_tflops = dw_fl / cls_s[2] / 1e12 if cls_s[2] > 0 else 0.0
-    dw_avg_s = prof_kern[2] / max(prof_cnt[2], 1) / 1e3
+    mb_mine = 2 * M // plan.stages[s_mine][2]  # minibatches of this replica in the profile pass
+    cfl = class_flops(layers, first_l, last_l, B)  # per minibatch, per kernel class
+    cls_s = prof_kern / 1e3
+    cls_tflops = [cfl[i] * mb_mine / cls_s[i] / 1e12 if cls_s[i] > 0 and cfl[i] > 0 else 0.0 for i in range(8)]
+    names = pd.KERNEL_CLASSES
     if args.config == "mlp4096":
         # HBM-bound: dW GEMM with the fused SGD update (K = 256), bytes per launch
+        dw_avg_s = prof_kern[2] / max(prof_cnt[2], 1) / 1e3
         dw_bytes = float(np.mean([dw_update_bytes(L, B) for L in lin]))
         achieved = dw_bytes / dw_avg_s / 1e9 if dw_avg_s > 0 else 0.0
         roof = {"bound": "hbm", "kernel": "dW GEMM + fused SGD update (tcgen05, EPI_SGD)",
@@ -556,17 +584,19 @@ def main():
                 "bytes_per_launch": dw_bytes, "avg_launch_us": dw_avg_s * 1e6,
                 "peak_source": peaks["source"] + " hbm_gbs (copy)"}
     else:
-        # tensor-bound stages (convolutions / LSTM / classifier GEMMs): the dominant GEMM class
-        names = ["forward GEMMs", "dX GEMMs", "dW GEMMs (+update)"]
-        tfl = [fw_tflops, dx_tflops, dw_tflops]
-        d = int(np.argmax(cls_s))
-        roof = {"bound": "tensor", "kernel": f"{names[d]} of the stage (tcgen05), class total",
-                "achieved": tfl[d], "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
-                "frac": tfl[d] / peaks["bf16_tflops_sustained"], "traffic": None,
-                "flops_per_minibatch": [fwd_fl / mb_mine, dx_fl / mb_mine, dw_fl / mb_mine][d],
+        # tensor-bound stages: the kernel class with the largest share of the step
+        d = int(np.argmax([cls_s[i] if cfl[i] > 0 else 0.0 for i in range(8)]))
+        avg_s = prof_kern[d] / max(prof_cnt[d], 1) / 1e3
+        per_launch = cfl[d] * mb_mine / max(prof_cnt[d], 1)
+        roof = {"bound": "tensor", "kernel": names[d], "achieved": cls_tflops[d],
+                "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
+                "frac": cls_tflops[d] / peaks["bf16_tflops_sustained"],
+                "traffic": ncu_traffic(names[d]),
+                "flops_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
+                "flops_per_minibatch": cfl[d],
                 "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"}
-    step_share = {cls: float(prof_kern[i] / max(prof_ms, 1e-9)) for i, cls in enumerate(["fwd_gemm", "dx_gemm",
-                                                                                           "dw_update_gemm", "other"])}
+    fw_tflops, dx_tflops, dw_tflops = cls_tflops[0], cls_tflops[1], cls_tflops[2]
+    step_share = {cls: float(prof_kern[i] / max(prof_ms, 1e-9)) for i, cls in enumerate(names)}
     step_share["note"] = "profile pass (2 steps, every kernel class event-timed); dW and dX overlap on two streams"
 
     # ---- end to end through the public API: host (pinned) inputs in, losses out, every step
@@ -624,12 +654,13 @@ def main():
             "roofline": dict(roof, timing="CUDA events around every launch of the class on its stream, "
                                           "instrumented profile pass (2 steps) right after the timed region; "
                                           "dW overlaps the next layer's dX"),
-            "tensor_pipe": {"fwd_gemm_tflops": fw_tflops, "dx_gemm_tflops": dx_tflops, "dw_gemm_tflops": dw_tflops,
+            "tensor_pipe": {"class_tflops": {n: t for n, t in zip(pd.KERNEL_CLASSES, cls_tflops) if t > 0},
+                            "class_frac": {n: t / peaks["bf16_tflops_sustained"]
+                                           for n, t in zip(pd.KERNEL_CLASSES, cls_tflops) if t > 0},
                             "peak_tflops": peaks["bf16_tflops_sustained"],
-                            "fwd_frac": fw_tflops / peaks["bf16_tflops_sustained"],
-                            "dx_frac": dx_tflops / peaks["bf16_tflops_sustained"],
-                            "dw_frac": dw_tflops / peaks["bf16_tflops_sustained"],
-                            "note": "class FLOPs / class device time (dW time includes the fused update)",
+                            "note": "algorithmic class FLOPs (bench.class_flops) / class device time (CUDA events, "
+                                    "profile pass); dW time includes a fused update; ncu tensor-pipe counters "
+                                    "per stage are in profiles/",
                             "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"},
             "step_share": step_share,
             "stage_tflops": stage_flops * args.steps * M / plan.stages[s_mine][2] / (total_ms / 1e3) / 1e12,

@@ -252,6 +252,7 @@ PD_API pd_status pd_get_version_map(pd_ctx *ctx, int32_t *out, size_t cap);
 PD_API pd_status pd_get_losses(pd_ctx *ctx, float *out, size_t cap);
 
 #define PD_MAX_LOCAL_WORKERS 64
+#define PD_KERNEL_CLASSES 8     /* pd_stats per-class kernel timing */
 typedef struct {
     double host_ms;               /* host wall time of the last pd_run                     */
     double device_ms;             /* device span of the last run over the local workers    */
@@ -265,16 +266,19 @@ typedef struct {
     double run_ms;                /* device time of the last run: max over local workers of
                                      the span between events recorded on the worker's stream
                                      before its first and after its last operation          */
-    double kern_ms[4];            /* record_trace 2: summed device time per kernel class:
-                                     0 forward GEMM, 1 dX GEMM, 2 dW GEMM (+fused update), 3 reserved */
-    uint64_t kern_count[4];       /* launches timed per class                                */
+    double kern_ms[PD_KERNEL_CLASSES]; /* record_trace 2: summed device time per kernel class:
+                                     0 forward GEMM, 1 dX GEMM, 2 dW GEMM (+fused update),
+                                     3 other (bias gradients, pooling, embedding, copies),
+                                     4 LSTM wavefront forward, 5 LSTM wavefront backward,
+                                     6 softmax-CE, 7 separate optimizer update pass        */
+    uint64_t kern_count[PD_KERNEL_CLASSES]; /* launches timed per class                      */
 } pd_stats;
 
 PD_API pd_status pd_get_stats(pd_ctx *ctx, pd_stats *out);
 
 /* Changes the instrumentation of later pd_run calls: record_trace as in pd_train_cfg;
  * kernel_timing_mask bit c times every kernel of class c with CUDA events on its stream
- * (0 forward GEMMs, 1 dX GEMMs, 2 dW GEMMs incl. the fused update, 3 bias / other); each timed
+ * (the PD_KERNEL_CLASSES classes of pd_stats.kern_ms); each timed
  * launch costs two event records, so time only what is needed inside a timed region. */
 PD_API pd_status pd_set_timing(pd_ctx *ctx, int record_trace, int kernel_timing_mask);
 

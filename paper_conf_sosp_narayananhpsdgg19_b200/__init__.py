@@ -32,6 +32,9 @@ PD_SYNC_STASH, PD_SYNC_VERTICAL = 0, 1
 PD_EPI_STORE, PD_EPI_MASK, PD_EPI_F32, PD_EPI_SGD, PD_EPI_ADAM = 0, 1, 2, 3, 4
 PD_MAX_STAGES = 64
 PD_MAX_LOCAL_WORKERS = 64
+PD_KERNEL_CLASSES = 8
+KERNEL_CLASSES = ["fwd_gemm", "dx_gemm", "dw_gemm", "other", "lstm_wave_fwd", "lstm_wave_bwd", "softmax_ce",
+                  "optimizer_update"]
 
 
 class PDError(RuntimeError):
@@ -79,7 +82,7 @@ class Stats(C.Structure):
                 ("kernel_launches", C.c_uint64), ("bytes_sent", C.c_uint64), ("num_local_workers", C.c_int),
                 ("worker_id", C.c_int * PD_MAX_LOCAL_WORKERS), ("busy_ms", C.c_double * PD_MAX_LOCAL_WORKERS),
                 ("span_ms", C.c_double * PD_MAX_LOCAL_WORKERS), ("run_ms", C.c_double),
-                ("kern_ms", C.c_double * 4), ("kern_count", C.c_uint64 * 4)]
+                ("kern_ms", C.c_double * PD_KERNEL_CLASSES), ("kern_count", C.c_uint64 * PD_KERNEL_CLASSES)]
 
 
 class LstmRecDesc(C.Structure):
@@ -335,7 +338,7 @@ def pd_get_stats(ctx) -> dict:
             "run_ms": s.run_ms, "kern_ms": list(s.kern_ms), "kern_count": [int(x) for x in s.kern_count]}
 
 
-def pd_set_timing(ctx, record_trace: int, kernel_timing_mask: int = 0xF):
+def pd_set_timing(ctx, record_trace: int, kernel_timing_mask: int = 0xFF):
     _check(lib.pd_set_timing(ctx, record_trace, kernel_timing_mask), ctx)
 
 

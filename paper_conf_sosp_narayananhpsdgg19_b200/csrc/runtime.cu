@@ -209,7 +209,7 @@ struct pd_ctx {
     double host_ms = 0;
     // op index of F / B / U of local index j in worker w's static list of this run (checker)
     std::vector<std::vector<int32_t>> opF, opB, opU;
-    int ktime_mask = 0xF;            // kernel classes timed when record_trace >= 2
+    int ktime_mask = 0xFF;           // kernel classes timed when record_trace >= 2
     int layer_prof = 0;              // per-layer F / B device times (pd_set_layer_profiling)
     std::vector<void *> solo_bufs;   // pd_stage_solo stand-in buffers (owned)
     std::atomic<bool> abort{false};
@@ -310,7 +310,7 @@ struct Worker {
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> op_ev;  // record_trace 2
     std::vector<cudaEvent_t> ev_pool;
     cudaEvent_t run_ev[2] = {nullptr, nullptr};  // start / end of this worker's part of a run
-    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev[4];  // per kernel class (record_trace 2)
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev[PD_KERNEL_CLASSES];  // per kernel class (record_trace 2)
     struct LayerEv {
         int layer;
         char dir;  // 'F' or 'B'
@@ -568,17 +568,27 @@ struct Exec {
         return elem_ptr(w->act[l - w->first], (long)(j % w->k) * dev_in_elems(c->layers, l, B()), esz);
     }
 
-    // per-kernel-class device time (0 fwd GEMM, 1 dX GEMM, 2 dW(+update) GEMM, 3 other)
+    // timing events: the pre-sized pool, grown on demand (never while capturing: the callers
+    // return before asking for one then)
+    cudaEvent_t pool_event() {
+        if (ev_used >= (int)w->ev_pool.size()) {
+            cudaEvent_t e;
+            CK(cudaEventCreate(&e));
+            w->ev_pool.push_back(e);
+        }
+        return w->ev_pool[ev_used++];
+    }
+    // per-kernel-class device time (pd_stats.kern_ms classes)
     bool capturing = false;
     cudaEvent_t kstart(int cls) {
         if (capturing || !timing || !((c->ktime_mask >> cls) & 1)) return nullptr;
-        cudaEvent_t a = w->ev_pool[ev_used++];
+        cudaEvent_t a = pool_event();
         CK(cudaEventRecord(a, w->stream));
         return a;
     }
     void kend(int cls, cudaEvent_t a) {
         if (!a) return;
-        cudaEvent_t b = w->ev_pool[ev_used++];
+        cudaEvent_t b = pool_event();
         CK(cudaEventRecord(b, w->stream));
         w->kev[cls].push_back({a, b});
     }
@@ -586,25 +596,25 @@ struct Exec {
     // an F or B op; the op then runs serialised on the worker's stream (no side stream, no graphs)
     cudaEvent_t lstart() {
         if (!c->layer_prof || capturing) return nullptr;
-        cudaEvent_t a = w->ev_pool[ev_used++];
+        cudaEvent_t a = pool_event();
         CK(cudaEventRecord(a, w->stream));
         return a;
     }
     void lend(int l, char dir, cudaEvent_t a) {
         if (!a) return;
-        cudaEvent_t b = w->ev_pool[ev_used++];
+        cudaEvent_t b = pool_event();
         CK(cudaEventRecord(b, w->stream));
         w->lev.push_back({l, dir, a, b});
     }
     void record_start() {
         if (!timing) return;
-        cudaEvent_t a = w->ev_pool[ev_used++];
+        cudaEvent_t a = pool_event();
         CK(cudaEventRecord(a, w->stream));
         w->op_ev.push_back({a, nullptr});
     }
     void record_end() {
         if (!timing) return;
-        cudaEvent_t b = w->ev_pool[ev_used++];
+        cudaEvent_t b = pool_event();
         CK(cudaEventRecord(b, w->stream));
         w->op_ev.back().second = b;
     }
@@ -701,9 +711,7 @@ struct Exec {
                                              (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz)
                                   : y_last;
             if (const int run = lstm_wave_run(l)) {
-                cudaEvent_t k0 = kstart(0);
                 lstm_wave_forward(l, run, t, j, slot, y_last);
-                kend(0, k0);
                 l += run - 1;
                 continue;
             }
@@ -733,7 +741,9 @@ struct Exec {
         }
         if (s + 1 == n()) {
             if (loss_dst == w->loss_scratch) CK(cudaMemsetAsync(loss_dst, 0, 4, w->stream));
+            cudaEvent_t k6 = kstart(6);
             CK(softmax_ce(w->logits, bf16, labels, lrows, layer(w->last).out, w->dlogits, loss_dst, w->stream));
+            kend(6, k6);
             lend(w->last, 'F', last_l0);
         }
         };
@@ -833,11 +843,15 @@ struct Exec {
             const bool adam = c->cfg.optimizer == PD_ADAM;
             g.epi = EPI_F32;
             g.out = w->gbuf + woff;
+            cudaEvent_t k0 = kstart(2);
             CK(run_gemm(bf16, g, w->stream));
+            kend(2, k0);
+            k0 = kstart(7);
             CK(update_from_grad(w->master + woff, static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], woff, esz)),
                                 w->gbuf + woff, (long)M * N, c->cfg.optimizer, adam ? w->adam_m + woff : nullptr,
                                 adam ? w->adam_v + woff : nullptr, c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps,
                                 w->updates_total + 1, w->stream));
+            kend(7, k0);
             return;
         }
         if (bc.fused) {
@@ -856,7 +870,9 @@ struct Exec {
             g.epi = EPI_F32;
             g.out = bc.gdst + woff;
         }
+        cudaEvent_t k0 = kstart(2);
         CK(run_gemm(bf16, g, w->stream));
+        kend(2, k0);
     }
 
     // bias gradient = column sums of G [rows][cols] (+ fused update)
@@ -902,10 +918,8 @@ struct Exec {
             gemm_dx(l, (int)rows, d.in, d.out, G, d.out, Wl(l, bc.sslot), d.in, x, dx);
             kend(1, k0);
         }
-        cudaEvent_t k0 = kstart(2);
         gemm_dw(bc, c->poff[l], d.out, d.in, (int)rows, G, d.out, x, d.in);
-        kend(2, k0);
-        k0 = kstart(3);
+        cudaEvent_t k0 = kstart(3);
         bias_update(bc, c->poff[l] + (long)d.out * d.in, G, rows, d.out);
         kend(3, k0);
     }
@@ -1097,7 +1111,10 @@ struct Exec {
             wd.b_hh[i] = param_f32(lstm_off(l, 3), slot);
             wd.gates[i] = st.gates, wd.c[i] = st.c, wd.h[i] = static_cast<__nv_bfloat16 *>(st.h);
         }
+        cudaEvent_t k0 = kstart(4);
         CK(lstm_wave(wd, w->stream));
+        kend(4, k0);
+        k0 = kstart(3);
         // each layer's output to the next layer's input stash (its backward reads it) / the
         // stage output
         for (int i = 0; i < L; ++i) {
@@ -1107,6 +1124,7 @@ struct Exec {
                                   : y_last;
             CK(cudaMemcpyAsync(y, lstm_state(l, j).h, (size_t)TB * H * esz, cudaMemcpyDeviceToDevice, w->stream));
         }
+        kend(3, k0);
     }
 
     void lstm_wave_backward(int l0, int L, int t, int j, const void *G, void *dx, const BwdCtx &bc) {
@@ -1130,19 +1148,19 @@ struct Exec {
             wd.da[i] = static_cast<__nv_bfloat16 *>(elem_ptr(w->lstm_wda, (long)i * TB * 4 * H, esz));
             wd.dc[i] = w->lstm_wdc + (long)i * Bn * H;
         }
-        cudaEvent_t k0 = kstart(1);
+        cudaEvent_t k0 = kstart(5);
         CK(lstm_wave(wd, w->stream));
+        kend(5, k0);
         // the bottom layer's input gradient (inner layers' are folded into the wavefront)
+        k0 = kstart(1);
         if (dx) gemm_dx(l0, (int)TB, H, 4 * H, wd.da[0], 4 * H, wd.W_ih[0], H, layer_input(l0, t, j), dx);
         kend(1, k0);
-        k0 = kstart(2);
         for (int i = L - 1; i >= 0; --i) {
             const int l = l0 + i;
             gemm_dw(bc, lstm_off(l, 0), 4 * H, H, (int)TB, wd.da[i], 4 * H, layer_input(l, t, j), H);
             gemm_dw(bc, lstm_off(l, 1), 4 * H, H, (int)((T - 1) * (long)Bn), elem_ptr(wd.da[i], (long)Bn * 4 * H, esz),
                     4 * H, lstm_state(l, j).h, H);
         }
-        kend(2, k0);
         k0 = kstart(3);
         for (int i = L - 1; i >= 0; --i) {
             bias_update_pair(bc, lstm_off(l0 + i, 2), lstm_off(l0 + i, 3), wd.da[i], TB, 4 * H);
@@ -1257,11 +1275,9 @@ struct Exec {
         });
         if (dx) gemm_dx(l, (int)TB, I, 4 * H, w->lstm_da, 4 * H, Wih, I, x, dx);
         kend(1, k0);
-        k0 = kstart(2);
         gemm_dw(bc, lstm_off(l, 0), 4 * H, I, (int)TB, w->lstm_da, 4 * H, x, I);
         gemm_dw(bc, lstm_off(l, 1), 4 * H, H, (int)((T - 1) * (long)Bn), elem_ptr(w->lstm_da, (long)Bn * 4 * H, esz),
                 4 * H, st.h, H);
-        kend(2, k0);
         k0 = kstart(3);
         bias_update_pair(bc, lstm_off(l, 2), lstm_off(l, 3), w->lstm_da, TB, 4 * H);
         kend(3, k0);
@@ -2556,7 +2572,7 @@ pd_status pd_get_stats(pd_ctx *c, pd_stats *out) {
         if (w->run_ev[0] && cudaEventElapsedTime(&run_ms, w->run_ev[0], w->run_ev[1]) == cudaSuccess)
             out->run_ms = std::max(out->run_ms, (double)run_ms);
         cudaGetLastError();
-        for (int cls = 0; cls < 4; ++cls)
+        for (int cls = 0; cls < PD_KERNEL_CLASSES; ++cls)
             for (auto &pr : w->kev[cls]) {
                 float ms = 0;
                 if (cudaEventElapsedTime(&ms, pr.first, pr.second) == cudaSuccess) {
@@ -2583,7 +2599,7 @@ pd_status pd_set_timing(pd_ctx *c, int record_trace, int mask) {
     CHECK_CTX(c);
     if (record_trace < 0 || record_trace > 2) return PD_EINVAL;
     c->cfg.record_trace = record_trace;
-    c->ktime_mask = mask & 0xF;
+    c->ktime_mask = mask & ((1 << PD_KERNEL_CLASSES) - 1);
     return PD_OK;
 }
 

@@ -96,7 +96,7 @@ class Pipeline:
     def stats(self):
         return pd_get_stats(self.ctx)
 
-    def set_timing(self, record_trace, kernel_timing_mask=0xF):
+    def set_timing(self, record_trace, kernel_timing_mask=0xFF):
         pd_set_timing(self.ctx, record_trace, kernel_timing_mask)
 
     def set_layer_profiling(self, on: bool):

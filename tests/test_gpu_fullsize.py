@@ -5,7 +5,13 @@ deltas (tests/golden/<case>.npz, written by tools/gen_golden_fullsize.py from or
 
 Tolerances: parameters within the north star's bf16 2e-2 (max relative error); the deltas
 (= -lr x gradient, where a version or indexing bug would show) within DELTA_TOL of the
-floored delta norm (R23, "bf16 tolerance"), and the first loss within 1e-2."""
+floored delta norm (R23, "bf16 tolerance"), and the first loss within 1e-2.
+DELTA_TOL: bf16 rounding alone (tools/bf16_emulate.py: torch fp64 with bf16 rounding where the
+CUDA path stores bf16) puts the first layer's gradient of these random-label problems 5.4 %
+(long-K W0) and 7.4 % (conv1 W) away from the exact one -- the gradient is a sum with heavy
+cancellation -- and the GPU lands on those floors to 3 digits (measured: 0.0539 / 0.0739);
+0.1 leaves room for accumulation order, not for a bug (a wrong version or index moves the
+delta by O(1))."""
 import os
 
 import numpy as np
@@ -19,7 +25,7 @@ from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline
 pytestmark = pytest.mark.gpu
 
 GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
-DELTA_TOL = 5e-2
+DELTA_TOL = 0.1
 
 
 @pytest.mark.parametrize("name", ["longk_dw", "vgg_conv1", "gnmt16_wave"])
