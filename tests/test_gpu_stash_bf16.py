@@ -31,8 +31,22 @@ def test_bf16_stash_discriminates(name):
     r = stash_cases.evaluate(name)
     print(r)
     assert r["trace_exact"], r
-    assert r["mutant_delta_err"] > 0.05, r  # the case makes stashing visible at all
+    assert r["mutant_l2"] > 0.04, r  # the case makes stashing visible at all
     assert stash_cases.discriminates(r), r
+
+
+def test_bf16_single_layer_first_stage():
+    """Stage 0 = one Linear layer: its overlapped backward has no dX, so only the fork event
+    orders the side stream's dW + update after the gradient arrives."""
+    import numpy as np
+    import paper_conf_sosp_narayananhpsdgg19_b200 as pd
+    from gpu_helpers import run_both, assert_schedule_exact, param_errors, BF16_TOL
+    wl, last, reps, M = stash_cases.case("mlp256_first1")
+    res = run_both(wl, last, reps, M, pd.PD_BF16, n_data=4)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < BF16_TOL, (perr, derr)
+    np.testing.assert_allclose(res["losses"], res["ref"].losses, rtol=2e-2)
 
 
 def _run_faulty(fault, name):
@@ -56,7 +70,10 @@ def test_fault_backward_reads_latest_version(name):
 def test_fault_side_stream_unordered(name):
     r = _run_faulty("fault_no_dxwait", name)
     print(r)
-    assert "error" in r or not r["discriminates"] or r["param_err"] > 2e-2, r
+    if name == "mlp256_first1":  # no stash effect at stage 0: the parity tolerance is the bar
+        assert "error" in r or r["param_err"] > 2e-2, r
+    else:
+        assert "error" in r or not r["discriminates"], r
 
 
 def test_fault_receive_ring_too_shallow():

@@ -46,6 +46,9 @@ def main(name, lrs, Ms, dtype):
             mut = oracle.run(wl.layers, last, reps, wl.batch, M, p0, synth.make_data(wl, 4), wl.optimizer, lr,
                              stash=False)
             print(json.dumps({"case": name, "lr": lr, "M": M, "dtype": dtype,
+                              "l2": {"gpu": stash_cases.rel_l2(res["got"], ref.params, p0),
+                                     "nost": stash_cases.rel_l2(res["got"], mut.params, p0),
+                                     "mut": stash_cases.rel_l2(mut.params, ref.params, p0)},
                               "gpu": per_tensor(res["got"], ref.params, p0),
                               "nost": per_tensor(res["got"], mut.params, p0),
                               "mut": per_tensor(mut.params, ref.params, p0)}), flush=True)
