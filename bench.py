@@ -410,7 +410,10 @@ def stage_table(args, wl, peaks, n_plan, only=-1):
             continue
         R = plan.stages[s][2]
         M_solo = 8 * R
-        r = solo_stage(plan, s, layers, wl, p0, data, n_data, M_solo)
+        quick = getattr(args, "solo_runs", 3) <= 1
+        r = solo_stage(plan, s, layers, wl, p0, data, n_data, M_solo, runs=max(1, getattr(args, "solo_runs", 3)),
+                       warm=1 if quick else 2, profile=not quick)
+        r.setdefault("class_ms_per_minibatch", {})
         r["gflop_per_minibatch"] = sum(layer_flops(layers[l], B) * (2.0 / 3.0 if l == 0 else 1.0)
                                        for l in range(plan.stages[s][0], plan.stages[s][1] + 1)) / 1e9
         r["tflops"] = r["gflop_per_minibatch"] / r["ms_per_minibatch"]
@@ -445,6 +448,8 @@ def main():
                          "alone on this GPU, projected N-GPU throughput = B min_s R_s / t_s (L775-777); 0 = off")
     ap.add_argument("--stage", type=int, default=-1,
                     help="measure only this stage of the --stage-plan plan in solo mode (for ncu) and exit")
+    ap.add_argument("--solo-runs", type=int, default=3,
+                    help="timed runs per stage in solo mode (1 = one warm-up + one run, no profile pass: for ncu)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-batch", type=int, default=0,
                     help="samples in the oracle's bounded sample (default: 8 for mlp4096, 1 otherwise -- ~10-60 s)")

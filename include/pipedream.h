@@ -258,7 +258,7 @@ typedef struct {
     double device_ms;             /* device span of the last run over the local workers    */
     double bubble;                /* 1 - sum(busy) / (local workers * span)  (record_trace 2) */
     uint64_t kernel_launches;     /* kernels this library launched during the last pd_run  */
-    uint64_t bytes_sent;          /* activation + gradient bytes written to other workers  */
+    uint64_t bytes_sent;          /* last pd_run: activation + gradient bytes written to other workers */
     int num_local_workers;
     int worker_id[PD_MAX_LOCAL_WORKERS];
     double busy_ms[PD_MAX_LOCAL_WORKERS];  /* sum of F/B op device durations per worker    */
@@ -272,6 +272,11 @@ typedef struct {
                                      4 LSTM wavefront forward, 5 LSTM wavefront backward,
                                      6 softmax-CE, 7 separate optimizer update pass        */
     uint64_t kern_count[PD_KERNEL_CLASSES]; /* launches timed per class                      */
+    uint64_t replica_bytes;       /* last pd_run, local workers: peer bytes of the sharded replica
+                                     sync -- per round and replica (R-1)/R of the parameters'
+                                     fp32 gradients read from the peers, and this replica's 1/R
+                                     shard of the new version (fp32 [+ bf16]) stored into each
+                                     of the R-1 peers                                        */
 } pd_stats;
 
 PD_API pd_status pd_get_stats(pd_ctx *ctx, pd_stats *out);

@@ -82,7 +82,8 @@ class Stats(C.Structure):
                 ("kernel_launches", C.c_uint64), ("bytes_sent", C.c_uint64), ("num_local_workers", C.c_int),
                 ("worker_id", C.c_int * PD_MAX_LOCAL_WORKERS), ("busy_ms", C.c_double * PD_MAX_LOCAL_WORKERS),
                 ("span_ms", C.c_double * PD_MAX_LOCAL_WORKERS), ("run_ms", C.c_double),
-                ("kern_ms", C.c_double * PD_KERNEL_CLASSES), ("kern_count", C.c_uint64 * PD_KERNEL_CLASSES)]
+                ("kern_ms", C.c_double * PD_KERNEL_CLASSES), ("kern_count", C.c_uint64 * PD_KERNEL_CLASSES),
+                ("replica_bytes", C.c_uint64)]
 
 
 class LstmRecDesc(C.Structure):
@@ -335,7 +336,8 @@ def pd_get_stats(ctx) -> dict:
     return {"host_ms": s.host_ms, "device_ms": s.device_ms, "bubble": s.bubble,
             "kernel_launches": int(s.kernel_launches), "bytes_sent": int(s.bytes_sent), "num_local_workers": n,
             "worker_id": list(s.worker_id[:n]), "busy_ms": list(s.busy_ms[:n]), "span_ms": list(s.span_ms[:n]),
-            "run_ms": s.run_ms, "kern_ms": list(s.kern_ms), "kern_count": [int(x) for x in s.kern_count]}
+            "run_ms": s.run_ms, "kern_ms": list(s.kern_ms), "kern_count": [int(x) for x in s.kern_count],
+            "replica_bytes": int(s.replica_bytes)}
 
 
 def pd_set_timing(ctx, record_trace: int, kernel_timing_mask: int = 0xFF):

@@ -64,31 +64,11 @@ struct EpiArgs {
     int ksplit;         // K is cut into ksplit contiguous ranges; work unit = (tile, split)
     ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
     int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
-    int l2_prefetch;    // producer L2-prefetch distance in K-blocks (0 = off; measured no gain so far)
-    int dbg;                    // tools only (PD_EPI_DEBUG): bit 5 = old per-row epilogue
-    // cluster split-K (csplit > 1): the csplit K-ranges of one output tile run as one thread-block
-    // cluster (CG * csplit CTAs); partial accumulators are summed through distributed shared
-    // memory (each CTA reduces a 64-column slice, in split order) and the final bf16 epilogue is
-    // applied in the same kernel -- no fp32 partials in HBM, no second launch
-    int csplit;
     unsigned long long *probe;  // tools only (PD_GEMM_PROBE): per-CTA %globaltimer phase stamps [grid][8]
-    // in-kernel split-K: each (tile, split) writes its fp32 partial to ws[split]; the last CTA
-    // to finish a tile (per-tile counter) sums the partials in split order and applies the
-    // final epilogue (final_epi = EPI_STORE or EPI_MASK) -- no separate reduction launch
-    void *ws;               // final output (bf16) when reducing in-kernel
-    long split_stride_out;  // its row stride
-    int *counters;
-    int final_epi;
-    // distributed in-kernel split-K (with counters): every split CTA of a tile, once all S
-    // partials are in L2, sums 1/S of the tile's columns and applies the final epilogue
-    // (needs all of a launch's CTAs co-resident: one unit per CTA, one such GEMM per GPU)
-    int dist;
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
     long ldm;
-    const void *l2_next;  // L2 prefetch of the next layer's operand (warp 3), nullptr = off
-    long l2_next_bytes;
     float *master;
     __nv_bfloat16 *slot;
     float *adam_m, *adam_v;
@@ -320,8 +300,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) PROBE(0);
-    uint32_t crank = 0;  // rank in the cluster (pair, or pair x cluster split)
-    if (CG == 2 || e.csplit > 1) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
+    uint32_t crank = 0;  // rank in the CTA pair's cluster
+    if (CG == 2) asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(crank));
     const uint32_t rank = CG == 2 ? (crank & 1u) : 0u;                  // rank in the CTA pair
     const uint16_t pmask = (uint16_t)(3u << (crank & ~1u));              // the pair's CTAs
     const int pair = blockIdx.x / CG, npairs = gridDim.x / CG;
@@ -330,11 +310,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int kblocks = (K + BK - 1) / BK;
     const int units = tiles * e.ksplit;
     const int kper = (kblocks + e.ksplit - 1) / e.ksplit;
-    // persistent loop over units (tile, split); cluster split-K: exactly one unit per CTA
-    const int csplit = e.csplit > 1 ? e.csplit : 1;
-    const int my_split = (int)(crank / CG) % csplit;
-    const int u0 = csplit > 1 ? my_split * tiles + (int)(blockIdx.x / (CG * csplit)) : pair;
-    const int ustep = csplit > 1 ? units : npairs;
+    // persistent loop over units (tile, split)
+    const int u0 = pair, ustep = npairs;
     constexpr uint32_t TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
 
     if (warp == 0 && lane == 0) {
@@ -387,30 +364,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const uint32_t tmem_base = *tmem_slot;
     if (threadIdx.x == 0) PROBE(1);
 
-    if (warp == 3 && lane == 0 && e.l2_next) {
-        // next layer's weights -> L2 while this GEMM streams its own: this CTA's contiguous
-        // share, 32 KB bulk prefetches (no smem, no completion to wait for)
-        const long share = ((e.l2_next_bytes + gridDim.x - 1) / gridDim.x + 15) & ~15L;
-        const long b0 = (long)blockIdx.x * share, b1 = min(e.l2_next_bytes, b0 + share);
-        for (long off = b0; off < b1; off += 32768) {
-            const uint32_t sz = (uint32_t)min(32768L, b1 - off) & ~15u;
-            if (sz)
-                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(
-                                 static_cast<const char *>(e.l2_next) + off),
-                             "r"(sz)
-                             : "memory");
-        }
-    }
-    // programmatic dependent launch: let the next kernel of the stream get scheduled now (its
-    // own wait holds it until this grid completes); everything above touched only on-chip state
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (warp == 0) {
         // ===== TMA producer =====
         if (lane == 0) {
-            // the previous kernel's outputs (operands, and the buffers this GEMM overwrites) are
-            // complete and visible from here on; every other role's global access is ordered
-            // after this thread's loads (mbarriers).  A no-op without the PDL launch attribute
-            asm volatile("griddepcontrol.wait;" ::: "memory");
             int stage = 0;
             uint32_t phase = 0;
             for (int unit = u0; unit < units; unit += ustep) {
@@ -431,20 +387,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     }
                     kbk += e.conv.b_kshift;
                 };
-                auto prefetch = [&](int kb) {
-                    int ka, ma, kbk, nb;
-                    coords(kb, ka, ma, kbk, nb);
-                    if (AMAJ == KMAJ) tma_prefetch_2d(&tmA, ka, ma);
-                    else
-                        for (int j = 0; j < BM / 64; ++j) tma_prefetch_2d(&tmA, ma + 64 * j, ka);
-                    if (BMAJ == KMAJ) tma_prefetch_2d(&tmB, kbk, nb);
-                    else
-                        for (int j = 0; j < BNC / 64; ++j) tma_prefetch_2d(&tmB, nb + 64 * j, kbk);
-                };
-                const int PF = e.l2_prefetch;  // L2 prefetch distance in K-blocks (0 = off)
-                for (int kb = kb0; kb < min(kb1, kb0 + PF); ++kb) prefetch(kb);
                 for (int kb = kb0; kb < kb1; ++kb) {
-                    if (PF && kb + PF < kb1) prefetch(kb + PF);
                     mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
                     if (kb == kb0 && unit == u0) PROBE(2);
                     // CG = 2: both CTAs' bytes land on the LEADER's full barrier (peer bit cleared)
@@ -580,25 +523,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             EpiArgs es = e;
             if (EPI == EPI_F32) es.out = static_cast<float *>(e.out) + (long)split * e.split_stride;
             const bool empty_range = split * kper >= kblocks;  // (host avoids it; be safe)
-            const bool reduce = EPI == EPI_F32 && e.counters != nullptr;  // in-kernel split-K
-            if (csplit > 1) {
-                // ---- cluster split-K: this split's partial accumulator -> own shared memory
-                // (the operand ring is idle now), row-major [128][BN + 4] fp32
-                const uint32_t pbase = smem_u32(smem) + (uint32_t)((q * 32 + lane) * (BN + 4) * 4);
-#pragma unroll 1
-                for (int c = 0; c < BN / 32; ++c) {
-                    float v[32];
-                    tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, v);
-                    if (empty_range) {
-#pragma unroll
-                        for (int i = 0; i < 32; ++i) v[i] = 0.f;
-                    }
-#pragma unroll
-                    for (int j = 0; j < 8; ++j)
-                        st_shared_v4(pbase + (uint32_t)((c * 32 + 4 * j) * 4), v[4 * j], v[4 * j + 1], v[4 * j + 2],
-                                     v[4 * j + 3]);
-                }
-            } else if ((EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) && !(e.dbg & 32)) {
+            if (EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) {
                 // ---- TMA-store epilogue: rows m0+32q.., one 32 x 32 chunk at a time
                 uint8_t *wst = epi_stg + q * C::WARP_STG;
                 const int r0 = m0 + q * 32;
@@ -653,7 +578,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     ++ocnt;
                     if (warp == 4 && lane == 0 && c < 2) PROBE(9 + c);
                 }
-                if (reduce && lane == 0) bulk_wait0();  // partials visible before the split counter
             } else {
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
@@ -675,183 +599,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 else mbar_arrive_cluster(smem_u32(&tempty[acc]) & 0xFEFFFFFFu);  // the leader's barrier
             }
             if (++acc == 2) { acc = 0; acc_phase ^= 1; }
-            if (reduce && e.dist) {
-                // publish this partial, wait for the tile's other splits, then reduce this split's
-                // share of the columns (32-column groups [g0, g1) of BN / 32) over all S partials
-                __threadfence();
-                asm volatile("bar.sync 1, 128;" ::: "memory");
-                const int cidx = tile * CG + (int)rank;
-                if (warp == 4 && lane == 0) {
-                    atomicAdd(e.counters + cidx, 1);
-                    unsigned v;
-                    do {
-                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(e.counters + cidx) : "memory");
-                    } while ((int)v < e.ksplit);
-                }
-                asm volatile("bar.sync 1, 128;" ::: "memory");
-                __threadfence();
-                const int ngr = BN / 32, g0 = split * ngr / e.ksplit, g1 = (split + 1) * ngr / e.ksplit;
-                const int nf4 = (g1 - g0) * 8;  // float4 per row of this share
-                const int et = (int)threadIdx.x - 128;
-                const float *part = static_cast<const float *>(e.out);
-                __nv_bfloat16 *dst = static_cast<__nv_bfloat16 *>(e.ws);
-#pragma unroll 2
-                for (int it = et; it < BM * nf4; it += 128) {
-                    const int r = it / nf4, f = it % nf4;
-                    const int grow = m0 + r, col = n0 + g0 * 32 + f * 4;
-                    if (grow >= M || col >= N) continue;
-                    const long off = (long)grow * e.ldo + col;
-                    float4 acc4 = __ldcg(reinterpret_cast<const float4 *>(part + off));
-                    for (int sp = 1; sp < e.ksplit; ++sp) {
-                        const float4 b4 = __ldcg(reinterpret_cast<const float4 *>(part + (long)sp * e.split_stride + off));
-                        acc4.x += b4.x; acc4.y += b4.y; acc4.z += b4.z; acc4.w += b4.w;
-                    }
-                    float v4[4] = {acc4.x, acc4.y, acc4.z, acc4.w};
-                    if (e.final_epi == EPI_STORE) {
-                        if (e.bias) {
-                            const float4 bb = *reinterpret_cast<const float4 *>(e.bias + col);
-                            v4[0] += bb.x; v4[1] += bb.y; v4[2] += bb.z; v4[3] += bb.w;
-                        }
-                        if (e.relu)
-#pragma unroll
-                            for (int i = 0; i < 4; ++i) v4[i] = fmaxf(v4[i], 0.f);
-                    } else {
-                        const uint2 mr = *reinterpret_cast<const uint2 *>(e.mask + (long)grow * e.ldm + col);
-                        const __nv_bfloat16 *mh = reinterpret_cast<const __nv_bfloat16 *>(&mr);
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) v4[i] = __bfloat162float(mh[i]) > 0.f ? v4[i] : 0.f;
-                    }
-                    uint2 o;
-                    o.x = pack_bf16(v4[0], v4[1]);
-                    o.y = pack_bf16(v4[2], v4[3]);
-                    *reinterpret_cast<uint2 *>(dst + (long)grow * e.split_stride_out + col) = o;
-                }
-                // the last split done reading resets both counters for the next launch
-                asm volatile("bar.sync 1, 128;" ::: "memory");
-                if (warp == 4 && lane == 0) {
-                    const int old = atomicAdd(e.counters + 4096 + cidx, 1);
-                    if (old == e.ksplit - 1) {
-                        e.counters[cidx] = 0;
-                        e.counters[4096 + cidx] = 0;
-                    }
-                }
-            } else if (reduce) {
-                // publish this partial; the tile's last arriving split reduces all of them
-                __threadfence();
-                asm volatile("bar.sync 1, 128;" ::: "memory");
-                __shared__ int s_last;
-                const int cidx = tile * CG + (int)rank;
-                if (warp == 4 && lane == 0) {
-                    const int old = atomicAdd(e.counters + cidx, 1);
-                    s_last = (old == e.ksplit - 1);
-                    if (s_last) e.counters[cidx] = 0;  // ready for the next launch (stream order)
-                }
-                asm volatile("bar.sync 1, 128;" ::: "memory");
-                if (s_last) {
-                    __threadfence();
-                    EpiArgs ef = e;
-                    for (int c = 0; c < BN / 32; ++c) {
-                        const int col = n0 + c * 32;
-                        if (col >= N || row >= M) continue;
-                        float v[32];
-                        const float *p0 = static_cast<const float *>(e.out) + (long)row * e.ldo + col;
-                        const bool fullc = col + 32 <= N;
-                        for (int sp = 0; sp < e.ksplit; ++sp) {
-                            const float *p = p0 + (long)sp * e.split_stride;
-                            if (fullc) {
-#pragma unroll
-                                for (int q4 = 0; q4 < 8; ++q4) {
-                                    const float4 f = __ldcg(reinterpret_cast<const float4 *>(p) + q4);
-                                    if (sp == 0) {
-                                        v[q4 * 4] = f.x; v[q4 * 4 + 1] = f.y; v[q4 * 4 + 2] = f.z; v[q4 * 4 + 3] = f.w;
-                                    } else {
-                                        v[q4 * 4] += f.x; v[q4 * 4 + 1] += f.y; v[q4 * 4 + 2] += f.z; v[q4 * 4 + 3] += f.w;
-                                    }
-                                }
-                            } else {
-                                for (int i = 0; i < 32; ++i) {
-                                    const float f = (col + i < N) ? __ldcg(p + i) : 0.f;
-                                    v[i] = sp == 0 ? f : v[i] + f;
-                                }
-                            }
-                        }
-                        ef.out = e.ws;  // the final bf16 output
-                        ef.ldo = e.split_stride_out;
-                        if (e.final_epi == EPI_MASK) epilogue_chunk<EPI_MASK>(ef, v, row, col, M, N);
-                        else epilogue_chunk<EPI_STORE>(ef, v, row, col, M, N);
-                    }
-                }
-            }
         }
         if (EPI == EPI_STORE || EPI == EPI_MASK || EPI == EPI_F32) {
             if (lane == 0) bulk_wait0();  // every bulk store complete before the CTA retires
         }
         if (warp == 4 && lane == 0) PROBE(6);
-    }
-    if (csplit > 1) {
-        // ---- cluster split-K reduction: every split's partial is in its CTA's shared memory;
-        // split s sums columns [64 s, 64 s + 64) of its pair-rank's 128 rows over all splits
-        // (in split order: deterministic), applies the epilogue and stores that bf16 slice
-        cluster_sync_all();
-        if ((EPI == EPI_STORE || EPI == EPI_MASK) && warp >= 4) {
-            const int t = threadIdx.x - 128;
-            const int tile = blockIdx.x / (CG * csplit);
-            const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM, n0 = (tile / m_blocks) * BN;
-            // this split's columns: 32-column chunks [ch0, ch1) of the BN-wide tile
-            const int nb = BN / 32, ch0 = my_split * nb / csplit, ch1 = (my_split + 1) * nb / csplit;
-            const int c_lo = ch0 * 32, groups = (ch1 - ch0) * 4;  // 8-column groups
-            const uint32_t part = smem_u32(smem), ost = smem_u32(epi_stg);
-#pragma unroll 1
-            for (int item = t; item < 128 * groups; item += 128) {
-                const int r = item / groups, g = item % groups, col = c_lo + g * 8;
-                float x[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-                const uint32_t la = part + (uint32_t)((r * (BN + 4) + col) * 4);
-                for (int sp = 0; sp < csplit; ++sp) {
-                    const uint32_t ra = mapa_cluster(la, (uint32_t)(sp * CG) + rank);
-                    const float4 a = ld_dsmem_v4(ra), b = ld_dsmem_v4(ra + 16);
-                    x[0] += a.x; x[1] += a.y; x[2] += a.z; x[3] += a.w;
-                    x[4] += b.x; x[5] += b.y; x[6] += b.z; x[7] += b.w;
-                }
-                const int grow = m0 + r, gcol = n0 + col;
-                if constexpr (EPI == EPI_STORE) {
-                    if (e.bias) {
-#pragma unroll
-                        for (int j = 0; j < 8; ++j) x[j] += (gcol + j < N) ? __ldg(e.bias + gcol + j) : 0.f;
-                    }
-                    if (e.relu) {
-#pragma unroll
-                        for (int j = 0; j < 8; ++j) x[j] = fmaxf(x[j], 0.f);
-                    }
-                } else if constexpr (EPI == EPI_MASK) {
-                    if (grow < M && gcol + 8 <= N) {
-                        const uint4 raw = __ldg(reinterpret_cast<const uint4 *>(e.mask + (long)grow * e.ldm + gcol));
-                        const __nv_bfloat16 *h = reinterpret_cast<const __nv_bfloat16 *>(&raw);
-#pragma unroll
-                        for (int j = 0; j < 8; ++j) x[j] = (__bfloat162float(h[j]) > 0.f) ? x[j] : 0.f;
-                    } else {
-                        for (int j = 0; j < 8; ++j)
-                            x[j] = (grow < M && gcol + j < N && __bfloat162float(e.mask[(long)grow * e.ldm + gcol + j]) > 0.f)
-                                       ? x[j] : 0.f;
-                    }
-                }
-                uint4 w;
-                w.x = pack_bf16(x[0], x[1]);
-                w.y = pack_bf16(x[2], x[3]);
-                w.z = pack_bf16(x[4], x[5]);
-                w.w = pack_bf16(x[6], x[7]);
-                // staging: one 64B-swizzled [128 rows][32 cols] bf16 box per 32-column chunk
-                const int cb = g >> 2, j = g & 3;
-                st_shared_v4u(ost + (uint32_t)(cb * 8192 + r * 64 + ((j ^ ((r >> 1) & 3)) << 4)), w);
-            }
-            fence_proxy_async();
-            asm volatile("bar.sync 1, 128;" ::: "memory");
-            if (t == 0) {
-                for (int cb = 0; cb < ch1 - ch0; ++cb) tma_store_2d(&tmO, ost + cb * 8192, n0 + c_lo + 32 * cb, m0);
-                bulk_commit();
-                bulk_wait0();
-            }
-        }
-        cluster_sync_all();  // no CTA leaves while a peer may still read its partial
     }
     tc_fence_before();
     if (CG == 2) {
@@ -1212,17 +964,6 @@ bool encode_map(CUtensorMap *map, const void *base, long inner, long outer, long
     return r == CUDA_SUCCESS;
 }
 
-// PD_PDL=1: GEMMs and split-K reductions that the caller marks (Gemm::pdl) launch with
-// programmatic stream serialization, so a kernel's launch and prologue overlap its predecessor's
-// tail (griddepcontrol.wait in the kernels holds every dependent access)
-bool g_pdl_enabled() {
-    static const int v = [] {
-        const char *e = getenv("PD_PDL");
-        return e ? atoi(e) : 0;
-    }();
-    return v != 0;
-}
-
 int num_sms() {
     static int n = 0;
     if (!n) {
@@ -1273,10 +1014,6 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
     using C = Cfg<BN / CG, EPI>;
     EpiArgs e = e0;
     e.probe = probe_buf();
-    {
-        static const int dbg = getenv("PD_EPI_DEBUG") ? atoi(getenv("PD_EPI_DEBUG")) : 0;
-        e.dbg = dbg;
-    }
     auto kern = tc_gemm_kernel<BN, AMAJ, BMAJ, EPI, CG>;
     static bool attr_set = false;  // per instantiation; benign race (idempotent)
     if (!attr_set) {
@@ -1287,11 +1024,7 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
     // epilogue tensor maps: output tile {32 cols, 32 rows} (bf16 64B-swizzled / fp32 128B-swizzled;
     // split-K partials stacked as [S*M][N]) and the ReLU-mask tile
     CUtensorMap mo = ma, mk = ma;
-    if (e.csplit > 1) {
-        // cluster split-K: each CTA stores a [128 rows][64 cols] bf16 slice
-        if (!(EPI == EPI_STORE || EPI == EPI_MASK) || !make_map(&mo, e.out, g.N, g.M, e.ldo, 32, 128, false, 64))
-            return cudaErrorInvalidValue;
-    } else if (EPI == EPI_STORE || EPI == EPI_MASK) {
+    if (EPI == EPI_STORE || EPI == EPI_MASK) {
         if (!make_map(&mo, e.out, g.N, g.M, e.ldo, 32, 32, false, 64)) return cudaErrorInvalidValue;
         if (EPI == EPI_MASK && !make_map(&mk, e.mask, g.N, g.M, e.ldm, 32, 32, false, 64))
             return cudaErrorInvalidValue;
@@ -1306,10 +1039,9 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
     }
     const int units = ((g.M + BM * CG - 1) / (BM * CG)) * ((g.N + BN - 1) / BN) * e.ksplit;
     const int slots = num_sms() / CG;
-    const int grid = e.csplit > 1 ? CG * units : CG * (units < slots ? units : slots);
-    const int cluster = e.csplit > 1 ? CG * e.csplit : CG;
-    const bool pdl = g_pdl_enabled() && g.pdl;
-    if (cluster == 1 && !pdl) {
+    const int grid = CG * (units < slots ? units : slots);
+    const int cluster = CG;
+    if (cluster == 1) {
         kern<<<grid, NUM_THREADS, C::SMEM, s>>>(ma, mb, mo, mk, e, g.M, g.N, g.K);
     } else {
         cudaLaunchConfig_t cfg{};
@@ -1317,22 +1049,13 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         cfg.blockDim = dim3(NUM_THREADS);
         cfg.dynamicSmemBytes = C::SMEM;
         cfg.stream = s;
-        cudaLaunchAttribute attr[2];
-        int na = 0;
-        if (cluster > 1) {
-            attr[na].id = cudaLaunchAttributeClusterDimension;
-            attr[na].val.clusterDim.x = cluster;
-            attr[na].val.clusterDim.y = 1;
-            attr[na].val.clusterDim.z = 1;
-            ++na;
-        }
-        if (pdl) {
-            attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-            attr[na].val.programmaticStreamSerializationAllowed = 1;
-            ++na;
-        }
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = cluster;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
         cfg.attrs = attr;
-        cfg.numAttrs = na;
+        cfg.numAttrs = 1;
         cudaError_t err = cudaLaunchKernelEx(&cfg, kern, ma, mb, mo, mk, e, g.M, g.N, g.K);
         if (err != cudaSuccess) return err;
     }
@@ -1405,7 +1128,7 @@ cudaError_t gemm_bf16_update(const Gemm &g, cudaStream_t s) {
     // tile width: the update streams master (+ Adam m, v) per output element, the GEMM streams
     // (128 + BN) x 64 operand elements per K-block into the SM; wider tiles raise the FLOPs per
     // ingested byte (the per-SM TMA ingest, ~60 GB/s, bounds these tiles -- tools/tma_bw.cu)
-    static const int bn_adam = getenv("PD_UPD_BN_ADAM") ? atoi(getenv("PD_UPD_BN_ADAM")) : 128;
+    constexpr int bn_adam = 128;
     const char *bs = getenv("PD_UPD_BN_SGD");  // read per call (tests toggle it)
     const int bn_sgd = bs && atoi(bs) == 256 ? 256 : 128;
     const int BN = adam ? bn_adam : bn_sgd;
@@ -1434,8 +1157,6 @@ __global__ void splitk_epilogue_kernel(const float *ws, int S, long split_stride
                                        const float *__restrict__ bias, int relu, const __nv_bfloat16 *__restrict__ mask,
                                        long ldm, __nv_bfloat16 *__restrict__ out, long ldo,
                                        float *__restrict__ zero_ws) {
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    asm volatile("griddepcontrol.wait;" ::: "memory");  // the GEMM's partials (no-op without PDL)
     const long n4 = N / 4;
     const long total = (long)M * n4;
     for (long i = (long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long)gridDim.x * blockDim.x) {
@@ -1489,44 +1210,6 @@ static int use_pairs(const Gemm &g) {
     if (env_int("PD_GEMM_CG", 2) == 1) return 1;
     // N <= 64 would leave the second CTA's half of B empty (zero columns): single CTAs there
     return (g.M >= 256 && g.N > 64 && (g.epi == EPI_STORE || g.epi == EPI_MASK || g.epi == EPI_F32)) ? 2 : 1;
-}
-
-// thread-block clusters of `csize` CTAs that can be resident at once (GPC-limited: 15 of 8
-// CTAs on a 148-SM B200), for the ~1-CTA-per-SM GEMM kernels; cached per (CG, size)
-static int max_active_clusters(int cg, int csize) {
-    static int cache[3][9] = {};
-    if (csize < 1 || csize > 8) return 0;
-    int &c = cache[cg][csize];
-    if (c) return c;
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = dim3(csize * 64);
-    cfg.blockDim = dim3(NUM_THREADS);
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = csize;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    int n = 0;
-    cudaError_t err;
-    if (cg == 2) {
-        auto k = tc_gemm_kernel<256, KMAJ, KMAJ, EPI_STORE, 2>;
-        cfg.dynamicSmemBytes = Cfg<128, EPI_STORE>::SMEM;
-        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cfg.dynamicSmemBytes);
-        err = cudaOccupancyMaxActiveClusters(&n, k, &cfg);
-    } else {
-        auto k = tc_gemm_kernel<256, KMAJ, KMAJ, EPI_STORE, 1>;
-        cfg.dynamicSmemBytes = Cfg<256, EPI_STORE>::SMEM;
-        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cfg.dynamicSmemBytes);
-        err = cudaOccupancyMaxActiveClusters(&n, k, &cfg);
-    }
-    if (err != cudaSuccess) {
-        cudaGetLastError();
-        n = 0;
-    }
-    c = n > 0 ? n : -1;
-    return c;
 }
 
 static int choose_ksplit(const Gemm &g, int sms) {
@@ -1589,45 +1272,6 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaErrorInvalidValue;
     {
         const int S = choose_ksplit(g, num_sms());
-        const int cg0 = use_pairs(g);
-        const long ctiles = (long)((g.M + BM * cg0 - 1) / (BM * cg0)) * ((g.N + 255) / 256);
-        int CS = 0;  // cluster split count: the largest of 4, 3, 2 whose clusters all fit in one wave
-        const int csenv = env_int("PD_GEMM_CSPLIT", 1);
-        // bit 0: forward (EPI_STORE) GEMMs, bit 1: dX (EPI_MASK) GEMMs.  Clusters need CG*CS free SMs
-        // in one GPC at launch: the dX GEMMs overlap the side stream's dW kernels, which keep SMs
-        // busy; measured in the MLP step: forward only -6 %, both -13 % -> off by default (kept for
-        // standalone GEMMs: PD_GEMM_CSPLIT_EPI=3)
-        const int csepi = env_int("PD_GEMM_CSPLIT_EPI", 0);
-        const bool epi_ok = (g.epi == EPI_STORE && (csepi & 1)) || (g.epi == EPI_MASK && (csepi & 2));
-        if (S >= 3 && csenv && epi_ok && g.N % 8 == 0)
-            for (int cs = csenv > 1 ? csenv : 4; cs >= 2 && !CS; --cs)
-                if ((g.K + BK - 1) / BK >= cs && ctiles <= max_active_clusters(cg0, cg0 * cs)) CS = cs;
-        if (getenv("PD_GEMM_CSPLIT_DEBUG"))
-            fprintf(stderr, "csplit: tiles %ld S %d maxclusters(%d)=%d (%d)=%d (%d)=%d -> CS %d\n", ctiles, S, cg0 * 4,
-                    max_active_clusters(cg0, cg0 * 4), cg0 * 3, max_active_clusters(cg0, cg0 * 3), cg0 * 2,
-                    max_active_clusters(cg0, cg0 * 2), CS);
-        if (CS) {
-            // cluster split-K: CS K-ranges of a 256-wide tile reduced through DSMEM, one launch
-            CUtensorMap ma, mbm;
-            const int cg = cg0;
-            const bool okA = g.amaj == KMAJ ? make_map(&ma, g.A, g.K, g.M, g.lda, 64, BM)
-                                            : make_map(&ma, g.A, g.M, g.K, g.lda, 64, BK);
-            const bool okB = g.bmaj == KMAJ ? make_map(&mbm, g.B, g.K, g.N, g.ldb, 64, 256 / cg)
-                                            : make_map(&mbm, g.B, g.N, g.K, g.ldb, 64, BK);
-            if (!okA || !okB) return cudaErrorInvalidValue;
-            EpiArgs e{};
-            e.out = g.out;
-            e.ldo = g.ldo;
-            e.ksplit = CS;
-            e.csplit = CS;
-            e.l2_next = g.l2_next;
-            e.l2_next_bytes = g.l2_next_bytes;
-            e.bias = g.epi == EPI_STORE ? g.bias : nullptr;
-            e.relu = g.epi == EPI_STORE ? g.relu : 0;
-            e.mask = g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr;
-            e.ldm = g.ldm;
-            return cg == 2 ? dispatch_major<256, 2>(g, ma, mbm, e, s) : dispatch_major<256>(g, ma, mbm, e, s);
-        }
         if (S > 1) {
             CUtensorMap ma, mbm;
             const int cg = use_pairs(g);
@@ -1642,27 +1286,10 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             e.ldo = g.N;
             e.ksplit = S;
             e.split_stride = (long)g.M * g.N;
-            e.l2_next = g.l2_next;
-            e.l2_next_bytes = g.l2_next_bytes;
-            // in-kernel reduction: PD_SPLIT_INKERNEL=1 last CTA of a tile sums the S partials;
-            // =2 (needs Gemm::split_dist: the caller's guarantee that no other co-residency-
-            // dependent kernel shares the GPU) every split sums 1/S of the columns
-            const int ik_mode = env_int("PD_SPLIT_INKERNEL", 0);
-            const bool inkernel = g.split_counters != nullptr && (ik_mode == 1 || (ik_mode == 2 && g.split_dist));
-            if (inkernel) {
-                e.dist = ik_mode == 2;
-                e.counters = g.split_counters;
-                e.ws = g.out;
-                e.split_stride_out = g.ldo;
-                e.final_epi = g.epi;
-                e.bias = g.epi == EPI_STORE ? g.bias : nullptr;
-                e.relu = g.epi == EPI_STORE ? g.relu : 0;
-                e.mask = g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr;
-                e.ldm = g.ldm;
-            }
-            // zeroed workspace: every split reduce-adds (TMA, in L2) into one fp32 partial set, the
-            // reduction kernel reads M*N instead of S*M*N floats and re-zeroes them
-            const bool atomic = g.ws_zeroed && !inkernel;
+            // zeroed workspace (kernel ABI workspace_zeroed): every split reduce-adds (TMA, in L2)
+            // into one fp32 partial set, the reduction kernel reads M*N instead of S*M*N floats
+            // and re-zeroes them
+            const bool atomic = g.ws_zeroed;
             if (atomic) {
                 e.atomic_out = 1;
                 e.split_stride = 0;
@@ -1670,25 +1297,17 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
             Gemm gf = g;
             gf.epi = EPI_F32;
             cudaError_t err = cg == 2 ? dispatch_major<256, 2>(gf, ma, mbm, e, s) : dispatch_major<256>(gf, ma, mbm, e, s);
-            if (err != cudaSuccess || inkernel) return err;
+            if (err != cudaSuccess) return err;
             const long total = (long)g.M * (g.N / 4);
             long blocks = (total + 255) / 256;
             if (blocks > 148L * 8) blocks = 148L * 8;
-            cudaLaunchConfig_t cfg{};
-            cfg.gridDim = dim3((unsigned)blocks);
-            cfg.blockDim = dim3(256);
-            cfg.stream = s;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-            attr[0].val.programmaticStreamSerializationAllowed = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = (g_pdl_enabled() && g.pdl) ? 1 : 0;
             ++tl_launches;
-            return cudaLaunchKernelEx(&cfg, splitk_epilogue_kernel, (const float *)g.workspace, atomic ? 1 : S,
-                                      (long)g.M * g.N, g.M, g.N, g.epi == EPI_STORE ? g.bias : nullptr,
-                                      g.epi == EPI_STORE ? g.relu : 0,
-                                      g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr, g.ldm,
-                                      static_cast<__nv_bfloat16 *>(g.out), g.ldo, atomic ? g.workspace : nullptr);
+            splitk_epilogue_kernel<<<(unsigned)blocks, 256, 0, s>>>(
+                (const float *)g.workspace, atomic ? 1 : S, (long)g.M * g.N, g.M, g.N,
+                g.epi == EPI_STORE ? g.bias : nullptr, g.epi == EPI_STORE ? g.relu : 0,
+                g.epi == EPI_MASK ? static_cast<const __nv_bfloat16 *>(g.mask) : nullptr, g.ldm,
+                static_cast<__nv_bfloat16 *>(g.out), g.ldo, atomic ? g.workspace : nullptr);
+            return cudaGetLastError();
         }
     }
     if ((g.epi == EPI_SGD || g.epi == EPI_ADAM) && g.ldo == g.N && g.N % 8 == 0) return gemm_bf16_update(g, s);
@@ -1702,15 +1321,11 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     if (cg == 2) {
         // pair tiles of 256 rows; BN >= 128 so each CTA holds >= 64 B columns
         const long pm = (g.M + 255) / 256;
-        if (env_int("PD_GEMM_BNSEL", 1)) {
-            // operand bytes each CTA ingests per K-block (32 KB at BN 256, 24 KB at BN 128) x
-            // waves of pair tiles: the per-SM TMA ingest bounds these GEMMs (tools/tma_bw.cu)
-            const long slots = sms / 2, t256 = pm * ((g.N + 255) / 256), t128 = pm * ((g.N + 127) / 128);
-            const long c256 = (t256 + slots - 1) / slots * 32, c128 = (t128 + slots - 1) / slots * 24;
-            if (c128 < c256 || g.N <= 128) BN = 128;
-        } else if (pm * ((g.N + 255) / 256) < sms / 2 || g.N <= 128) {
-            BN = 128;
-        }
+        // operand bytes each CTA ingests per K-block (32 KB at BN 256, 24 KB at BN 128) x
+        // waves of pair tiles: the per-SM TMA ingest bounds these GEMMs (tools/tma_bw.cu)
+        const long slots = sms / 2, t256 = pm * ((g.N + 255) / 256), t128 = pm * ((g.N + 127) / 128);
+        const long c256 = (t256 + slots - 1) / slots * 32, c128 = (t128 + slots - 1) / slots * 24;
+        if (c128 < c256 || g.N <= 128) BN = 128;
     } else {
         if ((long)mb * ((g.N + 255) / 256) < sms || g.N <= 128) BN = 128;
         if (BN == 128 && ((long)mb * ((g.N + 127) / 128) < sms || g.N <= 64)) BN = 64;
@@ -1732,7 +1347,6 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     EpiArgs e{};
     e.conv = g.conv;
     e.atomic_out = g.atomic_out;
-    e.l2_prefetch = env_int("PD_GEMM_PF", 0);
     e.out = g.out;
     e.ldo = g.ldo;
     e.ksplit = g.ksplit > 1 ? g.ksplit : 1;
@@ -1751,8 +1365,6 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         e.ksplit = (kb + kper - 1) / kper;
     }
     e.split_stride = 0;
-    e.l2_next = g.l2_next;
-    e.l2_next_bytes = g.l2_next_bytes;
     e.bias = g.bias;
     e.relu = g.relu;
     e.mask = static_cast<const __nv_bfloat16 *>(g.mask);

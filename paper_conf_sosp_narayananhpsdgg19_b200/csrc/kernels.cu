@@ -593,6 +593,74 @@ cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f
     return cudaGetLastError();
 }
 
+// Replica sync of one round, sharded (reduce-scatter -> update -> all-gather through peer
+// memory): this replica owns parameters [lo, hi) (16-byte multiples).  For each of them it
+// sums the R replicas' fp32 gradients in replica order (R7) over NVLink peer loads, applies
+// the optimizer to its own weights w_in (fp32 master on the bf16 path, the latest fp32 slot
+// on the fp32 path) and Adam state, and stores the new version into EVERY replica: fp32 into
+// out_f32[q] (masters / fp32 slots), bf16 into out_bf16[q] (bf16 slots).  Per replica and
+// round: (R-1)/R * 4 B/param of peer reads, (R-1)/R * (4 [+ 2]) B/param of peer stores,
+// instead of (R-1) * 4 B/param of reads and a redundant full update on every replica.
+template <bool ADAM>
+__global__ void __launch_bounds__(256) update_shard_kernel(const float *const *__restrict__ grads, int R, long lo,
+                                                           long n4, const float *w_in, float *const *__restrict__ out_f32,
+                                                           __nv_bfloat16 *const *__restrict__ out_bf16,
+                                                           float *__restrict__ m, float *__restrict__ v, float lr,
+                                                           float b1, float b2, float eps, float bc1, float bc2) {
+    const float invR = 1.0f / (float)R;
+    const long stride = (long)gridDim.x * blockDim.x;
+    for (long k = (long)blockIdx.x * blockDim.x + threadIdx.x; k < n4; k += stride) {
+        const long i = lo + 4 * k;
+        float4 g = *reinterpret_cast<const float4 *>(grads[0] + i);
+        for (int r = 1; r < R; ++r) {  // replica order
+            const float4 x = *reinterpret_cast<const float4 *>(grads[r] + i);
+            g.x += x.x, g.y += x.y, g.z += x.z, g.w += x.w;
+        }
+        if (R > 1) g.x *= invR, g.y *= invR, g.z *= invR, g.w *= invR;
+        float4 w = *reinterpret_cast<const float4 *>(w_in + i);
+        if constexpr (ADAM) {
+            float4 mm = *reinterpret_cast<const float4 *>(m + i), vv = *reinterpret_cast<const float4 *>(v + i);
+            w.x = adam_step(w.x, g.x, mm.x, vv.x, lr, b1, b2, eps, bc1, bc2);
+            w.y = adam_step(w.y, g.y, mm.y, vv.y, lr, b1, b2, eps, bc1, bc2);
+            w.z = adam_step(w.z, g.z, mm.z, vv.z, lr, b1, b2, eps, bc1, bc2);
+            w.w = adam_step(w.w, g.w, mm.w, vv.w, lr, b1, b2, eps, bc1, bc2);
+            *reinterpret_cast<float4 *>(m + i) = mm;
+            *reinterpret_cast<float4 *>(v + i) = vv;
+        } else {
+            w.x = w.x - lr * g.x, w.y = w.y - lr * g.y, w.z = w.z - lr * g.z, w.w = w.w - lr * g.w;
+        }
+        uint2 o;
+        if (out_bf16) {
+            __nv_bfloat162 a0 = __floats2bfloat162_rn(w.x, w.y), a1 = __floats2bfloat162_rn(w.z, w.w);
+            o.x = *reinterpret_cast<uint32_t *>(&a0);
+            o.y = *reinterpret_cast<uint32_t *>(&a1);
+        }
+        for (int r = 0; r < R; ++r) {
+            *reinterpret_cast<float4 *>(out_f32[r] + i) = w;
+            if (out_bf16) *reinterpret_cast<uint2 *>(out_bf16[r] + i) = o;
+        }
+    }
+}
+
+cudaError_t update_shard(const float *const *grads, int R, long lo, long hi, const float *w_in, float *const *out_f32,
+                         __nv_bfloat16 *const *out_bf16, int opt, float *m, float *v, float lr, float b1, float b2,
+                         float eps, int step, cudaStream_t s) {
+    if ((lo & 3) || (hi & 3) || hi < lo) return cudaErrorInvalidValue;
+    if (hi == lo) return cudaSuccess;
+    const float bc1 = 1.f - powf(b1, (float)step), bc2 = 1.f - powf(b2, (float)step);
+    const long n4 = (hi - lo) / 4;
+    long blocks = (n4 + 255) / 256;
+    if (blocks > 148L * 8) blocks = 148L * 8;
+    if (opt == PD_ADAM)
+        update_shard_kernel<true><<<(unsigned)blocks, 256, 0, s>>>(grads, R, lo, n4, w_in, out_f32, out_bf16, m, v, lr, b1,
+                                                                   b2, eps, bc1, bc2);
+    else
+        update_shard_kernel<false><<<(unsigned)blocks, 256, 0, s>>>(grads, R, lo, n4, w_in, out_f32, out_bf16, m, v, lr,
+                                                                    b1, b2, eps, bc1, bc2);
+    ++tl_launches;
+    return cudaGetLastError();
+}
+
 cudaError_t update_from_grad(float *master, __nv_bfloat16 *slot, const float *g, long n, int opt, float *m, float *v,
                              float lr, float b1, float b2, float eps, int step, cudaStream_t s) {
     if ((n & 3) || ((uintptr_t)master & 15) || ((uintptr_t)g & 15) || ((uintptr_t)slot & 7) ||

@@ -39,13 +39,71 @@ namespace pd {
 namespace {
 using namespace tcx;
 
-constexpr int NT = 256;
 constexpr int ATILE = 128 * 128;         // [128 rows][64 K] bf16 (or 2 x [64 K][64 rows] MN-major)
 constexpr int BTILE = 64 * 128;          // [<= 64 rows][64 K] bf16
 constexpr int STAGE = ATILE + BTILE;
-constexpr int STG_LD = 68;               // forward epilogue staging row stride (floats)
-constexpr int STG_BYTES = 128 * STG_LD * 4;
-constexpr int RECV_BYTES = 128 * 32 * 4;  // backward: the peer's partial for this CTA's batch half
+
+// Cluster K-split (CL CTAs per item, template parameter): the CTAs of a cluster split an
+// item's K-blocks, and each finishes R = 64 / CL of the 64 accumulator columns (batch rows,
+// on the 64-column grid: columns >= B are padding nobody uses).  Partials travel to the
+// owning CTA through DSMEM (st.async + mbarrier complete_tx) into its exchange buffer
+// xbuf[source slot][128 rows][row stride]:
+//   forward (CL 1 or 2): one slot per CTA of the cluster (own partial staged locally), row
+//                        stride R + 1 floats (bank-conflict-free staging stores by TMEM
+//                        row and cell-loop reads by hidden unit); the
+//                        forward's b_ih + b_hh per gate row in a separate 128-float array
+//   backward (CL 2, 4, 8): CL - 1 slots (own partial stays in registers), stride R
+// More CTAs per item = fewer weight / activation bytes each CTA ingests per wave (the per-SM
+// ingest, not the tensor pipe, bounds a wave), so short runs (a pipeline stage's 2-3 layers)
+// spread each wave over the whole machine.
+template <bool BWD, int CL>
+struct WaveCfg {
+    static constexpr int S = BWD ? 8 : 7;  // operand ring stages
+    static constexpr int R = 64 / CL;      // accumulator columns (batch rows) a CTA finishes
+    static constexpr int RP = BWD ? R : R + 1;  // forward: odd stride, conflict-free by row and by unit
+    static constexpr int SLOTS = BWD ? CL - 1 : CL;
+    static constexpr int XBYTES = (SLOTS > 0 ? SLOTS : 1) * 128 * RP * 4;
+    static constexpr int BIAS_BYTES = BWD ? 0 : 128 * 4;
+    // forward, CL = 2: the peer's chunk is staged here and moved by one bulk DSMEM copy
+    static constexpr int OUT_BYTES = (!BWD && CL > 1) ? 128 * RP * 4 : 0;
+    static constexpr int SMEM = S * STAGE + XBYTES + BIAS_BYTES + OUT_BYTES + 256 + 1024;
+    static_assert(64 % CL == 0 && (BWD ? (CL >= 2 && R / 2 >= 4) : CL <= 2), "unsupported cluster split");
+};
+
+// NC consecutive fp32 columns of this warp's 32 TMEM lanes (NC = 4, 8, 16), waited
+template <int NC>
+__device__ __forceinline__ void tmem_ldn(uint32_t taddr, float (&v)[NC]) {
+    uint32_t r[NC];
+    if constexpr (NC == 16) {
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+            : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+              "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+            : "r"(taddr));
+    } else if constexpr (NC == 8) {
+        asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                     : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                     : "r"(taddr));
+    } else {
+        static_assert(NC == 4, "tmem_ldn: 4, 8 or 16 columns");
+        asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+                     : "r"(taddr));
+    }
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < NC; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+__device__ __forceinline__ void st_async_v4(uint32_t dst, const float *v, uint32_t bar) {
+    asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(dst),
+                 "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "r"(bar)
+                 : "memory");
+}
+__device__ __forceinline__ void arrive_remote(uint32_t bar_local, int rank) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(mapa_cluster(bar_local, rank))
+                 : "memory");
+}
 
 __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
     unsigned v;
@@ -76,6 +134,7 @@ struct WaveLayer {
     const float *b_ih, *b_hh;  // forward
     float *gates, *c;          // saved state [T][B][4H], [T][B][H] (written fwd, read bwd)
     __nv_bfloat16 *h;          // forward output [T][B][H]
+    __nv_bfloat16 *h2;         // forward: optional second destination of h (top layer: the stage output)
     __nv_bfloat16 *da;         // backward output [T][B][4H]
     float *dc;                 // backward carry [B][H] (scratch)
 };
@@ -162,19 +221,20 @@ __device__ __forceinline__ uint32_t cluster_rank() {
 // 8 epilogue warps, two per TMEM lane quadrant: backward -- 16 batch rows each (the cell
 // backward is the latency-bound part of a wave); forward -- one 32-column accumulator chunk
 // each to stage, 8 of a thread's 16 units each in the cell
-template <bool BWD>
-__host__ __device__ constexpr int wave_threads() { return 384; }
+constexpr int WAVE_THREADS = 384;
 
-template <bool BWD>
-__global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
-    constexpr int NE = wave_threads<BWD>() - 128;  // epilogue threads
+template <bool BWD, int CL>
+__global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
+    constexpr int NE = WAVE_THREADS - 128;  // epilogue threads
+    using WC = WaveCfg<BWD, CL>;
+    constexpr int S = WC::S, R = WC::R, RP = WC::RP;
     auto epi_sync = [] { epi_sync_n<NE>(); };
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *sm = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    // backward: a cluster of 2 CTAs splits every item's K-blocks; each finishes half the batch
-    constexpr int S = BWD ? 8 : 7, CL = BWD ? 2 : 1;
-    float *stg = reinterpret_cast<float *>(sm + S * STAGE);  // fwd staging / bwd receive buffer
-    uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * STAGE + (BWD ? RECV_BYTES : STG_BYTES));
+    float *xbuf = reinterpret_cast<float *>(sm + S * STAGE);                 // exchange / staging
+    float *sbias = reinterpret_cast<float *>(sm + S * STAGE + WC::XBYTES);  // forward biases
+    float *outbox = reinterpret_cast<float *>(sm + S * STAGE + WC::XBYTES + WC::BIAS_BYTES);  // fwd, CL = 2
+    uint64_t *bars = reinterpret_cast<uint64_t *>(sm + S * STAGE + WC::XBYTES + WC::BIAS_BYTES + WC::OUT_BYTES);
     // bars: full_w[S], full_x[S], empty[S], acc_full[2], acc_empty[2], recv_full, recv_empty
     const uint32_t fw0 = smem_u32(bars), fx0 = smem_u32(bars + S), em0 = smem_u32(bars + 2 * S);
     const uint32_t af0 = smem_u32(bars + 3 * S), ae0 = smem_u32(bars + 3 * S + 2);
@@ -182,7 +242,7 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * S + 6);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int H = a.H, B = a.B, N = a.N;
-    const int rank = BWD ? (int)cluster_rank() : 0;
+    const int rank = CL > 1 ? (int)cluster_rank() : 0;
 
     if (tid == 0) {
         for (int s = 0; s < S; ++s) {
@@ -195,7 +255,7 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
             mbar_init(ae0 + 8 * b, NE);
         }
         mbar_init(rfull, 1);
-        mbar_init(rempty, 1);
+        mbar_init(rempty, CL > 1 ? CL - 1 : 1);  // every peer that receives from this CTA releases
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 3) {
@@ -204,7 +264,7 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
     }
     tc_fence_before();
     __syncthreads();
-    if (BWD) cluster_sync_all();  // the peer's barriers exist before any remote arrive / st.async
+    if (CL > 1) cluster_sync_all();  // the peers' barriers exist before any remote arrive / st.async
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
     // published (step, tile, CTA) items of a layer per completed step
@@ -314,28 +374,64 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
     } else if (warp >= 4) {
         // ---------------- epilogue
         const int q = (warp - 4) & 3;   // TMEM lane quadrant (warp % 4)
-        const int half = (warp - 4) >> 2;  // backward: which 16 of the 32 batch rows
+        const int half = (warp - 4) >> 2;  // which half of this CTA's columns (backward) / chunks (forward)
         const int et = tid - 128;
+        const uint32_t xb = smem_u32(xbuf);
         ItemIter<CL> it;
         int l, tile, t, acc = 0, pv = 0;
         uint32_t aph[2] = {0, 0}, rph = 0, eph = 0;
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             const bool mm = ik.hi > ik.lo;
-            if (BWD) {
-                // while the MMA runs: pull this item's cell-backward inputs (saved gates, c[t],
-                // c[t-1], the dc carry; written long before, mostly in HBM) into L2 -- lane i of
-                // warp q fetches the 128-byte lines of batch row hb + i for units q*32 .. q*32+31
-                const int b = rank * 32 + lane, jq = tile * 128 + q * 32;
-                if (half == 0 && b < B) {
-                    const WaveLayer &Lp = a.layer[l];
-                    const long r1 = ((long)t * B + b) * H + jq, r4 = ((long)t * B + b) * 4 * H + jq;
+            // while the MMA runs, load this thread's cell inputs (they do not depend on the
+            // accumulator): forward c[t-1] of its units; backward (one row chunk per thread,
+            // CL >= 4) the saved gates, c[t], c[t-1], the dc carry and the top layer's dy --
+            // for CL = 2 (two chunks, no registers to spare) only pulled into L2
+            constexpr bool PRE_B = BWD && R / 2 <= 8;
+            constexpr int PR = PRE_B ? R / 2 : 1, FC = BWD ? 1 : R / 8;
+            float pig[PR], pfg[PR], pgg[PR], pog[PR], pct[PR], pcp[PR], pdc[PR], pdy[PR];
+            float fcp[FC];
+            if constexpr (BWD) {
+                const WaveLayer &Lp = a.layer[l];
+                if constexpr (PRE_B) {
+                    const int j = tile * 128 + q * 32 + lane, hb2 = rank * R + half * (R / 2);
+                    const bool top = l == a.L - 1;
 #pragma unroll
-                    for (int g = 0; g < 4; ++g)
-                        asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.gates + r4 + (long)g * H));
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.c + r1));
-                    if (t > 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.c + r1 - (long)B * H));
-                    if (t < a.T - 1) asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.dc + (long)b * H + jq));
+                    for (int u = 0; u < PR; ++u) {
+                        const int b = hb2 + u;
+                        pig[u] = pfg[u] = pgg[u] = pog[u] = pct[u] = pcp[u] = pdc[u] = pdy[u] = 0.f;
+                        if (b < B) {
+                            const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
+                            pig[u] = __ldg(Lp.gates + r4);
+                            pfg[u] = __ldg(Lp.gates + r4 + H);
+                            pgg[u] = __ldg(Lp.gates + r4 + 2 * H);
+                            pog[u] = __ldg(Lp.gates + r4 + 3 * H);
+                            pct[u] = __ldg(Lp.c + r1);
+                            if (t > 0) pcp[u] = __ldg(Lp.c + r1 - (long)B * H);
+                            if (t < a.T - 1) pdc[u] = Lp.dc[(long)b * H + j];
+                            if (top) pdy[u] = __bfloat162float(a.dy_top[r1]);
+                        }
+                    }
+                } else {
+                    // lane i of warp q fetches the 128-byte lines of batch row rank * R + i
+                    const int b = rank * R + lane, jq = tile * 128 + q * 32;
+                    if (half == 0 && lane < R && b < B) {
+                        const long r1 = ((long)t * B + b) * H + jq, r4 = ((long)t * B + b) * 4 * H + jq;
+#pragma unroll
+                        for (int g = 0; g < 4; ++g)
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.gates + r4 + (long)g * H));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.c + r1));
+                        if (t > 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.c + r1 - (long)B * H));
+                        if (t < a.T - 1) asm volatile("prefetch.global.L2 [%0];" ::"l"(Lp.dc + (long)b * H + jq));
+                    }
+                }
+            } else {
+                // forward cell mapping: lane = hidden unit, warp w covers rows w, w + 8, ...
+                const int j = tile * 32 + lane;
+#pragma unroll
+                for (int i = 0; i < FC; ++i) {
+                    const int b = rank * R + (et >> 5) + 8 * i;
+                    fcp[i] = (t > 0 && b < B) ? a.layer[l].c[((long)(t - 1) * B + b) * H + j] : 0.f;
                 }
             }
             mbar_wait(af0 + 8 * acc, aph[acc]);
@@ -344,159 +440,193 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
             if (et == 0) probe(a, pv, 3);
             const uint32_t d = tmem + acc * 64 + ((uint32_t)(q * 32) << 16);
             const WaveLayer &Ly = a.layer[l];
-            if (!BWD) {
-                // stage D[row = g*32 + u][b] so one thread sees all four gates of (u, b)
+            if constexpr (!BWD) {
+                // stage D[row = g*32 + u][b] so one thread sees all four gates of (u, b): chunk ch
+                // (accumulator columns 32 ch .. 32 ch + 31) belongs to CTA ch of a pair (CL = 2)
+                // or to this CTA (CL = 1); it lands in the owner's slot `rank`
                 const int row = q * 32 + lane;
                 constexpr int NWQ = NE / 128;  // epilogue warps per TMEM lane quadrant
+                if (CL > 1) {
+                    mbar_wait(rempty, eph ^ 1);  // the peer has consumed what we sent it last item
+                    eph ^= 1;
+                }
 #pragma unroll
                 for (int ch = half; ch < 2; ch += NWQ) {
                     float v[32];
                     tmem_ld32(d + ch * 32, v);
+                    const int owner = CL == 1 ? 0 : ch;
+                    // own chunk: straight into this CTA's slot; the peer's: into the outbox
+                    const uint32_t base = owner == rank ? xb + (uint32_t)((rank * 128 + row) * RP * 4) +
+                                                              (CL == 1 ? ch * 32 * 4 : 0)
+                                                        : smem_u32(outbox) + (uint32_t)(row * RP * 4);
 #pragma unroll
-                    for (int i = 0; i < 8; ++i)
-                        *reinterpret_cast<float4 *>(stg + row * STG_LD + ch * 32 + i * 4) =
-                            make_float4(v[i * 4], v[i * 4 + 1], v[i * 4 + 2], v[i * 4 + 3]);
+                    for (int i = 0; i < 32; ++i)
+                        asm volatile("st.shared.f32 [%0], %1;" ::"r"(base + i * 4), "f"(v[i]) : "memory");
                 }
-                // gate row `row` = g*32 + u: b_ih + b_hh into the staging row's spare column 64
-                // (STG_LD = 68), so the cell loop below reads biases from shared memory
+                if (CL > 1) fence_proxy_async();  // the outbox, written by this thread, feeds a bulk copy
+                // gate row `row` = g*32 + u: b_ih + b_hh, so the cell loop reads biases from smem
                 if (half == 0) {
                     const int gi = row >> 5, uu = row & 31, jb = gi * H + tile * 32 + uu;
-                    stg[row * STG_LD + 64] = __ldg(Ly.b_ih + jb) + __ldg(Ly.b_hh + jb);
+                    sbias[row] = __ldg(Ly.b_ih + jb) + __ldg(Ly.b_hh + jb);
                 }
                 tc_fence_before();
                 mbar_arrive(ae0 + 8 * acc);
+                if (CL > 1) {
+                    // the whole outbox to the peer's slot `rank` in one bulk DSMEM copy
+                    epi_sync();
+                    if (et == 0) {
+                        const int peer = rank ^ 1;
+                        constexpr uint32_t bytes = 128 * RP * 4;
+                        asm volatile(
+                            "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                                mapa_cluster(xb + (uint32_t)(rank * 128 * RP * 4), peer)),
+                            "r"(smem_u32(outbox)), "r"(bytes), "r"(mapa_cluster(rfull, peer))
+                            : "memory");
+                        mbar_expect_tx(rfull, bytes);
+                    }
+                    mbar_wait(rfull, rph);
+                    rph ^= 1;
+                }
                 epi_sync();
                 if (et == 0) probe(a, pv, 4);
-                constexpr int UPT = 16 / NWQ;  // units per thread
-                const int b = et & 63, u0 = (et >> 6) * UPT, j0 = tile * 32 + u0;
-                if (b < B) {
-                    const long r1 = ((long)t * B + b) * H, r4 = ((long)t * B + b) * 4 * H;
-                    // c[t-1] of all this thread's units first: no load waits behind its stores
-                    float4 cpv[UPT / 4];
+                // cell: lane = hidden unit u (coalesced loads / stores along H), warp w = et / 32
+                // covers this CTA's rows w, w + 8, ... (R / 8 of them)
+                const int u = lane, j = tile * 32 + u;
 #pragma unroll
-                    for (int q4 = 0; q4 < UPT / 4; ++q4)
-                        cpv[q4] = t > 0 ? *reinterpret_cast<const float4 *>(Ly.c + r1 - (long)B * H + j0 + 4 * q4)
-                                        : make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int i = 0; i < R / 8; ++i) {
+                    const int br = (et >> 5) + 8 * i, b = rank * R + br;
+                    if (b >= B) break;
+                    float gv[4];
 #pragma unroll
-                    for (int u4 = 0; u4 < UPT; u4 += 4) {
-                        const int j = j0 + u4;
-                        float gv[4][4];
+                    for (int g = 0; g < 4; ++g) {
+                        const int gr = g * 32 + u;
+                        float x = sbias[gr];
 #pragma unroll
-                        for (int g = 0; g < 4; ++g)
-#pragma unroll
-                            for (int e = 0; e < 4; ++e) {
-                                const int gr = g * 32 + u0 + u4 + e;
-                                gv[g][e] = stg[gr * STG_LD + b] + stg[gr * STG_LD + 64];
-                            }
-                        const float cp[4] = {cpv[u4 / 4].x, cpv[u4 / 4].y, cpv[u4 / 4].z, cpv[u4 / 4].w};
-                        float ig[4], fg[4], gg[4], og[4], cc[4], hh[4];
-#pragma unroll
-                        for (int e = 0; e < 4; ++e) {
-                            ig[e] = sigm(gv[0][e]);
-                            fg[e] = sigm(gv[1][e]);
-                            gg[e] = tanhf(gv[2][e]);
-                            og[e] = sigm(gv[3][e]);
-                            cc[e] = fg[e] * cp[e] + ig[e] * gg[e];
-                            hh[e] = og[e] * tanhf(cc[e]);
-                        }
-                        uint2 p;
-                        p.x = pack_bf16(hh[0], hh[1]);
-                        p.y = pack_bf16(hh[2], hh[3]);
-                        *reinterpret_cast<uint2 *>(Ly.h + r1 + j) = p;
-                        *reinterpret_cast<float4 *>(Ly.c + r1 + j) = make_float4(cc[0], cc[1], cc[2], cc[3]);
-                        *reinterpret_cast<float4 *>(Ly.gates + r4 + j) = make_float4(ig[0], ig[1], ig[2], ig[3]);
-                        *reinterpret_cast<float4 *>(Ly.gates + r4 + H + j) = make_float4(fg[0], fg[1], fg[2], fg[3]);
-                        *reinterpret_cast<float4 *>(Ly.gates + r4 + 2 * H + j) = make_float4(gg[0], gg[1], gg[2], gg[3]);
-                        *reinterpret_cast<float4 *>(Ly.gates + r4 + 3 * H + j) = make_float4(og[0], og[1], og[2], og[3]);
+                        for (int src = 0; src < CL; ++src) x += xbuf[(src * 128 + gr) * RP + br];
+                        gv[g] = x;
                     }
+                    const float ig = sigm(gv[0]), fg = sigm(gv[1]), gg = tanhf(gv[2]), og = sigm(gv[3]);
+                    const float cc = fg * fcp[i] + ig * gg, hh = og * tanhf(cc);
+                    const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
+                    const __nv_bfloat16 hb16 = __float2bfloat16_rn(hh);
+                    Ly.h[r1] = hb16;
+                    if (Ly.h2) Ly.h2[r1] = hb16;
+                    Ly.c[r1] = cc;
+                    Ly.gates[r4] = ig;
+                    Ly.gates[r4 + H] = fg;
+                    Ly.gates[r4 + 2 * H] = gg;
+                    Ly.gates[r4 + 3 * H] = og;
                 }
             } else {
-                // thread = hidden unit (TMEM lane m); this CTA finishes batch rows [hb, hb + 32),
-                // this warp rows [hb + 16 half, +16), and swaps the matching 16 columns of the
-                // peer's half of its K-partial with the peer CTA
-                const int mrow = q * 32 + lane, j = tile * 128 + mrow, hb = rank * 32, c16 = half * 16;
-                float mine[16], other[16];
+                // thread = hidden unit (TMEM lane m); this CTA finishes batch rows [hb, hb + R),
+                // this warp the RH rows [hb + c0, hb + c0 + RH); the matching RH columns of every
+                // peer's share go to that peer (its slot for this CTA), and this CTA's own
+                // columns collect the CL - 1 partials the peers send
+                constexpr int RH = R / 2, RC = RH < 8 ? RH : 8;
+                const int mrow = q * 32 + lane, j = tile * 128 + mrow, hb = rank * R, c0 = half * RH;
+                float mine[RH];
                 if (mm) {
-                    tmem_ld16(d + hb + c16, mine);
-                    tmem_ld16(d + (32 - hb) + c16, other);
+                    tmem_ldn<RH>(d + hb + c0, mine);
                 } else {
 #pragma unroll
-                    for (int i = 0; i < 16; ++i) mine[i] = other[i] = 0.f;
+                    for (int i = 0; i < RH; ++i) mine[i] = 0.f;
+                }
+                const bool exch = ik.n0 + ik.n1 > 0;  // the same for every CTA of the cluster
+                if (exch) {
+                    mbar_wait(rempty, eph ^ 1);  // every peer consumed what we sent it last item
+                    eph ^= 1;
+#pragma unroll
+                    for (int pr = 0; pr < CL; ++pr) {
+                        if (pr == rank) continue;
+                        float other[RH];
+                        if (mm) {
+                            tmem_ldn<RH>(d + pr * R + c0, other);
+                        } else {
+#pragma unroll
+                            for (int i = 0; i < RH; ++i) other[i] = 0.f;
+                        }
+                        const int slot = rank < pr ? rank : rank - 1;
+                        const uint32_t dst = mapa_cluster(xb + (uint32_t)(((slot * 128 + mrow) * R + c0) * 4), pr);
+                        const uint32_t pbar = mapa_cluster(rfull, pr);
+#pragma unroll
+                        for (int i = 0; i < RH / 4; ++i) st_async_v4(dst + i * 16, other + i * 4, pbar);
+                    }
                 }
                 tc_fence_before();
                 mbar_arrive(ae0 + 8 * acc);
-                if (ik.n0 + ik.n1 > 0) {
-                    const int peer = rank ^ 1;
-                    mbar_wait(rempty, eph ^ 1);  // the peer consumed the previous exchange
-                    eph ^= 1;
-                    const uint32_t dst = mapa_cluster(smem_u32(stg) + (mrow * 32 + c16) * 4, peer);
-                    const uint32_t pbar = mapa_cluster(rfull, peer);
-#pragma unroll
-                    for (int i = 0; i < 4; ++i)
-                        asm volatile(
-                            "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.f32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
-                                dst + i * 16),
-                            "f"(other[i * 4]), "f"(other[i * 4 + 1]), "f"(other[i * 4 + 2]), "f"(other[i * 4 + 3]),
-                            "r"(pbar)
-                            : "memory");
-                    if (et == 0) mbar_expect_tx(rfull, 128 * 32 * 4);
+                if (exch) {
+                    if (et == 0) mbar_expect_tx(rfull, (uint32_t)(CL - 1) * 128 * R * 4);
                     mbar_wait(rfull, rph);
                     rph ^= 1;
 #pragma unroll
-                    for (int i = 0; i < 16; ++i) mine[i] += stg[mrow * 32 + c16 + i];
-                    epi_sync();  // every thread read its row: hand the buffer back to the peer
+                    for (int sl = 0; sl < CL - 1; ++sl)
+#pragma unroll
+                        for (int i = 0; i < RH; ++i) mine[i] += xbuf[(sl * 128 + mrow) * R + c0 + i];
+                    epi_sync();  // every thread read its row: hand the buffers back to the peers
                     if (et == 0) probe(a, pv, 4);
                     if (et == 0)
-                        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
-                                         mapa_cluster(rempty, peer))
-                                     : "memory");
+                        for (int pr = 0; pr < CL; ++pr)
+                            if (pr != rank) arrive_remote(rempty, pr);
                 }
-                const bool top = l == a.L - 1;
-                // cell backward over this warp's 16 batch rows, 8 rows at a time: every load of a
-                // chunk is issued before any store (the stores may alias the loads as far as the
-                // compiler knows, which otherwise serialises one memory latency per row); gates /
-                // c were written by the forward launch, so they take the read-only path
-                const int hb2 = hb + c16, nb = min(16, B - hb2);
+                // cell backward over this warp's RH batch rows
+                const int hb2 = hb + c0, nb = min(RH, B - hb2);
+                auto cell = [&](int u, float dh, float ig, float fg, float gg, float og, float ct, float cp, float dcn) {
+                    const int b = hb2 + u;
+                    const long r4 = ((long)t * B + b) * 4 * H + j;
+                    const float tc = tanhf(ct);
+                    const float dct = dh * og * (1.f - tc * tc) + dcn;
+                    Ly.dc[(long)b * H + j] = dct * fg;
+                    Ly.da[r4] = __float2bfloat16_rn(dct * gg * ig * (1.f - ig));
+                    Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp * fg * (1.f - fg));
+                    Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig * (1.f - gg * gg));
+                    Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og * (1.f - og));
+                };
+                if constexpr (PRE_B) {
 #pragma unroll
-                for (int i0 = 0; i0 < 16; i0 += 8) {  // unrolled: mine[] stays in registers
-                    if (i0 >= nb) break;
-                    float ig[8], fg[8], gg[8], og[8], ct[8], cp[8], dcn[8], dyv[8];
+                    for (int u = 0; u < RH; ++u)
+                        if (u < nb) cell(u, mine[u] + pdy[u], pig[u], pfg[u], pgg[u], pog[u], pct[u], pcp[u], pdc[u]);
+                } else {
+                    const bool top = l == a.L - 1;
+                    // RC rows at a time: every load of a chunk is issued before any store (the
+                    // stores may alias the loads as far as the compiler knows, which otherwise
+                    // serialises one memory latency per row); gates / c were written by the
+                    // forward launch, so they take the read-only path
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) {
-                        const int b = hb2 + i0 + u;
-                        ig[u] = fg[u] = gg[u] = og[u] = ct[u] = cp[u] = dcn[u] = dyv[u] = 0.f;
-                        if (i0 + u < nb) {
-                            const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
-                            ig[u] = __ldg(Ly.gates + r4);
-                            fg[u] = __ldg(Ly.gates + r4 + H);
-                            gg[u] = __ldg(Ly.gates + r4 + 2 * H);
-                            og[u] = __ldg(Ly.gates + r4 + 3 * H);
-                            ct[u] = __ldg(Ly.c + r1);
-                            if (t > 0) cp[u] = __ldg(Ly.c + r1 - (long)B * H);
-                            if (t < a.T - 1) dcn[u] = Ly.dc[(long)b * H + j];
-                            if (top) dyv[u] = __bfloat162float(a.dy_top[r1]);
+                    for (int i0 = 0; i0 < RH; i0 += RC) {  // unrolled: mine[] stays in registers
+                        if (i0 >= nb) break;
+                        float ig[RC], fg[RC], gg[RC], og[RC], ct[RC], cp[RC], dcn[RC], dyv[RC];
+#pragma unroll
+                        for (int u = 0; u < RC; ++u) {
+                            const int b = hb2 + i0 + u;
+                            ig[u] = fg[u] = gg[u] = og[u] = ct[u] = cp[u] = dcn[u] = dyv[u] = 0.f;
+                            if (i0 + u < nb) {
+                                const long r1 = ((long)t * B + b) * H + j, r4 = ((long)t * B + b) * 4 * H + j;
+                                ig[u] = __ldg(Ly.gates + r4);
+                                fg[u] = __ldg(Ly.gates + r4 + H);
+                                gg[u] = __ldg(Ly.gates + r4 + 2 * H);
+                                og[u] = __ldg(Ly.gates + r4 + 3 * H);
+                                ct[u] = __ldg(Ly.c + r1);
+                                if (t > 0) cp[u] = __ldg(Ly.c + r1 - (long)B * H);
+                                if (t < a.T - 1) dcn[u] = Ly.dc[(long)b * H + j];
+                                if (top) dyv[u] = __bfloat162float(a.dy_top[r1]);
+                            }
                         }
-                    }
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) {
-                        if (i0 + u >= nb) break;
-                        const int b = hb2 + i0 + u;
-                        const long r4 = ((long)t * B + b) * 4 * H + j;
-                        const float dh = mine[i0 + u] + dyv[u];
-                        const float tc = tanhf(ct[u]);
-                        const float dct = dh * og[u] * (1.f - tc * tc) + dcn[u];
-                        Ly.dc[(long)b * H + j] = dct * fg[u];
-                        Ly.da[r4] = __float2bfloat16_rn(dct * gg[u] * ig[u] * (1.f - ig[u]));
-                        Ly.da[r4 + H] = __float2bfloat16_rn(dct * cp[u] * fg[u] * (1.f - fg[u]));
-                        Ly.da[r4 + 2 * H] = __float2bfloat16_rn(dct * ig[u] * (1.f - gg[u] * gg[u]));
-                        Ly.da[r4 + 3 * H] = __float2bfloat16_rn(dh * tc * og[u] * (1.f - og[u]));
+                        for (int u = 0; u < RC; ++u) {
+                            if (i0 + u >= nb) break;
+                            cell(i0 + u, mine[i0 + u] + dyv[u], ig[u], fg[u], gg[u], og[u], ct[u], cp[u], dcn[u]);
+                        }
                     }
                 }
             }
             if (et == 0) probe(a, pv, 6);  // this thread's cell loop done
             epi_sync();
             if (et == 0) {
-                probe(a, pv, 7);  // all 128 epilogue threads done
+                // forward, CL = 2: the cell loop above read the peer's slot -- release it
+                if (!BWD && CL > 1)
+                    for (int pr = 0; pr < CL; ++pr)
+                        if (pr != rank) arrive_remote(rempty, pr);
+                probe(a, pv, 7);  // all epilogue threads done
                 asm volatile("fence.acq_rel.gpu;" ::: "memory");
                 asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(a.cnt + l) : "memory");
                 probe(a, pv, 5);
@@ -507,12 +637,9 @@ __global__ void __launch_bounds__(wave_threads<BWD>(), 1) lstm_wave_kernel(const
     }
     tc_fence_before();
     __syncthreads();
-    if (BWD) cluster_sync_all();  // no peer st.async / arrive may target an exited CTA
+    if (CL > 1) cluster_sync_all();  // no peer st.async / arrive may target an exited CTA
     if (warp == 3) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
 }
-
-int wave_smem(bool bwd) { return (bwd ? 8 * STAGE + RECV_BYTES : 7 * STAGE + STG_BYTES) + 256 + 1024; }
-
 
 int num_sm() {
     static int sms = 0;
@@ -525,23 +652,15 @@ int num_sm() {
     return sms;
 }
 
-// forward: one CTA per item up to one per SM; backward: a CTA pair per item up to one pair
-// per two SMs (and no more pairs than can be resident at once)
-int wave_grid(int L, int H, bool bwd, int max_pairs) {
-    const int items = L * (bwd ? H / 128 : H / 32);
-    if (!bwd) return items < num_sm() ? items : num_sm();
-    const int pairs = items < max_pairs ? items : max_pairs;
-    return 2 * pairs;
-}
-
-cudaLaunchConfig_t wave_cfg(bool bwd, int grid, cudaStream_t s, cudaLaunchAttribute *attr) {
+template <bool BWD, int CL>
+cudaLaunchConfig_t wave_cfg(int grid, cudaStream_t s, cudaLaunchAttribute *attr) {
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(bwd ? wave_threads<true>() : wave_threads<false>());
-    cfg.dynamicSmemBytes = wave_smem(bwd);
+    cfg.blockDim = dim3(WAVE_THREADS);
+    cfg.dynamicSmemBytes = WaveCfg<BWD, CL>::SMEM;
     cfg.stream = s;
     attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = bwd ? 2 : 1;
+    attr[0].val.clusterDim.x = CL;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
@@ -549,41 +668,61 @@ cudaLaunchConfig_t wave_cfg(bool bwd, int grid, cudaStream_t s, cudaLaunchAttrib
     return cfg;
 }
 
-int max_pairs_resident() {
+// clusters of this instantiation that can be resident at once (0 if it cannot launch); the
+// wavefront's spin-waits need every CTA of the grid resident, so grids never exceed this
+template <bool BWD, int CL>
+int max_clusters() {
     static int n = -1;
     if (n < 0) {
-        cudaLaunchAttribute attr[1];
-        cudaLaunchConfig_t cfg = wave_cfg(true, 2 * 64, nullptr, attr);
-        int c = 0;
-        if (cudaOccupancyMaxActiveClusters(&c, lstm_wave_kernel<true>, &cfg) != cudaSuccess) {
-            cudaGetLastError();
-            c = 0;
+        n = 0;
+        if (cudaFuncSetAttribute(lstm_wave_kernel<BWD, CL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 WaveCfg<BWD, CL>::SMEM) == cudaSuccess) {
+            cudaLaunchAttribute attr[1];
+            cudaLaunchConfig_t cfg = wave_cfg<BWD, CL>(CL * 64, nullptr, attr);
+            int c = 0;
+            if (cudaOccupancyMaxActiveClusters(&c, lstm_wave_kernel<BWD, CL>, &cfg) == cudaSuccess) n = c;
         }
-        n = c;
+        cudaGetLastError();
     }
     return n;
+}
+
+int max_clusters(bool bwd, int cl) {
+    if (!bwd) return cl == 2 ? max_clusters<false, 2>() : max_clusters<false, 1>();
+    return cl == 8 ? max_clusters<true, 8>() : cl == 4 ? max_clusters<true, 4>() : max_clusters<true, 2>();
+}
+
+// Cluster size: the widest K-split whose clusters all fit at once with one item each (every
+// SM ingesting a 1/CL share of an item per wave); when the items outnumber the resident
+// clusters (long runs), the narrowest split (forward 1, backward 2: the whole machine is busy
+// anyway and fewer, larger shares exchange less).
+int choose_cl(bool bwd, int items) {
+    const int sms = num_sm();
+    const int cands[2][3] = {{2, 1, 1}, {8, 4, 2}};
+    for (int cl : cands[bwd]) {
+        const int mc = max_clusters(bwd, cl);
+        if (mc >= items && cl * items <= sms) return cl;
+    }
+    return bwd ? 2 : 1;
 }
 
 }  // namespace
 
 bool lstm_wave_supported(int L, int B, int H, int I) {
     if (L < 1 || L > LSTM_WAVE_MAX_L || B < 1 || B > 64 || H < 128 || H % 128 || I != H) return false;
-    static int ok = 0;
-    if (!ok) {
-        int n = 0;
-        ok = 1;
-        if (cudaFuncSetAttribute(lstm_wave_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 wave_smem(false)) != cudaSuccess ||
-            cudaFuncSetAttribute(lstm_wave_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 wave_smem(true)) != cudaSuccess ||
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lstm_wave_kernel<false>, wave_threads<false>(), wave_smem(false)) !=
-                cudaSuccess ||
-            n < 1 || max_pairs_resident() < 1) {
-            cudaGetLastError();
-            ok = -1;
-        }
-    }
-    return ok > 0;
+    return max_clusters(false, 1) >= 1 && max_clusters(true, 2) >= 1;
+}
+
+// the smallest wave grid that runs every item: CL CTAs per item up to the resident clusters
+template <bool BWD, int CL>
+cudaError_t launch_wave(const WaveMaps &m, const WaveArgs &a, int items, cudaStream_t s) {
+    const int mc = max_clusters<BWD, CL>();
+    if (mc < 1) return cudaErrorNotSupported;
+    const int clusters = items < mc ? items : mc;
+    cudaLaunchAttribute attr[1];
+    cudaLaunchConfig_t cfg = wave_cfg<BWD, CL>(CL * clusters, s, attr);
+    ++tl_launches;
+    return cudaLaunchKernelEx(&cfg, lstm_wave_kernel<BWD, CL>, m, a);
 }
 
 cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
@@ -598,7 +737,7 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     std::memset(&m, 0, sizeof(m));
     const long TB = (long)T * B;
     for (int l = 0; l < L; ++l) {
-        a.layer[l] = {w.b_ih[l], w.b_hh[l], w.gates[l], w.c[l], w.h[l], w.da[l], w.dc[l]};
+        a.layer[l] = {w.b_ih[l], w.b_hh[l], w.gates[l], w.c[l], w.h[l], l == L - 1 ? w.h_out : nullptr, w.da[l], w.dc[l]};
         const int rows = w.bwd ? 64 : 32, cols = 64;
         if (!tma_map_bf16(&m.w_ih[l], w.W_ih[l], H, 4L * H, H, cols, rows) ||
             !tma_map_bf16(&m.w_hh[l], w.W_hh[l], H, 4L * H, H, cols, rows))
@@ -612,7 +751,9 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     if (!w.bwd && !tma_map_bf16(&m.act[0], w.x, H, TB, H, 64, a.N)) return cudaErrorInvalidValue;
     cudaError_t e = cudaMemsetAsync(w.cnt, 0, sizeof(unsigned) * L, s);
     if (e != cudaSuccess) return e;
-    const int grid = wave_grid(L, H, w.bwd, max_pairs_resident());
+    const int items = L * a.tiles;
+    const int cl = choose_cl(w.bwd, items);
+    const int grid = cl * std::min(items, max_clusters(w.bwd, cl));
     {
         // PD_WAVE_L2_MB: MB of the run's weights kept L2-resident (whole layers, evict_last; the
         // rest streams evict_first).  Measured GNMT-8 at N = 1: 0 -> 11.51k, 32 -> 11.80k,
@@ -634,11 +775,10 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
             pbuf = nullptr;
         if (pbuf && cudaMemsetAsync(pbuf, 0, pbytes, s) == cudaSuccess) a.probe = pbuf;
     }
-    cudaLaunchAttribute attr[1];
-    cudaLaunchConfig_t cfg = wave_cfg(w.bwd, grid, s, attr);
-    ++tl_launches;
-    e = w.bwd ? cudaLaunchKernelEx(&cfg, lstm_wave_kernel<true>, m, a)
-              : cudaLaunchKernelEx(&cfg, lstm_wave_kernel<false>, m, a);
+    if (!w.bwd) e = cl == 2 ? launch_wave<false, 2>(m, a, items, s) : launch_wave<false, 1>(m, a, items, s);
+    else if (cl == 8) e = launch_wave<true, 8>(m, a, items, s);
+    else if (cl == 4) e = launch_wave<true, 4>(m, a, items, s);
+    else e = launch_wave<true, 2>(m, a, items, s);
     if (e == cudaSuccess && a.probe) {
         std::vector<unsigned long long> h(pbytes / 8);
         if (cudaStreamSynchronize(s) == cudaSuccess && cudaMemcpy(h.data(), pbuf, pbytes, cudaMemcpyDeviceToHost) == cudaSuccess) {
@@ -646,7 +786,9 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
             for (auto x : h)
                 if (x && x < t0) t0 = x;
             if (FILE *f = fopen(pfile, "a")) {
-                fprintf(f, "%s L=%d T=%d B=%d H=%d grid=%d", w.bwd ? "bwd" : "fwd", L, T, B, H, grid);
+                fprintf(f, "%s L=%d T=%d B=%d H=%d grid=%d CL=%d max_clusters fwd1/2 %d/%d bwd2/4/8 %d/%d/%d",
+                        w.bwd ? "bwd" : "fwd", L, T, B, H, grid, cl, max_clusters(false, 1), max_clusters(false, 2),
+                        max_clusters(true, 2), max_clusters(true, 4), max_clusters(true, 8));
                 for (int c = 0; c < grid; ++c) {
                     fprintf(f, " |");
                     for (int v = 0; v < PROBE_V; ++v) {

@@ -108,18 +108,7 @@ struct Gemm {
     ConvGeom conv;        // implicit-GEMM convolution (bf16 path only)
     int ksplit = 1;       // explicit split-K (EPI_F32 with atomic_out)
     int max_ctas = 0;     // cap on resident CTAs (0 = every SM): leaves SMs to a concurrent kernel
-    int *split_counters = nullptr;  // >= 8192 zeroed ints: split-K tiles reduce in-kernel (last CTA)
     int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
-    // optional: bytes [l2_next, l2_next + l2_next_bytes) are prefetched into L2 by an idle warp
-    // while this GEMM runs (the next layer's weights on the forward / dX chains)
-    const void *l2_next = nullptr;
-    long l2_next_bytes = 0;
-    // programmatic dependent launch allowed for this GEMM's kernels (with PD_PDL=1): set by the
-    // runtime for the forward / dX chains, whose predecessor on the stream is another such kernel
-    int pdl = 0;
-    // the caller guarantees this GEMM's CTAs can all be co-resident (no other worker's spin-waiting
-    // kernel on the GPU): allows the distributed in-kernel split-K reduction (PD_SPLIT_INKERNEL=2)
-    int split_dist = 0;
 };
 
 // cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}
@@ -150,6 +139,13 @@ cudaError_t adam_f32(const float *in, const float *g, float *out, float *m, floa
 cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f32, const float *const *grads,
                           int R, long goff, long n, int opt, float *m, float *v, float lr, float b1, float b2,
                           float eps, int step, cudaStream_t s);
+// replica sync of one round, sharded: this replica's parameters [lo, hi) (multiples of 4):
+// g = (sum_r grads[r][i]) * (1/R) in r order (R7), optimizer step on w_in[i] (+ m, v), the
+// new value stored to out_f32[q][i] and (if out_bf16) bf16 to out_bf16[q][i] for every
+// replica q.  grads / out_f32 / out_bf16 are DEVICE arrays of R pointers (peer memory).
+cudaError_t update_shard(const float *const *grads, int R, long lo, long hi, const float *w_in, float *const *out_f32,
+                         __nv_bfloat16 *const *out_bf16, int opt, float *m, float *v, float lr, float b1, float b2,
+                         float eps, int step, cudaStream_t s);
 // bf16 path, one unreplicated fp32 gradient: master -= SGD/Adam step of g, slot = bf16(master);
 // vectorised (n % 4 == 0, 16-byte aligned arrays; else cudaErrorInvalidValue)
 cudaError_t update_from_grad(float *master, __nv_bfloat16 *slot, const float *g, long n, int opt, float *m, float *v,
@@ -194,6 +190,8 @@ struct LstmWaveDesc {
     const float *b_ih[LSTM_WAVE_MAX_L] = {}, *b_hh[LSTM_WAVE_MAX_L] = {};
     float *gates[LSTM_WAVE_MAX_L] = {}, *c[LSTM_WAVE_MAX_L] = {}, *dc[LSTM_WAVE_MAX_L] = {};
     __nv_bfloat16 *h[LSTM_WAVE_MAX_L] = {}, *da[LSTM_WAVE_MAX_L] = {};
+    __nv_bfloat16 *h_out = nullptr;  // forward: second destination of the top layer's h (the stage
+                                     // output: the consumer's receive slot, possibly peer memory)
     unsigned *cnt = nullptr;  // >= L uints (zeroed by lstm_wave on the stream)
 };
 bool lstm_wave_supported(int L, int B, int H, int I);

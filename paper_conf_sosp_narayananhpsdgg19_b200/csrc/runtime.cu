@@ -163,19 +163,27 @@ struct Link {
 };
 
 // ---------------------------------------------------------------- IPC blob
+constexpr int MAX_SYNC_SLOTS = 32;  // weight-stash slots a replicated worker exposes to its peers
 struct IpcBlob {
     uint32_t magic;
     int32_t stage, replica, device;
     int32_t has_recv, has_grad, has_rgrad;
     cudaIpcMemHandle_t recv, grad, rgrad0, rgrad1, flags;
+    // replicated stages: the weight-stash slots and the fp32 master, which the peers' sharded
+    // updates write (replica sync as reduce-scatter -> update -> all-gather)
+    int32_t nslots, has_master;
+    cudaIpcMemHandle_t wslot[MAX_SYNC_SLOTS], master;
 };
-constexpr uint32_t BLOB_MAGIC = 0x50443031u;  // "PD01"
+constexpr uint32_t BLOB_MAGIC = 0x50443032u;  // "PD02"
 
 // Buffers a worker exposes to others (local pointers, or IPC-mapped in this process).
 struct Shared {
     void *recv = nullptr;      // activation receive ring (stage > 0)
     void *grad = nullptr;      // gradient receive ring (stage < n-1)
     float *rgrad[2] = {};      // replica gradient buffers (R_s > 1), round parity
+    void *wslot[MAX_SYNC_SLOTS] = {};  // replicated stages: weight-stash slots (peers write their shards)
+    int nslots = 0;
+    float *master = nullptr;   // replicated stages, bf16 path: fp32 master (peers write their shards)
     uint32_t *flags = nullptr; // flag words (remote links)
     bool valid = false;
     bool standin = false;      // pd_stage_solo: local buffers standing in for an absent worker
@@ -212,6 +220,9 @@ struct pd_ctx {
     int ktime_mask = 0xFF;           // kernel classes timed when record_trace >= 2
     int layer_prof = 0;              // per-layer F / B device times (pd_set_layer_profiling)
     std::vector<void *> solo_bufs;   // pd_stage_solo stand-in buffers (owned)
+    std::mutex done_mu;              // worker threads of a pd_run finishing (watchdog wake-up)
+    std::condition_variable done_cv;
+    int running = 0;
     std::atomic<bool> abort{false};
     std::mutex err_mu;
     pd_status sticky = PD_OK;
@@ -265,11 +276,13 @@ struct Worker {
     float *gbuf = nullptr;      // fp32 gradient (unreplicated fp32 path / biases)
     float *ws = nullptr;        // split-K partials of the bf16 GEMMs
     long ws_bytes = 0;
-    int *split_counters = nullptr;  // per-tile arrival counters of in-kernel split-K
-    bool alone = false;  // the only worker on its GPU (all workers in this process): GEMMs may rely
-                         // on co-residency of their own CTAs (Gemm::split_dist)
     float *rgrad[2] = {};       // replicated stages: gradient per round parity
     const float **rgrad_ptrs = nullptr;  // device array [2][R]: peers' rgrad for each parity
+    // sharded replica sync: device arrays of every replica's destinations of a new version --
+    // sync_f32[slot][R]: fp32 masters (bf16 path, same for every slot) or fp32 slot `slot`;
+    // sync_bf16[slot][R]: bf16 slot `slot` (bf16 path)
+    float **sync_f32 = nullptr;
+    __nv_bfloat16 **sync_bf16 = nullptr;
     const float **self_grad_ptr = nullptr;  // device array [1]: gbuf
     // activations
     std::vector<void *> act;     // per inner layer l (index l-first, l>first): k slots of in_elems
@@ -319,11 +332,18 @@ struct Worker {
     std::vector<LayerEv> lev;  // layer profiling: one per layer per F / B op
     uint64_t launches = 0;
     uint64_t bytes_sent = 0;
+    uint64_t replica_bytes = 0;  // peer bytes of the sharded replica sync (gradient reads + pushes)
     int updates_total = 0;  // Adam step counter base (persists across runs)
     // slot-ownership checker: vc[w] = number of ops of worker w known (through the messages
     // this worker has awaited, transitively) to be complete before this worker's current op;
     // vc[id] counts this worker's own ops
     std::vector<int32_t> vc;
+    std::vector<char> wave_inner;  // per stage layer: inside an LSTM wavefront run (input = saved h below)
+    // watchdog state (pd_run reports a run that makes no progress): the op being issued and
+    // where the host thread is -- 0 issuing, 1 waiting for ring space in link_post, 2 waiting
+    // for a message in link_wait, 3 synchronising at the end of the run, 4 finished
+    std::atomic<int> st_op{-1}, st_where{4};
+    std::atomic<long> st_link{0};
 
     ~Worker();
 };
@@ -338,8 +358,9 @@ Worker::~Worker() {
     void *lb[] = {lstm_gx, lstm_gh, lstm_dh, lstm_dc, lstm_da, lstm_cnt, lstm_wda, lstm_wdc};
     for (void *p : lb)
         if (p) cudaFree(p);
-    void *bufs[] = {master, fbias, (void *)breg_off, (void *)breg_cnt, adam_m, adam_v, gbuf, ws, (void *)split_counters, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
-                    dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr};
+    void *bufs[] = {master, fbias, (void *)breg_off, (void *)breg_cnt, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
+                    dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr,
+                    (void *)sync_f32, (void *)sync_bf16};
     for (void *p : bufs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
@@ -406,6 +427,8 @@ Link &get_link(pd_ctx *c, int type, int src, int dst) {
     return *it->second;
 }
 
+thread_local Worker *tl_worker = nullptr;  // the worker this host thread runs (watchdog state)
+
 // `vc`: the posting worker's vector clock (snapshotted with the message, local links only)
 void link_post(pd_ctx *c, Link &L, cudaStream_t s, const std::vector<int32_t> &vc) {
     if (L.remote) {
@@ -414,11 +437,13 @@ void link_post(pd_ctx *c, Link &L, cudaStream_t s, const std::vector<int32_t> &v
         return;
     }
     const int E = (int)L.ev.size();
+    if (tl_worker) tl_worker->st_where = 1, tl_worker->st_link = L.posted;
     {
         std::unique_lock<std::mutex> g(L.mu);
         L.cv.wait(g, [&] { return L.posted - L.waited < E || c->abort.load(); });
         if (c->abort) throw Abort{};
     }
+    if (tl_worker) tl_worker->st_where = 0;
     CK(cudaEventRecord(L.ev[L.posted % E], s));
     {
         std::lock_guard<std::mutex> g(L.mu);
@@ -442,11 +467,13 @@ void link_wait(pd_ctx *c, Link &L, cudaStream_t s, int64_t idx, std::vector<int3
     }
     if (idx < 0) return;  // same process: the previous pd_run joined every worker's stream
     const int E = (int)L.ev.size();
+    if (tl_worker) tl_worker->st_where = 2, tl_worker->st_link = idx;
     {
         std::unique_lock<std::mutex> g(L.mu);
         L.cv.wait(g, [&] { return L.posted > idx || c->abort.load(); });
         if (c->abort) throw Abort{};
     }
+    if (tl_worker) tl_worker->st_where = 0;
     CK(cudaStreamWaitEvent(s, L.ev[idx % E], 0));
     {
         std::lock_guard<std::mutex> g(L.mu);
@@ -470,28 +497,8 @@ void *elem_ptr(void *base, long idx, int esz) { return static_cast<char *>(base)
 cudaError_t run_gemm(int bf16, const Gemm &g, cudaStream_t s) { return bf16 ? gemm_bf16(g, s) : gemm_f32(g, s); }
 
 // y = act(x W^T + b)
-// PD_SPLIT_ATOMIC=1: the M = B split-K GEMMs sum their partials by TMA reduce-add into the
-// zeroed workspace (Gemm::ws_zeroed).  Measured (MLP-4096 M = 256 GEMMs): 27.6 -> 29.7 us
-// isolated, -1 % in the step, so per-split partials stay the default
-int split_atomic() {
-    static const int v = [] {
-        const char *e = getenv("PD_SPLIT_ATOMIC");
-        return e ? atoi(e) : 0;
-    }();
-    return v;
-}
-
-// PD_L2_PF bit 0: forward GEMMs prefetch the next layer's weights into L2; bit 1: dX GEMMs
-int l2_pf_mask() {
-    static const int v = [] {
-        const char *e = getenv("PD_L2_PF");
-        return e ? atoi(e) : 0;
-    }();
-    return v;
-}
-
 void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, const float *bias_f32, const void *x,
-                    void *y, float *ws, long ws_bytes, const void *next_w = nullptr, long next_bytes = 0) {
+                    void *y, float *ws, long ws_bytes) {
     const int B = L.c->cfg.minibatch;
     Gemm g;
     g.M = (int)rows_of(d, B);
@@ -510,12 +517,6 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.relu = d.act == PD_ACT_RELU;
     g.workspace = ws;
     g.workspace_bytes = ws_bytes;
-    g.ws_zeroed = split_atomic();  // w->ws is zero-filled at allocation and re-zeroed by every reduce-add use
-    g.split_counters = L.w->split_counters;
-    g.split_dist = L.w->alone;
-    g.l2_next = next_w;
-    g.l2_next_bytes = next_bytes;
-    g.pdl = 1;
     CK(run_gemm(L.bf16, g, L.w->stream));
 }
 
@@ -557,6 +558,7 @@ struct Exec {
     // input of layer l for local index j
     const void *layer_input(int l, int t, int j) const {
         const pd_layer_desc &d = layer(l);
+        if (l > w->first && w->wave_inner[l - w->first]) return lstm_state(l - 1, j).h;
         if (l == w->first) {
             if (w->stage == 0) {
                 const int di = t % c->n_data;
@@ -719,9 +721,7 @@ struct Exec {
             cudaEvent_t k0 = kstart(0);
             if (d.kind == PD_LINEAR) {
                 LayerCtx lc{c, w, bf16};
-                const bool pf = bf16 && (l2_pf_mask() & 1) && l < w->last && layer(l + 1).kind == PD_LINEAR;
-                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes,
-                               pf ? Wl(l + 1, slot) : nullptr, pf ? (long)layer(l + 1).in * layer(l + 1).out * esz : 0);
+                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes);
             } else if (d.kind == PD_LSTM) {
                 lstm_forward(l, j, slot, x, y);
             } else if (d.kind == PD_EMBEDDING) {
@@ -783,8 +783,7 @@ struct Exec {
     };
 
     // dX = G W (B(n,k) given by the caller) fused with the previous layer's ReLU derivative
-    void gemm_dx(int l, int M, int N, int K, const void *G, long ldg, const void *W, long ldw, const void *x, void *dx,
-                 const void *next_w = nullptr, long next_bytes = 0) {
+    void gemm_dx(int l, int M, int N, int K, const void *G, long ldg, const void *W, long ldw, const void *x, void *dx) {
         const bool prev_relu = l > 0 && layer(l - 1).act == PD_ACT_RELU;
         Gemm g;
         g.M = M;
@@ -803,12 +802,6 @@ struct Exec {
         g.ldm = N;
         g.workspace = w->ws;
         g.workspace_bytes = w->ws_bytes;
-        g.ws_zeroed = split_atomic();
-        g.split_counters = w->split_counters;
-        g.split_dist = w->alone;
-        g.l2_next = next_w;
-        g.l2_next_bytes = next_bytes;
-        g.pdl = 1;
         CK(run_gemm(bf16, g, w->stream));
     }
 
@@ -1013,11 +1006,7 @@ struct Exec {
     // whole-op graphs: bf16 fused all-linear SGD stages (the launch-bound MLP path), and only
     // when no per-kernel timing is requested (event timing cannot live inside a graph)
     bool op_graphs_ok() const {
-        static const int env = [] {
-            const char *e = getenv("PD_OP_GRAPHS");
-            return e ? atoi(e) : 1;
-        }();
-        if (!env || !bf16 || c->cfg.optimizer != PD_SGD || c->layer_prof) return false;
+        if (!bf16 || c->cfg.optimizer != PD_SGD || c->layer_prof) return false;
         if (c->plan.stage[w->stage].replicas != 1) return false;
         if (timing && c->ktime_mask) return false;
         for (int l = w->first; l <= w->last; ++l)
@@ -1102,6 +1091,15 @@ struct Exec {
         wd.bwd = 0, wd.L = L, wd.T = T, wd.B = Bn, wd.H = H;
         wd.x = static_cast<const __nv_bfloat16 *>(layer_input(l0, t, j));
         wd.cnt = w->lstm_cnt;
+        // the run's inner layers read their input straight from the previous layer's saved h
+        // (layer_input); the top layer's epilogue also stores h into the next layer's input
+        // stash or the stage output -- the consumer's receive slot, over NVLink when the
+        // consumer is another GPU -- so no copy follows the kernel
+        const int top = l0 + L - 1;
+        wd.h_out = static_cast<__nv_bfloat16 *>(
+            top < w->last ? elem_ptr(w->act[top + 1 - w->first], (long)(j % w->k) * dev_in_elems(c->layers, top + 1, B()),
+                                     esz)
+                          : y_last);
         for (int i = 0; i < L; ++i) {
             const int l = l0 + i;
             LstmState st = lstm_state(l, j);
@@ -1114,17 +1112,6 @@ struct Exec {
         cudaEvent_t k0 = kstart(4);
         CK(lstm_wave(wd, w->stream));
         kend(4, k0);
-        k0 = kstart(3);
-        // each layer's output to the next layer's input stash (its backward reads it) / the
-        // stage output
-        for (int i = 0; i < L; ++i) {
-            const int l = l0 + i;
-            void *y = l < w->last ? elem_ptr(w->act[l + 1 - w->first],
-                                             (long)(j % w->k) * dev_in_elems(c->layers, l + 1, B()), esz)
-                                  : y_last;
-            CK(cudaMemcpyAsync(y, lstm_state(l, j).h, (size_t)TB * H * esz, cudaMemcpyDeviceToDevice, w->stream));
-        }
-        kend(3, k0);
     }
 
     void lstm_wave_backward(int l0, int L, int t, int j, const void *G, void *dx, const BwdCtx &bc) {
@@ -1294,22 +1281,6 @@ struct Exec {
         return g;
     }
 
-    static bool packed_taps() {
-        static const int v = [] {
-            const char *e = getenv("PD_CONV_C8");
-            return e ? atoi(e) : 1;
-        }();
-        return v != 0;
-    }
-
-    static bool tapchunk_dw() {
-        static const int v = [] {
-            const char *e = getenv("PD_CONV_DW_ONEGEMM");
-            return e ? atoi(e) : 1;
-        }();
-        return v != 0;
-    }
-
     void conv_forward(int l, int slot, const void *x, void *y) {
         const pd_layer_desc &d = layer(l);
         const int Cp = cpad8(d.in), Co = d.out, Hp = d.height + 2, Wp = d.width + 2;
@@ -1323,7 +1294,7 @@ struct Exec {
         }
         Gemm g;
         g.conv = conv_geom(d, +1);
-        if (Cp == 8 && Co <= 64 && packed_taps()) {
+        if (Cp == 8 && Co <= 64) {
             // RGB first layer: 9 taps x 8 channels packed into one K = 80 block
             g.conv.c8 = 1;
             g.M = (int)M;
@@ -1404,7 +1375,7 @@ struct Exec {
         if (!bf16) {
             CK(conv_dw_f32(static_cast<const float *>(G), static_cast<const float *>(x), gW, B(), d.height, d.width,
                            Cp, Co, w->stream));
-        } else if (Cp == 8 && packed_taps()) {
+        } else if (Cp == 8) {
             // dW[co][tap*8 + ci] for all 9 taps of an 8-channel input in ONE GEMM (N = 72)
             Gemm g;
             g.M = Co;
@@ -1423,7 +1394,7 @@ struct Exec {
             g.out = gW;
             g.ldo = 72;
             CK(run_gemm(1, g, w->stream));
-        } else if (Cp % 64 == 0 && tapchunk_dw()) {
+        } else if (Cp % 64 == 0) {
             // dW[co][tap*Cp + ci] for all 9 taps in ONE GEMM (N = 9*Cp): the dY tile is loaded
             // once per K-block for every tap of the tile instead of once per tap
             Gemm g;
@@ -1501,21 +1472,6 @@ struct Exec {
         kend(2, k0);
     }
 
-    static bool concurrent_dw() {
-        static const int v = [] {
-            const char *e = getenv("PD_OVERLAP_DW");
-            return e ? atoi(e) : 1;
-        }();
-        return v != 0;
-    }
-    static int dw_ctas() {
-        static const int v = [] {
-            const char *e = getenv("PD_DW_CTAS");
-            return e ? atoi(e) : 0;
-        }();
-        return v;
-    }
-
     // Backward of an all-linear stage on the bf16 fused path with the weight-gradient GEMM +
     // optimizer update of layer l (HBM-bound) on a side stream, overlapping the input-gradient
     // GEMM of layer l-1 (L2/latency-bound) on the main stream.  Hazards: dW_l rewrites W_l
@@ -1548,9 +1504,7 @@ struct Exec {
                     if (l + 2 <= last) CK(cudaStreamWaitEvent(w->stream, w->ev_dw[l + 2 - first], 0));
                 }
                 cudaEvent_t k0 = kstart(1);
-                const bool pf = (l2_pf_mask() & 2) && l - 1 >= first && !(s == 0 && l - 1 == 0);
-                gemm_dx(l, (int)rows, d.in, d.out, Gl, d.out, Wl(l, bc.sslot), d.in, x, dx,
-                        pf ? Wl(l - 1, bc.sslot) : nullptr, pf ? (long)layer(l - 1).in * layer(l - 1).out * esz : 0);
+                gemm_dx(l, (int)rows, d.in, d.out, Gl, d.out, Wl(l, bc.sslot), d.in, x, dx);
                 kend(1, k0);
 #ifndef PD_FAULT_NO_DXWAIT
                 // dW_l + update rewrites W_l in place when k_s = 1: after dX_l has read it
@@ -1561,8 +1515,13 @@ struct Exec {
             // side stream: dW_l + fused update, bias
             cudaStream_t main = w->stream;
             w->stream = w->side;
-            cudaEvent_t k0 = kstart(2);
-            {
+            cudaEvent_t k0 = nullptr;
+            if (split_dw(d.out, d.in, (int)rows)) {
+                // long-K weight gradient (the classifier over T*B rows): 2-CTA GEMM -> fp32
+                // gradient -> vectorised update (gemm_dw), not the single-CTA fused epilogue
+                gemm_dw(bc, c->poff[l], d.out, d.in, (int)rows, Gl, d.out, x, d.in);
+            } else {
+                k0 = kstart(2);
                 Gemm g;
                 g.M = d.out;
                 g.N = d.in;
@@ -1586,10 +1545,9 @@ struct Exec {
                 g.b2 = c->cfg.beta2;
                 g.eps = c->cfg.eps;
                 g.step = w->updates_total + 1;
-                g.max_ctas = dw_ctas();
                 CK(run_gemm(1, g, w->stream));
+                kend(2, k0);
             }
-            kend(2, k0);
             k0 = kstart(3);
             bias_update(bc, c->poff[l] + (long)d.out * d.in, Gl, rows, d.out);
             kend(3, k0);
@@ -1647,7 +1605,7 @@ struct Exec {
         BwdCtx bc{fused, gdst, nslot, sslot};
         bool all_linear = true;
         for (int l = w->first; l <= w->last; ++l) all_linear = all_linear && layer(l).kind == PD_LINEAR;
-        if (fused && all_linear && concurrent_dw() && !c->layer_prof) {
+        if (fused && all_linear && !c->layer_prof) {
             const void *dx_first = nullptr;
             if (!(s == 0 && w->first == 0)) {
                 const int Rp = c->plan.stage[s - 1].replicas;
@@ -1730,31 +1688,34 @@ struct Exec {
         const bool adam = c->cfg.optimizer == PD_ADAM;
         const int step = w->updates_total + 1;
         if (Rs > 1) {
-            // round j: wait for every peer's gradient, then one fused reduce + update kernel
+            // round j: reduce-scatter -> update -> all-gather through peer memory.  Every replica
+            // waits for the others' gradients, reduces and updates its 1/R shard of the
+            // parameters (sum in replica order, R7) and stores the new version of that shard
+            // into every replica's next slot (and fp32 master); the round completes when every
+            // replica has posted DONE -- the next forward reads the whole new version
             for (int r = 0; r < Rs; ++r) {
                 if (r == w->replica) continue;
                 Link &L = get_link(c, L_READY, c->worker_id(s, r), w->id);
                 link_wait(c, L, w->stream, j, w->vc);
                 hb_require(c->worker_id(s, r), c->opB, j, "replica gradient reduced before its backward", t);
             }
-            if (bf16) {
-                CK(update_master(w->master, static_cast<__nv_bfloat16 *>(w->wslot[nslot]), nullptr,
-                                 w->rgrad_ptrs + (j & 1) * Rs, Rs, 0, w->P, c->cfg.optimizer, w->adam_m, w->adam_v,
-                                 c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, step, w->stream));
-            } else {
-                // fp32 path: master == latest slot; new version into the next slot
-                const int lslot = vin % w->k;
-                if (nslot != lslot)
-                    CK(cudaMemcpyAsync(w->wslot[nslot], w->wslot[lslot], w->P * 4, cudaMemcpyDeviceToDevice,
-                                       w->stream));
-                CK(update_master(static_cast<float *>(w->wslot[nslot]), nullptr, nullptr, w->rgrad_ptrs + (j & 1) * Rs,
-                                 Rs, 0, w->P, c->cfg.optimizer, w->adam_m, w->adam_v, c->cfg.lr, c->cfg.beta1,
-                                 c->cfg.beta2, c->cfg.eps, step, w->stream));
-            }
+            auto shard_lo = [&](int r) { return (w->P * r / Rs) / 64 * 64; };
+            const long lo = shard_lo(w->replica), hi = w->replica + 1 == Rs ? w->P : shard_lo(w->replica + 1);
+            const float *w_in = bf16 ? w->master : static_cast<const float *>(w->wslot[vin % w->k]);
+            CK(update_shard(w->rgrad_ptrs + (j & 1) * Rs, Rs, lo, hi, w_in, w->sync_f32 + (size_t)nslot * Rs,
+                            bf16 ? w->sync_bf16 + (size_t)nslot * Rs : nullptr, c->cfg.optimizer, w->adam_m, w->adam_v,
+                            c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, step, w->stream));
+            w->replica_bytes += (uint64_t)(Rs - 1) * (hi - lo) * (4 + 4 + (bf16 ? 2 : 0));
             for (int r = 0; r < Rs; ++r) {
                 if (r == w->replica) continue;
                 Link &L = get_link(c, L_DONE, w->id, c->worker_id(s, r));
                 link_post(c, L, w->stream, w->vc);
+            }
+            for (int r = 0; r < Rs; ++r) {
+                if (r == w->replica) continue;
+                Link &L = get_link(c, L_DONE, c->worker_id(s, r), w->id);
+                link_wait(c, L, w->stream, j, w->vc);
+                hb_require(c->worker_id(s, r), c->opU, j, "new version used before every shard was written", t);
             }
         } else if (!bf16) {
             const float *latest = static_cast<const float *>(w->wslot[vin % w->k]);
@@ -1771,15 +1732,31 @@ struct Exec {
         w->fwd_version.erase(j);
     }
 
+    // PD_OP_TRACE=1: every op a worker issues, on stderr (diagnosing a stuck run)
+    static bool op_trace() {
+        static const bool v = getenv("PD_OP_TRACE") != nullptr;
+        return v;
+    }
     void run_ops() {
         const int Rs = c->plan.stage[w->stage].replicas;
         std::vector<Op> ops = worker_ops(Rs, w->replica, k[w->stage], M);
         w->run_base = w->version;
         w->vc.assign(c->nw, 0);
+        // layers inside (not at the bottom of) an LSTM wavefront run: their input is the
+        // previous layer's saved h (decided per run: it depends on the dtype, layer profiling
+        // and the wavefront's co-residency rule)
+        w->wave_inner.assign(w->last - w->first + 1, 0);
+        for (int l = w->first; l <= w->last; ++l) {
+            int st = l;
+            if (lstm_wave_run_of(l, st) > 0 && st < l) w->wave_inner[l - w->first] = 1;
+        }
         for (size_t i = 0; i < ops.size(); ++i) {
             const Op &op = ops[i];
             if (c->abort) throw Abort{};
             w->vc[w->id] = (int32_t)i + 1;  // a post during op i claims ops 0..i complete
+            w->st_op = (int)i;
+            if (op_trace()) fprintf(stderr, "[pd] worker %d op %zu %c t=%d j=%d v=%d\n", w->id, i, op.kind, op.t, op.j,
+                                    w->version);
             if (op.kind == 'F') forward(op.t, op.j);
             else if (op.kind == 'B') backward(op.t, op.j);
             else update(op.t, op.j);
@@ -1789,13 +1766,18 @@ struct Exec {
 
 void worker_thread(pd_ctx *c, Worker *w, int M, std::vector<int> k) {
     tl_launches = 0;
+    tl_worker = w;
+    w->st_where = 0;
     try {
         CK(cudaSetDevice(w->device));
         Exec ex{c, w, M, k, c->cfg.dtype == PD_BF16, c->esz, c->cfg.record_trace >= 2};
         CK(cudaEventRecord(w->run_ev[0], w->stream));
         ex.run_ops();
         CK(cudaEventRecord(w->run_ev[1], w->stream));
+        if (Exec::op_trace()) fprintf(stderr, "[pd] worker %d issued everything, synchronizing\n", w->id);
+        w->st_where = 3;
         CK(cudaStreamSynchronize(w->stream));
+        if (Exec::op_trace()) fprintf(stderr, "[pd] worker %d done\n", w->id);
     } catch (const CudaFail &f) {
         char buf[256];
         snprintf(buf, sizeof buf, "worker %d: %s failed: %s", w->id, f.what, cudaGetErrorString(f.e));
@@ -1807,6 +1789,13 @@ void worker_thread(pd_ctx *c, Worker *w, int M, std::vector<int> k) {
         if (w->stream) cudaStreamSynchronize(w->stream);
     }
     w->launches = tl_launches;
+    w->st_where = 4;
+    tl_worker = nullptr;
+    {
+        std::lock_guard<std::mutex> g(c->done_mu);
+        --c->running;
+    }
+    c->done_cv.notify_all();
 }
 
 }  // namespace
@@ -2031,6 +2020,9 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             w->rgrad[0] = dalloc<float>(P * 4);
             w->rgrad[1] = dalloc<float>(P * 4);
             w->rgrad_ptrs = dalloc<const float *>(sizeof(float *) * 2 * Rs);
+            if (w->k > MAX_SYNC_SLOTS) throw CudaFail{cudaErrorInvalidValue, "too many stash slots on a replicated stage"};
+            w->sync_f32 = dalloc<float *>(sizeof(float *) * w->k * Rs);
+            w->sync_bf16 = dalloc<__nv_bfloat16 *>(sizeof(void *) * w->k * Rs);
         }
         // activation stash for inner layers
         w->act.assign(w->last - w->first + 1, nullptr);
@@ -2072,7 +2064,6 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         if (bf16) {
             w->ws_bytes = 8L * max_elems * 4;  // up to 8 K-splits of the widest activation
             w->ws = dalloc<float>(w->ws_bytes);
-            w->split_counters = dalloc<int>(8192 * sizeof(int));
             w->loss_scratch = dalloc<float>(256);
         }
         if (stage > 0) w->recv = dalloc<void>((size_t)w->D * dev_in_elems(c->layers, w->first, B) * esz);
@@ -2090,6 +2081,11 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
         sh.grad = w->gring;
         sh.rgrad[0] = w->rgrad[0];
         sh.rgrad[1] = w->rgrad[1];
+        if (Rs > 1) {
+            sh.nslots = w->k;
+            for (int q = 0; q < w->k; ++q) sh.wslot[q] = w->wslot[q];
+            sh.master = w->master;
+        }
         sh.flags = w->flags;
         sh.valid = true;
     } catch (const CudaFail &f) {
@@ -2126,6 +2122,13 @@ pd_status pd_export_worker(pd_ctx *c, int stage, int replica, void *blob, size_t
         b.has_rgrad = 1;
         if (cudaIpcGetMemHandle(&b.rgrad0, w->rgrad[0]) != cudaSuccess) return PD_ECUDA;
         if (cudaIpcGetMemHandle(&b.rgrad1, w->rgrad[1]) != cudaSuccess) return PD_ECUDA;
+        b.nslots = w->k;
+        for (int q = 0; q < w->k; ++q)
+            if (cudaIpcGetMemHandle(&b.wslot[q], w->wslot[q]) != cudaSuccess) return PD_ECUDA;
+        if (w->master) {
+            b.has_master = 1;
+            if (cudaIpcGetMemHandle(&b.master, w->master) != cudaSuccess) return PD_ECUDA;
+        }
     }
     if (cudaIpcGetMemHandle(&b.flags, w->flags) != cudaSuccess) return PD_ECUDA;
     std::memcpy(blob, &b, sizeof b);
@@ -2159,6 +2162,10 @@ pd_status pd_import_worker(pd_ctx *c, const void *blob, size_t len) {
     if (b.has_rgrad) {
         ok = ok && open(b.rgrad0, reinterpret_cast<void **>(&sh.rgrad[0]));
         ok = ok && open(b.rgrad1, reinterpret_cast<void **>(&sh.rgrad[1]));
+        if (b.nslots < 0 || b.nslots > MAX_SYNC_SLOTS) ok = false;
+        sh.nslots = ok ? b.nslots : 0;
+        for (int q = 0; q < sh.nslots; ++q) ok = ok && open(b.wslot[q], &sh.wslot[q]);
+        if (b.has_master) ok = ok && open(b.master, reinterpret_cast<void **>(&sh.master));
     }
     ok = ok && open(b.flags, reinterpret_cast<void **>(&sh.flags));
     if (!ok) {
@@ -2248,18 +2255,9 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
     if (c->n_data < 1) return PD_ESTATE;
     for (int id = 0; id < c->nw; ++id)
         if (!c->shared[id].valid) return PD_ESTATE;
-    bool any_local = false, all_local = true;
-    for (auto &w : c->W) {
-        any_local = any_local || (bool)w;
-        all_local = all_local && (bool)w;
-    }
+    bool any_local = false;
+    for (auto &w : c->W) any_local = any_local || (bool)w;
     if (!any_local) return PD_ESTATE;
-    for (auto &w : c->W) {
-        if (!w) continue;
-        int same = 0;
-        for (auto &o : c->W) same += o && o->device == w->device;
-        w->alone = all_local && same == 1;
-    }
     // with a depth override the stash ring must still hold k_s versions at every worker
     try {
         // links (created once; local when both ends are in this process)
@@ -2376,9 +2374,26 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
                 for (int par = 0; par < 2; ++par)
                     for (int r = 0; r < Rs; ++r) ptrs[par * Rs + r] = c->shared[c->worker_id(w->stage, r)].rgrad[par];
                 CK(cudaMemcpy(w->rgrad_ptrs, ptrs.data(), sizeof(float *) * ptrs.size(), cudaMemcpyHostToDevice));
+                std::vector<float *> f32((size_t)w->k * Rs);
+                std::vector<__nv_bfloat16 *> b16((size_t)w->k * Rs);
+                for (int q = 0; q < w->k; ++q)
+                    for (int r = 0; r < Rs; ++r) {
+                        const Shared &ps = c->shared[c->worker_id(w->stage, r)];
+                        if (ps.nslots != w->k) throw CudaFail{cudaErrorInvalidValue, "replica stash depth mismatch"};
+                        if (c->esz == 2) {
+                            f32[(size_t)q * Rs + r] = ps.master;
+                            b16[(size_t)q * Rs + r] = static_cast<__nv_bfloat16 *>(ps.wslot[q]);
+                        } else {
+                            f32[(size_t)q * Rs + r] = static_cast<float *>(ps.wslot[q]);
+                            b16[(size_t)q * Rs + r] = nullptr;
+                        }
+                    }
+                CK(cudaMemcpy(w->sync_f32, f32.data(), sizeof(float *) * f32.size(), cudaMemcpyHostToDevice));
+                CK(cudaMemcpy(w->sync_bf16, b16.data(), sizeof(void *) * b16.size(), cudaMemcpyHostToDevice));
             }
             w->events.clear();
             w->op_ev.clear();
+            w->bytes_sent = w->replica_bytes = 0;
             for (auto &kv : w->kev) kv.clear();
             for (auto &e : w->run_ev)
                 if (!e) CK(cudaEventCreate(&e));
@@ -2402,8 +2417,47 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
     c->vmap.assign((size_t)c->n * M, -1);
     auto t0 = std::chrono::steady_clock::now();
     std::vector<std::thread> th;
+    c->running = 0;
+    for (auto &wp : c->W) c->running += wp ? 1 : 0;
     for (auto &wp : c->W)
-        if (wp) th.emplace_back(worker_thread, c, wp.get(), M, k);
+        if (wp) {
+            wp->st_where = 0;
+            wp->st_op = -1;
+            th.emplace_back(worker_thread, c, wp.get(), M, k);
+        }
+    // watchdog: a run that makes no progress for 60 s is reported once on stderr (per worker:
+    // the op it issues and where its host thread waits) -- diagnosis only, it does not abort
+    {
+        const auto start = std::chrono::steady_clock::now();
+        std::vector<int> last_op(c->nw, -2);
+        auto last_change = start;
+        bool reported = false;
+        for (;;) {
+            {
+                std::unique_lock<std::mutex> g(c->done_mu);
+                if (c->done_cv.wait_for(g, std::chrono::seconds(1), [&] { return c->running == 0; })) break;
+            }
+            bool changed = false;
+            for (auto &wp : c->W)
+                if (wp) {
+                    const int op = wp->st_op.load();
+                    if (op != last_op[wp->id]) last_op[wp->id] = op, changed = true;
+                }
+            const auto now = std::chrono::steady_clock::now();
+            if (changed) last_change = now;
+            if (!reported && now - last_change > std::chrono::seconds(60)) {
+                reported = true;
+                static const char *where[] = {"issuing", "link_post (ring full)", "link_wait", "stream sync", "done"};
+                for (auto &wp : c->W)
+                    if (wp) {
+                        const int wh = wp->st_where.load();
+                        fprintf(stderr, "[pd] watchdog: no progress for 60 s: worker %d (stage %d) op %d, %s (message %ld)\n",
+                                wp->id, wp->stage, wp->st_op.load(), where[wh < 0 || wh > 4 ? 0 : wh],
+                                (long)wp->st_link.load());
+                    }
+            }
+        }
+    }
     for (auto &t : th) t.join();
     c->host_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     if (c->sticky != PD_OK) return c->sticky;
@@ -2440,6 +2494,9 @@ pd_status pd_stage_solo(pd_ctx *c) {
                 const long P = c->poff[last] + (long)align_up(c->pcount[last], 64);
                 sh.rgrad[0] = static_cast<float *>(own((size_t)P * 4));
                 sh.rgrad[1] = static_cast<float *>(own((size_t)P * 4));
+                sh.nslots = c->kalloc[s];
+                for (int q = 0; q < sh.nslots; ++q) sh.wslot[q] = own((size_t)P * esz);
+                if (esz == 2) sh.master = static_cast<float *>(own((size_t)P * 4));
             }
             sh.flags = static_cast<uint32_t *>(own(sizeof(uint32_t) * std::max(1, c->flag_count(s))));
             sh.valid = sh.standin = true;
@@ -2558,6 +2615,7 @@ pd_status pd_get_stats(pd_ctx *c, pd_stats *out) {
         if (!w) continue;
         out->kernel_launches += w->launches;
         out->bytes_sent += w->bytes_sent;
+        out->replica_bytes += w->replica_bytes;
         double busy = 0, span = 0;
         if (!w->op_ev.empty() && w->op_ev.back().second) {
             cudaSetDevice(w->device);
@@ -2706,9 +2764,11 @@ void pd_destroy(pd_ctx *c) {
     for (int id = 0; id < c->nw; ++id) {
         if (c->W[id] || !c->shared[id].valid || c->shared[id].standin) continue;
         Shared &sh = c->shared[id];
-        void *ps[] = {sh.recv, sh.grad, sh.rgrad[0], sh.rgrad[1], sh.flags};
+        void *ps[] = {sh.recv, sh.grad, sh.rgrad[0], sh.rgrad[1], sh.flags, sh.master};
         for (void *p : ps)
             if (p) cudaIpcCloseMemHandle(p);
+        for (int q = 0; q < sh.nslots; ++q)
+            if (sh.wslot[q]) cudaIpcCloseMemHandle(sh.wslot[q]);
     }
     c->W.clear();
     delete c;
@@ -2735,13 +2795,6 @@ extern "C" PD_API pd_status pd_kernel_gemm(const pd_gemm_desc *d, void *stream) 
     g.lr = d->lr; g.b1 = d->beta1; g.b2 = d->beta2; g.eps = d->eps; g.step = d->step;
     g.workspace = d->workspace; g.workspace_bytes = d->workspace_bytes;
     g.ws_zeroed = d->workspace_zeroed;
-    static int *counters = nullptr;  // kernel-level API: one zeroed counter array per process
-    if (d->dtype == PD_BF16 && d->workspace && !counters) {
-        if (cudaMalloc(&counters, 8192 * sizeof(int)) != cudaSuccess || cudaMemset(counters, 0, 8192 * sizeof(int)) != cudaSuccess ||
-            cudaDeviceSynchronize() != cudaSuccess)
-            return PD_ECUDA;
-    }
-    g.split_counters = counters;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     cudaError_t e = d->dtype == PD_BF16 ? gemm_bf16(g, s) : gemm_f32(g, s);
     if (e == cudaErrorInvalidValue) return PD_EINVAL;

@@ -7,7 +7,7 @@ PAPER.md L1225-1231) through exactly the kernel path the full-size bench takes:
                 the 16-layer wavefront (lstm_wave.cu) with its L2-residency split, the
                 long-K (T*B rows) 2-CTA weight-gradient GEMMs, the fused bias updates.
                 The oracle needs ~8 min single-threaded for it, so its expected values are
-                computed once by tools/gen_golden_fullsize.py (which calls only oracle/ and
+                computed once by tests/gen_golden_fullsize.py (which calls only oracle/ and
                 synth/) and stored, sampled, under tests/golden/.
   longk_dw      Linear(256, 256)+ReLU -> Linear(256, 256) applied per token over T = 50,
                 B = 64 (K = T*B = 3200 rows): the default long-K weight-gradient path

@@ -3,7 +3,7 @@
 (tests/fullsize_cases.py), sampled.  Calls only oracle/ and synth/ -- no value here comes
 from the CUDA path.  The oracle is single-threaded; gnmt16_wave takes ~8 minutes.
 
-    python tools/gen_golden_fullsize.py gnmt16_wave [more cases]
+    python tests/gen_golden_fullsize.py gnmt16_wave [more cases]
 """
 import os
 import sys
@@ -11,9 +11,9 @@ import time
 
 import numpy as np
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))  # repo root
 sys.path.insert(0, ROOT)
-sys.path.insert(0, os.path.join(ROOT, "tests"))
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 
 import oracle  # noqa: E402
 import synth  # noqa: E402

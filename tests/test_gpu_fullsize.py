@@ -1,7 +1,7 @@
 """Parity at the bench's full sizes (VERDICT r1 "next round" #2): the 16-layer H = 1024
 wavefront, the default long-K weight-gradient path (K = T*B = 3200) and the packed-tap VGG
 conv1 at 224 x 224, each one bf16 SGD step of a single stage against the oracle's sampled
-deltas (tests/golden/<case>.npz, written by tools/gen_golden_fullsize.py from oracle/ only).
+deltas (tests/golden/<case>.npz, written by tests/gen_golden_fullsize.py from oracle/ only).
 
 Tolerances: parameters within the north star's bf16 2e-2 (max relative error); the deltas
 (= -lr x gradient, where a version or indexing bug would show) within DELTA_TOL of the

@@ -22,7 +22,7 @@ pytestmark = pytest.mark.gpu
 # One layer runs the persistent per-layer kernels; runs of >= 2 layers the wavefront kernel
 # (lstm_wave.cu) unless PD_LSTM_WAVE=0.
 SHAPES = [(2, 256, 16, 6), (1, 512, 40, 5), (1, 1024, 64, 4), (2, 1024, 64, 3)]
-WAVE_SHAPES = [(4, 256, 16, 6), (3, 512, 40, 5), (8, 128, 8, 4), (4, 1024, 64, 3)]
+WAVE_SHAPES = [(4, 256, 16, 6), (3, 512, 40, 5), (8, 128, 8, 4), (4, 1024, 64, 3), (3, 1024, 64, 3)]
 
 
 def _workload(n, H, B, T):

@@ -272,3 +272,23 @@ def test_vertical_sync_second_run_fp32():
     r1 = oracle.run(wl.layers, last, [1] * 4, wl.batch, 9, p0, data, lr=wl.lr, vertical_sync=True)
     r2 = oracle.run(wl.layers, last, [1] * 4, wl.batch, 9, r1.params, data, lr=wl.lr, vertical_sync=True)
     assert torchref.max_rel_err([got[l] for l in range(len(wl.layers))], r2.params) < FP32_TOL
+
+
+@pytest.mark.parametrize("reps,dtype", [([2, 1], pd.PD_FP32), ([3, 1], pd.PD_BF16), ([4], pd.PD_FP32), ([4], pd.PD_BF16)])
+def test_sharded_replica_sync_bytes(reps, dtype):
+    """Replica sync as reduce-scatter -> update -> all-gather (each worker
+    sends and receives (m-1)/m |w| per round): per round every replica reads the other
+    replicas' fp32 gradients for its 1/R shard and stores its shard of the new version into
+    the R-1 peers (fp32 master or fp32 slot, + bf16 slot on the bf16 path), so the whole
+    stage moves (R-1) * P * (4 + 4 [+ 2]) bytes per round -- 2 (R-1)/R |g| per replica on the
+    fp32 path (|g| = 4 P) -- and the parameters still match the oracle's round mean."""
+    wl = synth.workload("mlp4096", reduced=True)
+    last = [7, 15] if len(reps) == 2 else [15]
+    R, M = reps[0], 4 * reps[0]
+    res = run_both(wl, last, reps, M, dtype, lr=0.05 if dtype == pd.PD_BF16 else None)
+    assert_schedule_exact(res)
+    perr, derr = param_errors(res)
+    assert perr < (BF16_TOL if dtype == pd.PD_BF16 else FP32_TOL), (perr, derr)
+    P = sum(-(-synth.param_count(wl.layers[l]) // 64) * 64 for l in range(last[0] + 1))  # 256-byte layer blocks
+    per_param = 4 + 4 + (2 if dtype == pd.PD_BF16 else 0)
+    assert res["stats"]["replica_bytes"] == (M // R) * (R - 1) * P * per_param

@@ -8,6 +8,11 @@
    straight (max_replicas = 1) -- with the predicted throughput B / A(0 -> N, m).
 3. Predicted vs real (Fig. 15) where this host can run the plan: the 1-GPU
    plan is run at full speed and its samples/s set against the prediction.
+3b. Predicted vs real beyond one GPU with --real-stages: every stage of each straight plan is
+   run alone on this GPU (pd_stage_solo: neighbours replaced by infinitely fast stand-ins),
+   and B * min_s R_s / t_s of the measured stage times is set against the optimizer's
+   B / A(0 -> N, m) (the pipeline's throughput is its slowest stage's, L775-777; transfers
+   and the fill/drain bubble are not in either number).
 4. Depth sweep (Fig. 18) with --depth-sweep: a straight pipeline of the
    largest --gpus count run as virtual workers on this GPU with pd_run(M, D) for
    D = 1 .. n+2 -- per-stage stash memory (weight versions k_s(D) and activation rings, from
@@ -74,6 +79,7 @@ def main():
     ap.add_argument("--gpus", type=int, nargs="+", default=[1, 2, 4, 8])
     ap.add_argument("--profile-minibatches", type=int, default=8)
     ap.add_argument("--depth-sweep", action="store_true")
+    ap.add_argument("--real-stages", action="store_true")
     ap.add_argument("--json", default="")
     a = ap.parse_args()
     wl = synth.workload(a.config)
@@ -112,6 +118,25 @@ def main():
     print(f"1 GPU: predicted {pred:.1f} samples/s (sum of serialised per-layer times), real {real:.1f} "
           f"(ratio {real / pred:.2f}; the real run overlaps dW with dX and replays graphs)")
     res["predicted_vs_real_1gpu"] = {"predicted": pred, "real": real, "ratio": real / pred}
+
+    if a.real_stages:
+        import bench
+        p0 = synth.init_params(L)
+        data = synth.make_data(wl, 8)
+        for pl in plans:
+            if pl["kind"] != "straight" or pl["gpus"] < 2:
+                continue
+            p = pd.Plan(pl["stages"], pl["noam"], 0.0)
+            ts = []
+            for s_ in range(len(p.stages)):
+                r = bench.solo_stage(p, s_, L, wl, p0, data, 8, 8 * p.stages[s_][2], runs=2, warm=1, profile=False)
+                ts.append(r["ms_per_minibatch"])
+            real = B * min(st[2] / (t / 1e3) for st, t in zip(p.stages, ts))
+            pl["stage_ms_solo"] = ts
+            pl["real_from_stages_samples_per_s"] = real
+            pl["real_over_predicted"] = real / pl["predicted_samples_per_s"]
+            print(f"N={pl['gpus']} straight: stage ms {[round(t, 3) for t in ts]} -> {real:10.1f} samples/s "
+                  f"(predicted {pl['predicted_samples_per_s']:10.1f}, ratio {real / pl['predicted_samples_per_s']:.2f})")
 
     if a.depth_sweep:
         N = max(a.gpus)
