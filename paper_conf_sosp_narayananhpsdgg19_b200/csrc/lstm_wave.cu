@@ -100,23 +100,6 @@ __device__ __forceinline__ void st_async_v4(uint32_t dst, const float *v, uint32
                  "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "r"(bar)
                  : "memory");
 }
-// TMEM-resident weights (forward): the accumulators take TMEM columns [0, 128); K-block i of
-// the resident set occupies columns 128 + 32 i (128 lanes = gate rows, 64 bf16 of K packed two
-// per 32-bit column -- the tcgen05 A-operand layout, filled by tcgen05.cp from the same
-// 128B-swizzled K-major smem tile the MMA would read)
-constexpr int MAX_KRES = 12;
-__device__ __forceinline__ void tc_cp_128x256b(uint32_t taddr, uint64_t sdesc) {
-    asm volatile("tcgen05.cp.cta_group::1.128x256b [%0], %1;" ::"r"(taddr), "l"(sdesc) : "memory");
-}
-// D += A (TMEM) x B (smem)
-__device__ __forceinline__ void tc_mma_ta(uint32_t d_tmem, uint32_t a_tmem, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}" ::"r"(d_tmem),
-        "r"(a_tmem), "l"(bdesc), "r"(idesc), "r"(acc));
-}
-
 __device__ __forceinline__ void arrive_remote(uint32_t bar_local, int rank) {
     asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(mapa_cluster(bar_local, rank))
                  : "memory");
@@ -167,8 +150,6 @@ struct WaveArgs {
     const __nv_bfloat16 *dy_top;  // backward: gradient w.r.t. the top layer's output [T][B][H]
     unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
     unsigned long long *probe;    // tools only (PD_WAVE_PROBE): [CTA][visit < PROBE_V][8] %globaltimer
-    int kres;                     // forward, one item per cluster: K-blocks of the item's weights kept in
-                                  // TMEM for the whole launch (0 = off, <= MAX_KRES)
     int keep_layers;              // weights of layers < keep_layers load with L2 evict_last, the rest
                                   // evict_first (0: no hint): a fixed subset stays L2-resident across
                                   // waves instead of the whole run thrashing the 126 MB L2
@@ -277,21 +258,8 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
         mbar_init(rempty, CL > 1 ? CL - 1 : 1);  // every peer that receives from this CTA releases
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    // resident weights (forward, one item per cluster): global K-blocks [r_lo, r_lo + nres) of
-    // the item's t > 0 range (x part W_ih, then h part W_hh)
-    int r_l = 0, r_tile = 0, r_lo = 0, nres = 0;
-    if (!BWD && a.kres > 0 && (int)(gridDim.x / CL) >= a.L * a.tiles) {
-        const int i = (int)(blockIdx.x / CL);
-        r_l = i / a.tiles;
-        r_tile = i % a.tiles;
-        const int tot = 2 * (a.H / 64);
-        r_lo = tot * rank / CL;
-        nres = min(a.kres, tot * (rank + 1) / CL - r_lo);
-    }
-    const uint32_t tmem_cols = nres > 0 ? 512u : 128u;
     if (warp == 3) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "r"(tmem_cols));
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" ::"r"(smem_u32(tmem_slot)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     tc_fence_before();
@@ -308,27 +276,11 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
         int l, tile, t, s = 0, pv = 0;
         uint32_t ph = 0;
         const uint64_t pol_last = l2_policy_evict_last(), pol_first = l2_policy_evict_first();
-        // the resident K-blocks' weights, once: they pass through the ring into TMEM
-        for (int i = 0; i < nres; ++i) {
-            mbar_wait(em0 + 8 * s, ph ^ 1);
-            const uint32_t dst = smem_u32(sm + s * STAGE);
-            mbar_expect_tx(fw0 + 8 * s, ATILE);
-            const int kb = r_lo + i, n0 = a.H / 64;
-            const CUtensorMap *w = kb >= n0 ? &m.w_hh[r_l] : &m.w_ih[r_l];
-            const int k = (kb >= n0 ? kb - n0 : kb) * 64;
-            for (int g = 0; g < 4; ++g) tma_load_2d(dst + g * 4096, w, fw0 + 8 * s, k, g * H + r_tile * 32);
-            if (++s == S) s = 0, ph ^= 1;
-        }
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             for (int kb = ik.lo; kb < ik.hi; ++kb) {
                 mbar_wait(em0 + 8 * s, ph ^ 1);
                 if (kb == ik.lo) probe(a, pv, 0);
-                if (kb >= r_lo && kb < r_lo + nres) {  // in TMEM: the stage carries only the activations
-                    mbar_arrive(fw0 + 8 * s);
-                    if (++s == S) s = 0, ph ^= 1;
-                    continue;
-                }
                 const uint32_t dst = smem_u32(sm + s * STAGE);
                 mbar_expect_tx(fw0 + 8 * s, ATILE);
                 const bool p1 = kb >= ik.n0;
@@ -358,11 +310,6 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
         ItemIter<CL> it;
         int l, tile, t, s = 0, pv = -1;
         uint32_t ph = 0;
-        for (int i = 0; i < nres; ++i) {  // the resident weights' ring stages carry no activations
-            mbar_wait(em0 + 8 * s, ph ^ 1);
-            mbar_arrive(fx0 + 8 * s);
-            if (++s == S) s = 0, ph ^= 1;
-        }
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             ++pv;
@@ -399,16 +346,6 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
         ItemIter<CL> it;
         int l, tile, t, s = 0, acc = 0, pv = 0;
         uint32_t ph = 0, aph[2] = {0, 0};
-        for (int i = 0; i < nres; ++i) {  // resident weights: smem -> TMEM columns 128 + 32 i
-            mbar_wait(fw0 + 8 * s, ph);
-            mbar_wait(fx0 + 8 * s, ph);
-            tc_fence_after();
-            const uint32_t sa = smem_u32(sm + s * STAGE);
-#pragma unroll
-            for (int kk = 0; kk < 4; ++kk) tc_cp_128x256b(tmem + 128 + i * 32 + kk * 8, smem_desc(sa + kk * 32, 16, 1024));
-            tc_commit(em0 + 8 * s);
-            if (++s == S) s = 0, ph ^= 1;
-        }
         while (it.next(a, BWD, l, tile, t)) {
             const ItemK ik = item_k(a, BWD, l, t, rank, CL);
             mbar_wait(ae0 + 8 * acc, aph[acc] ^ 1);  // epilogue drained this accumulator
@@ -419,17 +356,11 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
                 mbar_wait(fx0 + 8 * s, ph);
                 tc_fence_after();
                 const uint32_t sa = smem_u32(sm + s * STAGE), sb = sa + ATILE;
-                const bool res = kb >= r_lo && kb < r_lo + nres;
 #pragma unroll
                 for (int kk = 0; kk < 4; ++kk) {
+                    const uint64_t ad = BWD ? smem_desc(sa + kk * 2048, 8192, 1024) : smem_desc(sa + kk * 32, 16, 1024);
                     const uint64_t bd = smem_desc(sb + kk * 32, 16, 1024);
-                    const uint32_t accf = (kb > ik.lo || kk) ? 1u : 0u;
-                    if (res) {
-                        tc_mma_ta(d, tmem + 128 + (kb - r_lo) * 32 + kk * 8, bd, idesc, accf);
-                    } else {
-                        const uint64_t ad = BWD ? smem_desc(sa + kk * 2048, 8192, 1024) : smem_desc(sa + kk * 32, 16, 1024);
-                        tc_mma(d, ad, bd, idesc, accf);
-                    }
+                    tc_mma(d, ad, bd, idesc, (kb > ik.lo || kk) ? 1u : 0u);
                 }
                 tc_commit(em0 + 8 * s);
                 if (++s == S) s = 0, ph ^= 1;
@@ -707,7 +638,7 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
     tc_fence_before();
     __syncthreads();
     if (CL > 1) cluster_sync_all();  // no peer st.async / arrive may target an exited CTA
-    if (warp == 3) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(tmem_cols));
+    if (warp == 3) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tmem));
 }
 
 int num_sm() {
@@ -822,13 +753,6 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     const int items = L * a.tiles;
     const int cl = choose_cl(w.bwd, items);
-    // forward with one item per cluster (a pipeline stage's short run): keep MAX_KRES K-blocks of
-    // each item's weights in TMEM for the whole launch (PD_WAVE_KRES overrides, 0 = off)
-    {
-        const char *ek = getenv("PD_WAVE_KRES");
-        const int kres = ek ? atoi(ek) : MAX_KRES;
-        a.kres = (!w.bwd && items <= max_clusters(false, cl)) ? std::max(0, std::min(kres, MAX_KRES)) : 0;
-    }
     const int grid = cl * std::min(items, max_clusters(w.bwd, cl));
     {
         // PD_WAVE_L2_MB: MB of the run's weights kept L2-resident (whole layers, evict_last; the
