@@ -443,9 +443,11 @@ def main():
     ap.add_argument("--minibatches", type=int, default=0,
                     help="minibatches per step (default 8 for one stage; 1024 for n > 1 stages: steady state, "
                          "fill/drain bubble (n-1)/(M+n-1) < 1 %%)")
-    ap.add_argument("--stage-plan", type=int, default=8,
+    ap.add_argument("--stage-plan", type=int, default=-1,
                     help="per-stage table (solo mode, pd_stage_solo): each stage of the N-GPU plan measured "
-                         "alone on this GPU, projected N-GPU throughput = B min_s R_s / t_s (L775-777); 0 = off")
+                         "alone on this GPU, projected N-GPU throughput = B min_s R_s / t_s (L775-777); 0 = off; "
+                         "default: the GPU count BASELINE.json names for the config (GNMT-16 8, GNMT-8 4, "
+                         "MLP-4096 4, VGG-16 8 as 7-1)")
     ap.add_argument("--stage", type=int, default=-1,
                     help="measure only this stage of the --stage-plan plan in solo mode (for ncu) and exit")
     ap.add_argument("--solo-runs", type=int, default=3,
@@ -461,6 +463,8 @@ def main():
     ap.add_argument("--sync", default="stash", choices=["stash", "vertical"],
                     help="weight stashing (default) or vertical sync (§3.3; straight plans)")
     args = ap.parse_args()
+    if args.stage_plan < 0:
+        args.stage_plan = {"gnmt16": 8, "gnmt8": 4, "mlp4096": 4, "vgg16": 8}[args.config]
     if args.cpu_batch <= 0:
         args.cpu_batch = 8 if args.config == "mlp4096" else 1
     if args.impl == "reference":

@@ -37,7 +37,7 @@ def load(path):
     for r in rows[1:]:
         d = launches.setdefault(r[ii], {"name": r[ki]})
         v = float(r[vi].replace(",", "")) if r[vi] not in ("", "n/a") else 0.0
-        scale = {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "byte": 1e-9, "Kbyte": 1e-6, "Mbyte": 1e-3,
+        scale = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3, "byte": 1e-9, "Kbyte": 1e-6, "Mbyte": 1e-3,
                  "Gbyte": 1.0}.get(r[ui], 1.0)
         d[r[mi]] = v * scale
     return list(launches.values())
