@@ -409,7 +409,7 @@ def stage_table(args, wl, peaks, n_plan, only=-1):
         if only >= 0 and s != only:
             continue
         R = plan.stages[s][2]
-        M_solo = 8 * R
+        M_solo = 8 * int(np.lcm.reduce([st[2] for st in plan.stages]))  # pd_run: a multiple of every R_s
         quick = getattr(args, "solo_runs", 3) <= 1
         r = solo_stage(plan, s, layers, wl, p0, data, n_data, M_solo, runs=max(1, getattr(args, "solo_runs", 3)),
                        warm=1 if quick else 2, profile=not quick)

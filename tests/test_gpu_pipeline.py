@@ -292,3 +292,30 @@ def test_sharded_replica_sync_bytes(reps, dtype):
     P = sum(-(-synth.param_count(wl.layers[l]) // 64) * 64 for l in range(last[0] + 1))  # 256-byte layer blocks
     per_param = 4 + 4 + (2 if dtype == pd.PD_BF16 else 0)
     assert res["stats"]["replica_bytes"] == (M // R) * (R - 1) * P * per_param
+
+
+@pytest.mark.parametrize("stage", [0, 1, 2])
+def test_stage_solo_mode(stage):
+    """pd_stage_solo (the bench's per-stage table): one stage of a 3-stage plan runs its static
+    op list alone -- absent neighbours replaced by stand-ins, incoming flags pre-posted -- and
+    completes with the trace the schedule prescribes for that worker (same F/B/U order and
+    versions as the oracle's trace of the full pipeline)."""
+    import oracle
+    from paper_conf_sosp_narayananhpsdgg19_b200.session import Pipeline, workers_of
+    wl = synth.workload("mlp4096", reduced=True)
+    last, M = [4, 9, 15], 9
+    plan = pd.Plan.manual(last, [1, 1, 1])
+    wid = [w for w, s, r, g in workers_of(plan) if s == stage][0]
+    p0 = synth.init_params(wl.layers)
+    data = synth.make_data(wl, 3)
+    with Pipeline(plan, wl.layers, p0, dtype=pd.PD_BF16, lr=0.05, minibatch=wl.batch, local=lambda w: w == wid,
+                  solo=True) as P:
+        P.set_data(*data, 3)
+        P.run(M)
+        P.run(M)  # a second run continues from the stand-ins' pre-posted flags
+        got = [t[:8] for t in P.trace()]
+    ref = oracle.run(wl.layers, last, [1, 1, 1], wl.batch, M, p0, data, lr=0.05, math=False)
+    want = [e for e in ref.events if e[1] == stage]
+    # versions continue from the first run: M updates per run on every stage
+    want = [(a, b, c, d, k, t, vi + M, vo + M) for (a, b, c, d, k, t, vi, vo) in want]
+    assert got == want
