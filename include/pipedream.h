@@ -60,10 +60,26 @@ typedef struct {
     uint64_t param_bytes;
 } pd_layer_profile;
 
+#define PD_MAX_LEVELS 4
+
 typedef struct {
     double bandwidth_Bps; /* B_1 of the single topology level (R13); <= 0 => 900e9 (NVLink 5)   */
     int max_replicas;     /* 0 = unconstrained; 1 = straight pipeline; k = at most k per stage  */
     int comm_model;       /* 0 = literal L903-927 formula (default), 1 = per-link ring (R11)    */
+    /* Hierarchical topology (Fig. 7), lowest level first: level k = 1..num_levels
+     * is level_size[k-1] components of level k-1 joined by links of level_bw[k-1] bytes/s
+     * (level 0 = one GPU).  num_levels 0 = one level (level_size = num_gpus, level_bw =
+     * bandwidth_Bps); otherwise the product of level_size must equal num_gpus.  The DP runs
+     * from the lowest level up (A^k built on A^{k-1}); max_replicas bounds the replication
+     * chosen at every level.  The plan comes back flattened: a level-k stage replicated m'
+     * times over level-(k-1) components runs its layers' level-(k-1) plan inside each
+     * component, so each of those sub-stages is one stage replicated m' x (its own factor).
+     * first_gpu stays consecutive (R18); routing t mod R_s keeps a minibatch inside one
+     * component if replica rho is placed on component rho mod m' (multi-node placement is
+     * the caller's). */
+    int num_levels;
+    int level_size[PD_MAX_LEVELS];
+    double level_bw[PD_MAX_LEVELS];
 } pd_plan_opts;
 
 #define PD_MAX_STAGES 64

@@ -66,6 +66,8 @@ def lib():
         L.orc_plan.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int, C.c_int, C.c_double,
                                C.c_int, C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p,
                                C.c_void_p]
+        L.orc_plan_levels.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int, C.c_int, C.c_void_p, C.c_void_p,
+                                      C.c_int, C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
         _lib = L
     return _lib
 
@@ -229,5 +231,29 @@ def plan(T, a, w, gpus, bandwidth=900e9, max_replicas=0, comm_model=0) -> Plan:
         raise ValueError("infeasible")
     if rc != 0:
         raise ValueError(f"orc_plan returned {rc}")
+    n = ns.value
+    return Plan([int(x) for x in sl[:n]], [int(x) for x in sr[:n]], noam.value, slow.value)
+
+
+def plan_levels(T, a, w, levels, max_replicas=0, comm_model=0) -> Plan:
+    """Hierarchical §3.1 partitioner (Fig. 7): levels = [(m_1, B_1), ..., (m_L, B_L)], lowest
+    level first; GPUs = prod m_k.  The plan comes back flattened (see oracle.cpp)."""
+    T = np.ascontiguousarray(T, np.float64)
+    a = np.ascontiguousarray(a, np.uint64)
+    w = np.ascontiguousarray(w, np.uint64)
+    N = len(T)
+    lm = np.ascontiguousarray([m for m, _ in levels], np.int32)
+    lb = np.ascontiguousarray([b for _, b in levels], np.float64)
+    ns = C.c_int(0)
+    sl = np.zeros(N, np.int32)
+    sr = np.zeros(N, np.int32)
+    noam = C.c_int(0)
+    slow = C.c_double(0)
+    rc = lib().orc_plan_levels(_ptr(T), _ptr(a), _ptr(w), N, len(levels), _ptr(lm), _ptr(lb), max_replicas, comm_model,
+                               C.byref(ns), _ptr(sl), _ptr(sr), C.byref(noam), C.byref(slow))
+    if rc == -7:
+        raise ValueError("infeasible")
+    if rc != 0:
+        raise ValueError(f"orc_plan_levels returned {rc}")
     n = ns.value
     return Plan([int(x) for x in sl[:n]], [int(x) for x in sr[:n]], noam.value, slow.value)

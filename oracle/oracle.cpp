@@ -29,6 +29,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <functional>
 #include <vector>
 
 extern "C" {
@@ -920,6 +921,113 @@ int orc_plan(const double *T, const unsigned long long *a, const unsigned long l
     }
     int n = (int)lasts.size();
     for (int q = 0; q < n; q++) { stage_last[q] = lasts[n - 1 - q]; stage_replicas[q] = reps[n - 1 - q]; }
+    *n_stages = n;
+    *noam = ceil_div(gpus, stage_replicas[0]);
+    *slowest = best;
+    return 0;
+}
+
+/*
+ * §3.1 partitioner over a hierarchical topology (Fig. 7): level k (k = 1..L) is
+ * made of m_k components of level k-1 joined by links of bandwidth B_k; level 0 is one GPU
+ * (m_0 = 1).  Solved from the lowest level up (L881-885):
+ *   A^0(i->j, m_0) = sum_{l=i..j} T_l                                         (L967-971)
+ *   T^k(i->j, m) = max( A^{k-1}(i->j, m_{k-1}), C_k ) / m,  C_k = 2 (m-1) sum w_l / B_k
+ *                                          (comm_model 1: C_k / m)             (L903-927)
+ *   A^k(i->j, m) = min( T^k(i->j, m),
+ *                  min_{i<=s<j} min_{1<=m'<m} max( A^k(i->s, m-m'), 2 a_s / B_k, T^k(s+1->j, m') ) )
+ *                                                                              (L931-941)
+ *   A^k(i->j, 1) = A^{k-1}(i->j, m_{k-1}) follows from T^k(i->j, 1) (L971-975).
+ * Ties as in orc_plan.  max_replicas bounds the m chosen at every level.  The plan is
+ * returned flattened: a level-k stage replicated m' times over level-(k-1) components runs
+ * the level-(k-1) plan of its layers inside each component, so each of those sub-stages
+ * becomes one stage replicated m' x (its own replication).  gpus = prod m_k.
+ */
+int orc_plan_levels(const double *T, const unsigned long long *a, const unsigned long long *w, int N, int n_levels,
+                    const int *level_m, const double *level_bw, int max_replicas, int comm_model, int *n_stages,
+                    int *stage_last, int *stage_replicas, int *noam, double *slowest) {
+    if (N < 1 || n_levels < 1) return -1;
+    int gpus = 1;
+    for (int k = 0; k < n_levels; k++) {
+        if (level_m[k] < 1 || !(level_bw[k] > 0)) return -1;
+        gpus *= level_m[k];
+    }
+    const double INF = 1e300;
+    /* per level: A[i][j][m], argmin split and m' */
+    struct Level { int mk; double bw; std::vector<double> A; std::vector<int> bs, bm; };
+    std::vector<Level> lev(n_levels);
+    std::vector<double> below((long)N * N, 0.0);  /* A^{k-1}(i->j, m_{k-1}) */
+    for (int i = 0; i < N; i++)
+        for (int j = i; j < N; j++) {
+            double s = 0.0;
+            for (int l = i; l <= j; l++) s += T[l];
+            below[(long)i * N + j] = s;
+        }
+    for (int k = 0; k < n_levels; k++) {
+        Level &L = lev[k];
+        L.mk = level_m[k];
+        L.bw = level_bw[k];
+        const int M1 = L.mk + 1;
+        L.A.assign((long)N * N * M1, INF);
+        L.bs.assign((long)N * N * M1, -1);
+        L.bm.assign((long)N * N * M1, -1);
+        auto id = [&](int i, int j, int m) { return ((long)i * N + j) * M1 + m; };
+        auto Tk = [&](int i, int j, int m) -> double {
+            if (max_replicas > 0 && m > max_replicas) return INF;
+            double wsum = 0.0;
+            for (int l = i; l <= j; l++) wsum += (double)w[l];
+            double comm = comm_model == 1 ? 2.0 * (m - 1) * wsum / ((double)m * L.bw) : 2.0 * (m - 1) * wsum / L.bw;
+            double comp = below[(long)i * N + j];
+            if (!(comp < INF)) return INF;  /* no level-(k-1) plan for these layers: none here either */
+            return (comp > comm ? comp : comm) / (double)m;
+        };
+        for (int len = 1; len <= N; len++)
+            for (int i = 0; i + len - 1 < N; i++) {
+                int j = i + len - 1;
+                for (int m = 1; m <= L.mk; m++) {
+                    double best = Tk(i, j, m);
+                    int bsv = -1, bmv = -1;
+                    for (int s = i; s < j; s++)
+                        for (int mp = 1; mp < m; mp++) {
+                            double v = L.A[id(i, s, m - mp)];
+                            double c = 2.0 * (double)a[s] / L.bw;
+                            double y = Tk(s + 1, j, mp);
+                            if (c > v) v = c;
+                            if (y > v) v = y;
+                            if (v < best) { best = v; bsv = s; bmv = mp; }
+                        }
+                    L.A[id(i, j, m)] = best; L.bs[id(i, j, m)] = bsv; L.bm[id(i, j, m)] = bmv;
+                }
+            }
+        for (int i = 0; i < N; i++)
+            for (int j = i; j < N; j++) below[(long)i * N + j] = L.A[id(i, j, L.mk)];
+    }
+    const Level &top = lev[n_levels - 1];
+    double best = top.A[((long)0 * N + (N - 1)) * (top.mk + 1) + top.mk];
+    if (!(best < INF)) return -7;
+    /* expand level k's plan of layers i..j on m components, each stage replicated `mult` more times */
+    std::vector<int> lasts, reps;
+    std::function<void(int, int, int, int, int)> expand = [&](int k, int i, int j, int m, int mult) {
+        const Level &L = lev[k];
+        auto id = [&](int ii, int jj, int mm) { return ((long)ii * N + jj) * (L.mk + 1) + mm; };
+        std::vector<int> sl, sr;  /* this level's stages, last first */
+        int jj = j, mm = m;
+        for (;;) {
+            int s = L.bs[id(i, jj, mm)], mp = L.bm[id(i, jj, mm)];
+            if (s < 0) { sl.push_back(jj); sr.push_back(mm); break; }
+            sl.push_back(jj); sr.push_back(mp);
+            jj = s; mm -= mp;
+        }
+        int first = i;
+        for (int q = (int)sl.size() - 1; q >= 0; q--) {
+            if (k == 0) { lasts.push_back(sl[q]); reps.push_back(mult * sr[q]); }
+            else expand(k - 1, first, sl[q], lev[k - 1].mk, mult * sr[q]);
+            first = sl[q] + 1;
+        }
+    };
+    expand(n_levels - 1, 0, N - 1, top.mk, 1);
+    int n = (int)lasts.size();
+    for (int q = 0; q < n; q++) { stage_last[q] = lasts[q]; stage_replicas[q] = reps[q]; }
     *n_stages = n;
     *noam = ceil_div(gpus, stage_replicas[0]);
     *slowest = best;

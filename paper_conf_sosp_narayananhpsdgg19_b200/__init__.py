@@ -47,8 +47,13 @@ class LayerProfile(C.Structure):
     _fields_ = [("compute_s", C.c_double), ("act_bytes", C.c_uint64), ("param_bytes", C.c_uint64)]
 
 
+PD_MAX_LEVELS = 4
+
+
 class PlanOpts(C.Structure):
-    _fields_ = [("bandwidth_Bps", C.c_double), ("max_replicas", C.c_int), ("comm_model", C.c_int)]
+    _fields_ = [("bandwidth_Bps", C.c_double), ("max_replicas", C.c_int), ("comm_model", C.c_int),
+                ("num_levels", C.c_int), ("level_size", C.c_int * PD_MAX_LEVELS),
+                ("level_bw", C.c_double * PD_MAX_LEVELS)]
 
 
 class StageDesc(C.Structure):
@@ -212,12 +217,21 @@ class Plan:
         return plan
 
 
-def pd_plan(compute_s, act_bytes, param_bytes, num_gpus, bandwidth_Bps=0.0, max_replicas=0, comm_model=0) -> Plan:
+def pd_plan(compute_s, act_bytes, param_bytes, num_gpus, bandwidth_Bps=0.0, max_replicas=0, comm_model=0,
+            levels=None) -> Plan:
+    """levels: optional [(m_1, B_1), ..., (m_L, B_L)] hierarchy (Fig. 7), lowest level first."""
     n = len(compute_s)
     prof = (LayerProfile * n)()
     for k in range(n):
         prof[k] = LayerProfile(float(compute_s[k]), int(act_bytes[k]), int(param_bytes[k]))
     opts = PlanOpts(bandwidth_Bps, max_replicas, comm_model)
+    if levels:
+        if len(levels) > PD_MAX_LEVELS:
+            raise ValueError("too many topology levels")
+        opts.num_levels = len(levels)
+        for k, (m, bw) in enumerate(levels):
+            opts.level_size[k] = int(m)
+            opts.level_bw[k] = float(bw)
     out = PlanT()
     _check(lib.pd_plan(prof, n, num_gpus, C.byref(opts), C.byref(out)))
     return Plan.from_c(out)

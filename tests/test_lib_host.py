@@ -203,3 +203,37 @@ def test_stage_solo_needs_a_local_worker():
         pd.pd_stage_solo(ctx)
     assert ei.value.status == pd.PD_ESTATE
     pd.pd_destroy(ctx)
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_pd_plan_hierarchical_bit_exact_with_oracle(seed):
+    """Fig. 7 multi-level topology: the library's level-by-level DP and
+    flattened plan equal the oracle's (itself pinned to hierarchical brute force)."""
+    rng = np.random.default_rng(300 + seed)
+    N = int(rng.integers(1, 12))
+    T, a, w = synth.random_profile(rng, N)
+    levels = [[(4, 900e9), (2, 25e9)], [(2, 900e9), (2, 50e9), (2, 12.5e9)], [(8, 900e9)], [(3, 600e9), (3, 10e9)]][seed % 4]
+    G = int(np.prod([m for m, _ in levels]))
+    for max_rep in (0, 1, 2):
+        for cm in (0, 1):
+            try:
+                ref = oracle.plan_levels(T, a, w, levels, max_rep, cm)
+            except ValueError:
+                with pytest.raises(pd.PDError) as ei:
+                    pd.pd_plan(T, a, w, G, 0.0, max_rep, cm, levels=levels)
+                assert ei.value.status == pd.PD_EINFEASIBLE
+                continue
+            got = pd.pd_plan(T, a, w, G, 0.0, max_rep, cm, levels=levels)
+            assert (got.stage_last, got.replicas, got.noam) == (ref.stage_last, ref.replicas, ref.noam)
+            assert got.slowest_stage_s == ref.slowest
+            assert sum(got.replicas) == G
+
+
+def test_pd_plan_hierarchy_validation():
+    T, a, w = [1e-3] * 4, [1 << 20] * 4, [1 << 20] * 4
+    with pytest.raises(pd.PDError) as ei:  # product of level sizes must be the GPU count
+        pd.pd_plan(T, a, w, 8, levels=[(4, 900e9), (3, 25e9)])
+    assert ei.value.status == pd.PD_EINVAL
+    one = pd.pd_plan(T, a, w, 8, 900e9)
+    same = pd.pd_plan(T, a, w, 8, levels=[(8, 900e9)])
+    assert (one.stages, one.slowest_stage_s) == (same.stages, same.slowest_stage_s)
