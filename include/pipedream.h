@@ -242,6 +242,20 @@ PD_API pd_status pd_run(pd_ctx *ctx, int num_minibatches, int noam);
  *         PD_ECUDA. */
 PD_API pd_status pd_stage_solo(pd_ctx *ctx);
 
+/* Per-stage checkpointing (L1407-1413): every LOCAL worker writes its own state to
+ * `<dir>/stage<s>_replica<r>.pdckpt` -- the latest weights in fp32 (the master on the bf16
+ * path), the Adam m and v, its version and update count -- with no coordination across
+ * workers ("each stage dumps its model parameters locally").  Call between pd_run calls: a
+ * run ends drained, so the latest version is the only live one.  pd_load_checkpoint restores
+ * a context created with the same plan, layers and config (after pd_stage_init, before the
+ * next pd_run): every version slot gets the checkpointed weights, training continues as if
+ * uninterrupted (same versions, same optimizer step).  A worker whose file is missing or
+ * does not match (stage, replica, parameter count, dtype, optimizer) fails the call.
+ * Errors: PD_EINVAL (NULL dir, mismatching file), PD_ESTATE, PD_ECUDA, PD_ENOMEM; an I/O
+ * failure returns PD_EINVAL with the path in pd_last_error. */
+PD_API pd_status pd_save_checkpoint(pd_ctx *ctx, const char *dir);
+PD_API pd_status pd_load_checkpoint(pd_ctx *ctx, const char *dir);
+
 /* Copies the LATEST fp32 parameters of `layer` (master weights) to host_out.  The layer's
  * stage must have a local worker (replica 0 preferred).  count must equal the layer's
  * parameter count (PD_EINVAL otherwise). */

@@ -138,6 +138,8 @@ def _load():
         "pd_set_layer_profiling": [vp, i],
         "pd_get_layer_times": [vp, vp, vp, st],
         "pd_stage_solo": [vp],
+        "pd_save_checkpoint": [vp, C.c_char_p],
+        "pd_load_checkpoint": [vp, C.c_char_p],
     }
     for name, args in sigs.items():
         f = getattr(L, name)
@@ -158,7 +160,7 @@ EXPORTED = ["pd_plan", "pd_create", "pd_stage_init", "pd_export_worker", "pd_imp
             "pd_get_params", "pd_get_trace", "pd_get_version_map", "pd_get_losses", "pd_get_stats", "pd_destroy",
             "pd_strerror", "pd_last_error", "pd_inflight", "pd_kernel_gemm", "pd_kernel_softmax_ce",
             "pd_kernel_lstm_rec", "pd_profile", "pd_set_layer_profiling", "pd_get_layer_times",
-            "pd_set_timing", "pd_kernel_bias_grad", "pd_stage_solo"]
+            "pd_set_timing", "pd_kernel_bias_grad", "pd_stage_solo", "pd_save_checkpoint", "pd_load_checkpoint"]
 
 
 def _strerror(s):
@@ -368,6 +370,15 @@ def pd_get_layer_times(ctx, num_layers: int):
     b = np.zeros(num_layers, np.float64)
     _check(lib.pd_get_layer_times(ctx, _ptr(f), _ptr(b), num_layers), ctx)
     return f, b
+
+
+def pd_save_checkpoint(ctx, directory: str):
+    """Every local worker writes <dir>/stage<s>_replica<r>.pdckpt (L1407-1413)."""
+    _check(lib.pd_save_checkpoint(ctx, os.fsencode(directory)), ctx)
+
+
+def pd_load_checkpoint(ctx, directory: str):
+    _check(lib.pd_load_checkpoint(ctx, os.fsencode(directory)), ctx)
 
 
 def pd_stage_solo(ctx):

@@ -301,6 +301,7 @@ struct Worker {
     void *lstm_da = nullptr;
     unsigned *lstm_cnt = nullptr;  // step counters of the persistent recurrence kernels
     void *lstm_wda = nullptr;      // wavefront backward: da of every layer of an LSTM run
+    int lstm_wmax = 0;             // ... for runs of up to this many layers
     float *lstm_wdc = nullptr;     // ... and their dc carries
     int lstm_rec = -1;             // persistent recurrences usable (-1 = not decided yet)
     // CUDA graphs of the LSTM recurrences (T steps of small GEMM + cell kernels), keyed by
@@ -1086,7 +1087,6 @@ struct Exec {
     void lstm_wave_forward(int l0, int L, int t, int j, int slot, void *y_last) {
         const pd_layer_desc &d = layer(l0);
         const int T = d.seq_len, Bn = B(), H = d.out;
-        const long TB = (long)T * Bn;
         LstmWaveDesc wd;
         wd.bwd = 0, wd.L = L, wd.T = T, wd.B = Bn, wd.H = H;
         wd.x = static_cast<const __nv_bfloat16 *>(layer_input(l0, t, j));
@@ -1118,10 +1118,8 @@ struct Exec {
         const pd_layer_desc &d = layer(l0);
         const int T = d.seq_len, Bn = B(), H = d.out;
         const long TB = (long)T * Bn;
-        if (!w->lstm_wda) {
-            w->lstm_wda = dalloc<void>((size_t)LSTM_WAVE_MAX_L * TB * 4 * H * esz);
-            w->lstm_wdc = dalloc<float>((size_t)LSTM_WAVE_MAX_L * Bn * H * 4);
-        }
+        if (!w->lstm_wda || L > w->lstm_wmax)  // sized in pd_stage_init: no allocation while others capture
+            throw CudaFail{cudaErrorInvalidValue, "wavefront scratch not allocated"};
         LstmWaveDesc wd;
         wd.bwd = 1, wd.L = L, wd.T = T, wd.B = Bn, wd.H = H;
         wd.dy_top = static_cast<const __nv_bfloat16 *>(G);
@@ -2062,6 +2060,30 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             gx_elems = std::max(gx_elems, TB * 4 * H);
             bh_elems = std::max(bh_elems, (long)B * H);
         }
+        // wavefront backward scratch (da and the dc carry of every layer of the longest chain of
+        // equal LSTMs this stage can run as one wavefront), allocated here: an allocation inside
+        // pd_run would device-synchronise while another worker captures a graph
+        if (bf16) {
+            int chain = 1, longest = 1;
+            for (int l = w->first + 1; l <= w->last; ++l) {
+                const pd_layer_desc &p = c->layers[l - 1], &q = c->layers[l];
+                const bool link = p.kind == PD_LSTM && q.kind == PD_LSTM && p.in == p.out && q.in == p.out &&
+                                  q.out == p.out && q.seq_len == p.seq_len;
+                chain = link ? chain + 1 : 1;
+                longest = std::max(longest, chain);
+            }
+            if (longest >= 2) {
+                long tb4h = 0, bh = 0;  // the largest LSTM of the stage bounds every run's per-layer scratch
+                for (int l = w->first; l <= w->last; ++l)
+                    if (c->layers[l].kind == PD_LSTM) {
+                        tb4h = std::max(tb4h, (long)c->layers[l].seq_len * B * 4 * c->layers[l].out);
+                        bh = std::max(bh, (long)B * c->layers[l].out);
+                    }
+                w->lstm_wmax = std::min(longest, LSTM_WAVE_MAX_L);
+                w->lstm_wda = dalloc<void>((size_t)w->lstm_wmax * tb4h * esz);
+                w->lstm_wdc = dalloc<float>((size_t)w->lstm_wmax * bh * 4);
+            }
+        }
         if (gx_elems) {
             w->lstm_gx = dalloc<float>(gx_elems * 4);
             w->lstm_da = dalloc<void>(gx_elems * esz);
@@ -2528,6 +2550,104 @@ pd_status pd_stage_solo(pd_ctx *c) {
     } catch (const CudaFail &f) {
         c->fail(PD_ECUDA, std::string("pd_stage_solo: ") + f.what + ": " + cudaGetErrorString(f.e));
         return f.e == cudaErrorMemoryAllocation ? PD_ENOMEM : PD_ECUDA;
+    }
+    return PD_OK;
+}
+
+namespace {
+struct CkptHeader {
+    char magic[8];  // "PDCKPT1"
+    int32_t stage, replica, dtype, optimizer;
+    int32_t version, updates_total;
+    int64_t params;  // device-layout parameter count of the stage (P)
+    int32_t has_adam, pad;
+};
+std::string ckpt_path(const char *dir, int s, int r) {
+    return std::string(dir) + "/stage" + std::to_string(s) + "_replica" + std::to_string(r) + ".pdckpt";
+}
+}  // namespace
+
+pd_status pd_save_checkpoint(pd_ctx *c, const char *dir) {
+    CHECK_CTX(c);
+    if (!dir) return PD_EINVAL;
+    for (auto &wp : c->W) {
+        Worker *w = wp.get();
+        if (!w) continue;
+        const std::string path = ckpt_path(dir, w->stage, w->replica);
+        if (cudaSetDevice(w->device) != cudaSuccess || cudaStreamSynchronize(w->stream) != cudaSuccess) {
+            c->fail(PD_ECUDA, "pd_save_checkpoint: device");
+            return PD_ECUDA;
+        }
+        const bool adam = c->cfg.optimizer == PD_ADAM;
+        std::vector<float> buf((size_t)w->P * (adam ? 3 : 1));
+        // the latest weights: the fp32 master (bf16 path) or the latest fp32 version slot
+        const float *src = c->esz == 2 ? w->master : static_cast<const float *>(w->wslot[w->version % w->k]);
+        bool ok = cudaMemcpy(buf.data(), src, (size_t)w->P * 4, cudaMemcpyDeviceToHost) == cudaSuccess;
+        if (adam)
+            ok = ok && cudaMemcpy(buf.data() + w->P, w->adam_m, (size_t)w->P * 4, cudaMemcpyDeviceToHost) == cudaSuccess &&
+                 cudaMemcpy(buf.data() + 2 * w->P, w->adam_v, (size_t)w->P * 4, cudaMemcpyDeviceToHost) == cudaSuccess;
+        if (!ok) {
+            c->fail(PD_ECUDA, "pd_save_checkpoint: copy");
+            return PD_ECUDA;
+        }
+        CkptHeader h{};
+        std::memcpy(h.magic, "PDCKPT1", 8);
+        h.stage = w->stage, h.replica = w->replica, h.dtype = c->cfg.dtype, h.optimizer = c->cfg.optimizer;
+        h.version = w->version, h.updates_total = w->updates_total, h.params = w->P, h.has_adam = adam;
+        FILE *f = fopen((path + ".tmp").c_str(), "wb");
+        const bool wrote = f && fwrite(&h, sizeof h, 1, f) == 1 && fwrite(buf.data(), 4, buf.size(), f) == buf.size();
+        if (f) fclose(f);
+        if (!wrote || rename((path + ".tmp").c_str(), path.c_str()) != 0) {
+            std::lock_guard<std::mutex> g(c->err_mu);
+            c->err = "pd_save_checkpoint: cannot write " + path;
+            return PD_EINVAL;
+        }
+    }
+    return PD_OK;
+}
+
+pd_status pd_load_checkpoint(pd_ctx *c, const char *dir) {
+    CHECK_CTX(c);
+    if (!dir) return PD_EINVAL;
+    for (auto &wp : c->W) {
+        Worker *w = wp.get();
+        if (!w) continue;
+        const std::string path = ckpt_path(dir, w->stage, w->replica);
+        const bool adam = c->cfg.optimizer == PD_ADAM;
+        CkptHeader h{};
+        std::vector<float> buf((size_t)w->P * (adam ? 3 : 1));
+        FILE *f = fopen(path.c_str(), "rb");
+        const bool read = f && fread(&h, sizeof h, 1, f) == 1 && std::memcmp(h.magic, "PDCKPT1", 8) == 0 &&
+                          h.stage == w->stage && h.replica == w->replica && h.dtype == c->cfg.dtype &&
+                          h.optimizer == c->cfg.optimizer && h.params == w->P && h.has_adam == (int)adam &&
+                          fread(buf.data(), 4, buf.size(), f) == buf.size();
+        if (f) fclose(f);
+        if (!read) {
+            std::lock_guard<std::mutex> g(c->err_mu);
+            c->err = "pd_load_checkpoint: missing or mismatching " + path;
+            return PD_EINVAL;
+        }
+        try {
+            CK(cudaSetDevice(w->device));
+            CK(cudaStreamSynchronize(w->stream));
+            if (c->esz == 2) {
+                CK(cudaMemcpy(w->master, buf.data(), (size_t)w->P * 4, cudaMemcpyHostToDevice));
+                for (void *slot : w->wslot)
+                    CK(f32_to_bf16(w->master, static_cast<__nv_bfloat16 *>(slot), w->P, w->stream));
+            } else {
+                for (void *slot : w->wslot) CK(cudaMemcpy(slot, buf.data(), (size_t)w->P * 4, cudaMemcpyHostToDevice));
+            }
+            if (adam) {
+                CK(cudaMemcpy(w->adam_m, buf.data() + w->P, (size_t)w->P * 4, cudaMemcpyHostToDevice));
+                CK(cudaMemcpy(w->adam_v, buf.data() + 2 * w->P, (size_t)w->P * 4, cudaMemcpyHostToDevice));
+            }
+            CK(cudaStreamSynchronize(w->stream));
+        } catch (const CudaFail &e) {
+            c->fail(PD_ECUDA, std::string("pd_load_checkpoint: ") + e.what);
+            return PD_ECUDA;
+        }
+        w->version = h.version;
+        w->updates_total = h.updates_total;
     }
     return PD_OK;
 }

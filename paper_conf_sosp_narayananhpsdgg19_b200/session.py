@@ -10,7 +10,8 @@ import numpy as np
 
 from . import (PD_BF16, PD_SGD, Plan, pd_create, pd_destroy, pd_export_worker, pd_get_layer_times, pd_get_losses,
                pd_get_params, pd_get_stats, pd_get_trace, pd_get_version_map, pd_import_worker, pd_set_data,
-               pd_set_layer_profiling, pd_set_timing, pd_stage_init, pd_stage_solo, pd_run)
+               pd_set_layer_profiling, pd_set_timing, pd_stage_init, pd_stage_solo, pd_run, pd_save_checkpoint,
+               pd_load_checkpoint)
 
 
 def workers_of(plan: Plan):
@@ -73,6 +74,12 @@ class Pipeline:
                     if blob_worker(b) in local_sr:
                         continue
                     pd_import_worker(self.ctx, b)
+
+    def save_checkpoint(self, directory):
+        pd_save_checkpoint(self.ctx, directory)
+
+    def load_checkpoint(self, directory):
+        pd_load_checkpoint(self.ctx, directory)
 
     def set_data(self, inputs, tokens, labels, n):
         pd_set_data(self.ctx, inputs, tokens, labels, n)
