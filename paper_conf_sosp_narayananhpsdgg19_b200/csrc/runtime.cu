@@ -2582,10 +2582,14 @@ pd_status pd_save_checkpoint(pd_ctx *c, const char *dir) {
         std::vector<float> buf((size_t)w->P * (adam ? 3 : 1));
         // the latest weights: the fp32 master (bf16 path) or the latest fp32 version slot
         const float *src = c->esz == 2 ? w->master : static_cast<const float *>(w->wslot[w->version % w->k]);
-        bool ok = cudaMemcpy(buf.data(), src, (size_t)w->P * 4, cudaMemcpyDeviceToHost) == cudaSuccess;
+        bool ok = cudaMemcpyAsync(buf.data(), src, (size_t)w->P * 4, cudaMemcpyDeviceToHost, w->stream) == cudaSuccess;
         if (adam)
-            ok = ok && cudaMemcpy(buf.data() + w->P, w->adam_m, (size_t)w->P * 4, cudaMemcpyDeviceToHost) == cudaSuccess &&
-                 cudaMemcpy(buf.data() + 2 * w->P, w->adam_v, (size_t)w->P * 4, cudaMemcpyDeviceToHost) == cudaSuccess;
+            ok = ok &&
+                 cudaMemcpyAsync(buf.data() + w->P, w->adam_m, (size_t)w->P * 4, cudaMemcpyDeviceToHost, w->stream) ==
+                     cudaSuccess &&
+                 cudaMemcpyAsync(buf.data() + 2 * w->P, w->adam_v, (size_t)w->P * 4, cudaMemcpyDeviceToHost,
+                                 w->stream) == cudaSuccess;
+        ok = ok && cudaStreamSynchronize(w->stream) == cudaSuccess;
         if (!ok) {
             c->fail(PD_ECUDA, "pd_save_checkpoint: copy");
             return PD_ECUDA;
@@ -2628,18 +2632,22 @@ pd_status pd_load_checkpoint(pd_ctx *c, const char *dir) {
             return PD_EINVAL;
         }
         try {
+            // every copy and conversion on the worker's stream: a pageable cudaMemcpy may return
+            // before its DMA lands, and the conversion kernel must not read the master before
             CK(cudaSetDevice(w->device));
             CK(cudaStreamSynchronize(w->stream));
             if (c->esz == 2) {
-                CK(cudaMemcpy(w->master, buf.data(), (size_t)w->P * 4, cudaMemcpyHostToDevice));
+                CK(cudaMemcpyAsync(w->master, buf.data(), (size_t)w->P * 4, cudaMemcpyHostToDevice, w->stream));
                 for (void *slot : w->wslot)
                     CK(f32_to_bf16(w->master, static_cast<__nv_bfloat16 *>(slot), w->P, w->stream));
             } else {
-                for (void *slot : w->wslot) CK(cudaMemcpy(slot, buf.data(), (size_t)w->P * 4, cudaMemcpyHostToDevice));
+                for (void *slot : w->wslot)
+                    CK(cudaMemcpyAsync(slot, buf.data(), (size_t)w->P * 4, cudaMemcpyHostToDevice, w->stream));
             }
             if (adam) {
-                CK(cudaMemcpy(w->adam_m, buf.data() + w->P, (size_t)w->P * 4, cudaMemcpyHostToDevice));
-                CK(cudaMemcpy(w->adam_v, buf.data() + 2 * w->P, (size_t)w->P * 4, cudaMemcpyHostToDevice));
+                CK(cudaMemcpyAsync(w->adam_m, buf.data() + w->P, (size_t)w->P * 4, cudaMemcpyHostToDevice, w->stream));
+                CK(cudaMemcpyAsync(w->adam_v, buf.data() + 2 * w->P, (size_t)w->P * 4, cudaMemcpyHostToDevice,
+                                   w->stream));
             }
             CK(cudaStreamSynchronize(w->stream));
         } catch (const CudaFail &e) {
