@@ -157,14 +157,16 @@ class RunResult:
 
 def run(layers, stage_last, replicas, B, M, params=None, data=None, optimizer=0, lr=0.05,
         beta1=0.9, beta2=0.999, eps=1e-8, depth=0, math=True, stash=True,
-        fwd_time=None, bwd_time=None, vertical_sync=False) -> RunResult:
+        fwd_time=None, bwd_time=None, vertical_sync=False, gpipe=False) -> RunResult:
     """Simulate PipeDream training.  ``params`` is a list of per-layer flat arrays.
-    ``vertical_sync``: every stage uses the version the input stage tagged t with (§3.3)."""
+    ``vertical_sync``: every stage uses the version the input stage tagged t with (§3.3).
+    ``gpipe``: the §5.4 comparison schedule -- flush every D = ``depth`` (0 => n) minibatches,
+    one update per group with the group's mean gradient (L1277-1279, R27)."""
     n = len(stage_last)
     lay = _layers(layers)
     sl = np.ascontiguousarray(stage_last, np.int32)
     rp = np.ascontiguousarray(replicas, np.int32)
-    mode = (1 if math else 0) | (0 if stash else 2) | (4 if vertical_sync else 0)
+    mode = (1 if math else 0) | (0 if stash else 2) | (4 if vertical_sync else 0) | (8 if gpipe else 0)
     inputs = tokens = labels = None
     n_data = 1
     if data is not None:

@@ -16,6 +16,8 @@
  *   - an event-driven executor with explicit per-stage activation/gradient queues,
  *     weight stashing (§3.3), updates applied to the latest weights
  *     (L1341-1353) and replica rounds averaged in replica order (L1345-1347, L1373-1381);
+ *   - the GPipe comparison schedule (§5.4): pipeline flushes every D minibatches with the
+ *     group's gradients aggregated into one update (L1277-1279);
  *   - an optional timeline (start/end per op, bubble) for Fig. 2/4/8-style pins;
  *   - the §3.1 dynamic-programming partitioner (L899-985) as read in DESIGN.md R10-R16.
  *
@@ -447,6 +449,7 @@ struct Worker {
     int f_done = 0;                /* forwards completed                                     */
     int last_tag = 0;              /* version used by the latest forward (vertical sync)     */
     int max_live = 1;              /* widest version window held (pin P10)                   */
+    std::vector<std::vector<float>> group_g; /* GPipe: the gradients of the current group, in t order */
 };
 
 struct Sim {
@@ -458,6 +461,8 @@ struct Sim {
     OptCfg opt;
     bool math, stash;
     bool vsync;             /* vertical sync (§3.3): every stage uses the tag version */
+    bool gpipe;             /* GPipe-style flush (§5.4) with gradient aggregation (L1277-1279) */
+    int group;              /* GPipe: minibatches per flush group (the pipeline depth D)          */
     std::map<std::pair<int, int>, int> act_tag; /* (stage, t) -> version tag travelling with the activation */
     const float *inputs; const int *tokens, *labels; int n_data;
     const double *ftime, *btime;
@@ -483,6 +488,23 @@ long sample_in_size(const orc_layer &L) { return in_size(L, 1); }
  * then (B U)* for the remaining minibatches.  U immediately follows B (L237-241). */
 void build_ops(Sim &S, Worker &w) {
     int s = w.stage, Rs = S.R[s];
+    if (S.gpipe) {
+        /* GPipe (R27): minibatches in groups of D; every stage but the last forwards
+         * the whole group, then runs its backwards in t order; the last stage runs F(t) B(t)
+         * back to back (its backward starts immediately, L719-721); one U per group applies
+         * the aggregated gradient (the flush).  Op.round = group index. */
+        for (int g = 0; g * S.group < S.M; g++) {
+            int t0 = g * S.group, t1 = t0 + S.group;
+            if (s + 1 < S.n_stages) {
+                for (int t = t0; t < t1; t++) w.ops.push_back({'F', t, g});
+                for (int t = t0; t < t1; t++) w.ops.push_back({'B', t, g});
+            } else {
+                for (int t = t0; t < t1; t++) { w.ops.push_back({'F', t, g}); w.ops.push_back({'B', t, g}); }
+            }
+            w.ops.push_back({'U', t1 - 1, g});
+        }
+        return;
+    }
     std::vector<int> ts;
     for (int t = w.replica; t < S.M; t += Rs) ts.push_back(t);
     int Mr = (int)ts.size();
@@ -623,6 +645,7 @@ void exec(Sim &S, Worker &w, const Op &op) {
         if (s > 0) S.grad_t[{s - 1, t}] = en;
         S.grad_q.erase({s, t});
         w.last_b_t = t;
+        if (S.gpipe && S.math) w.group_g.push_back(w.grad);
         if (S.R[s] > 1) {
             auto key = std::make_pair(s, op.round);
             if (!S.round_t.count(key)) {
@@ -656,6 +679,20 @@ void exec(Sim &S, Worker &w, const Op &op) {
             g = S.round_mean[key].data();
         }
         ev_t = op.round;
+    } else if (S.gpipe) {
+        /* gradient aggregation (L1277-1279): the group's D gradients added in t order into one
+         * buffer, times 1/D -- the mean over the group, so that a flush group of D minibatches
+         * of B samples is one SGD step on D*B samples (R27) */
+        if (S.math) {
+            mean.assign(np, 0.0f);
+            for (auto &gt : w.group_g)
+                for (long k2 = 0; k2 < np; k2++) mean[k2] += gt[k2];
+            float inv = 1.0f / (float)w.group_g.size();
+            for (long k2 = 0; k2 < np; k2++) mean[k2] = mean[k2] * inv;
+            g = mean.data();
+            w.group_g.clear();
+        }
+        ev_t = op.round;
     } else if (S.math) {
         g = w.grad.data();
     }
@@ -672,9 +709,17 @@ void exec(Sim &S, Worker &w, const Op &op) {
 
     /* the stashed version of the backward just applied is released; a version is discarded
      * once no pending backward references it and it is not the latest (L1349-1353) */
-    int vb = w.fwd_version[t];
-    w.refcount[vb]--;
-    w.fwd_version.erase(t);
+    if (S.gpipe) {
+        /* the flush: every minibatch of the group has finished its backward */
+        for (int t2 = op.round * S.group; t2 <= t; t2++) {
+            w.refcount[w.fwd_version[t2]]--;
+            w.fwd_version.erase(t2);
+        }
+    } else {
+        int vb = w.fwd_version[t];
+        w.refcount[vb]--;
+        w.fwd_version.erase(t);
+    }
     /* vertical sync: a minibatch not yet forwarded here carries a tag >= the tag of the
      * last one forwarded here (the input stage's version only grows and it forwards in t
      * order; straight pipelines), so versions from that tag on are kept */
@@ -757,6 +802,9 @@ int orc_inflight(const int *R, int n, int depth, int *k_out) {
  *   mode bit0      : 1 = do the math, 0 = schedule only
  *   mode bit1      : 1 = disable weight stashing (negative control; backward uses latest)
  *   mode bit2      : 1 = vertical sync (§3.3; straight pipelines only)
+ *   mode bit3      : 1 = GPipe-style flush schedule with gradient aggregation (§5.4,
+ *                    L1277-1279; R27): groups of D = depth (0 => n) minibatches, one
+ *                    update per group with the mean of the group's gradients; straight only
  *   inputs/tokens/labels: n_data minibatches, minibatch t uses data t mod n_data
  *   params         : in = initial flat params (layer order), out = final latest params
  *                    (replica 0 of every stage; replicas are identical by construction)
@@ -773,7 +821,7 @@ int orc_run(const orc_layer *layers, int n_layers, const int *stage_last, const 
     Sim S;
     S.layers = layers; S.n_layers = n_layers; S.n_stages = n_stages; S.B = B; S.M = M; S.depth = depth;
     S.opt = OptCfg{opt_kind, lr, b1, b2, eps};
-    S.math = (mode & 1) != 0; S.stash = (mode & 2) == 0; S.vsync = (mode & 4) != 0;
+    S.math = (mode & 1) != 0; S.stash = (mode & 2) == 0; S.vsync = (mode & 4) != 0; S.gpipe = (mode & 8) != 0;
     S.inputs = inputs; S.tokens = tokens; S.labels = labels; S.n_data = n_data > 0 ? n_data : 1;
     S.ftime = fwd_time; S.btime = bwd_time;
     if (n_stages < 1 || stage_last[n_stages - 1] != n_layers - 1) return -1;
@@ -789,6 +837,15 @@ int orc_run(const orc_layer *layers, int n_layers, const int *stage_last, const 
         for (int s = 0; s < n_stages; s++) if (S.R[s] != 1) return -1; /* straight pipelines only */
     }
     S.k.assign(n_stages, 0);
+    if (S.gpipe) {
+        /* GPipe: straight plans, no vertical sync; group D = depth, or NOAM = n when depth = 0
+         * (the paper's "pipeline depth equivalent to NOAM", L1955-1958); M a multiple of D */
+        if (S.vsync) return -1;
+        for (int s = 0; s < n_stages; s++) if (S.R[s] != 1) return -1;
+        S.group = depth > 0 ? depth : n_stages;
+        if (M % S.group != 0) return -1;
+        depth = 0;
+    }
     if (orc_inflight(replicas, n_stages, depth, S.k.data()) != 0) return -1;
     S.poff.assign(n_layers + 1, 0);
     for (int l = 0; l < n_layers; l++) S.poff[l + 1] = S.poff[l] + param_count(layers[l]);
