@@ -137,8 +137,19 @@ typedef enum { PD_SGD = 0, PD_ADAM = 1 } pd_optimizer;
  *   PD_SYNC_VERTICAL  vertical sync: the input stage tags minibatch t with its latest
  *                     version v and EVERY stage runs F(s,t) and B(s,t) with its own stashed
  *                     version v (L1175-1186; update rule L1247-1253).  Straight plans only
- *                     (every R_s = 1, else PD_EUNSUPPORTED); every stage keeps k_0 versions. */
-typedef enum { PD_SYNC_STASH = 0, PD_SYNC_VERTICAL = 1 } pd_sync_mode;
+ *                     (every R_s = 1, else PD_EUNSUPPORTED); every stage keeps k_0 versions.
+ *   PD_SYNC_GPIPE     the paper's comparison schedule (§5.4) with gradient
+ *                     aggregation (L1277-1279): minibatches in flush groups of D (the pd_run
+ *                     `noam` argument; 0 => NOAM = n).  Every stage but the last forwards the
+ *                     whole group and then runs its backwards in t order (the last stage runs
+ *                     F(t) B(t) back to back); each backward writes its weight gradient into
+ *                     its own fp32 buffer, and one update per group applies the mean of the D
+ *                     gradients (summed in t order, times 1/D) -- a pipeline flush per group,
+ *                     one weight version per group (v(s,t) = floor(t/D), R27).
+ *                     Straight plans only (else PD_EUNSUPPORTED); D <= max(n, cfg.max_depth)
+ *                     and num_minibatches % D == 0 (else PD_EINVAL).  Trace: one 'U' per
+ *                     group with minibatch = the group index. */
+typedef enum { PD_SYNC_STASH = 0, PD_SYNC_VERTICAL = 1, PD_SYNC_GPIPE = 2 } pd_sync_mode;
 
 typedef struct {
     int dtype;        /* PD_FP32: fp32 SIMT parity path (no tensor cores, tf32 off);

@@ -28,7 +28,7 @@ PD_LINEAR, PD_LSTM, PD_CONV3X3, PD_MAXPOOL2, PD_EMBEDDING = 0, 1, 2, 3, 4
 PD_ACT_NONE, PD_ACT_RELU = 0, 1
 PD_FP32, PD_BF16 = 0, 1
 PD_SGD, PD_ADAM = 0, 1
-PD_SYNC_STASH, PD_SYNC_VERTICAL = 0, 1
+PD_SYNC_STASH, PD_SYNC_VERTICAL, PD_SYNC_GPIPE = 0, 1, 2
 PD_EPI_STORE, PD_EPI_MASK, PD_EPI_F32, PD_EPI_SGD, PD_EPI_ADAM = 0, 1, 2, 3, 4
 PD_MAX_STAGES = 64
 PD_MAX_LOCAL_WORKERS = 64
@@ -269,7 +269,8 @@ def _layer_descs(layers):
 
 def pd_create(plan: Plan, layers, dtype=PD_BF16, optimizer=PD_SGD, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8,
               minibatch=1, record_trace=1, max_depth=0, sync_mode=0):
-    """sync_mode: PD_SYNC_STASH (weight stashing) or PD_SYNC_VERTICAL (vertical sync, §3.3)."""
+    """sync_mode: PD_SYNC_STASH (weight stashing), PD_SYNC_VERTICAL (vertical sync, §3.3) or
+    PD_SYNC_GPIPE (the §5.4 flush schedule with gradient aggregation, R27)."""
     ctx = C.c_void_p()
     cfg = TrainCfg(dtype, optimizer, lr, beta1, beta2, eps, minibatch, record_trace, max_depth, sync_mode)
     _check(lib.pd_create(C.byref(ctx), C.byref(plan.to_c()), _layer_descs(layers), len(layers), C.byref(cfg)))

@@ -593,6 +593,9 @@ cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f
     return cudaGetLastError();
 }
 
+// (GPipe flush update: the same kernel with R = D gradient buffers of one worker -- the
+// group's gradients summed in t order, times 1/D -- and nout = 1 destination.)
+//
 // Replica sync of one round, sharded (reduce-scatter -> update -> all-gather through peer
 // memory): this replica owns parameters [lo, hi) (16-byte multiples).  For each of them it
 // sums the R replicas' fp32 gradients in replica order (R7) over NVLink peer loads, applies
@@ -604,7 +607,7 @@ cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f
 template <bool ADAM>
 __global__ void __launch_bounds__(256) update_shard_kernel(const float *const *__restrict__ grads, int R, long lo,
                                                            long n4, const float *w_in, float *const *__restrict__ out_f32,
-                                                           __nv_bfloat16 *const *__restrict__ out_bf16,
+                                                           __nv_bfloat16 *const *__restrict__ out_bf16, int nout,
                                                            float *__restrict__ m, float *__restrict__ v, float lr,
                                                            float b1, float b2, float eps, float bc1, float bc2) {
     const float invR = 1.0f / (float)R;
@@ -635,7 +638,7 @@ __global__ void __launch_bounds__(256) update_shard_kernel(const float *const *_
             o.x = *reinterpret_cast<uint32_t *>(&a0);
             o.y = *reinterpret_cast<uint32_t *>(&a1);
         }
-        for (int r = 0; r < R; ++r) {
+        for (int r = 0; r < nout; ++r) {
             *reinterpret_cast<float4 *>(out_f32[r] + i) = w;
             if (out_bf16) *reinterpret_cast<uint2 *>(out_bf16[r] + i) = o;
         }
@@ -643,7 +646,7 @@ __global__ void __launch_bounds__(256) update_shard_kernel(const float *const *_
 }
 
 cudaError_t update_shard(const float *const *grads, int R, long lo, long hi, const float *w_in, float *const *out_f32,
-                         __nv_bfloat16 *const *out_bf16, int opt, float *m, float *v, float lr, float b1, float b2,
+                         __nv_bfloat16 *const *out_bf16, int nout, int opt, float *m, float *v, float lr, float b1, float b2,
                          float eps, int step, cudaStream_t s) {
     if ((lo & 3) || (hi & 3) || hi < lo) return cudaErrorInvalidValue;
     if (hi == lo) return cudaSuccess;
@@ -652,10 +655,10 @@ cudaError_t update_shard(const float *const *grads, int R, long lo, long hi, con
     long blocks = (n4 + 255) / 256;
     if (blocks > 148L * 8) blocks = 148L * 8;
     if (opt == PD_ADAM)
-        update_shard_kernel<true><<<(unsigned)blocks, 256, 0, s>>>(grads, R, lo, n4, w_in, out_f32, out_bf16, m, v, lr, b1,
+        update_shard_kernel<true><<<(unsigned)blocks, 256, 0, s>>>(grads, R, lo, n4, w_in, out_f32, out_bf16, nout, m, v, lr, b1,
                                                                    b2, eps, bc1, bc2);
     else
-        update_shard_kernel<false><<<(unsigned)blocks, 256, 0, s>>>(grads, R, lo, n4, w_in, out_f32, out_bf16, m, v, lr,
+        update_shard_kernel<false><<<(unsigned)blocks, 256, 0, s>>>(grads, R, lo, n4, w_in, out_f32, out_bf16, nout, m, v, lr,
                                                                     b1, b2, eps, bc1, bc2);
     ++tl_launches;
     return cudaGetLastError();

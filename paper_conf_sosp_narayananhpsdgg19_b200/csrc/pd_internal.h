@@ -27,6 +27,7 @@ struct Op {
 pd_status inflight_counts(const pd_plan_t &plan, int depth, std::vector<int> &k);
 // F(t_0..t_{k-1}) then (B(t_j) U F(t_{j+k}))* then (B U)* (L1023-1065, L237-241).
 std::vector<Op> worker_ops(int R_s, int replica, int k_s, int M);
+std::vector<Op> gpipe_ops(bool last_stage, int D, int M);
 // receive-ring depth of stage s >= 1: ceil(k_{s-1} R_{s-1} / R_s).
 int recv_ring_depth(const pd_plan_t &plan, const std::vector<int> &k, int s);
 
@@ -144,7 +145,7 @@ cudaError_t update_master(float *master, __nv_bfloat16 *slot_bf16, float *slot_f
 // new value stored to out_f32[q][i] and (if out_bf16) bf16 to out_bf16[q][i] for every
 // replica q.  grads / out_f32 / out_bf16 are DEVICE arrays of R pointers (peer memory).
 cudaError_t update_shard(const float *const *grads, int R, long lo, long hi, const float *w_in, float *const *out_f32,
-                         __nv_bfloat16 *const *out_bf16, int opt, float *m, float *v, float lr, float b1, float b2,
+                         __nv_bfloat16 *const *out_bf16, int nout, int opt, float *m, float *v, float lr, float b1, float b2,
                          float eps, int step, cudaStream_t s);
 // bf16 path, one unreplicated fp32 gradient: master -= SGD/Adam step of g, slot = bf16(master);
 // vectorised (n % 4 == 0, 16-byte aligned arrays; else cudaErrorInvalidValue)

@@ -284,6 +284,13 @@ struct Worker {
     float **sync_f32 = nullptr;
     __nv_bfloat16 **sync_bf16 = nullptr;
     const float **self_grad_ptr = nullptr;  // device array [1]: gbuf
+    // GPipe flush schedule (PD_SYNC_GPIPE): one fp32 gradient buffer per minibatch of a flush
+    // group (gp_grad[i] for the group's i-th minibatch), their device pointer array, and the
+    // update's destinations per weight slot (fp32: master on the bf16 path / slot q; bf16: slot q)
+    std::vector<float *> gp_grad;
+    const float **gp_ptrs = nullptr;
+    float **gp_out_f32 = nullptr;
+    __nv_bfloat16 **gp_out_bf16 = nullptr;
     // activations
     std::vector<void *> act;     // per inner layer l (index l-first, l>first): k slots of in_elems
     void *recv = nullptr;        // D slots (stage > 0)
@@ -353,6 +360,7 @@ Worker::~Worker() {
     if (device >= 0) cudaSetDevice(device);
     if (stream) cudaStreamSynchronize(stream);
     for (void *p : wslot) cudaFree(p);
+    for (void *p : gp_grad) cudaFree(p);
     for (void *p : act) cudaFree(p);
     for (void *p : aux)
         if (p) cudaFree(p);
@@ -361,7 +369,7 @@ Worker::~Worker() {
         if (p) cudaFree(p);
     void *bufs[] = {master, fbias, (void *)breg_off, (void *)breg_cnt, adam_m, adam_v, gbuf, ws, stage_in, rgrad[0], rgrad[1], recv, gring, scratch[0], scratch[1], scratch[2], logits,
                     dlogits, data_in, tokens, labels, losses, flags, (void *)rgrad_ptrs, (void *)self_grad_ptr,
-                    (void *)sync_f32, (void *)sync_bf16};
+                    (void *)sync_f32, (void *)sync_bf16, (void *)gp_ptrs, (void *)gp_out_f32, (void *)gp_out_bf16};
     for (void *p : bufs)
         if (p) cudaFree(p);
     for (cudaEvent_t e : ev_pool) cudaEventDestroy(e);
@@ -538,6 +546,7 @@ struct Exec {
 
     const pd_layer_desc &layer(int l) const { return c->layers[l]; }
     int B() const { return c->cfg.minibatch; }
+    bool gpipe() const { return c->cfg.sync_mode == PD_SYNC_GPIPE; }  // flush groups of k[0] (R27)
     int n() const { return c->n; }
 
     // weights of layer l in stash slot `slot` (path dtype)
@@ -1604,11 +1613,13 @@ struct Exec {
         const void *G = (s + 1 == n()) ? w->dlogits
                                        : elem_ptr(w->gring, (long)(j % w->G) * dev_out_elems(c->layers, w->last, B()), esz);
         int cur = 0;
-        const bool fused = bf16 && Rs == 1;  // dW + optimizer update in one GEMM epilogue
-        float *gdst = Rs > 1 ? w->rgrad[jr & 1] : w->gbuf;
+        // dW + optimizer update in one GEMM epilogue; GPipe: the weight gradient of the group's
+        // i-th minibatch into its own fp32 buffer, aggregated by the group's update (L1277-1279)
+        const bool fused = bf16 && Rs == 1 && !gpipe();
+        float *gdst = Rs > 1 ? w->rgrad[jr & 1] : gpipe() ? w->gp_grad[t % k[0]] : w->gbuf;
         const int next_version = w->version + 1;
         const int nslot = next_version % w->k;
-        check_weight_slot(nslot, j, t);
+        if (!gpipe()) check_weight_slot(nslot, j, t);  // (GPipe: the group's update follows every B)
         BwdCtx bc{fused, gdst, nslot, sslot};
         bool all_linear = true;
         for (int l = w->first; l <= w->last; ++l) all_linear = all_linear && layer(l).kind == PD_LINEAR;
@@ -1691,7 +1702,7 @@ struct Exec {
         const int Rs = c->plan.stage[s].replicas;
         const int vin = w->version;
         const int nslot = (vin + 1) % w->k;
-        trace('U', Rs > 1 ? j : t, vin, vin + 1);
+        trace('U', Rs > 1 || gpipe() ? j : t, vin, vin + 1);
         const bool adam = c->cfg.optimizer == PD_ADAM;
         const int step = w->updates_total + 1;
         if (Rs > 1) {
@@ -1710,7 +1721,7 @@ struct Exec {
             const long lo = shard_lo(w->replica), hi = w->replica + 1 == Rs ? w->P : shard_lo(w->replica + 1);
             const float *w_in = bf16 ? w->master : static_cast<const float *>(w->wslot[vin % w->k]);
             CK(update_shard(w->rgrad_ptrs + (j & 1) * Rs, Rs, lo, hi, w_in, w->sync_f32 + (size_t)nslot * Rs,
-                            bf16 ? w->sync_bf16 + (size_t)nslot * Rs : nullptr, c->cfg.optimizer, w->adam_m, w->adam_v,
+                            bf16 ? w->sync_bf16 + (size_t)nslot * Rs : nullptr, Rs, c->cfg.optimizer, w->adam_m, w->adam_v,
                             c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, step, w->stream));
             w->replica_bytes += (uint64_t)(Rs - 1) * (hi - lo) * (4 + 4 + (bf16 ? 2 : 0));
             for (int r = 0; r < Rs; ++r) {
@@ -1724,6 +1735,14 @@ struct Exec {
                 link_wait(c, L, w->stream, j, w->vc);
                 hb_require(c->worker_id(s, r), c->opU, j, "new version used before every shard was written", t);
             }
+        } else if (gpipe()) {
+            // the flush: every backward of group j is done (stream order); mean of its D
+            // gradients (t order, times 1/D) applied to the latest weights, new version into
+            // slot nslot (the only other version alive is the one this group used)
+            const float *w_in = bf16 ? w->master : static_cast<const float *>(w->wslot[vin % w->k]);
+            CK(update_shard(w->gp_ptrs, k[0], 0, w->P, w_in, w->gp_out_f32 + nslot,
+                            bf16 ? w->gp_out_bf16 + nslot : nullptr, 1, c->cfg.optimizer, w->adam_m, w->adam_v,
+                            c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps, step, w->stream));
         } else if (!bf16) {
             const float *latest = static_cast<const float *>(w->wslot[vin % w->k]);
             float *next = static_cast<float *>(w->wslot[nslot]);
@@ -1736,7 +1755,8 @@ struct Exec {
         // (bf16 unreplicated: the update was fused into B's dW epilogues)
         w->version = vin + 1;
         w->updates_total += 1;
-        w->fwd_version.erase(j);
+        if (gpipe()) w->fwd_version.clear();  // every minibatch of the group is done
+        else w->fwd_version.erase(j);
     }
 
     // PD_OP_TRACE=1: every op a worker issues, on stderr (diagnosing a stuck run)
@@ -1746,7 +1766,7 @@ struct Exec {
     }
     void run_ops() {
         const int Rs = c->plan.stage[w->stage].replicas;
-        std::vector<Op> ops = worker_ops(Rs, w->replica, k[w->stage], M);
+        std::vector<Op> ops = gpipe() ? gpipe_ops(w->stage + 1 == n(), k[0], M) : worker_ops(Rs, w->replica, k[w->stage], M);
         w->run_base = w->version;
         w->vc.assign(c->nw, 0);
         // layers inside (not at the bottom of) an LSTM wavefront run: their input is the
@@ -1881,10 +1901,15 @@ pd_status pd_create(pd_ctx **out, const pd_plan_t *plan, const pd_layer_desc *la
     }
     // plan.noam is derived, not chosen: 0, or exactly k_0 = ceil(W / R_0) (L1021, R1)
     if (plan->noam != 0 && plan->noam != kdef[0]) return PD_EINVAL;
-    if (cfg->sync_mode != PD_SYNC_STASH && cfg->sync_mode != PD_SYNC_VERTICAL) return PD_EINVAL;
-    if (cfg->sync_mode == PD_SYNC_VERTICAL)
+    if (cfg->sync_mode != PD_SYNC_STASH && cfg->sync_mode != PD_SYNC_VERTICAL && cfg->sync_mode != PD_SYNC_GPIPE)
+        return PD_EINVAL;
+    if (cfg->sync_mode != PD_SYNC_STASH)
         for (int s = 0; s < n; ++s)
-            if (plan->stage[s].replicas != 1) return PD_EUNSUPPORTED;  // straight pipelines (§3.3)
+            if (plan->stage[s].replicas != 1) return PD_EUNSUPPORTED;  // straight pipelines (§3.3, §5.4)
+    // GPipe: every stage holds a whole flush group of D <= max(n, max_depth) minibatches (its
+    // activation stash and receive rings); one weight version at a time (R27)
+    if (cfg->sync_mode == PD_SYNC_GPIPE)
+        for (int s = 0; s < n; ++s) kmax[s] = std::max({kmax[s], n, cfg->max_depth});
     pd_ctx *c = new pd_ctx;
     c->plan = *plan;
     c->layers.assign(layers, layers + num_layers);
@@ -2022,6 +2047,22 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
             const float *one[1] = {w->gbuf};
             w->self_grad_ptr = dalloc<const float *>(sizeof(one));
             CK(cudaMemcpy(w->self_grad_ptr, one, sizeof(one), cudaMemcpyHostToDevice));
+        }
+        if (c->cfg.sync_mode == PD_SYNC_GPIPE) {
+            // one fp32 gradient buffer per minibatch of the largest flush group
+            for (int q = 0; q < w->k; ++q) w->gp_grad.push_back(dalloc<float>(P * 4));
+            w->gp_ptrs = dalloc<const float *>(sizeof(float *) * w->k);
+            CK(cudaMemcpy(w->gp_ptrs, w->gp_grad.data(), sizeof(float *) * w->k, cudaMemcpyHostToDevice));
+            std::vector<float *> f32(w->k);
+            std::vector<__nv_bfloat16 *> b16(w->k);
+            for (int q = 0; q < w->k; ++q) {
+                f32[q] = bf16 ? w->master : static_cast<float *>(w->wslot[q]);
+                b16[q] = bf16 ? static_cast<__nv_bfloat16 *>(w->wslot[q]) : nullptr;
+            }
+            w->gp_out_f32 = dalloc<float *>(sizeof(float *) * w->k);
+            w->gp_out_bf16 = dalloc<__nv_bfloat16 *>(sizeof(void *) * w->k);
+            CK(cudaMemcpy(w->gp_out_f32, f32.data(), sizeof(float *) * w->k, cudaMemcpyHostToDevice));
+            CK(cudaMemcpy(w->gp_out_bf16, b16.data(), sizeof(void *) * w->k, cudaMemcpyHostToDevice));
         }
         if (Rs > 1) {
             w->rgrad[0] = dalloc<float>(P * 4);
@@ -2280,7 +2321,19 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
     for (int s = 0; s < c->n; ++s)
         if (M % c->plan.stage[s].replicas) return PD_EINVAL;
     std::vector<int> k;
-    if (inflight_counts(c->plan, noam, k) != PD_OK) return PD_EINVAL;
+    const bool gpipe = c->cfg.sync_mode == PD_SYNC_GPIPE;
+    if (gpipe) {
+        // flush groups of D = noam (0 => NOAM = n) minibatches; k_s = D (a whole group in
+        // flight at every stage but the last, which runs F B back to back), R27
+        const int D = noam > 0 ? noam : c->n;
+        if (M % D) return PD_EINVAL;
+        k.assign(c->n, D);
+        k[c->n - 1] = 1;
+        for (int s = 0; s < c->n; ++s)
+            if (D > c->kalloc[s]) return PD_EINVAL;
+    } else {
+        if (inflight_counts(c->plan, noam, k) != PD_OK) return PD_EINVAL;
+    }
     for (int s = 0; s < c->n; ++s)
         if (k[s] > c->kalloc[s]) return PD_EINVAL;
     if (c->n_data < 1) return PD_ESTATE;
@@ -2380,11 +2433,11 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
             const int Rs = c->plan.stage[s].replicas;
             for (int r = 0; r < Rs; ++r) {
                 const int id = c->worker_id(s, r);
-                const std::vector<Op> ops = worker_ops(Rs, r, k[s], M);
-                const int Mr = (int)(ops.size() / 3);
+                const std::vector<Op> ops = gpipe ? gpipe_ops(s + 1 == c->n, k[0], M) : worker_ops(Rs, r, k[s], M);
+                const int Mr = M / Rs;
                 c->opF[id].assign(Mr, -1);
                 c->opB[id].assign(Mr, -1);
-                c->opU[id].assign(Mr, -1);
+                c->opU[id].assign(Mr, -1);  // (GPipe: M / D updates, indexed by group)
                 for (size_t i = 0; i < ops.size(); ++i)
                     (ops[i].kind == 'F' ? c->opF : ops[i].kind == 'B' ? c->opB : c->opU)[id][ops[i].j] = (int32_t)i;
             }

@@ -47,6 +47,30 @@ std::vector<Op> worker_ops(int R_s, int replica, int k_s, int M) {
     return ops;
 }
 
+// GPipe comparison schedule (§5.4; R27), straight plans: flush groups of
+// D minibatches.  Stages s < n-1: F(t) for the group, then B(t) for the group in t order; the
+// last stage: F(t) B(t) back to back (its backward starts immediately, L719-721); one U per
+// group (Op.j = group index, Op.t = the group's last minibatch) applies the aggregated
+// gradient (L1277-1279).  F / B carry j = t (one replica).
+std::vector<Op> gpipe_ops(bool last_stage, int D, int M) {
+    std::vector<Op> ops;
+    ops.reserve(2 * M + M / D + 1);
+    for (int g = 0; g * D < M; ++g) {
+        const int t0 = g * D, t1 = t0 + D;
+        if (last_stage) {
+            for (int t = t0; t < t1; ++t) {
+                ops.push_back({'F', t, t});
+                ops.push_back({'B', t, t});
+            }
+        } else {
+            for (int t = t0; t < t1; ++t) ops.push_back({'F', t, t});
+            for (int t = t0; t < t1; ++t) ops.push_back({'B', t, t});
+        }
+        ops.push_back({'U', t1 - 1, g});
+    }
+    return ops;
+}
+
 int recv_ring_depth(const pd_plan_t &plan, const std::vector<int> &k, int s) {
     // An activation for t lives in stage s's ring from F(s-1, t) until B(s, t).  The
     // producer replica runs F(t_{j+k}) only after B(t_j), which waits for B(s, t_j), so at

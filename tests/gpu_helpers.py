@@ -33,7 +33,8 @@ def run_both(wl, stage_last, replicas, M, dtype, n_data=5, noam=0, lr=None, reco
         losses = P.losses(M)
         stats = P.stats()
     ref = oracle.run(wl.layers, stage_last, replicas, wl.batch, M, p0, data, wl.optimizer, lr, wl.beta1,
-                     wl.beta2, wl.eps, depth=noam, vertical_sync=sync_mode == pd.PD_SYNC_VERTICAL)
+                     wl.beta2, wl.eps, depth=noam, vertical_sync=sync_mode == pd.PD_SYNC_VERTICAL,
+                     gpipe=sync_mode == pd.PD_SYNC_GPIPE)
     return dict(p0=p0, got=got, trace=trace, vmap=vmap, losses=losses, stats=stats, ref=ref)
 
 

@@ -118,6 +118,27 @@ def test_create_sync_mode_validation():
     assert ei.value.status == pd.PD_EUNSUPPORTED
 
 
+def test_gpipe_mode_validation():
+    # PD_SYNC_GPIPE (§5.4, R27): straight plans only; pd_run's group size D must divide M and
+    # fit the rings sized at pd_create (D <= max(n, max_depth)) -- checked before any device work
+    wl = synth.workload("mlp_small")
+    with pytest.raises(pd.PDError) as ei:
+        pd.pd_create(pd.Plan.manual([1, 2], [2, 1]), wl.layers, pd.PD_FP32, minibatch=16, sync_mode=pd.PD_SYNC_GPIPE)
+    assert ei.value.status == pd.PD_EUNSUPPORTED
+    ctx = pd.pd_create(pd.Plan.manual([1, 2], [1, 1]), wl.layers, pd.PD_FP32, minibatch=16,
+                       sync_mode=pd.PD_SYNC_GPIPE, max_depth=4)
+    try:
+        for M, D in ((7, 0), (9, 2), (8, 8)):
+            with pytest.raises(pd.PDError) as ei:
+                pd.pd_run(ctx, M, D)
+            assert ei.value.status == pd.PD_EINVAL, (M, D)
+        with pytest.raises(pd.PDError) as ei:  # valid sizes, but no worker initialised
+            pd.pd_run(ctx, 8, 4)
+        assert ei.value.status == pd.PD_ESTATE
+    finally:
+        pd.pd_destroy(ctx)
+
+
 @pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU failure mode")
 def test_device_calls_fail_loudly_without_gpu():
     wl = synth.workload("mlp_small")
