@@ -57,12 +57,17 @@ def _ws(split, M, N):
 
 
 @pytest.mark.parametrize("split", [0, 1, 2])
+@pytest.mark.parametrize("csplit", [0, 1, 2])
 @pytest.mark.parametrize("M,N,K,amn,bmn", SHAPES[:4] + [
     (32, 4096, 4096, 0, 0),    # small-M split-K: 8 splits of a 128-row tile holding 32 rows
     (40, 4096, 2048, 0, 1),    # ragged rows inside an epilogue warp's 32-row slab
     (256, 4096, 4096, 0, 0),   # the MLP-4096 forward shape (2-CTA, 4 splits)
 ])
-def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split):
+def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split, csplit, monkeypatch):
+    # csplit 2 (default): small-M shapes take the pair cluster split-K kernel, 1: the single-CTA
+    # cluster split-K kernel (DSMEM reductions); 0: the workspace split-K path (PD_GEMM_CSPLIT,
+    # read per call)
+    monkeypatch.setenv("PD_GEMM_CSPLIT", str(csplit))
     A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16, seed=1)
     bias = torch.randn(N, device="cuda")
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
@@ -77,8 +82,10 @@ def test_tc_gemm_store_bias_relu(M, N, K, amn, bmn, split):
 
 
 @pytest.mark.parametrize("split", [0, 1, 2])
+@pytest.mark.parametrize("csplit", [0, 1, 2])
 @pytest.mark.parametrize("M,N,K", [(256, 1024, 4096), (40, 4096, 4096), (256, 4096, 4096)])
-def test_tc_gemm_mask_epilogue(split, M, N, K):
+def test_tc_gemm_mask_epilogue(split, M, N, K, csplit, monkeypatch):
+    monkeypatch.setenv("PD_GEMM_CSPLIT", str(csplit))
     A, B, As, Bs = _operands(M, N, K, 0, 1, torch.bfloat16, seed=2)
     mask = torch.relu(torch.randn(M, N, device="cuda")).to(torch.bfloat16)
     out = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
@@ -207,11 +214,53 @@ def test_bias_grad_kernel(rows, cols, mode):
     assert torch.equal(slot, master.to(torch.bfloat16))
 
 
-def test_split_k_reduction_in_the_pipeline():
-    # an M = 256 all-linear bf16 stage whose forward / dX GEMMs split K (2-CTA 256-row tiles,
-    # 2 splits at K = 1024), reduced in split order by the separate reduction kernel.  Schedule
-    # exact, parameters vs the fp32 oracle within the bf16 tolerance.  (The in-kernel and
-    # cluster split-K reductions were measured slower in the step and are gone.)
+@pytest.mark.parametrize("M,N,K,amn,bmn,S", [
+    (256, 4096, 4096, 0, 0, 4),   # MLP-4096 forward: 32 tiles x 4 splits = 128 CTAs
+    (256, 4096, 4096, 0, 1, 4),   # MLP-4096 dX (MN-major weights)
+    (512, 4096, 4096, 0, 0, 2),   # 64 tiles: 2 splits fit the machine
+    (200, 1000, 1000, 0, 1, 4),   # ragged rows / columns / K tail inside the last split
+    (40, 2056, 776, 0, 0, 4),     # ragged everything, K not a multiple of 64
+    (256, 1024, 512, 0, 0, 2),    # K = 8 blocks: 4 splits would leave 2 blocks each
+])
+def test_cluster_splitk_gemm(M, N, K, amn, bmn, S, monkeypatch):
+    # the cluster split-K kernels (the K-splits of a tile = one cluster, partials summed in
+    # split order through DSMEM; mode 2: CTA pairs x 2 K halves, mode 1: S single CTAs)
+    # against torch fp32, and against the workspace split-K path (mode 0)
+    A, B, As, Bs = _operands(M, N, K, amn, bmn, torch.bfloat16, seed=5)
+    bias = torch.randn(N, device="cuda")
+    mask = torch.relu(torch.randn(M, N, device="cuda")).to(torch.bfloat16)
+    ws = torch.zeros(8 * M * N, device="cuda")
+    outs = {}
+    for cs in (2, 1, 0):
+        monkeypatch.setenv("PD_GEMM_CSPLIT", str(cs))
+        o1 = torch.full((M, N), 7.0, device="cuda", dtype=torch.bfloat16)
+        o2 = torch.full((M, N), 7.0, device="cuda", dtype=torch.bfloat16)
+        pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], o1.data_ptr(),
+                          N, amn, bmn, pd.PD_EPI_STORE, bias=bias.data_ptr(), relu=1, workspace=ws.data_ptr(),
+                          workspace_bytes=ws.numel() * 4)
+        pd.pd_kernel_gemm(pd.PD_BF16, M, N, K, As.data_ptr(), As.shape[1], Bs.data_ptr(), Bs.shape[1], o2.data_ptr(),
+                          N, amn, bmn, pd.PD_EPI_MASK, mask=mask.data_ptr(), ldm=N, workspace=ws.data_ptr(),
+                          workspace_bytes=ws.numel() * 4)
+        torch.cuda.synchronize()
+        outs[cs] = (o1, o2)
+    acc = A.float() @ B.float().t()
+    for cs in (2, 1):
+        o1, o2 = outs[cs]
+        assert _rel(o1, torch.relu(acc + bias)) < 1e-2, cs
+        assert _rel(o2, acc * (mask.float() > 0)) < 1e-2, cs
+        assert bool(((o2.float() == 0) | (mask.float() > 0)).all())
+        # the reductions sum fp32 partials: equal up to bf16 output rounding
+        for a, b in zip(outs[cs], outs[0]):
+            assert _rel(a, b.float()) < 1e-2, cs
+
+
+@pytest.mark.parametrize("csplit", [2, 1, 0])
+def test_split_k_reduction_in_the_pipeline(csplit, monkeypatch):
+    # an M = 256 all-linear bf16 stage whose forward / dX GEMMs split K: the cluster split-K
+    # kernels (csplit 2, the default: CTA pairs x 2 K halves; 1: single CTAs; DSMEM reduction
+    # in split order) or the 2-CTA workspace split-K + reduction kernel (csplit 0).  Schedule exact, parameters vs the fp32 oracle
+    # within the bf16 tolerance.
+    monkeypatch.setenv("PD_GEMM_CSPLIT", str(csplit))
     import synth
     from gpu_helpers import run_both, assert_schedule_exact, param_errors, BF16_TOL
     wl = synth.Workload("mlp1024", synth.mlp([1024, 1024, 1024, 1024], 256), 256, synth.SGD, 0.05)
