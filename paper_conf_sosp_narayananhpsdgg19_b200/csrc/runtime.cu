@@ -2323,12 +2323,11 @@ pd_status pd_run(pd_ctx *c, int M, int noam) {
     std::vector<int> k;
     const bool gpipe = c->cfg.sync_mode == PD_SYNC_GPIPE;
     if (gpipe) {
-        // flush groups of D = noam (0 => NOAM = n) minibatches; k_s = D (a whole group in
-        // flight at every stage but the last, which runs F B back to back), R27
+        // flush groups of D = noam (0 => NOAM = n) minibatches: k_s = D at every stage (a whole
+        // group in flight; the last stage runs F B back to back), R27; Exec reads D as k[0]
         const int D = noam > 0 ? noam : c->n;
         if (M % D) return PD_EINVAL;
         k.assign(c->n, D);
-        k[c->n - 1] = 1;
         for (int s = 0; s < c->n; ++s)
             if (D > c->kalloc[s]) return PD_EINVAL;
     } else {

@@ -70,9 +70,11 @@ def test_gpipe_bf16_discriminates_the_schedule():
     ref = res["ref"]
     other = oracle.run(wl.layers, last, [1] * 4, wl.batch, M, res["p0"], synth.make_data(wl, 4), wl.optimizer,
                        wl.lr)
+    # distances relative to the GPipe trajectory's delta: the 1F1B oracle is `gap` away, the
+    # run must be within gap/4 (so, by the triangle inequality, >= 3 gap/4 from 1F1B's)
     gap = rel_l2(other.params, ref.params, res["p0"])
+    assert gap > 1.0, gap
     assert rel_l2(res["got"], ref.params, res["p0"]) <= gap / 4, gap
-    assert rel_l2(res["got"], other.params, res["p0"]) > gap / 4
 
 
 def test_gpipe_second_run_continues():
@@ -88,6 +90,7 @@ def test_gpipe_second_run_continues():
         P.run(M)
         P.run(M)
         got = P.params([synth.param_count(L) for L in wl.layers])
+        got = [got[l] for l in range(len(wl.layers))]
     ref = oracle.run(wl.layers, last, [1] * 4, wl.batch, 2 * M, p0, data, wl.optimizer, wl.lr, gpipe=True)
     import torchref
     assert torchref.max_rel_err(got, ref.params) < FP32_TOL
