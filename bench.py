@@ -460,8 +460,9 @@ def main():
     ap.add_argument("--plan", default="pipeline", choices=["pipeline", "dp"],
                     help="pipeline: pd_plan straight pipeline (VGG: (N-1)-1); dp: one stage x N replicas "
                          "(pure data parallelism, SURVEY §8(f) NEXT #1)")
-    ap.add_argument("--sync", default="stash", choices=["stash", "vertical"],
-                    help="weight stashing (default) or vertical sync (§3.3; straight plans)")
+    ap.add_argument("--sync", default="stash", choices=["stash", "vertical", "gpipe"],
+                    help="weight stashing (default), vertical sync (§3.3; straight plans) or the GPipe "
+                         "comparison schedule (§5.4: flush every NOAM minibatches, aggregated update)")
     args = ap.parse_args()
     if args.stage_plan < 0:
         args.stage_plan = {"gnmt16": 8, "gnmt8": 4, "mlp4096": 4, "vgg16": 8}[args.config]
@@ -520,7 +521,7 @@ def main():
     p0 = synth.init_params(layers) if True else None
     n_data = 8
     data = synth.make_data(wl, n_data)
-    sync = pd.PD_SYNC_VERTICAL if args.sync == "vertical" else pd.PD_SYNC_STASH
+    sync = {"stash": pd.PD_SYNC_STASH, "vertical": pd.PD_SYNC_VERTICAL, "gpipe": pd.PD_SYNC_GPIPE}[args.sync]
     P = Pipeline(plan, layers, p0, dtype=pd.PD_BF16, optimizer=wl.optimizer, lr=wl.lr, minibatch=B, sync_mode=sync,
                  record_trace=int(os.environ.get("PD_BENCH_TRACE", "2")), device_of=lambda g: g if world > 1 else local_rank,
                  local=(lambda wid: wid == rank) if world > 1 else None,
