@@ -923,27 +923,53 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const uint32_t tmem_base = *tmem_slot;
     if (threadIdx.x == 0) PROBE(1);
     if (warp == 0 && lane == 0) mbar_expect_tx(smem_u32(rbar), SLICE);
+    // programmatic dependent launch: the next GEMM of the chain may be scheduled now (it only
+    // prefetches its weights before its own griddepcontrol.wait)
+    if (threadIdx.x == 0) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 
     if (warp == 0) {
         if (lane == 0) {  // ===== TMA producer: this CTA's A rows and B half land on the leader's barrier
             int stage = 0;
             uint32_t phase = 0;
-            for (int kb = kb0; kb < kb1; kb += KS) {
+            auto load_a = [&](uint32_t sa, uint32_t fb, int k0) {
+                if (AMAJ == KMAJ) {
+                    tma_load_2d_cg<2>(sa, &tmA, fb, k0, m0);
+                } else {
+#pragma unroll
+                    for (int j = 0; j < BM / 64; ++j) tma_load_2d_cg<2>(sa + j * BK * 128, &tmA, fb, m0 + 64 * j, k0);
+                }
+            };
+            auto load_b = [&](uint32_t sb, uint32_t fb, int k0) {
+                if (BMAJ == KMAJ) tma_load_2d_cg<2>(sb, &tmB, fb, k0, n0 + (int)prank * 64);
+                else tma_load_2d_cg<2>(sb, &tmB, fb, n0 + (int)prank * 64, k0);
+            };
+            // prologue: the weights (B) of the first ring stages do not depend on the previous
+            // kernel -- issue them before griddepcontrol.wait, the activations (A) after it
+            const int npre = min(NST, (kb1 - kb0 + KS - 1) / KS);
+            for (int st = 0; st < npre; ++st) {
+                const uint32_t fb = smem_u32(&full[st]) & 0xFEFFFFFFu;
+                const int kb = kb0 + st * KS, nk = min(KS, kb1 - kb);
+                if (prank == 0) mbar_expect_tx(fb, 2 * nk * C::STAGE_BYTES);
+                for (int h = 0; h < nk; ++h)
+                    load_b(smem_u32(smem + (st * KS + h) * C::STAGE_BYTES) + C::A_BYTES, fb, (kb + h) * BK);
+            }
+            asm volatile("griddepcontrol.wait;" ::: "memory");
+            for (int st = 0; st < npre; ++st) {
+                const uint32_t fb = smem_u32(&full[st]) & 0xFEFFFFFFu;
+                const int kb = kb0 + st * KS, nk = min(KS, kb1 - kb);
+                for (int h = 0; h < nk; ++h) load_a(smem_u32(smem + (st * KS + h) * C::STAGE_BYTES), fb, (kb + h) * BK);
+            }
+            stage = npre % NST;
+            phase = npre == NST ? 1u : 0u;
+            for (int kb = kb0 + npre * KS; kb < kb1; kb += KS) {
                 mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
                 const uint32_t fb = smem_u32(&full[stage]) & 0xFEFFFFFFu;
                 const int nk = min(KS, kb1 - kb);
                 if (prank == 0) mbar_expect_tx(fb, 2 * nk * C::STAGE_BYTES);
                 for (int h = 0; h < nk; ++h) {
-                    const uint32_t sa = smem_u32(smem + (stage * KS + h) * C::STAGE_BYTES), sb = sa + C::A_BYTES;
-                    const int k0 = (kb + h) * BK;
-                    if (AMAJ == KMAJ) {
-                        tma_load_2d_cg<2>(sa, &tmA, fb, k0, m0);
-                    } else {
-#pragma unroll
-                        for (int j = 0; j < BM / 64; ++j) tma_load_2d_cg<2>(sa + j * BK * 128, &tmA, fb, m0 + 64 * j, k0);
-                    }
-                    if (BMAJ == KMAJ) tma_load_2d_cg<2>(sb, &tmB, fb, k0, n0 + (int)prank * 64);
-                    else tma_load_2d_cg<2>(sb, &tmB, fb, n0 + (int)prank * 64, k0);
+                    const uint32_t sa = smem_u32(smem + (stage * KS + h) * C::STAGE_BYTES);
+                    load_a(sa, fb, (kb + h) * BK);
+                    load_b(sa + C::A_BYTES, fb, (kb + h) * BK);
                 }
                 if (++stage == NST) { stage = 0; phase ^= 1; }
             }
@@ -1605,13 +1631,16 @@ cudaError_t launch_csplit2(const Gemm &g, const CUtensorMap &ma, const CUtensorM
     cfg.blockDim = dim3(NUM_THREADS);
     cfg.dynamicSmemBytes = C::SMEM;
     cfg.stream = s;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 4;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
-    cfg.numAttrs = 1;
+    const char *pv = getenv("PD_GEMM_PDL");  // 0: no programmatic dependent launch (A/B measurement)
+    cfg.numAttrs = g.pdl && !(pv && atoi(pv) == 0) ? 2 : 1;
     EpiArgs ep = e;
     ep.probe = probe_buf();
     cudaError_t err = cudaLaunchKernelEx(&cfg, kern, ma, mb, mo, mk, ep, g.M, g.N, g.K);

@@ -110,6 +110,11 @@ struct Gemm {
     int ksplit = 1;       // explicit split-K (EPI_F32 with atomic_out)
     int max_ctas = 0;     // cap on resident CTAs (0 = every SM): leaves SMs to a concurrent kernel
     int atomic_out = 0;   // EPI_F32: fp32 atomic accumulation into out
+    // programmatic dependent launch (cluster split-K path): the kernel may start while the
+    // previous kernel of the stream is still running; it loads only B (the weights) before
+    // griddepcontrol.wait.  Only for a GEMM whose predecessor is the previous layer's GEMM of
+    // the same chain (whose first kernel launched normally), so B is never being written.
+    int pdl = 0;
 };
 
 // cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}

@@ -507,7 +507,7 @@ cudaError_t run_gemm(int bf16, const Gemm &g, cudaStream_t s) { return bf16 ? ge
 
 // y = act(x W^T + b)
 void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, const float *bias_f32, const void *x,
-                    void *y, float *ws, long ws_bytes) {
+                    void *y, float *ws, long ws_bytes, int pdl = 0) {
     const int B = L.c->cfg.minibatch;
     Gemm g;
     g.M = (int)rows_of(d, B);
@@ -526,6 +526,7 @@ void linear_forward(const LayerCtx &L, const pd_layer_desc &d, const void *W, co
     g.relu = d.act == PD_ACT_RELU;
     g.workspace = ws;
     g.workspace_bytes = ws_bytes;
+    g.pdl = pdl;
     CK(run_gemm(L.bf16, g, L.w->stream));
 }
 
@@ -731,7 +732,10 @@ struct Exec {
             cudaEvent_t k0 = kstart(0);
             if (d.kind == PD_LINEAR) {
                 LayerCtx lc{c, w, bf16};
-                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes);
+                // the previous kernel on the stream is the previous layer's GEMM: this one may
+                // start early and prefetch its weights (Gemm::pdl)
+                const int pdl = bf16 && l > w->first && layer(l - 1).kind == PD_LINEAR && !w->fbias;
+                linear_forward(lc, d, Wl(l, slot), bias_f32(l, slot), x, y, w->ws, w->ws_bytes, pdl);
             } else if (d.kind == PD_LSTM) {
                 lstm_forward(l, j, slot, x, y);
             } else if (d.kind == PD_EMBEDDING) {
