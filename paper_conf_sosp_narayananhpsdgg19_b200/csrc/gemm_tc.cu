@@ -1946,6 +1946,11 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         if ((long)mb * ((g.N + 255) / 256) < sms || g.N <= 128) BN = 128;
         if (BN == 128 && ((long)mb * ((g.N + 127) / 128) < sms || g.N <= 64)) BN = 64;
     }
+    // long-K reductions split K to fill the machine (atomic_out, ksplit 0: conv weight
+    // gradients over N*H*W pixels), so narrow tiles buy no parallelism -- only ingest: the
+    // widest tile has the most FLOPs per streamed byte (128 x 256 x 64 per 48 KB vs 128 x 64 x 64
+    // per 24 KB; the ingest of ~90 GB/s per SM bounds these tiles)
+    if (g.atomic_out && g.ksplit == 0 && g.N >= 256 && !g.conv.c8) BN = 256;
     BN = env_int("PD_GEMM_BN", BN);  // tuning override (tools/gemm_bench.py)
     if (cg == 2 && BN < 128) BN = 128;
     CUtensorMap ma, mbm;
