@@ -1853,7 +1853,7 @@ static cudaError_t gemm_c8(const Gemm &g, cudaStream_t s) {
     const int sms = num_sms();
     const long tiles = (g.M + BM - 1) / BM;
     const int kb = (g.K + BK - 1) / BK;
-    long S = (2L * sms + tiles - 1) / tiles;
+    long S = (2L * sms + tiles - 1) / tiles;  // (2, 4 and 8 units per SM measured equal here)
     if (S > kb / 4) S = kb / 4;
     if (S < 1) S = 1;
     const long kper = (kb + S - 1) / S;
@@ -1974,7 +1974,10 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     if (g.atomic_out && g.ksplit == 0) {  // long-K reductions (conv dW): fill the machine
         const long tiles = (long)mb * ((g.N + BN - 1) / BN);
         const int kb = (g.K + BK - 1) / BK;
-        long S = (2L * sms + tiles - 1) / tiles;
+        // ~8 (tile, K-range) units per SM: shorter ranges balance the persistent CTAs and keep
+        // the concurrently streamed pixel windows close together in L2 (measured on VGG-16: 2 ->
+        // 4 -> 8 -> 16 -> 32 units per SM: 5.85k, 6.16k, 6.32k, 6.30k, 6.09k samples/s)
+        long S = (8L * sms + tiles - 1) / tiles;
         if (S > kb / 4) S = kb / 4;
         if (S < 1) S = 1;
         const long kper = (kb + S - 1) / S;
