@@ -1109,6 +1109,152 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
 }
 
+// ---------------------------------------------------------------- RGB first conv layer, forward
+// Packed-tap forward of a Cp = 8 input (the RGB layer: 3 channels padded to 8, 16 bytes per
+// padded-grid pixel).  Output pixel m, tap t reads input row m + shift[t]; the 9 shifted
+// 128-row windows of a tile are all inside ONE contiguous span of rows
+// [m0 - (Wp+1), m0 + 128 + (Wp+1)), so a tile's whole A operand is one 1-D bulk copy of
+// (128 + 2 (Wp+1)) x 16 B instead of 9 TMA boxes of 128 16-byte rows (the row count, not the
+// bytes, bounded the box version: 566 us for 418 MB of output at 224^2, B = 64).  [px][8]
+// bf16 IS the unswizzled K-major core-matrix layout (8 rows x 16 B), so tap t's operand is the
+// span at row offset shift[t] + Wp + 1 -- two taps per K = 16 MMA, their distance as the
+// descriptor's leading byte offset.  The weights W [Co][72] (+ a zero K = 72..79 slot) stay
+// resident in shared memory for the whole persistent launch.
+constexpr int C8_NS = 6;  // span ring depth
+__global__ void __launch_bounds__(NUM_THREADS, 1)
+    conv_c8_fwd_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__ CUtensorMap tmO,
+                       const __nv_bfloat16 *__restrict__ X, EpiArgs e, int M, int N, int span_bytes) {
+    constexpr int BNW = 64;  // output channels (N <= 64)
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *sB = smem;                                   // 10 slots x 64 rows x 16 B
+    uint8_t *ring = smem + 10 * 1024;                     // C8_NS spans
+    uint8_t *epi_stg = ring + C8_NS * span_bytes;         // 4 warps x 2 x 2 KB (1024-aligned: span_bytes % 1024 == 0)
+    uint64_t *bars = reinterpret_cast<uint64_t *>(epi_stg + 4 * 4096);
+    uint64_t *full = bars, *empty = bars + C8_NS, *tfull = bars + 2 * C8_NS, *tempty = tfull + 2, *bbar = tempty + 2;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bbar + 1);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int Wp = e.conv.Wp, halo = Wp + 1;
+    const int tiles = (M + BM - 1) / BM;
+
+    if (warp == 0 && lane == 0) {
+        asm volatile("prefetch.tensormap [%0];" ::"l"(&tmB) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(&tmO) : "memory");
+        for (int s = 0; s < C8_NS; ++s) {
+            mbar_init(smem_u32(&full[s]), 1);
+            mbar_init(smem_u32(&empty[s]), 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(smem_u32(&tfull[a]), 1);
+            mbar_init(smem_u32(&tempty[a]), 4);
+        }
+        mbar_init(smem_u32(bbar), 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(2 * BNW));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    // zero the span ring once: window rows a clipped copy leaves unwritten (the image's first /
+    // last halo) then hold finite values -- they only feed border outputs, which are zeroed
+    for (int i = threadIdx.x; i < C8_NS * span_bytes / 16; i += NUM_THREADS)
+        reinterpret_cast<uint4 *>(ring)[i] = make_uint4(0, 0, 0, 0);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {  // ===== producer: the weights once, then one span per tile
+            mbar_expect_tx(smem_u32(bbar), 10 * BNW * 16);
+            for (int j = 0; j < 10; ++j) tma_load_2d(smem_u32(sB + j * 1024), &tmB, smem_u32(bbar), 8 * j, 0);
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                long r0 = (long)tile * BM - halo, r1 = (long)tile * BM + BM + halo;  // span rows [r0, r1)
+                uint32_t dst = smem_u32(ring + stage * span_bytes);
+                if (r0 < 0) { dst += (uint32_t)(-r0) * 16; r0 = 0; }
+                if (r1 > M) r1 = M;
+                const uint32_t bytes = (uint32_t)(r1 - r0) * 16;
+                mbar_expect_tx(smem_u32(&full[stage]), bytes);
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                                 dst),
+                             "l"(X + r0 * 8), "r"(bytes), "r"(smem_u32(&full[stage]))
+                             : "memory");
+                if (++stage == C8_NS) { stage = 0; phase ^= 1; }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {  // ===== MMA: K = 80 as 5 x K16, taps (2k, 2k+1); tap 9 = zero weights
+            constexpr uint32_t idesc = make_idesc(BM, BNW, KMAJ, KMAJ);
+            mbar_wait(smem_u32(bbar), 0);
+            int off[10];
+#pragma unroll
+            for (int t = 0; t < 9; ++t) off[t] = (e.conv.a_shift[t] + halo) * 16;
+            off[9] = off[8];  // (any finite rows: its weights are zero)
+            int stage = 0, acc = 0;
+            uint32_t phase = 0, acc_phase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
+                mbar_wait(smem_u32(&full[stage]), phase);
+                tc_fence_after();
+                const uint32_t sp = smem_u32(ring + stage * span_bytes), sb = smem_u32(sB);
+#pragma unroll
+                for (int k = 0; k < 5; ++k) {
+                    const uint64_t ad = smem_desc_ns(sp + off[2 * k], off[2 * k + 1] - off[2 * k], 128);
+                    const uint64_t bd = smem_desc_ns(sb + 2 * k * 1024, 1024, 128);
+                    tc_mma(tmem_base + acc * BNW, ad, bd, idesc, k > 0 ? 1u : 0u);
+                }
+                tc_commit(smem_u32(&empty[stage]));
+                tc_commit(smem_u32(&tfull[acc]));
+                if (++stage == C8_NS) { stage = 0; phase ^= 1; }
+                if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+            }
+        }
+    } else if (warp >= 4) {  // ===== epilogue: bias + ReLU + zero border, bf16 TMA stores
+        const int q = warp & 3;
+        uint8_t *wst = epi_stg + q * 4096;
+        int acc = 0;
+        uint32_t acc_phase = 0, ocnt = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            mbar_wait(smem_u32(&tfull[acc]), acc_phase);
+            tc_fence_after();
+            const int r0 = tile * BM + q * 32;
+#pragma unroll 1
+            for (int c = 0; c < BNW / 32 && c * 32 < N; ++c) {
+                float v[32];
+                tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BNW + c * 32, v);
+                epi_math<EPI_STORE>(e, v, r0 + lane, c * 32, N, nullptr, lane);
+                if (lane == 0) bulk_wait_read1();
+                __syncwarp();
+                uint8_t *ot = wst + (ocnt & 1) * 2048;
+                epi_stage<EPI_STORE>(ot, v, lane);
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) {
+                    tma_store_2d(&tmO, smem_u32(ot), c * 32, r0);
+                    bulk_commit();
+                }
+                ++ocnt;
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
+            if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+        }
+        if (lane == 0) bulk_wait_read0();
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(2 * BNW));
+    }
+}
+
 // ---------------------------------------------------------------- dW GEMM + fused optimizer update
 // The weight-gradient GEMM of an unreplicated stage never leaves the chip: its accumulator
 // tile is consumed in TMEM by the update, which reads the fp32 master tile (and Adam m, v),
@@ -1834,8 +1980,31 @@ static cudaError_t gemm_c8(const Gemm &g, cudaStream_t s) {
     e.bias = g.bias;
     e.relu = g.relu;
     e.ksplit = 1;
+    if (g.conv.c8 == 1 && g.lda == 8 && g.conv.Wp > 0) {
+        // forward: one contiguous span of X rows per tile (conv_c8_fwd_kernel); W resident
+        if (g.N > 64 || g.amaj != KMAJ || g.bmaj != KMAJ || g.epi != EPI_STORE) return cudaErrorInvalidValue;
+        CUtensorMap mo;
+        if (!make_map(&mbm, g.B, 72, g.N, g.ldb, 8, 64, false, 0) || !make_map(&mo, g.out, g.N, g.M, g.ldo, 32, 32, false, 64))
+            return cudaErrorInvalidValue;
+        const int span = ((BM + 2 * (g.conv.Wp + 1)) * 16 + 1023) / 1024 * 1024;
+        const int smem = 10 * 1024 + C8_NS * span + 4 * 4096 + 256 + 1024;
+        if (smem > 232448) return cudaErrorInvalidValue;
+        static int attr_smem = 0;
+        if (smem > attr_smem) {
+            cudaError_t err = cudaFuncSetAttribute(conv_c8_fwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+            if (err != cudaSuccess) return err;
+            attr_smem = smem;
+        }
+        const int tiles = (g.M + BM - 1) / BM;
+        const int grid = tiles < num_sms() ? tiles : num_sms();
+        conv_c8_fwd_kernel<<<grid, NUM_THREADS, smem, s>>>(mbm, mo, static_cast<const __nv_bfloat16 *>(g.A), e, g.M, g.N,
+                                                          span);
+        ++tl_launches;
+        return cudaGetLastError();
+    }
     if (g.conv.c8 == 1) {
-        // forward: A = X [M][8] (box {8, 128}), B = W [N][72] (box {8, N}); N <= 64
+        // forward without the output grid (no halo geometry): A = X [M][8] (box {8, 128}),
+        // B = W [N][72] (box {8, N}); N <= 64
         if (g.N > 64 || g.amaj != KMAJ || g.bmaj != KMAJ || g.epi != EPI_STORE) return cudaErrorInvalidValue;
         if (!make_map(&ma, g.A, 8, g.M, g.lda, 8, BM, false, 0) ||
             !make_map(&mbm, g.B, 72, g.N, g.ldb, 8, 64, false, 0))
