@@ -605,6 +605,15 @@ def main():
                 "flops_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
                 "flops_per_minibatch": cfl[d],
                 "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"}
+        if roof["traffic"] and avg_s > 0:
+            # the same launch against the memory roof: DRAM bytes of one launch (ncu --set full)
+            # over its live average duration -- a wavefront kernel re-streams every layer's
+            # weights once per wave (they exceed the on-chip capacity at N = 1), so it is bound
+            # by HBM / per-SM ingest, not by the tensor pipe
+            gbs = roof["traffic"] / avg_s / 1e9
+            roof["memory_view"] = {"dram_gbs": gbs, "frac_hbm": gbs / peaks["hbm_gbs"],
+                                   "hbm_peak_gbs": peaks["hbm_gbs"],
+                                   "note": "ncu dram__bytes_read+write per launch / live avg launch time"}
     fw_tflops, dx_tflops, dw_tflops = cls_tflops[0], cls_tflops[1], cls_tflops[2]
     step_share = {cls: float(prof_kern[i] / max(prof_ms, 1e-9)) for i, cls in enumerate(names)}
     step_share["note"] = "profile pass (2 steps, every kernel class event-timed); dW and dX overlap on two streams"
