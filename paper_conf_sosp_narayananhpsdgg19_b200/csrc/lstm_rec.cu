@@ -68,11 +68,9 @@ __device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence
 // split cluster barrier: arrive after the DSMEM reads of a step, wait before this CTA next
 // overwrites what its peers read (its staging buffer / the tiles the staging aliases)
 __device__ __forceinline__ void cl_arrive() { asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory"); }
-__device__ __forceinline__ void cl_sync(int dbg) {
-    if (!(dbg & 2)) {
-        asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-        asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-    }
+__device__ __forceinline__ void cl_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 __device__ __forceinline__ void cl_wait() { asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory"); }
 __device__ __forceinline__ void st_dsmem_v4(uint32_t addr, float a, float b, float c, float d) {
@@ -116,8 +114,6 @@ struct RecArgs {
     const __nv_bfloat16 *dy;
     const float *gates_in, *c_in;
     __nv_bfloat16 *da;
-    int dbg;                    // tools only (PD_LSTM_DBG): 1 no dependency waits, 2 no cluster barriers,
-                                // 4 relaxed publish (no release), 8 no MMA -- timing experiments, wrong results
     unsigned long long *probe;  // tools: [grid][T][8] %globaltimer stamps by thread 0 (nullptr = off)
 };
 
@@ -251,11 +247,10 @@ __global__ void __launch_bounds__(RT, 1)
         float acc[4][4] = {};
         if (t > 0) {
             const uint32_t par = (uint32_t)(t - 1) & 1;
-            if (t > 1 && !(a.dbg & 2)) cl_wait();  // every owner finished reading the previous step's partials
+            if (t > 1) cl_wait();  // every owner finished reading the previous step's partials
             if (tid == 0) {
                 // 64 units of h = 8 producer CTAs per K-block
-                if (!(a.dbg & 1))
-                    for (int kb = 0; kb < KB; ++kb) wait_count(a.cnt + (k0 >> 6) + kb, 8u * t);
+                for (int kb = 0; kb < KB; ++kb) wait_count(a.cnt + (k0 >> 6) + kb, 8u * t);
                 fence_proxy_async_global();
                 for (int kb = 0; kb < KB; ++kb) {
                     mbar_expect_tx(full0 + kb * 8, (uint32_t)N * 128);
@@ -263,8 +258,7 @@ __global__ void __launch_bounds__(RT, 1)
                 }
                 stamp(a, t, 1);
             } else if (tid == 32) {
-                if (a.dbg & 8) tc_commit(mma_bar);
-                else issue_mmas<0>(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
+                issue_mmas<0>(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
             }
             __syncwarp();
             mbar_wait(mma_bar, par);
@@ -283,7 +277,7 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
                         for (int u = 0; u < 4; ++u) acc[g][u] += recv[((src * 4 + g) * 8 + u4 + u) * 64 + b];
             }
-            if (!(a.dbg & 2)) cl_arrive();
+            cl_arrive();
             stamp(a, t, 4);
         }
         float ig[4], fg[4], gg[4], og[4], cc[4], hh[4];
@@ -307,8 +301,7 @@ __global__ void __launch_bounds__(RT, 1)
         }
         __syncthreads();
         if (tid == 0 && t + 1 < T) {
-            if (a.dbg & 4) atomicAdd(a.cnt + (U0 >> 6), 1u);
-            else red_release_add(a.cnt + (U0 >> 6), 1u);
+            red_release_add(a.cnt + (U0 >> 6), 1u);
         }
         if (act) {
             const long r4 = ((long)t * B + b) * 4 * H + j;
@@ -321,7 +314,7 @@ __global__ void __launch_bounds__(RT, 1)
         stamp(a, t, 5);
     }
     tc_fence_before();
-    if (T > 1 && !(a.dbg & 2)) cl_wait();  // no peer may push into / read from an exited CTA
+    if (T > 1) cl_wait();  // no peer may push into / read from an exited CTA
     if (warp == 0) tmem_free(tmem, 64);
 }
 
@@ -419,11 +412,10 @@ __global__ void __launch_bounds__(RT, 1)
         }
         if (s > 0) {
             const uint32_t par = (uint32_t)(s - 1) & 1;
-            if (s > 1 && !(a.dbg & 2)) cl_wait();  // every owner finished reading the previous step's partials
+            if (s > 1) cl_wait();  // every owner finished reading the previous step's partials
             if (tid == 0) {
                 // 64 gate rows of da = 4 producer CTAs per K-block
-                if (!(a.dbg & 1))
-                    for (int kb = 0; kb < KB; ++kb) wait_count(a.cnt + (k0 >> 6) + kb, 4u * s);
+                for (int kb = 0; kb < KB; ++kb) wait_count(a.cnt + (k0 >> 6) + kb, 4u * s);
                 fence_proxy_async_global();
                 for (int kb = 0; kb < KB; ++kb) {
                     mbar_expect_tx(full0 + kb * 8, (uint32_t)N * 128);
@@ -431,8 +423,7 @@ __global__ void __launch_bounds__(RT, 1)
                 }
                 stamp(a, s, 1);
             } else if (tid == 32) {
-                if (a.dbg & 8) tc_commit(mma_bar);
-                else issue_mmas<1>(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
+                issue_mmas<1>(tmem, smem_u32(sW), smem_u32(sX), full0, mma_bar, KB, N, par);
             }
             __syncwarp();
             mbar_wait(mma_bar, par);
@@ -452,7 +443,7 @@ __global__ void __launch_bounds__(RT, 1)
 #pragma unroll
                 for (int u = 0; u < 8; ++u) dh[u] += rec[u];
             }
-            if (!(a.dbg & 2)) cl_arrive();
+            cl_arrive();
             stamp(a, s, 4);
         }
         if (act) {
@@ -488,7 +479,7 @@ __global__ void __launch_bounds__(RT, 1)
         stamp(a, s, 5);
     }
     tc_fence_before();
-    if (T > 1 && !(a.dbg & 2)) cl_wait();
+    if (T > 1) cl_wait();
     if (warp == 0) tmem_free(tmem, 64);
 }
 
@@ -562,7 +553,6 @@ cudaError_t lstm_rec_fwd(const float *gx, const float *b_ih, const float *b_hh, 
     a.T = T, a.B = B, a.H = H, a.N = (B + 15) / 16 * 16;
     a.cnt = cnt, a.W = Whh, a.gx = gx, a.b_ih = b_ih, a.b_hh = b_hh, a.gates = gates, a.c = c, a.h = h;
     a.probe = probe;
-    if (const char *e = getenv("PD_LSTM_DBG")) a.dbg = atoi(e);
     CUtensorMap map;
     CUtensorMap wmap;
     if (!tma_map_bf16(&map, h, H, (long)T * B, H, 64, a.N) || !tma_map_bf16(&wmap, Whh, H, 4L * H, H, 64, 32))
@@ -579,7 +569,6 @@ cudaError_t lstm_rec_bwd(const __nv_bfloat16 *dy, const float *gates, const floa
     a.T = T, a.B = B, a.H = H, a.N = (B + 15) / 16 * 16;
     a.cnt = cnt, a.W = Whh, a.dy = dy, a.gates_in = gates, a.c_in = c, a.da = da;
     a.probe = probe;
-    if (const char *e = getenv("PD_LSTM_DBG")) a.dbg = atoi(e);
     CUtensorMap map;
     CUtensorMap wmap;
     if (!tma_map_bf16(&map, da, 4L * H, (long)T * B, 4L * H, 64, a.N) || !tma_map_bf16(&wmap, Whh, H, 4L * H, H, 64, 64))
