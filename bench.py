@@ -135,13 +135,14 @@ def model_profile(layers, B, peaks):
     return T, a, w
 
 
-def ncu_traffic(key):
+def ncu_traffic(key, config):
     """dram__bytes_read.sum + dram__bytes_write.sum per launch (bytes) of kernel `key` from the
-    committed `ncu --set full` capture (profiles/ncu_traffic_r*.json, tools/ncu_traffic.py), or None."""
+    committed `ncu --set full` capture (profiles/ncu_traffic_r*.json, tools/ncu_traffic.py) of
+    this config's launch, or None (a capture of another config's launch does not apply)."""
     import glob
     for path in sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_traffic_r*.json")), reverse=True):
         d = json.load(open(path))
-        if key in d:
+        if key in d and d[key].get("config", config) == config:
             return d[key]["traffic_MB"] * 1e6
     return None
 
@@ -588,7 +589,7 @@ def main():
         achieved = dw_bytes / dw_avg_s / 1e9 if dw_avg_s > 0 else 0.0
         roof = {"bound": "hbm", "kernel": "dW GEMM + fused SGD update (tcgen05, EPI_SGD)",
                 "achieved": achieved, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / peaks["hbm_gbs"], "traffic": ncu_traffic("dw_update_sgd"),
+                "frac": achieved / peaks["hbm_gbs"], "traffic": ncu_traffic("dw_update_sgd", args.config),
                 "traffic_source": "ncu --set full capture of one launch (profiles/ncu_traffic_r*.json); "
                                   "writes still dirty in L2 at kernel end are not in dram__bytes_write",
                 "bytes_per_launch": dw_bytes, "avg_launch_us": dw_avg_s * 1e6,
@@ -601,7 +602,7 @@ def main():
         roof = {"bound": "tensor", "kernel": names[d], "achieved": cls_tflops[d],
                 "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
                 "frac": cls_tflops[d] / peaks["bf16_tflops_sustained"],
-                "traffic": ncu_traffic(names[d]),
+                "traffic": ncu_traffic(names[d], args.config),
                 "flops_per_launch": per_launch, "avg_launch_us": avg_s * 1e6,
                 "flops_per_minibatch": cfl[d],
                 "peak_source": peaks["source"] + " bf16_tflops_sustained (cuBLAS)"}

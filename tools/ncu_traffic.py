@@ -1,12 +1,14 @@
 """Per-launch DRAM traffic of an `ncu --set full` capture (raw page CSV) -> JSON that bench.py
-reports as roofline.traffic.  usage: ncu_traffic.py RAW.csv KEY OUT.json [ROW]  (merges into OUT.json; ROW = the launch, default 0)"""
+reports as roofline.traffic.  usage: ncu_traffic.py RAW.csv KEY OUT.json [ROW] [CONFIG]
+(merges into OUT.json; ROW = the launch, default 0; CONFIG = the bench config the launch came
+from -- bench.py uses the record only for that config)"""
 import csv
 import json
 import os
 import sys
 
 
-def main(raw, key, out, row="0"):
+def main(raw, key, out, row="0", config=None):
     rows = list(csv.reader(open(raw)))
     h, units, vals = rows[0], rows[1], rows[2 + int(row)]
     col = {n: i for i, n in enumerate(h)}
@@ -25,6 +27,8 @@ def main(raw, key, out, row="0"):
            "duration_us": us("gpu__time_duration.sum"),
            "source": os.path.basename(raw)}
     rec["traffic_MB"] = rec["dram_read_MB"] + rec["dram_write_MB"]
+    if config:
+        rec["config"] = config
     d = json.load(open(out)) if os.path.exists(out) else {}
     d[key] = rec
     json.dump(d, open(out, "w"), indent=1)
@@ -32,4 +36,4 @@ def main(raw, key, out, row="0"):
 
 
 if __name__ == "__main__":
-    main(*sys.argv[1:5])
+    main(*sys.argv[1:6])
