@@ -65,6 +65,9 @@ struct EpiArgs {
     ConvGeom conv;      // implicit-GEMM 3x3 convolution geometry (conv.taps == 0: plain GEMM)
     int atomic_out;     // EPI_F32: accumulate with fp32 atomics (split-K / per-tap dW)
     unsigned long long *probe;  // tools only (PD_GEMM_PROBE): per-CTA %globaltimer phase stamps [grid][8]
+    const unsigned *wait_cnt;   // Gemm::wait_cnt (splits run in reverse, each waits for its rows)
+    int wait_T, wait_B;
+    unsigned wait_per;
     const float *bias;
     int relu;
     const __nv_bfloat16 *mask;
@@ -370,10 +373,25 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             int stage = 0;
             uint32_t phase = 0;
             for (int unit = u0; unit < units; unit += ustep) {
-                const int tile = unit % tiles, split = unit / tiles;
+                const int tile = unit % tiles, split = e.wait_cnt ? e.ksplit - 1 - unit / tiles : unit / tiles;
                 const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM;
                 const int n0 = (tile / m_blocks) * BN + (int)rank * BNC;
                 const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
+                if (e.wait_cnt && kb1 > kb0) {
+                    // the rows of this split were produced by a kernel still running (the LSTM
+                    // backward wave): wait for the producer's step counter, then the async proxy
+                    const unsigned target = (unsigned)(e.wait_T - (kb0 * BK) / e.wait_B) * e.wait_per;
+                    unsigned v;
+                    const unsigned long long t0 = gtimer();
+                    do {
+                        asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(e.wait_cnt) : "memory");
+                        if (gtimer() - t0 > 4000000000ull) {
+                            printf("tc_gemm: producer wait timeout (%u < %u)\n", v, target);
+                            __trap();
+                        }
+                    } while (v < target);
+                    asm volatile("fence.proxy.async.global;" ::: "memory");
+                }
                 // coordinates of K-block kb for this CTA (plain GEMM, implicit conv, shifted dW)
                 auto coords = [&](int kb, int &ka, int &ma, int &kbk, int &nb) {
                     const int k0 = kb * BK;
@@ -454,7 +472,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             int acc = 0;
             uint32_t acc_phase = 0;
             for (int unit = u0; unit < units; unit += ustep) {
-                const int split = unit / tiles;
+                const int split = e.wait_cnt ? e.ksplit - 1 - unit / tiles : unit / tiles;
                 const int kb0 = split * kper, kb1 = min(kblocks, kb0 + kper);
                 mbar_wait(smem_u32(&tempty[acc]), acc_phase ^ 1);
                 tc_fence_after();
@@ -514,7 +532,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         uint32_t acc_phase = 0;
         uint32_t ocnt = 0, mcnt = 0, mph = 0;  // staging-buffer / mask-buffer counters and phases
         for (int unit = u0; unit < units; unit += ustep) {
-            const int tile = unit % tiles, split = unit / tiles;
+            const int tile = unit % tiles, split = e.wait_cnt ? e.ksplit - 1 - unit / tiles : unit / tiles;
             const int m0 = (tile % m_blocks) * (BM * CG) + (int)rank * BM, n0 = (tile / m_blocks) * BN;
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
             tc_fence_after();
@@ -1672,7 +1690,8 @@ cudaError_t launch(const Gemm &g, const CUtensorMap &ma, const CUtensorMap &mb, 
         }
     }
     const int units = ((g.M + BM * CG - 1) / (BM * CG)) * ((g.N + BN - 1) / BN) * e.ksplit;
-    const int slots = num_sms() / CG;
+    int slots = num_sms() / CG;
+    if (g.max_ctas > 0 && g.max_ctas / CG < slots) slots = g.max_ctas / CG > 0 ? g.max_ctas / CG : 1;
     const int grid = CG * (units < slots ? units : slots);
     const int cluster = CG;
     if (cluster == 1) {
@@ -2157,6 +2176,11 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         e.ksplit = (kb + kper - 1) / kper;
     }
     e.split_stride = 0;
+    e.wait_cnt = g.wait_cnt;
+    e.wait_T = g.wait_T;
+    e.wait_B = g.wait_B > 0 ? g.wait_B : 1;
+    e.wait_per = g.wait_per;
+    if (g.wait_cnt && (g.epi != EPI_F32 || !g.atomic_out || g.conv.taps)) return cudaErrorInvalidValue;
     e.bias = g.bias;
     e.relu = g.relu;
     e.mask = static_cast<const __nv_bfloat16 *>(g.mask);

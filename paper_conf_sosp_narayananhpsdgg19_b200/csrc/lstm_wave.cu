@@ -149,6 +149,9 @@ struct WaveArgs {
     WaveLayer layer[LSTM_WAVE_MAX_L];
     const __nv_bfloat16 *dy_top;  // backward: gradient w.r.t. the top layer's output [T][B][H]
     unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
+    unsigned *started;            // optional: +1 per CTA at its start (residency signal) ...
+    volatile unsigned *started_host;  // ... the last CTA writes `epoch` here (mapped host memory)
+    unsigned epoch;
     unsigned long long *probe;    // tools only (PD_WAVE_PROBE): [CTA][visit < PROBE_V][8] %globaltimer
     int keep_layers;              // weights of layers < keep_layers load with L2 evict_last, the rest
                                   // evict_first (0: no hint): a fixed subset stays L2-resident across
@@ -267,6 +270,13 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
     if (CL > 1) cluster_sync_all();  // the peers' barriers exist before any remote arrive / st.async
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    if (tid == 0 && a.started) {  // this CTA is resident; the last one tells the host
+        if (atomicAdd(a.started, 1u) == gridDim.x - 1 && a.started_host) {
+            __threadfence_system();
+            *a.started_host = a.epoch;
+            __threadfence_system();
+        }
+    }
     // published (step, tile, CTA) items of a layer per completed step
     const unsigned per_step = (unsigned)a.tiles * CL;
 
@@ -708,6 +718,13 @@ int choose_cl(bool bwd, int items) {
 
 }  // namespace
 
+int lstm_wave_grid(bool bwd, int L, int H, int *cl_out) {
+    const int items = L * (bwd ? H / 128 : H / 32);
+    const int cl = choose_cl(bwd, items);
+    if (cl_out) *cl_out = cl;
+    return cl * std::min(items, max_clusters(bwd, cl));
+}
+
 bool lstm_wave_supported(int L, int B, int H, int I) {
     if (L < 1 || L > LSTM_WAVE_MAX_L || B < 1 || B > 64 || H < 128 || H % 128 || I != H) return false;
     return max_clusters(false, 1) >= 1 && max_clusters(true, 2) >= 1;
@@ -751,6 +768,10 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
     if (!w.bwd && !tma_map_bf16(&m.act[0], w.x, H, TB, H, 64, a.N)) return cudaErrorInvalidValue;
     cudaError_t e = cudaMemsetAsync(w.cnt, 0, sizeof(unsigned) * L, s);
     if (e != cudaSuccess) return e;
+    a.started = w.started;
+    a.started_host = w.started_host;
+    a.epoch = w.epoch;
+    if (w.started && (e = cudaMemsetAsync(w.started, 0, sizeof(unsigned), s)) != cudaSuccess) return e;
     const int items = L * a.tiles;
     const int cl = choose_cl(w.bwd, items);
     const int grid = cl * std::min(items, max_clusters(w.bwd, cl));

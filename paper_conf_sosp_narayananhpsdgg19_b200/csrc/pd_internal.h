@@ -115,6 +115,13 @@ struct Gemm {
     // griddepcontrol.wait.  Only for a GEMM whose predecessor is the previous layer's GEMM of
     // the same chain (whose first kernel launched normally), so B is never being written.
     int pdl = 0;
+    // wait for a producer kernel running concurrently (EPI_F32 with explicit ksplit): before
+    // loading the K-blocks [kb0, kb1) of a unit, wait until *wait_cnt >= (wait_T - kb0*64 /
+    // wait_B) * wait_per (acquire) -- rows r of A belong to step r / wait_B, and the producer
+    // completes steps in descending order; the splits then run last-rows first
+    const unsigned *wait_cnt = nullptr;
+    int wait_T = 0, wait_B = 1;
+    unsigned wait_per = 0;
 };
 
 // cached 2-D bf16 tensor map (128B swizzle), row-major [outer][ld_elems], box {box_inner, box_outer}
@@ -199,8 +206,17 @@ struct LstmWaveDesc {
     __nv_bfloat16 *h_out = nullptr;  // forward: second destination of the top layer's h (the stage
                                      // output: the consumer's receive slot, possibly peer memory)
     unsigned *cnt = nullptr;  // >= L uints (zeroed by lstm_wave on the stream)
+    // optional residency signal: every CTA of the wave adds 1 to *started (device, zeroed by
+    // lstm_wave) at its start; the last one writes `epoch` to *started_host (mapped pinned host
+    // memory), so the host can launch work that must not take the wave's SMs first
+    unsigned *started = nullptr;
+    volatile unsigned *started_host = nullptr;  // device pointer of the mapped host word
+    unsigned epoch = 0;
 };
 bool lstm_wave_supported(int L, int B, int H, int I);
+// CTAs of the wave launch lstm_wave would issue for an L-layer run (H hidden units); *cl =
+// its cluster K-split (a layer's timestep counts as done at cnt >= (done steps) * (H/128) * cl)
+int lstm_wave_grid(bool bwd, int L, int H, int *cl = nullptr);
 cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s);
 cudaError_t lstm_cell_bwd(int bf16, const void *dy, const float *dh_rec, const float *gates, const float *c,
                           const float *c_prev, float *dc, void *da, int B, int H, cudaStream_t s);

@@ -310,6 +310,12 @@ struct Worker {
     void *lstm_wda = nullptr;      // wavefront backward: da of every layer of an LSTM run
     int lstm_wmax = 0;             // ... for runs of up to this many layers
     float *lstm_wdc = nullptr;     // ... and their dc carries
+    // weight gradients of a short wavefront run computed while its backward wave runs (one
+    // stream + completion event per GEMM: 2 per layer, runs of <= 3 layers)
+    cudaStream_t dw_stream[6] = {};
+    cudaEvent_t dw_ev[6] = {};
+    unsigned *wave_flag = nullptr;  // mapped pinned host word: the backward wave is resident (epoch)
+    unsigned wave_epoch = 0;
     int lstm_rec = -1;             // persistent recurrences usable (-1 = not decided yet)
     // CUDA graphs of the LSTM recurrences (T steps of small GEMM + cell kernels), keyed by
     // (layer, direction, saved-state slot, weight slot, dY pointer): replayed instead of
@@ -379,6 +385,11 @@ Worker::~Worker() {
     for (auto &kv : opgraphs) cudaGraphExecDestroy(kv.second.first);
     if (loss_scratch) cudaFree(loss_scratch);
     for (cudaEvent_t e : ev_dx) cudaEventDestroy(e);
+    for (int i = 0; i < 6; ++i) {
+        if (dw_ev[i]) cudaEventDestroy(dw_ev[i]);
+        if (dw_stream[i]) cudaStreamDestroy(dw_stream[i]);
+    }
+    if (wave_flag) cudaFreeHost(wave_flag);
     for (cudaEvent_t e : ev_dw) cudaEventDestroy(e);
     if (ev_fork) cudaEventDestroy(ev_fork);
     if (side) cudaStreamDestroy(side);
@@ -1127,6 +1138,126 @@ struct Exec {
         kend(4, k0);
     }
 
+    // Backward wave of a short run (<= 3 layers: the wave leaves >= 52 SMs idle) with the run's
+    // weight gradients computed WHILE the wave runs, on the idle SMs: the W_ih / W_hh GEMMs of
+    // every layer (6 streams) split K = T*B into chunks of timesteps, run the chunks last
+    // timesteps first, and wait per chunk for the wave's step counter of that layer (the wave
+    // finishes timesteps in descending order), reduce-adding fp32 partials into the zeroed
+    // gradient; the optimizer updates follow the wave.  The GEMM streams launch only once
+    // every CTA of the wave is resident (a stream wait on the wave's start counter), so they
+    // can never take SMs the spinning wave needs.  Only for a worker alone on its GPU.
+    // Returns false (nothing issued) when not applicable.
+    bool wave_dw_overlap(int l0, int L, int t, int j, LstmWaveDesc &wd, void *dx, const BwdCtx &bc) {
+        if (!bc.fused || L > 3 || !w->dw_stream[0]) return false;
+        if (const char *e = getenv("PD_WAVE_DW")) {  // 0: weight gradients after the wave (tests)
+            if (atoi(e) == 0) return false;
+        }
+        for (auto &o : c->W)
+            if (o && o.get() != w && o->device == w->device) return false;
+        const int T = wd.T, Bn = wd.B, H = wd.H;
+        int wcl = 0;
+        const int wgrid = lstm_wave_grid(true, L, H, &wcl);
+        int sms = 0;
+        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, w->device));
+        const int ng = 2 * L;
+        const int cap = (sms - wgrid) / ng / 2 * 2;  // CTAs per GEMM (pairs)
+        if (cap < 4) return false;
+        const long TB = (long)T * Bn;
+        unsigned *started = w->lstm_cnt + LSTM_WAVE_MAX_L;
+        unsigned *flag_dev = nullptr;
+        CK(cudaHostGetDevicePointer(reinterpret_cast<void **>(&flag_dev), w->wave_flag, 0));
+        // zeroed gradients (reduce-add targets), then the wave; the gradient GEMMs are launched
+        // only once the host sees every wave CTA resident (a device-side gate could let them
+        // take the SMs the wave's clusters need first)
+        for (int i = 0; i < L; ++i)
+            for (int m = 0; m < 2; ++m)
+                CK(cudaMemsetAsync(w->gbuf + lstm_off(l0 + i, m), 0, (size_t)4 * H * H * 4, w->stream));
+        CK(cudaEventRecord(w->ev_fork, w->stream));
+        wd.started = started;
+        wd.started_host = flag_dev;
+        wd.epoch = ++w->wave_epoch;
+        cudaEvent_t k0 = kstart(5);
+        CK(lstm_wave(wd, w->stream));
+        kend(5, k0);
+        {
+            const auto t0 = std::chrono::steady_clock::now();
+            while (*reinterpret_cast<volatile unsigned *>(w->wave_flag) != wd.epoch) {
+                if (c->abort) throw Abort{};
+                if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(20))
+                    throw CudaFail{cudaErrorLaunchTimeout, "backward wave never became resident"};
+                std::this_thread::yield();
+            }
+        }
+        const int chunk_steps = 10;  // availability granularity (the chunk's K = 10 * B rows)
+        // the new version goes to another slot than the one the wave reads (k_s >= 2): each
+        // matrix's optimizer update can follow its gradient GEMM on the same stream, under the
+        // wave; with k_s = 1 (in place) the updates wait for the wave and the bottom layer's dX
+        const bool early = bc.nslot != bc.sslot;
+        const bool adam = c->cfg.optimizer == PD_ADAM;
+        int g = 0;
+        for (int i = L - 1; i >= 0; --i)
+            for (int m = 0; m < 2; ++m, ++g) {
+                const int l = l0 + i;
+                cudaStream_t st = w->dw_stream[g];
+                CK(cudaStreamWaitEvent(st, w->ev_fork, 0));
+                const int steps = m == 0 ? T : T - 1;  // W_hh pairs da[t+1] with h[t]
+                Gemm gg;
+                gg.M = 4 * H;
+                gg.N = H;
+                gg.K = (int)((long)steps * Bn);
+                gg.A = m == 0 ? static_cast<const void *>(wd.da[i]) : elem_ptr(wd.da[i], (long)Bn * 4 * H, esz);
+                gg.lda = 4 * H;
+                gg.amaj = MNMAJ;
+                gg.B = m == 0 ? layer_input(l, t, j) : lstm_state(l, j).h;
+                gg.ldb = H;
+                gg.bmaj = MNMAJ;
+                gg.epi = EPI_F32;
+                gg.atomic_out = 1;
+                gg.ksplit = (steps + chunk_steps - 1) / chunk_steps;
+                gg.out = w->gbuf + lstm_off(l, m);
+                gg.ldo = H;
+                gg.max_ctas = cap;
+                gg.wait_cnt = w->lstm_cnt + i;
+                gg.wait_T = steps;  // row r of A is step r / B (+1 for W_hh), done at cnt >= (T - step) * per
+                gg.wait_B = Bn;
+                gg.wait_per = (unsigned)(H / 128) * (unsigned)wcl;
+                CK(run_gemm(1, gg, st));
+                if (early) {  // this matrix's update right behind its gradient (still under the wave)
+                    const long woff = lstm_off(l, m);
+                    CK(update_from_grad(w->master + woff,
+                                        static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], woff, esz)),
+                                        w->gbuf + woff, 4L * H * H, c->cfg.optimizer, adam ? w->adam_m + woff : nullptr,
+                                        adam ? w->adam_v + woff : nullptr, c->cfg.lr, c->cfg.beta1, c->cfg.beta2,
+                                        c->cfg.eps, w->updates_total + 1, st));
+                }
+                CK(cudaEventRecord(w->dw_ev[g], st));
+            }
+        // the bottom layer's input gradient, then (after every gradient GEMM) the updates: with
+        // k_s = 1 the W_ih update is in place and dX reads W_ih
+        k0 = kstart(1);
+        if (dx) gemm_dx(l0, (int)TB, H, 4 * H, wd.da[0], 4 * H, wd.W_ih[0], H, layer_input(l0, t, j), dx);
+        kend(1, k0);
+        for (int i = L - 1; i >= 0; --i) {  // biases: sums over the whole da, after the wave
+            k0 = kstart(3);
+            bias_update_pair(bc, lstm_off(l0 + i, 2), lstm_off(l0 + i, 3), wd.da[i], TB, 4 * H);
+            kend(3, k0);
+        }
+        for (int k = 0; k < ng; ++k) CK(cudaStreamWaitEvent(w->stream, w->dw_ev[k], 0));
+        if (!early)
+            for (int i = L - 1; i >= 0; --i)
+                for (int m = 0; m < 2; ++m) {
+                    const long woff = lstm_off(l0 + i, m);
+                    k0 = kstart(7);
+                    CK(update_from_grad(w->master + woff,
+                                        static_cast<__nv_bfloat16 *>(elem_ptr(w->wslot[bc.nslot], woff, esz)),
+                                        w->gbuf + woff, 4L * H * H, c->cfg.optimizer, adam ? w->adam_m + woff : nullptr,
+                                        adam ? w->adam_v + woff : nullptr, c->cfg.lr, c->cfg.beta1, c->cfg.beta2,
+                                        c->cfg.eps, w->updates_total + 1, w->stream));
+                    kend(7, k0);
+                }
+        return true;
+    }
+
     void lstm_wave_backward(int l0, int L, int t, int j, const void *G, void *dx, const BwdCtx &bc) {
         const pd_layer_desc &d = layer(l0);
         const int T = d.seq_len, Bn = B(), H = d.out;
@@ -1146,6 +1277,7 @@ struct Exec {
             wd.da[i] = static_cast<__nv_bfloat16 *>(elem_ptr(w->lstm_wda, (long)i * TB * 4 * H, esz));
             wd.dc[i] = w->lstm_wdc + (long)i * Bn * H;
         }
+        if (wave_dw_overlap(l0, L, t, j, wd, dx, bc)) return;
         cudaEvent_t k0 = kstart(5);
         CK(lstm_wave(wd, w->stream));
         kend(5, k0);
@@ -2127,6 +2259,12 @@ pd_status pd_stage_init(pd_ctx *c, int stage, int replica, int dev, const float 
                 w->lstm_wmax = std::min(longest, LSTM_WAVE_MAX_L);
                 w->lstm_wda = dalloc<void>((size_t)w->lstm_wmax * tb4h * esz);
                 w->lstm_wdc = dalloc<float>((size_t)w->lstm_wmax * bh * 4);
+                for (int i = 0; i < 6; ++i) {
+                    CK(cudaStreamCreateWithFlags(&w->dw_stream[i], cudaStreamNonBlocking));
+                    CK(cudaEventCreateWithFlags(&w->dw_ev[i], cudaEventDisableTiming));
+                }
+                CK(cudaHostAlloc(reinterpret_cast<void **>(&w->wave_flag), 64, cudaHostAllocMapped));
+                *w->wave_flag = 0;
             }
         }
         if (gx_elems) {

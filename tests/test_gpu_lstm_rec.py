@@ -140,3 +140,23 @@ def test_split_weight_gradient_path_matches_oracle(opt):
     else:  # Adam moves every weight by ~lr*sign(g): compare parameters, not deltas
         assert torchref.max_rel_err(a["got"], b["got"]) < 2e-2
     np.testing.assert_allclose(a["losses"], b["losses"], rtol=2e-3)
+
+
+# Weight gradients of a short wavefront run computed on the idle SMs WHILE the backward wave
+# runs (runtime wave_dw_overlap: chunks of 10 timesteps, last first, each waiting for the
+# wave's step counter; reduce-added fp32 partials): against the oracle, and against the
+# gradients computed after the wave (PD_WAVE_DW=0) -- equal up to the fp32 order of the chunk
+# sums.  (3, 512, 32, 21): 3 chunks per GEMM; (2, 256, 40, 23): chunk boundaries inside a
+# 64-row K-block (B = 40).
+@pytest.mark.parametrize("n,H,B,T", [(3, 512, 32, 21), (2, 256, 40, 23)])
+def test_wave_weight_gradients_overlapped(n, H, B, T):
+    wl = _workload(n, H, B, T)
+    last = [len(wl.layers) - 1]
+    a = _run_env(wl, last, 2, {"PD_LSTM_REC": "1", "PD_LSTM_WAVE": "1", "PD_WAVE_DW": "1"})
+    b = _run_env(wl, last, 2, {"PD_LSTM_REC": "1", "PD_LSTM_WAVE": "1", "PD_WAVE_DW": "0"})
+    assert_schedule_exact(a)
+    perr, derr = param_errors(a)
+    assert perr < BF16_TOL and derr < 5e-2, (perr, derr)
+    d = torchref.delta_err(a["got"], b["got"], a["p0"])
+    assert d < 1e-2, d
+    np.testing.assert_allclose(a["losses"], b["losses"], rtol=1e-5)
