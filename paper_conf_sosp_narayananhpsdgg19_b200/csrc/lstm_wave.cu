@@ -149,8 +149,8 @@ struct WaveArgs {
     WaveLayer layer[LSTM_WAVE_MAX_L];
     const __nv_bfloat16 *dy_top;  // backward: gradient w.r.t. the top layer's output [T][B][H]
     unsigned *cnt;                // per-layer completed (step, tile) items, zeroed by the caller
-    unsigned *started;            // optional: +1 per CTA at its start (residency signal) ...
-    volatile unsigned *started_host;  // ... the last CTA writes `epoch` here (mapped host memory)
+    unsigned *started;            // optional residency signal (LstmWaveDesc::started)
+    volatile unsigned *started_host;
     unsigned epoch;
     unsigned long long *probe;    // tools only (PD_WAVE_PROBE): [CTA][visit < PROBE_V][8] %globaltimer
     int keep_layers;              // weights of layers < keep_layers load with L2 evict_last, the rest
@@ -226,7 +226,9 @@ __device__ __forceinline__ uint32_t cluster_rank() {
 // each to stage, 8 of a thread's 16 units each in the cell
 constexpr int WAVE_THREADS = 384;
 
-template <bool BWD, int CL>
+// SIG: the residency signal (WaveArgs::started) is compiled in only where a caller asks for it --
+// the few instructions at the top measured 4.5 % slower waves when present in every instantiation
+template <bool BWD, int CL, bool SIG = false>
 __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid_constant__ WaveMaps m, const WaveArgs a) {
     constexpr int NE = WAVE_THREADS - 128;  // epilogue threads
     using WC = WaveCfg<BWD, CL>;
@@ -270,8 +272,8 @@ __global__ void __launch_bounds__(WAVE_THREADS, 1) lstm_wave_kernel(const __grid
     if (CL > 1) cluster_sync_all();  // the peers' barriers exist before any remote arrive / st.async
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
-    if (tid == 0 && a.started) {  // this CTA is resident; the last one tells the host
-        if (atomicAdd(a.started, 1u) == gridDim.x - 1 && a.started_host) {
+    if (SIG && tid == 0) {  // this CTA is resident; the last one tells the host
+        if (atomicAdd(a.started, 1u) == gridDim.x - 1) {
             __threadfence_system();
             *a.started_host = a.epoch;
             __threadfence_system();
@@ -731,7 +733,7 @@ bool lstm_wave_supported(int L, int B, int H, int I) {
 }
 
 // the smallest wave grid that runs every item: CL CTAs per item up to the resident clusters
-template <bool BWD, int CL>
+template <bool BWD, int CL, bool SIG = false>
 cudaError_t launch_wave(const WaveMaps &m, const WaveArgs &a, int items, cudaStream_t s) {
     const int mc = max_clusters<BWD, CL>();
     if (mc < 1) return cudaErrorNotSupported;
@@ -739,7 +741,16 @@ cudaError_t launch_wave(const WaveMaps &m, const WaveArgs &a, int items, cudaStr
     cudaLaunchAttribute attr[1];
     cudaLaunchConfig_t cfg = wave_cfg<BWD, CL>(CL * clusters, s, attr);
     ++tl_launches;
-    return cudaLaunchKernelEx(&cfg, lstm_wave_kernel<BWD, CL>, m, a);
+    if (SIG) {
+        static bool attr = false;  // (max_clusters set the attribute of the SIG = false twin)
+        if (!attr) {
+            const cudaError_t e = cudaFuncSetAttribute(lstm_wave_kernel<BWD, CL, true>,
+                                                       cudaFuncAttributeMaxDynamicSharedMemorySize, WaveCfg<BWD, CL>::SMEM);
+            if (e != cudaSuccess) return e;
+            attr = true;
+        }
+    }
+    return cudaLaunchKernelEx(&cfg, lstm_wave_kernel<BWD, CL, SIG>, m, a);
 }
 
 cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
@@ -797,6 +808,9 @@ cudaError_t lstm_wave(const LstmWaveDesc &w, cudaStream_t s) {
         if (pbuf && cudaMemsetAsync(pbuf, 0, pbytes, s) == cudaSuccess) a.probe = pbuf;
     }
     if (!w.bwd) e = cl == 2 ? launch_wave<false, 2>(m, a, items, s) : launch_wave<false, 1>(m, a, items, s);
+    else if (a.started && a.started_host) e = cl == 8 ? launch_wave<true, 8, true>(m, a, items, s)
+                          : cl == 4 ? launch_wave<true, 4, true>(m, a, items, s)
+                                    : launch_wave<true, 2, true>(m, a, items, s);
     else if (cl == 8) e = launch_wave<true, 8>(m, a, items, s);
     else if (cl == 4) e = launch_wave<true, 4>(m, a, items, s);
     else e = launch_wave<true, 2>(m, a, items, s);

@@ -206,11 +206,12 @@ struct LstmWaveDesc {
     __nv_bfloat16 *h_out = nullptr;  // forward: second destination of the top layer's h (the stage
                                      // output: the consumer's receive slot, possibly peer memory)
     unsigned *cnt = nullptr;  // >= L uints (zeroed by lstm_wave on the stream)
-    // optional residency signal: every CTA of the wave adds 1 to *started (device, zeroed by
-    // lstm_wave) at its start; the last one writes `epoch` to *started_host (mapped pinned host
-    // memory), so the host can launch work that must not take the wave's SMs first
+    // optional residency signal (backward): every CTA of the wave adds 1 to *started (device,
+    // zeroed by lstm_wave) when it starts and the last one writes `epoch` to *started_host (device
+    // pointer of a mapped pinned host word), so the host can launch work that must not take the
+    // wave's SMs before all of them are resident
     unsigned *started = nullptr;
-    volatile unsigned *started_host = nullptr;  // device pointer of the mapped host word
+    volatile unsigned *started_host = nullptr;
     unsigned epoch = 0;
 };
 bool lstm_wave_supported(int L, int B, int H, int I);

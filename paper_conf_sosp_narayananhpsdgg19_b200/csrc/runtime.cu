@@ -1163,7 +1163,6 @@ struct Exec {
         const int cap = (sms - wgrid) / ng / 2 * 2;  // CTAs per GEMM (pairs)
         if (cap < 4) return false;
         const long TB = (long)T * Bn;
-        unsigned *started = w->lstm_cnt + LSTM_WAVE_MAX_L;
         unsigned *flag_dev = nullptr;
         CK(cudaHostGetDevicePointer(reinterpret_cast<void **>(&flag_dev), w->wave_flag, 0));
         // zeroed gradients (reduce-add targets), then the wave; the gradient GEMMs are launched
@@ -1173,7 +1172,7 @@ struct Exec {
             for (int m = 0; m < 2; ++m)
                 CK(cudaMemsetAsync(w->gbuf + lstm_off(l0 + i, m), 0, (size_t)4 * H * H * 4, w->stream));
         CK(cudaEventRecord(w->ev_fork, w->stream));
-        wd.started = started;
+        wd.started = w->lstm_cnt + LSTM_WAVE_MAX_L;
         wd.started_host = flag_dev;
         wd.epoch = ++w->wave_epoch;
         cudaEvent_t k0 = kstart(5);
