@@ -1154,6 +1154,9 @@ struct Exec {
         }
         for (auto &o : c->W)
             if (o && o.get() != w && o->device == w->device) return false;
+        cudaStreamCaptureStatus cap_st = cudaStreamCaptureStatusNone;  // (the host gate cannot be captured)
+        CK(cudaStreamIsCapturing(w->stream, &cap_st));
+        if (cap_st != cudaStreamCaptureStatusNone) return false;
         const int T = wd.T, Bn = wd.B, H = wd.H;
         int wcl = 0;
         const int wgrid = lstm_wave_grid(true, L, H, &wcl);
