@@ -1136,7 +1136,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 // descriptor's leading byte offset.  The weights W [Co][72] (+ a zero K = 72..79 slot) stay
 // resident in shared memory for the whole persistent launch.
 constexpr int C8_NS = 6;  // span ring depth
-__global__ void __launch_bounds__(NUM_THREADS, 1)
+constexpr int C8_THREADS = 384;  // two epilogue groups of 4 warps: even / odd tiles (accumulator 0 / 1)
+__global__ void __launch_bounds__(C8_THREADS, 1)
     conv_c8_fwd_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__ CUtensorMap tmO,
                        const __nv_bfloat16 *__restrict__ X, EpiArgs e, int M, int N, int span_bytes) {
     constexpr int BNW = 64;  // output channels (N <= 64)
@@ -1144,8 +1145,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint8_t *sB = smem;                                   // 10 slots x 64 rows x 16 B
     uint8_t *ring = smem + 10 * 1024;                     // C8_NS spans
-    uint8_t *epi_stg = ring + C8_NS * span_bytes;         // 4 warps x 2 x 2 KB (1024-aligned: span_bytes % 1024 == 0)
-    uint64_t *bars = reinterpret_cast<uint64_t *>(epi_stg + 4 * 4096);
+    uint8_t *epi_stg = ring + C8_NS * span_bytes;         // 8 warps x 2 x 2 KB (1024-aligned: span_bytes % 1024 == 0)
+    uint64_t *bars = reinterpret_cast<uint64_t *>(epi_stg + 8 * 4096);
     uint64_t *full = bars, *empty = bars + C8_NS, *tfull = bars + 2 * C8_NS, *tempty = tfull + 2, *bbar = tempty + 2;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bbar + 1);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -1173,7 +1174,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     // zero the span ring once: window rows a clipped copy leaves unwritten (the image's first /
     // last halo) then hold finite values -- they only feed border outputs, which are zeroed
-    for (int i = threadIdx.x; i < C8_NS * span_bytes / 16; i += NUM_THREADS)
+    for (int i = threadIdx.x; i < C8_NS * span_bytes / 16; i += C8_THREADS)
         reinterpret_cast<uint4 *>(ring)[i] = make_uint4(0, 0, 0, 0);
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     tc_fence_before();
@@ -1230,11 +1231,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             }
         }
     } else if (warp >= 4) {  // ===== epilogue: bias + ReLU + zero border, bf16 TMA stores
-        const int q = warp & 3;
-        uint8_t *wst = epi_stg + q * 4096;
-        int acc = 0;
+        // group g = (warp - 4) / 4 takes this CTA's tiles of parity g (accumulator g): two tiles'
+        // epilogues in flight, the epilogue (not the loads or the MMAs) bounds this kernel
+        const int q = warp & 3, grp = (warp - 4) >> 2;
+        uint8_t *wst = epi_stg + (warp - 4) * 4096;
+        const int acc = grp;
         uint32_t acc_phase = 0, ocnt = 0;
-        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        for (int tile = blockIdx.x + grp * gridDim.x; tile < tiles; tile += 2 * gridDim.x) {
             mbar_wait(smem_u32(&tfull[acc]), acc_phase);
             tc_fence_after();
             const int r0 = tile * BM + q * 32;
@@ -1258,7 +1261,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
-            if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+            acc_phase ^= 1;
         }
         if (lane == 0) bulk_wait_read0();
     }
@@ -2002,7 +2005,7 @@ static cudaError_t gemm_c8(const Gemm &g, cudaStream_t s) {
         if (!make_map(&mbm, g.B, 72, g.N, g.ldb, 8, 64, false, 0) || !make_map(&mo, g.out, g.N, g.M, g.ldo, 32, 32, false, 64))
             return cudaErrorInvalidValue;
         const int span = ((BM + 2 * (g.conv.Wp + 1)) * 16 + 1023) / 1024 * 1024;
-        const int smem = 10 * 1024 + C8_NS * span + 4 * 4096 + 256 + 1024;
+        const int smem = 10 * 1024 + C8_NS * span + 8 * 4096 + 256 + 1024;
         if (smem > 232448) return cudaErrorInvalidValue;
         static int attr_smem = 0;
         if (smem > attr_smem) {
@@ -2012,7 +2015,7 @@ static cudaError_t gemm_c8(const Gemm &g, cudaStream_t s) {
         }
         const int tiles = (g.M + BM - 1) / BM;
         const int grid = tiles < num_sms() ? tiles : num_sms();
-        conv_c8_fwd_kernel<<<grid, NUM_THREADS, smem, s>>>(mbm, mo, static_cast<const __nv_bfloat16 *>(g.A), e, g.M, g.N,
+        conv_c8_fwd_kernel<<<grid, C8_THREADS, smem, s>>>(mbm, mo, static_cast<const __nv_bfloat16 *>(g.A), e, g.M, g.N,
                                                           span);
         ++tl_launches;
         return cudaGetLastError();
