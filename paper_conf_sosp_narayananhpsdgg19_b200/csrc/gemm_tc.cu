@@ -1943,7 +1943,10 @@ static int env_int(const char *name, int dflt) {
 // 2-CTA pairs (M = 256 per MMA) for every plain GEMM with at least 256 rows
 static int use_pairs(const Gemm &g) {
     if (env_int("PD_GEMM_CG", 2) == 1) return 1;
-    // N <= 64 would leave the second CTA's half of B empty (zero columns): single CTAs there
+    // N <= 64 would leave the second CTA's half of B empty (zero columns) with 128-wide pair
+    // tiles -- except the implicit-GEMM conv forward at N = 64 (K-major weights), which runs
+    // 256 x 64 pair tiles (each CTA stages 32 weight rows: 20 KB per K-block instead of 24)
+    if (g.M >= 256 && g.N == 64 && g.conv.taps && g.bmaj == KMAJ && g.epi == EPI_STORE && !g.conv.c8) return 2;
     return (g.M >= 256 && g.N > 64 && (g.epi == EPI_STORE || g.epi == EPI_MASK || g.epi == EPI_F32)) ? 2 : 1;
 }
 
@@ -2129,6 +2132,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
         const long slots = sms / 2, t256 = pm * ((g.N + 255) / 256), t128 = pm * ((g.N + 127) / 128);
         const long c256 = (t256 + slots - 1) / slots * 32, c128 = (t128 + slots - 1) / slots * 24;
         if (c128 < c256 || g.N <= 128) BN = 128;
+        if (g.N <= 64) BN = 64;  // (use_pairs allows it for the conv forward only)
     } else {
         if ((long)mb * ((g.N + 255) / 256) < sms || g.N <= 128) BN = 128;
         if (BN == 128 && ((long)mb * ((g.N + 127) / 128) < sms || g.N <= 64)) BN = 64;
@@ -2139,7 +2143,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     // per 24 KB; the ingest of ~90 GB/s per SM bounds these tiles)
     if (g.atomic_out && g.ksplit == 0 && g.N >= 256 && !g.conv.c8) BN = 256;
     BN = env_int("PD_GEMM_BN", BN);  // tuning override (tools/gemm_bench.py)
-    if (cg == 2 && BN < 128) BN = 128;
+    if (cg == 2 && BN < 128 && g.N > 64) BN = 128;
     CUtensorMap ma, mbm;
     // implicit-GEMM conv: the tensors are [rows][channels] / [Cout][9*Cp]; the K walk over
     // (tap, channel block) is done by the producer's coordinates, not by the map extents
@@ -2197,6 +2201,7 @@ cudaError_t gemm_bf16(const Gemm &g, cudaStream_t s) {
     e.bc2 = 1.f - powf(g.b2, (float)g.step);
     if (cg == 2) {
         if (BN == 256) return dispatch_major<256, 2>(g, ma, mbm, e, s);
+        if (BN == 64) return launch<64, KMAJ, KMAJ, EPI_STORE, 2>(g, ma, mbm, e, s);  // (use_pairs: conv fwd only)
         return dispatch_major<128, 2>(g, ma, mbm, e, s);
     }
     if (BN == 256) return dispatch_major<256>(g, ma, mbm, e, s);
